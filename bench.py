@@ -1,0 +1,362 @@
+#!/usr/bin/env python3
+"""Benchmark of the WinRS fused Winograd BFC on B200 (BASELINE.json metric:
+effective TFLOPS = direct-conv FLOPs 2*N*C*K*Ho*Wo*R*S / device time, plus
+workspace bytes).
+
+A "step" is one pass of the whole hot path (plan is prebuilt; fused kernels +
+bucket reduction) over every layer of the workload, inputs resident in HBM.
+Default workload: configs[1] of BASELINE.json — the four ResNet-50 3x3 layers
+at N=64 (C=K=64/128/256/512, H=W=56/28/14/7, pad 1).  L2 is flushed (a
+256 MiB write) before every layer call and each call is timed with CUDA events
+on the launch stream (the flush is outside the timed events).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--dtype f16|f32] [--impl winrs|reference]
+
+N > 1 (torchrun): each rank runs the same per-rank workload on its own batch
+shard (weak scaling: global batch = N * 64) followed by one NCCL all_reduce of
+each layer's dW — the batch-sharded data-parallel BFC; time = max over ranks.
+--impl reference runs the FP64 CPU oracle (the only reference this paper-only
+tier has) on a bounded sample of the same workload, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "effective TFLOPS (direct-conv FLOPs) + workspace bytes per BFC layer"
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+def _workload(name: str, dtype: str):
+    from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+    if name == "r50":
+        return wl.RESNET50_F32 if dtype == "f32" else wl.RESNET50_F16
+    if name == "vgg":
+        return wl.VGG16_F16
+    if name == "wide":
+        return wl.WIDE_F32
+    if name == "r50l3":
+        return [wl.LAYERS["r50_l3_n512_f16"]]
+    raise ValueError(name)
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+        self.t = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        sm = [float(r[0]) for r in self.rows if len(r) >= 7 and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) >= 7 and r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            if len(r) >= 7:
+                for nme, v in zip(names, r[3:7]):
+                    if v.lower() == "active":
+                        reasons.add(nme)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def run_winrs(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_zhangc0zx0025_b200 as W
+    from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    layers = _workload(args.workload, args.dtype)
+    tdt = torch.float32 if args.dtype == "f32" else torch.float16
+
+    # Inputs resident in HBM (seeded, per-rank shard offset), plans prebuilt.
+    items = []
+    for l in layers:
+        X, dY = wl.make_inputs(l, seed_offset=1000 * rank)
+        p = W.plan(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype)
+        Xg = torch.from_numpy(X).to(dev)
+        Gg = torch.from_numpy(dY).to(dev)
+        dW = torch.empty((l.K, l.R, l.S, l.C), dtype=torch.float32, device=dev)
+        ws = torch.empty(max(p.workspace_bytes, 16), dtype=torch.uint8, device=dev)
+        items.append(dict(layer=l, plan=p, X=Xg, dY=Gg, dW=dW, ws=ws, Xh=torch.from_numpy(X).pin_memory(),
+                          Gh=torch.from_numpy(dY).pin_memory(), dWh=torch.empty(dW.shape).pin_memory()))
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    def one_step(timed_events=None):
+        for j, it in enumerate(items):
+            flush.fill_(j & 0xFF)                                  # evict L2 (outside the events)
+            if timed_events is not None:
+                timed_events[j][0].record(stream)
+            W.bfc(it["plan"], it["X"], it["dY"], it["dW"], it["ws"], stream)
+            if world > 1:
+                dist.all_reduce(it["dW"])
+            if timed_events is not None:
+                timed_events[j][1].record(stream)
+
+    for _ in range(args.warmup):
+        one_step()
+    torch.cuda.synchronize()
+
+    clocks = ClockSampler(local)
+    if rank == 0:
+        clocks.start()
+    ev = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)] for _ in items]
+          for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for s in range(args.steps):
+        one_step(ev[s])
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop() if rank == 0 else None
+
+    per_layer_ms = [sum(ev[s][j][0].elapsed_time(ev[s][j][1]) for s in range(args.steps)) / args.steps
+                    for j in range(len(items))]
+    step_ms = sum(per_layer_ms)
+    if world > 1:
+        t = torch.tensor([step_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        step_ms = float(t.item())
+
+    # Dominant kernel's live duration: time the fused kernel alone (no
+    # all_reduce) for the layer with the largest share, CUDA events on the stream.
+    dom = max(range(len(items)), key=lambda j: per_layer_ms[j])
+    it = items[dom]
+    p = it["plan"]
+    info = p.info
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    kt = []
+    for _ in range(max(3, args.steps)):
+        flush.fill_(1)
+        e0.record(stream)
+        W.bfc(p, it["X"], it["dY"], it["dW"], it["ws"], stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        kt.append(e0.elapsed_time(e1))
+    dom_ms = statistics.median(kt)
+
+    # End to end through the C ABI with host buffers (pinned), copies inside.
+    e2e_ms = []
+    for _ in range(max(2, min(args.steps, 5))):
+        tot = 0.0
+        for it2 in items:
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            dX = torch.empty_like(it2["X"])
+            dG = torch.empty_like(it2["dY"])
+            a.record(stream)
+            W.bfc_host(it2["plan"], it2["Xh"], it2["Gh"], it2["dWh"], dX, dG, it2["dW"], it2["ws"], stream)
+            b.record(stream)
+            torch.cuda.synchronize()
+            tot += a.elapsed_time(b)
+        e2e_ms.append(tot)
+    e2e = statistics.median(e2e_ms)
+    if world > 1:
+        t = torch.tensor([e2e], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e = float(t.item())
+
+    if rank == 0:
+        flops = sum(it["layer"].direct_flops for it in items) * world
+        value = flops / (step_ms * 1e-3) / 1e12
+        peaks, src = _peaks()
+        esz = 4 if args.dtype == "f32" else 2
+        l = it["layer"]
+        alg_bytes = esz * (l.N * l.H * l.W * l.C + l.N * l.Ho * l.Wo * l.K) + 4 * l.K * l.R * l.S * l.C * (
+            1 if info["Z"] == 1 else 2 * info["Z"] + 1)
+        if args.dtype == "f32":
+            peak = 148 * 128 * 2 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6 / 1e12
+            roof = {"bound": "alu", "achieved": info["ewm_flops"] / (dom_ms * 1e-3) / 1e12, "peak": peak,
+                    "unit": "TFLOP/s", "peak_source": "148 SMs x 128 FP32 lanes x 2 x sm_max_mhz (DESIGN.md)",
+                    "kernel": p.kernel_name, "layer": l.name}
+        else:
+            t_hbm = alg_bytes / (peaks["hbm_gbs"] * 1e9)
+            t_tc = info["ewm_flops"] / (peaks["bf16_tflops"] * 1e12)
+            if t_hbm >= t_tc:
+                roof = {"bound": "hbm", "achieved": alg_bytes / (dom_ms * 1e-3) / 1e9, "peak": peaks["hbm_gbs"],
+                        "unit": "GB/s", "peak_source": src}
+            else:
+                roof = {"bound": "tensor", "achieved": info["ewm_flops"] / (dom_ms * 1e-3) / 1e12,
+                        "peak": peaks["bf16_tflops"], "unit": "TFLOP/s", "peak_source": src + " (fp16 = bf16 rate)"}
+            roof.update(kernel=p.kernel_name, layer=l.name)
+        roof["frac"] = roof["achieved"] / roof["peak"]
+        roof["traffic"] = None
+        roof["alg_bytes"] = alg_bytes
+        roof["ewm_flops"] = info["ewm_flops"]
+        roof["kernel_ms"] = dom_ms
+        h2d = sum(it2["X"].numel() * it2["X"].element_size() + it2["dY"].numel() * it2["dY"].element_size()
+                  for it2 in items)
+        d2h = sum(it2["dW"].numel() * 4 for it2 in items)
+        out = {
+            "metric": METRIC,
+            "value": value,
+            "unit": "TFLOPS",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": step_ms,
+            "higher_is_better": True,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": args.dtype,
+            "data": "synthetic (seeded U[0,1), dY x 1e-2 for f16; PAPER.md P@50685)",
+            "config": {"workload": f"{args.workload}_{args.dtype}: " + ", ".join(x["layer"].name for x in items),
+                       "global_batch": layers[0].N * world, "parallelism": f"dp{world}" if world > 1 else "single",
+                       "l2": "flushed (256 MiB write) before every layer call; flush outside timed events",
+                       "layers": [{"name": x["layer"].name, "ms": per_layer_ms[j],
+                                   "tflops": x["layer"].direct_flops / (per_layer_ms[j] * 1e-3) / 1e12,
+                                   "workspace_bytes": x["plan"].workspace_bytes, "plan": repr(x["plan"]),
+                                   "kernel": x["plan"].kernel_name} for j, x in enumerate(items)]},
+            "roofline": roof,
+            "e2e": {"value": flops / (e2e * 1e-3) / 1e12, "unit": "TFLOPS", "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": d2h, "ms_per_step": e2e},
+            "gpu_launches": sum(x["plan"].launch_count for x in items) * args.steps,
+            "clocks": clk,
+        }
+        if not args.no_cpu_baseline:
+            out["cpu_baseline"] = cpu_baseline(layers, budget_s=args.cpu_seconds)
+        print(json.dumps(out))
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def cpu_baseline(layers, budget_s: float = 8.0):
+    """The FP64 oracle (oracle/, as it stands) on a bounded sample of the same
+    workload: each layer with its batch cut to the first n images, n grown
+    until the CPU time budget is used.  Reported in the same metric."""
+    from oracle import oracle as O
+    from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+    threads = len(os.sched_getaffinity(0))
+    n = 1
+    flops = 0.0
+    elapsed = 0.0
+    while True:
+        t0 = time.perf_counter()
+        f = 0.0
+        for l in layers:
+            s = l.with_(N=n)
+            X, dY = wl.make_inputs(s)
+            O.bfc_c(X, dY, s.R, s.S, s.pad, threads=threads)
+            f += s.direct_flops
+        dt = time.perf_counter() - t0
+        flops, elapsed = f, dt
+        if dt * 2 > budget_s or n * 2 > layers[0].N:
+            break
+        n *= 2
+    return {"value": flops / elapsed / 1e12, "unit": "TFLOPS", "cores": threads, "kind": "oracle",
+            "sample": f"every layer of the workload with N cut to {n} image(s) ({flops / 1e9:.2f} GFLOP, "
+                      f"{elapsed:.1f} s, FP64 C loop, OpenMP over k)"}
+
+
+def run_reference(args):
+    """--impl reference: the FP64 CPU oracle timed on the box's host cores on a
+    bounded sample per step; rank 0 only."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle import oracle as O
+    from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+    layers = _workload(args.workload, args.dtype)
+    threads = len(os.sched_getaffinity(0))
+    sample = [l.with_(N=1) for l in layers]
+    inputs = [wl.make_inputs(s) for s in sample]
+    for _ in range(args.warmup):
+        O.bfc_c(*inputs[0], sample[0].R, sample[0].S, sample[0].pad, threads=threads)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        for s, (X, dY) in zip(sample, inputs):
+            O.bfc_c(X, dY, s.R, s.S, s.pad, threads=threads)
+    dt = (time.perf_counter() - t0) / args.steps
+    flops = sum(s.direct_flops for s in sample)
+    v = flops / dt / 1e12
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "TFLOPS", "n_gpus": int(os.environ.get("WORLD_SIZE", "1")),
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{args.workload}_{args.dtype} (each layer at N=1)"},
+        "cpu_baseline": {"value": v, "unit": "TFLOPS", "cores": threads, "kind": "oracle",
+                         "sample": "every layer of the workload at N=1 per step"},
+        "e2e": {"value": v, "unit": "TFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="winrs", choices=["winrs", "reference"])
+    ap.add_argument("--workload", default="r50", choices=["r50", "vgg", "wide", "r50l3"])
+    ap.add_argument("--dtype", default=os.environ.get("WINRS_BENCH_DTYPE", "f32"), choices=["f32", "f16"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=8.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.workload in ("wide",):
+        args.dtype = "f32"
+    if args.workload in ("vgg", "r50l3"):
+        args.dtype = "f16"
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_winrs(args)
+
+
+if __name__ == "__main__":
+    main()

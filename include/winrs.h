@@ -1,0 +1,155 @@
+/*
+ * winrs.h — C ABI of the B200-native WinRS fused Winograd backward-filter
+ * convolution (BFC).  Implemented by libwinrs.so
+ * (paper_conf_icpp_zhangc0zx0025_b200/csrc/).
+ *
+ * Citations are character offsets into the single-line PAPER.md ("P@offset")
+ * plus the section; DESIGN.md lists every reading of the paper taken here.
+ *
+ * The operation (§2.2 P@10786 "BFC convolves X with nabla Y to
+ * compute filter gradients nabla W"; Table 1 P@14515 §3 for shapes/layouts):
+ *
+ *   Ho = H + 2*pad - R + 1,   Wo = W + 2*pad - S + 1
+ *   dW[k][r][s][c] = sum_{n,h,w} Xp[n][h+r-pad][w+s-pad][c] * dY[n][h][w][k]
+ *   (Xp = X with zero padding; stride 1, dilation 1, one group)
+ *
+ * Layouts (Table 1): X is NHWC [N][H][W][C]; dY is NHWC [N][Ho][Wo][K]; dW is
+ * KRSC [K][R][S][C] and is ALWAYS float32.  X and dY are both float32
+ * (WINRS_F32) or both IEEE binary16 (WINRS_F16).  These are exactly the
+ * physical orders of PyTorch channels_last activations and channels_last
+ * 4-D weights.
+ *
+ * Method (§3 P@15252-17405): a plan fixes the kernel pair
+ * Omega_a0(n0,r0) / Omega_a1(n1,r1) (§4.1 P@20377), the segment count and
+ * segment shape (§4.2 Alg. 1, §4.3 Alg. 2).  winrs_bfc launches the fused
+ * kernels over the segments of dY; each writes one of Z dW "buckets" (bucket 0
+ * is dW itself, buckets 1..Z-1 live in the workspace, P@15661), then one
+ * reduction kernel sums the buckets into dW in fixed order with FP32 Kahan
+ * summation (P@17126, P@39101).
+ *
+ * Ownership and threading:
+ *   - The caller owns X, dY, dW and the workspace.  The library never
+ *     allocates or frees device memory and never synchronises a stream.
+ *   - A plan is immutable after creation and may be used concurrently from
+ *     several host threads / streams as long as each concurrent call has its
+ *     own dW and workspace.
+ *   - dW is overwritten (beta = 0).  For a fixed plan and device the result
+ *     is bitwise deterministic (no floating-point atomics).
+ * Errors: status codes only; nothing is thrown across the ABI and the
+ * library never calls exit/abort.  Asynchronous device faults surface at the
+ * caller's next synchronisation (as with cuBLAS).
+ */
+#ifndef WINRS_H
+#define WINRS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define WINRS_API __attribute__((visibility("default")))
+#else
+#define WINRS_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum { WINRS_F32 = 0, WINRS_F16 = 1 } winrs_dtype_t;
+
+typedef enum {
+    WINRS_OK = 0,
+    WINRS_ERR_INVALID_ARG = 1,   /* bad dimension, null/unaligned pointer      */
+    WINRS_ERR_UNSUPPORTED = 2,   /* no kernel for S/dtype, channel alignment,
+                                    or the device is not sm_100                */
+    WINRS_ERR_WORKSPACE = 3,     /* workspace == NULL but workspace_bytes > 0  */
+    WINRS_ERR_CUDA = 4,          /* a CUDA launch/runtime error                */
+    WINRS_ERR_HOST_ALLOC = 5     /* host allocation of the plan failed         */
+} winrs_status_t;
+
+/* Opaque, host-owned plan. */
+typedef struct winrs_plan_s* winrs_plan_t;
+
+/* Device properties the planner uses (winrs_plan queries the current device;
+ * winrs_plan_for_device takes them explicitly, e.g. for host-only tests). */
+typedef struct {
+    int num_sms;      /* streaming multiprocessors (148 on B200)            */
+    int cc_major;     /* compute capability; the kernels are built for 10.0 */
+    int cc_minor;
+} winrs_device_t;
+
+/* Read-only description of a plan (all sizes in elements unless noted). */
+typedef struct {
+    int N, C, H, W, K, R, S, pad;
+    int dtype;                     /* winrs_dtype_t                                       */
+    int Ho, Wo;
+    int alpha0, n0, r0, k0;        /* bulk kernel Omega_alpha0(n0,r0), k0 units per row   */
+    int alpha1, n1, r1, k1;        /* residual kernel (alpha1 == 0: none), k1 units       */
+    int masked_cols;               /* zero-masked dY columns in the last residual unit    */
+    int z_hat;                     /* Alg. 1 estimate after Alg. 2 line 1                 */
+    int Z;                         /* number of dW buckets (block groups of Omega_alpha0) */
+    int seg_h, seg_w;              /* S^_H (rows per band), S^_W (dY columns per segment) */
+    int bands, seg_cols;           /* segment grid: bands x seg_cols Omega_alpha0 segments */
+    int tile_k0, tile_c0;          /* CTA tile B_N x B_M of the bulk kernel               */
+    int tile_k1, tile_c1;          /* CTA tile of the residual kernel                     */
+    long long ctas_main, ctas_resid, ctas_reduce;
+    size_t workspace_bytes;        /* (Z-1) * 4 * K*R*S*C, 0 when Z == 1                  */
+    double direct_flops;           /* 2*N*C*K*Ho*Wo*R*S (P@43462)                         */
+    double ewm_flops;              /* Winograd-domain EWM flops actually issued           */
+} winrs_plan_info_t;
+
+/* Create a plan for the current CUDA device.
+ *   dims: N,C,H,W (X), K (dY channels), R,S (dW height/width), pad (>= 0).
+ * Returns INVALID_ARG for a dimension <= 0, pad < 0, Ho < 1, Wo < 1 or a null
+ * `out`; UNSUPPORTED when S has no divisor n in {2..9} of the kernel set
+ * (§5 P@28451: F_W in {n*k : 2 <= k <= 9}), when C % 4 or K % 4 != 0
+ * (FP32) / C % 8 or K % 8 != 0 (FP16), or when the device is not sm_100.
+ * On success *out owns a new plan (free with winrs_plan_destroy). */
+WINRS_API winrs_status_t winrs_plan(int N, int C, int H, int W, int K, int R, int S, int pad,
+                          winrs_dtype_t dtype, winrs_plan_t* out);
+
+/* Same, for explicitly given device properties (no CUDA call is made). */
+WINRS_API winrs_status_t winrs_plan_for_device(int N, int C, int H, int W, int K, int R, int S, int pad,
+                                     winrs_dtype_t dtype, const winrs_device_t* dev,
+                                     winrs_plan_t* out);
+
+/* Copy the plan description into *info (host memory). */
+WINRS_API winrs_status_t winrs_plan_info(winrs_plan_t plan, winrs_plan_info_t* info);
+
+/* Workspace bytes winrs_bfc needs for this plan (0 when Z == 1); 0 for NULL. */
+WINRS_API size_t winrs_workspace_bytes(winrs_plan_t plan);
+
+/* Run the BFC asynchronously on `stream` (a cudaStream_t; NULL = legacy
+ * default stream).  X, dY: device pointers in the plan's dtype, NHWC;
+ * dW: device float32 KRSC, overwritten; workspace: device buffer of at least
+ * winrs_workspace_bytes(plan) bytes (may be NULL when that is 0).  All device
+ * pointers must be 16-byte aligned; X and dY must not alias dW or workspace.
+ * Returns INVALID_ARG (null plan/pointer, misalignment), WORKSPACE, or CUDA. */
+WINRS_API winrs_status_t winrs_bfc(winrs_plan_t plan, const void* X, const void* dY, float* dW,
+                         void* workspace, void* stream);
+
+/* Same computation with HOST buffers: copies X and dY host->device into
+ * caller-provided device staging buffers, runs winrs_bfc and copies dW back to
+ * host_dW, all on `stream`, then synchronises that stream.  Used for the
+ * end-to-end measurement.  dev_X/dev_dY/dev_dW are device buffers of the
+ * respective sizes. */
+WINRS_API winrs_status_t winrs_bfc_host(winrs_plan_t plan, const void* host_X, const void* host_dY,
+                              float* host_dW, void* dev_X, void* dev_dY, float* dev_dW,
+                              void* workspace, void* stream);
+
+/* Destroy a plan (NULL is a no-op). */
+WINRS_API void winrs_plan_destroy(winrs_plan_t plan);
+
+/* Static, human-readable name of a status code. */
+WINRS_API const char* winrs_status_string(winrs_status_t s);
+
+/* Library version string (static). */
+WINRS_API const char* winrs_version(void);
+
+/* Number of GPU kernel launches one winrs_bfc call of this plan issues. */
+WINRS_API int winrs_launch_count(winrs_plan_t plan);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* WINRS_H */

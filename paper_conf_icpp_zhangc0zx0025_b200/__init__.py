@@ -1,1 +1,192 @@
-"""WinRS on B200 — fused Winograd backward-filter convolution (placeholder; binding lands with the C ABI)."""
+"""WinRS on B200: fused Winograd backward-filter convolution (PAPER.md, ICPP'25).
+
+Thin Python binding over libwinrs.so (include/winrs.h) — argument marshalling
+only; every step of the method runs in the library's sm_100a kernels.  PyTorch
+supplies device memory, streams and process groups.
+
+    p = plan(N, C, H, W, K, R, S, pad, "f32")     # winrs_plan
+    dW = bfc(p, X, dY)                            # winrs_bfc  (dW: [K,R,S,C] fp32)
+
+X is [N,H,W,C] (NHWC) or a logical [N,C,H,W] channels_last tensor; dY likewise
+with (Ho, Wo, K).  dW is returned as a contiguous KRSC float32 tensor (use
+`as_kcrs(dW)` for PyTorch's logical [K,C,R,S] weight view, channels_last).
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass
+
+from . import _lib
+from ._lib import WinrsError, DTYPES
+
+__all__ = ["Plan", "plan", "plan_for_device", "bfc", "bfc_host", "as_kcrs", "bfc_data_parallel",
+           "WinrsError", "version", "emulate", "transform", "kernel_names"]
+
+
+class Plan:
+    """Owns a winrs_plan_t.  `info` mirrors winrs_plan_info_t."""
+
+    def __init__(self, handle: ctypes.c_void_p):
+        self._h = handle
+        inf = _lib.PlanInfoT()
+        _lib.check(_lib.lib().winrs_plan_info(self._h, ctypes.byref(inf)), "winrs_plan_info")
+        self.info = {name: getattr(inf, name) for name, _ in _lib.PlanInfoT._fields_}
+
+    @property
+    def handle(self):
+        return self._h
+
+    @property
+    def workspace_bytes(self) -> int:
+        return int(_lib.lib().winrs_workspace_bytes(self._h))
+
+    @property
+    def launch_count(self) -> int:
+        return int(_lib.lib().winrs_launch_count(self._h))
+
+    @property
+    def kernel_name(self) -> str:
+        return _lib.lib().winrs_debug_plan_kernel(self._h).decode()
+
+    @property
+    def dtype(self) -> str:
+        return "f32" if self.info["dtype"] == 0 else "f16"
+
+    def __del__(self):
+        h, self._h = getattr(self, "_h", None), None
+        if h and _lib._lib is not None:
+            _lib._lib.winrs_plan_destroy(h)
+
+    def __repr__(self):
+        i = self.info
+        s = (f"Plan(Omega_{i['alpha0']}({i['n0']},{i['r0']})x{i['k0']}")
+        if i["alpha1"]:
+            s += f" + Omega_{i['alpha1']}({i['n1']},{i['r1']})x{i['k1']}"
+        return s + (f", Z={i['Z']}, tile={i['tile_k0']}x{i['tile_c0']}, ws={i['workspace_bytes']}B)")
+
+
+def plan(N, C, H, W, K, R, S, pad, dtype: str = "f32") -> Plan:
+    """winrs_plan on the current CUDA device."""
+    h = ctypes.c_void_p()
+    _lib.check(_lib.lib().winrs_plan(N, C, H, W, K, R, S, pad, DTYPES[dtype], ctypes.byref(h)), "winrs_plan")
+    return Plan(h)
+
+
+def plan_for_device(N, C, H, W, K, R, S, pad, dtype: str = "f32", num_sms: int = 148,
+                    cc=(10, 0)) -> Plan:
+    """winrs_plan_for_device: plan without touching a GPU (host tests)."""
+    dev = _lib.DeviceT(num_sms, cc[0], cc[1])
+    h = ctypes.c_void_p()
+    _lib.check(_lib.lib().winrs_plan_for_device(N, C, H, W, K, R, S, pad, DTYPES[dtype], ctypes.byref(dev),
+                                                ctypes.byref(h)), "winrs_plan_for_device")
+    return Plan(h)
+
+
+def _as_nhwc(t, n, h, w, c, name):
+    """Return a tensor whose memory is NHWC [n,h,w,c] (no copy)."""
+    if tuple(t.shape) == (n, h, w, c) and t.is_contiguous():
+        return t
+    if tuple(t.shape) == (n, c, h, w):
+        import torch
+        if t.is_contiguous(memory_format=torch.channels_last):
+            return t.permute(0, 2, 3, 1)
+    raise ValueError(f"{name}: expected NHWC [{n},{h},{w},{c}] contiguous or channels_last "
+                     f"[{n},{c},{h},{w}], got shape {tuple(t.shape)} strides {t.stride()}")
+
+
+def bfc(p: Plan, X, dY, dW=None, workspace=None, stream=None):
+    """winrs_bfc on torch CUDA tensors; returns dW [K,R,S,C] float32."""
+    import torch
+    i = p.info
+    tdt = torch.float32 if p.dtype == "f32" else torch.float16
+    Xn = _as_nhwc(X, i["N"], i["H"], i["W"], i["C"], "X")
+    Gn = _as_nhwc(dY, i["N"], i["Ho"], i["Wo"], i["K"], "dY")
+    if Xn.dtype != tdt or Gn.dtype != tdt:
+        raise TypeError(f"X and dY must be {tdt} for this plan")
+    if not (Xn.is_cuda and Gn.is_cuda):
+        raise ValueError("X and dY must be CUDA tensors (use bfc_host for host buffers)")
+    if dW is None:
+        dW = torch.empty((i["K"], i["R"], i["S"], i["C"]), dtype=torch.float32, device=Xn.device)
+    elif not (dW.dtype == torch.float32 and dW.is_contiguous() and dW.numel() == i["K"] * i["R"] * i["S"] * i["C"]):
+        raise ValueError("dW must be a contiguous float32 KRSC tensor")
+    wsb = p.workspace_bytes
+    if wsb and workspace is None:
+        workspace = torch.empty(wsb, dtype=torch.uint8, device=Xn.device)
+    if stream is None:
+        stream = torch.cuda.current_stream(Xn.device)
+    sp = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+    _lib.check(_lib.lib().winrs_bfc(p.handle, Xn.data_ptr(), Gn.data_ptr(), dW.data_ptr(),
+                                    workspace.data_ptr() if wsb else None, sp), "winrs_bfc")
+    return dW
+
+
+def bfc_host(p: Plan, X_host, dY_host, dW_host, dev_X, dev_dY, dev_dW, workspace=None, stream=None):
+    """winrs_bfc_host: host (ideally pinned) tensors in, host dW out; the
+    H2D copies, the BFC and the D2H copy all run on `stream`, which is then
+    synchronised."""
+    import torch
+    wsb = p.workspace_bytes
+    if wsb and workspace is None:
+        workspace = torch.empty(wsb, dtype=torch.uint8, device=dev_X.device)
+    if stream is None:
+        stream = torch.cuda.current_stream(dev_X.device)
+    _lib.check(_lib.lib().winrs_bfc_host(p.handle, X_host.data_ptr(), dY_host.data_ptr(), dW_host.data_ptr(),
+                                         dev_X.data_ptr(), dev_dY.data_ptr(), dev_dW.data_ptr(),
+                                         workspace.data_ptr() if wsb else None, stream.cuda_stream),
+               "winrs_bfc_host")
+    return dW_host
+
+
+def as_kcrs(dW):
+    """KRSC storage -> logical [K,C,R,S] view (channels_last strides), no copy."""
+    return dW.permute(0, 3, 1, 2)
+
+
+def bfc_data_parallel(X_shard, dY_shard, R: int, S: int, pad: int, dtype: str = "f32", group=None,
+                      p: Plan | None = None):
+    """Batch-sharded BFC: each rank runs the fused BFC on
+    its contiguous N-slice, then ONE all_reduce(SUM) of dW over the process
+    group — the sum over n is the only exchange the method needs."""
+    import torch.distributed as dist
+    N, H, W, C = X_shard.shape
+    K = dY_shard.shape[-1]
+    if p is None:
+        p = plan(N, C, H, W, K, R, S, pad, dtype)
+    dW = bfc(p, X_shard, dY_shard)
+    if dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(dW, op=dist.ReduceOp.SUM, group=group)
+    return dW
+
+
+def version() -> str:
+    return _lib.lib().winrs_version().decode()
+
+
+def kernel_names():
+    L = _lib.lib()
+    return [L.winrs_debug_kernel_name(i).decode() for i in range(L.winrs_debug_kernel_count())]
+
+
+def emulate(p: Plan, X, dY):
+    """winrs_debug_emulate: FP64 host emulation of the plan's decomposition
+    (numpy float64 NHWC in, KRSC out)."""
+    import numpy as np
+    i = p.info
+    Xd = np.ascontiguousarray(X, dtype=np.float64)
+    Gd = np.ascontiguousarray(dY, dtype=np.float64)
+    assert Xd.shape == (i["N"], i["H"], i["W"], i["C"]) and Gd.shape == (i["N"], i["Ho"], i["Wo"], i["K"])
+    out = np.empty((i["K"], i["R"], i["S"], i["C"]), dtype=np.float64)
+    _lib.check(_lib.lib().winrs_debug_emulate(p.handle, Xd.ctypes.data, Gd.ctypes.data, out.ctypes.data),
+               "winrs_debug_emulate")
+    return out
+
+
+def transform(alpha: int, n: int, r: int, which: str, vec):
+    """winrs_debug_transform: apply the generated FT/IT/OT of Omega_alpha(n,r) in double."""
+    import numpy as np
+    w = {"ft": 0, "it": 1, "ot": 2}[which]
+    x = np.ascontiguousarray(vec, dtype=np.float64)
+    out = np.empty(n if w == 2 else alpha, dtype=np.float64)
+    _lib.check(_lib.lib().winrs_debug_transform(alpha, n, r, w, x.ctypes.data, out.ctypes.data),
+               "winrs_debug_transform")
+    return out

@@ -1,0 +1,253 @@
+// Host planner: the three-step configuration adaptation of PAPER.md §4
+// (P@20113-28371), integer-only and deterministic, restricted to the kernel
+// instantiations present in the registry.
+//
+//   1. Fastest kernel pair (§4.1 P@20377, criteria (1)-(3), Figure 5): n0 and
+//      n1 divide F_W; k0*r0 + k1*r1 covers O_W (the last unit may carry
+//      zero-masked columns, R6); minimal Winograd-domain EWM work
+//      sum k_i*alpha_i*(S/n_i)/tau_i (R7).
+//   2. Baseline segment count Z^ (§4.2 Algorithm 1; the unspecified functions
+//      are read as in DESIGN.md R8).
+//   3. Segment shape S^_H x S^_W and the final segment count (§4.3 Algorithm 2,
+//      eq. (5); readings R9, R10).
+//
+// Debug overrides (tests only): WINRS_FORCE_Z=<z>, WINRS_FORCE_TILE=<bn>x<bm>,
+// WINRS_FORCE_PAIR=a0,n0,r0,a1,n1,r1.
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <vector>
+#include "planner.h"
+
+namespace winrs {
+
+static long long cdiv(long long a, long long b) { return (a + b - 1) / b; }
+
+struct PairChoice {
+    const KernelEntry* proto = nullptr;   // any entry of the pair (tile chosen later)
+    int k0 = 0, k1 = 0, masked = 0;
+    double cost = 0;
+};
+
+// "Throughput coefficients" tau (P@20823): relative efficiency of a kernel on
+// B200.  Default 1 (pure alpha-count model, R7).
+static double tau(int /*alpha*/, int /*n*/, int /*r*/) { return 1.0; }
+
+static bool same_pair(const KernelEntry& a, const KernelEntry& b) {
+    return a.dtype == b.dtype && a.a0 == b.a0 && a.n0 == b.n0 && a.r0 == b.r0 && a.a1 == b.a1 &&
+           a.n1 == b.n1 && a.r1 == b.r1;
+}
+
+static bool parse_force_pair(int out[6]) {
+    const char* s = getenv("WINRS_FORCE_PAIR");
+    if (!s || !*s) return false;
+    return sscanf(s, "%d,%d,%d,%d,%d,%d", &out[0], &out[1], &out[2], &out[3], &out[4], &out[5]) == 6;
+}
+
+// Step 1: kernel-pair selection.
+static bool choose_pair(const Problem& p, const KernelEntry* es, int ne, PairChoice* best) {
+    int forced[6];
+    const bool force = parse_force_pair(forced);
+    bool found = false;
+    for (int i = 0; i < ne; ++i) {
+        const KernelEntry& e = es[i];
+        if (e.dtype != p.dtype) continue;
+        bool dup = false;   // evaluate each pair once (tile variants share it)
+        for (int j = 0; j < i; ++j)
+            if (same_pair(es[j], e)) { dup = true; break; }
+        if (dup) continue;
+        if (force && !(e.a0 == forced[0] && e.n0 == forced[1] && e.r0 == forced[2] && e.a1 == forced[3] &&
+                       e.n1 == forced[4] && e.r1 == forced[5]))
+            continue;
+        if (p.S % e.n0 != 0) continue;                       // criterion (1)
+        if (e.a1 && (p.S % e.n1 != 0 || e.n0 % e.n1 != 0)) continue;
+        auto consider = [&](int k0, int k1, int masked) {
+            const double c = k0 * (double)e.a0 * (p.S / e.n0) / tau(e.a0, e.n0, e.r0) +
+                             (e.a1 ? k1 * (double)e.a1 * (p.S / e.n1) / tau(e.a1, e.n1, e.r1) : 0.0);
+            bool better = !found;
+            if (!better) {
+                if (c != best->cost) better = c < best->cost;
+                else if (masked != best->masked) better = masked < best->masked;
+                else if (k0 != best->k0) better = k0 > best->k0;
+                else if (e.a0 != best->proto->a0) better = e.a0 > best->proto->a0;
+                else better = e.a1 < best->proto->a1;
+            }
+            if (better) {
+                best->proto = &e;
+                best->k0 = k0; best->k1 = k1; best->masked = masked; best->cost = c;
+                found = true;
+            }
+        };
+        if (e.a1 == 0) {
+            const int k0 = (int)cdiv(p.Wo, e.r0);             // criterion (2) with masking
+            consider(k0, 0, k0 * e.r0 - p.Wo);
+        } else {
+            for (int k0 = p.Wo / e.r0; k0 >= 1; --k0) {
+                const int rem = p.Wo - k0 * e.r0;
+                if (rem <= 0) continue;
+                const int k1 = (int)cdiv(rem, e.r1);
+                const int masked = k1 * e.r1 - rem;
+                consider(k0, k1, masked);
+            }
+        }
+    }
+    return found;
+}
+
+// Step 2: Algorithm 1 (R8).
+static int alg1(const Problem& p, const KernelEntry& e, int num_sms, int* zmax_out) {
+    const long long b2 = cdiv(p.K, e.bn) * cdiv(p.C, e.bm) * (long long)p.R * (p.S / e.n0);
+    const long long b0 = cdiv(p.K, 64) * cdiv((long long)p.N * cdiv(p.Ho, 2) * cdiv(p.Wo, 2), 32);
+    const long long b1 = cdiv(p.C, 64) * cdiv((long long)p.N * cdiv(p.H, 2) * cdiv(p.W, 2), 32);
+    double zh = (double)(b0 + b1) / (1.45 * (double)b2);                          // line 1
+    const long long bhat2 = (long long)e.occ * num_sms;                             // line 2
+    const double esz = p.dtype == 0 ? 4.0 : 2.0;
+    const double data = esz * ((double)p.N * p.H * p.W * p.C + (double)p.N * p.Ho * p.Wo * p.K);
+    const double dw_bytes = 4.0 * (double)p.K * p.R * p.S * p.C;
+    const int zmax = 1 + (int)std::floor(0.04 * data / dw_bytes);
+    *zmax_out = zmax;
+    if (zh < 2.0 && b2 >= bhat2) return 1;                                          // line 3
+    const long long z1 = cdiv(2LL * e.occ * num_sms, b2);                          // line 4
+    const double direct = 2.0 * p.N * p.C * p.K * (double)p.Ho * p.Wo * p.R * p.S;
+    const long long z2 = std::max(1LL, (long long)std::floor(direct / 1073741824.0));   // line 5
+    const long long z3 = std::max(1LL, (long long)p.N * p.Ho * p.Wo / 512);
+    long long z = std::min(std::min((long long)std::ceil(zh), z1), std::min(z2, z3));   // line 6
+    if (z < 1) z = 1;
+    long long P = 1;                                                                // line 7
+    while (P < z) P <<= 1;
+    if (P > 8) P = 8;
+    z = P * cdiv(z, P);
+    if (z > zmax) z = zmax;
+    return (int)std::max(1LL, z);
+}
+
+// Step 3: Algorithm 2 on the Omega_a0 region (width k0*r0, W_max = k0 units).
+static void alg2(const Problem& p, int r0, int k0, int z, int* z_used, int* seg_h, int* seg_w) {
+    const int Ho = p.Ho;
+    const int Hmax = p.pad > 0 ? std::max(1, Ho / p.pad) : Ho;
+    const int Wmax = k0;
+    z = std::min<long long>(z, (long long)Hmax * Wmax);                            // line 1
+    if (z < 1) z = 1;
+    *z_used = z;
+    int sh, sw;
+    if (z == 1) {                                                                   // line 2
+        sh = Ho; sw = k0 * r0;
+    } else if (z >= Wmax) {                                                         // line 3
+        // S^_H ~ Ho*W_max/Z^; the band count floor(Ho/S^_H) is rounded to the
+        // nearest integer of Z^/W_max instead of truncated (R9).
+        const long long nb = std::max(1LL, ((long long)z + Wmax / 2) / Wmax);
+        sh = (int)(Ho / nb); sw = r0;
+    } else if (Wmax % z == 0) {                                                     // line 4
+        sh = Ho; sw = r0 * (Wmax / z);
+    } else {                                                                        // lines 5-7
+        const int lo = (int)cdiv(Wmax, z), hi = (int)((long long)Hmax * Wmax / z);
+        int x = 0;
+        for (int c = lo; c <= hi && c <= Wmax; ++c)
+            if (Wmax % c == 0) { x = c; break; }
+        if (x) { sh = (int)((long long)Ho * Wmax / ((long long)z * x)); sw = x * r0; }
+        else { sh = Ho; sw = k0 * r0; }
+    }
+    *seg_h = std::min(std::max(sh, 1), Ho);
+    *seg_w = std::max(sw, r0);
+}
+
+static void fill_geometry(const Problem& p, const KernelEntry& e, const PairChoice& pc, int seg_h, int seg_w,
+                          Geometry* g) {
+    memset(g, 0, sizeof(*g));
+    g->N = p.N; g->C = p.C; g->H = p.H; g->W = p.W; g->K = p.K; g->R = p.R; g->S = p.S; g->pad = p.pad;
+    g->Ho = p.Ho; g->Wo = p.Wo;
+    g->a0 = e.a0; g->n0 = e.n0; g->r0 = e.r0; g->k0 = pc.k0;
+    g->seg_h = seg_h;
+    g->bands = std::max(1, p.Ho / seg_h);
+    g->seg_w = seg_w;
+    g->seg_cols = (int)cdiv((long long)pc.k0 * e.r0, seg_w);
+    g->a1 = e.a1; g->n1 = e.n1; g->r1 = e.r1; g->k1 = pc.k1;
+    g->res_col0 = pc.k0 * e.r0;
+    g->tile_k = e.bn; g->tile_c = e.bm;
+    g->kblocks = (int)cdiv(p.K, e.bn);
+    g->cblocks = (int)cdiv(p.C, e.bm);
+    g->ftiles = p.S / e.n0;
+    g->Z = g->bands * g->seg_cols;
+    g->dw_elems = (long long)p.K * p.R * p.S * p.C;
+}
+
+// Winograd-domain EWM flops the kernels issue (clipped rows, masked columns
+// counted as work): 2*K*C*N * sum_{fh, band} rows_valid * (units*alpha*S/n).
+static double ewm_flops(const Geometry& g) {
+    double tot = 0;
+    for (int band = 0; band < g.bands; ++band)
+        for (int fh = 0; fh < g.R; ++fh) {
+            int hs, he;
+            band_rows(g, band, fh, &hs, &he);
+            const double rows = he - hs;
+            double per_row = (double)g.k0 * g.a0 * (g.S / g.n0);
+            if (g.a1 && g.k1) per_row += (double)g.k1 * g.a1 * (g.S / g.n1);
+            tot += rows * per_row;
+        }
+    return 2.0 * g.K * g.C * (double)g.N * tot;
+}
+
+static void plan_with_tile(const Problem& p, const KernelEntry& e, const PairChoice& pc, int num_sms,
+                           PlanResult* out) {
+    int zmax = 1;
+    int z = alg1(p, e, num_sms, &zmax);
+    if (const char* fz = getenv("WINRS_FORCE_Z")) {
+        const int v = atoi(fz);
+        if (v >= 1) { z = v; zmax = 1 << 30; }
+    }
+    int z_used = 1, seg_h = p.Ho, seg_w = pc.k0 * e.r0;
+    Geometry g;
+    for (;;) {
+        alg2(p, e.r0, pc.k0, z, &z_used, &seg_h, &seg_w);
+        fill_geometry(p, e, pc, seg_h, seg_w, &g);
+        if (g.Z <= zmax || z <= 1) break;     // enforce the workspace cap (R11)
+        z = std::min(z_used, z) - 1;
+    }
+    out->geom = g;
+    out->entry = &e;
+    out->z_hat = z_used;
+    out->masked = pc.masked;
+}
+
+static int parse_force_tile(int* bn, int* bm) {
+    const char* s = getenv("WINRS_FORCE_TILE");
+    if (!s || !*s) return 0;
+    return sscanf(s, "%dx%d", bn, bm) == 2;
+}
+
+winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
+    int ne = 0;
+    const KernelEntry* es = kernel_entries(&ne);
+    PairChoice pc;
+    if (!choose_pair(p, es, ne, &pc)) return WINRS_ERR_UNSUPPORTED;
+    // Step 1b (B200): CTA tile.  Largest tile that still fills one wave of
+    // the SMs at its occupancy, else the variant giving the most CTAs.
+    std::vector<const KernelEntry*> tiles;
+    for (int i = 0; i < ne; ++i)
+        if (same_pair(es[i], *pc.proto)) tiles.push_back(&es[i]);
+    std::sort(tiles.begin(), tiles.end(), [](const KernelEntry* a, const KernelEntry* b) {
+        if (a->bn * a->bm != b->bn * b->bm) return a->bn * a->bm > b->bn * b->bm;
+        return a->bn > b->bn;
+    });
+    int fbn = 0, fbm = 0;
+    const bool force_tile = parse_force_tile(&fbn, &fbm);
+    PlanResult best;
+    bool have = false;
+    long long best_ctas = -1;
+    for (const KernelEntry* e : tiles) {
+        if (force_tile && (e->bn != fbn || e->bm != fbm)) continue;
+        PlanResult r;
+        plan_with_tile(p, *e, pc, num_sms, &r);
+        const long long ctas = num_ctas(r.geom);
+        if (!have || ctas > best_ctas) { best = r; best_ctas = ctas; have = true; }
+        if (ctas >= (long long)e->occ * num_sms) { best = r; have = true; break; }
+    }
+    if (!have) return WINRS_ERR_UNSUPPORTED;
+    best.ewm_flops = ewm_flops(best.geom);
+    *out = best;
+    return WINRS_OK;
+}
+
+}  // namespace winrs

@@ -1,0 +1,24 @@
+// Planner interface (host only).
+#pragma once
+#include "../../include/winrs.h"
+#include "registry.h"
+#include "winrs_internal.h"
+
+namespace winrs {
+
+struct Problem {
+    int N, C, H, W, K, R, S, pad, Ho, Wo;
+    int dtype;
+};
+
+struct PlanResult {
+    Geometry geom;
+    const KernelEntry* entry = nullptr;
+    int z_hat = 1;
+    int masked = 0;
+    double ewm_flops = 0;
+};
+
+winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out);
+
+}  // namespace winrs

@@ -1,0 +1,32 @@
+// Registry of compiled fused-kernel instantiations.  The planner only ever
+// chooses a (kernel pair, CTA tile) that is present here, so every plan is
+// runnable; there is no fallback path.
+#pragma once
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include "winrs_internal.h"
+
+namespace winrs {
+
+typedef cudaError_t (*LaunchFn)(const Geometry& g, const void* X, const void* dY, float* dW,
+                                float* ws, cudaStream_t stream);
+
+struct KernelEntry {
+    int dtype;                 // 0 = FP32 CUDA-core, 1 = FP16 tensor-core
+    int a0, n0, r0;            // bulk kernel Omega_a0(n0, r0)
+    int a1, n1, r1;            // residual kernel (a1 == 0: none)
+    int bn, bm;                // CTA tile B_N (k) x B_M (c)
+    int threads;
+    int occ;                   // planner's CTAs/SM hint
+    size_t smem;               // dynamic shared memory bytes
+    LaunchFn launch;
+    const char* name;
+};
+
+// All entries (FP32 and FP16), terminated by count.
+const KernelEntry* kernel_entries(int* count);
+
+cudaError_t launch_bucket_reduce(float* dW, const float* ws, long long n, int Z, int num_sms,
+                                 cudaStream_t stream);
+
+}  // namespace winrs

@@ -1,0 +1,303 @@
+// C ABI of libwinrs (include/winrs.h, include/winrs_debug.h): plan objects,
+// argument validation and the launch sequence of PAPER.md §3 (P@15252-17405):
+// (2) Kernel Execution — one fused launch over all segments (both kernels of
+// the pair), (3) Reduction — the bucket reduction kernel when Z > 1.
+#include <cuda_runtime.h>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <vector>
+#include "../../include/winrs.h"
+#include "../../include/winrs_debug.h"
+#include "planner.h"
+#include "winograd_generated.cuh"
+
+struct winrs_plan_s {
+    winrs::PlanResult pr;
+    winrs_plan_info_t info;
+    int num_sms;
+};
+
+using namespace winrs;
+
+static winrs_status_t build_plan(int N, int C, int H, int W, int K, int R, int S, int pad,
+                                 winrs_dtype_t dtype, const winrs_device_t* dev, winrs_plan_t* out) {
+    if (!out) return WINRS_ERR_INVALID_ARG;
+    *out = nullptr;
+    if (N <= 0 || C <= 0 || H <= 0 || W <= 0 || K <= 0 || R <= 0 || S <= 0 || pad < 0)
+        return WINRS_ERR_INVALID_ARG;
+    if (dtype != WINRS_F32 && dtype != WINRS_F16) return WINRS_ERR_INVALID_ARG;
+    const int Ho = H + 2 * pad - R + 1, Wo = W + 2 * pad - S + 1;
+    if (Ho < 1 || Wo < 1) return WINRS_ERR_INVALID_ARG;
+    if (!dev || dev->num_sms <= 0) return WINRS_ERR_INVALID_ARG;
+    if (dev->cc_major != 10 || dev->cc_minor != 0) return WINRS_ERR_UNSUPPORTED;   // sm_100a build
+    const int align = dtype == WINRS_F32 ? 4 : 8;                                  // 16-byte vectors
+    if (C % align || K % align) return WINRS_ERR_UNSUPPORTED;
+    Problem p{N, C, H, W, K, R, S, pad, Ho, Wo, (int)dtype};
+    PlanResult pr;
+    const winrs_status_t st = make_plan(p, dev->num_sms, &pr);
+    if (st != WINRS_OK) return st;
+    winrs_plan_s* pl = new (std::nothrow) winrs_plan_s;
+    if (!pl) return WINRS_ERR_HOST_ALLOC;
+    pl->pr = pr;
+    pl->num_sms = dev->num_sms;
+    const Geometry& g = pr.geom;
+    winrs_plan_info_t& in = pl->info;
+    memset(&in, 0, sizeof(in));
+    in.N = N; in.C = C; in.H = H; in.W = W; in.K = K; in.R = R; in.S = S; in.pad = pad;
+    in.dtype = dtype; in.Ho = Ho; in.Wo = Wo;
+    in.alpha0 = g.a0; in.n0 = g.n0; in.r0 = g.r0; in.k0 = g.k0;
+    in.alpha1 = g.a1; in.n1 = g.n1; in.r1 = g.r1; in.k1 = g.k1;
+    in.masked_cols = pr.masked;
+    in.z_hat = pr.z_hat;
+    in.Z = g.Z;
+    in.seg_h = g.seg_h; in.seg_w = g.seg_w; in.bands = g.bands; in.seg_cols = g.seg_cols;
+    in.tile_k0 = g.tile_k; in.tile_c0 = g.tile_c;
+    in.tile_k1 = g.a1 ? g.tile_k : 0; in.tile_c1 = g.a1 ? g.tile_c : 0;
+    in.ctas_main = num_ctas(g);
+    in.ctas_resid = 0;   // the residual phase runs inside the main launch's last-column CTAs
+    in.ctas_reduce = g.Z > 1 ? 1 : 0;
+    in.workspace_bytes = g.Z > 1 ? (size_t)(g.Z - 1) * 4u * (size_t)g.dw_elems : 0;
+    in.direct_flops = 2.0 * N * (double)C * K * Ho * Wo * R * S;
+    in.ewm_flops = pr.ewm_flops;
+    *out = pl;
+    return WINRS_OK;
+}
+
+extern "C" {
+
+winrs_status_t winrs_plan_for_device(int N, int C, int H, int W, int K, int R, int S, int pad,
+                                     winrs_dtype_t dtype, const winrs_device_t* dev, winrs_plan_t* out) {
+    return build_plan(N, C, H, W, K, R, S, pad, dtype, dev, out);
+}
+
+winrs_status_t winrs_plan(int N, int C, int H, int W, int K, int R, int S, int pad,
+                          winrs_dtype_t dtype, winrs_plan_t* out) {
+    if (!out) return WINRS_ERR_INVALID_ARG;
+    int d = 0;
+    if (cudaGetDevice(&d) != cudaSuccess) { cudaGetLastError(); return WINRS_ERR_CUDA; }
+    winrs_device_t dev{};
+    if (cudaDeviceGetAttribute(&dev.num_sms, cudaDevAttrMultiProcessorCount, d) != cudaSuccess ||
+        cudaDeviceGetAttribute(&dev.cc_major, cudaDevAttrComputeCapabilityMajor, d) != cudaSuccess ||
+        cudaDeviceGetAttribute(&dev.cc_minor, cudaDevAttrComputeCapabilityMinor, d) != cudaSuccess) {
+        cudaGetLastError();
+        return WINRS_ERR_CUDA;
+    }
+    return build_plan(N, C, H, W, K, R, S, pad, dtype, &dev, out);
+}
+
+winrs_status_t winrs_plan_info(winrs_plan_t plan, winrs_plan_info_t* info) {
+    if (!plan || !info) return WINRS_ERR_INVALID_ARG;
+    *info = plan->info;
+    return WINRS_OK;
+}
+
+size_t winrs_workspace_bytes(winrs_plan_t plan) { return plan ? plan->info.workspace_bytes : 0; }
+
+int winrs_launch_count(winrs_plan_t plan) {
+    if (!plan) return 0;
+    return 1 + (plan->pr.geom.Z > 1 ? 1 : 0);
+}
+
+static bool misaligned(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) != 0; }
+
+winrs_status_t winrs_bfc(winrs_plan_t plan, const void* X, const void* dY, float* dW, void* workspace,
+                         void* stream) {
+    if (!plan || !X || !dY || !dW) return WINRS_ERR_INVALID_ARG;
+    if (misaligned(X) || misaligned(dY) || misaligned(dW)) return WINRS_ERR_INVALID_ARG;
+    const Geometry& g = plan->pr.geom;
+    if (plan->info.workspace_bytes > 0) {
+        if (!workspace) return WINRS_ERR_WORKSPACE;
+        if (misaligned(workspace)) return WINRS_ERR_INVALID_ARG;
+    }
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    cudaError_t e = plan->pr.entry->launch(g, X, dY, dW, static_cast<float*>(workspace), s);
+    if (e != cudaSuccess) return WINRS_ERR_CUDA;
+    if (g.Z > 1) {
+        e = launch_bucket_reduce(dW, static_cast<const float*>(workspace), g.dw_elems, g.Z, plan->num_sms, s);
+        if (e != cudaSuccess) return WINRS_ERR_CUDA;
+    }
+    return WINRS_OK;
+}
+
+winrs_status_t winrs_bfc_host(winrs_plan_t plan, const void* host_X, const void* host_dY, float* host_dW,
+                              void* dev_X, void* dev_dY, float* dev_dW, void* workspace, void* stream) {
+    if (!plan || !host_X || !host_dY || !host_dW || !dev_X || !dev_dY || !dev_dW) return WINRS_ERR_INVALID_ARG;
+    const winrs_plan_info_t& in = plan->info;
+    const size_t esz = in.dtype == WINRS_F32 ? 4 : 2;
+    const size_t bx = esz * (size_t)in.N * in.H * in.W * in.C;
+    const size_t by = esz * (size_t)in.N * in.Ho * in.Wo * in.K;
+    const size_t bw = 4 * (size_t)in.K * in.R * in.S * in.C;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    if (cudaMemcpyAsync(dev_X, host_X, bx, cudaMemcpyHostToDevice, s) != cudaSuccess ||
+        cudaMemcpyAsync(dev_dY, host_dY, by, cudaMemcpyHostToDevice, s) != cudaSuccess) {
+        cudaGetLastError();
+        return WINRS_ERR_CUDA;
+    }
+    const winrs_status_t st = winrs_bfc(plan, dev_X, dev_dY, dev_dW, workspace, stream);
+    if (st != WINRS_OK) return st;
+    if (cudaMemcpyAsync(host_dW, dev_dW, bw, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess) {
+        cudaGetLastError();
+        return WINRS_ERR_CUDA;
+    }
+    return WINRS_OK;
+}
+
+void winrs_plan_destroy(winrs_plan_t plan) { delete plan; }
+
+const char* winrs_status_string(winrs_status_t s) {
+    switch (s) {
+        case WINRS_OK: return "WINRS_OK";
+        case WINRS_ERR_INVALID_ARG: return "WINRS_ERR_INVALID_ARG";
+        case WINRS_ERR_UNSUPPORTED: return "WINRS_ERR_UNSUPPORTED";
+        case WINRS_ERR_WORKSPACE: return "WINRS_ERR_WORKSPACE";
+        case WINRS_ERR_CUDA: return "WINRS_ERR_CUDA";
+        case WINRS_ERR_HOST_ALLOC: return "WINRS_ERR_HOST_ALLOC";
+    }
+    return "WINRS_ERR_UNKNOWN";
+}
+
+const char* winrs_version(void) { return "winrs-b200 0.1.0 (sm_100a)"; }
+
+}  // extern "C"
+
+// ----------------------------------------------------------------------------
+// Host FP64 emulator of the plan's decomposition (include/winrs_debug.h).
+// Walks exactly the CTA/segment/unit/row structure the kernels walk (same
+// index helpers from winrs_internal.h, same generated transforms instantiated
+// for double), so host-only tests can check the decomposition — pair split,
+// masked tail, clipping, segments, buckets, residual phase, reduction —
+// against the oracle before any GPU is involved.
+
+namespace {
+
+template <int A, int NN, int RR>
+void emu_phase(const Geometry& g, const double* X, const double* dY, double* bucket, const CtaCoord& cc,
+               int hs, int he, int w_first, int units, int fw0, bool accumulate) {
+    using WT = Wino<A, NN, RR>;
+    const int BN = g.tile_k, BM = g.tile_c;
+    const int k0 = cc.kb * BN, c0 = cc.cb * BM;
+    std::vector<double> v((size_t)A * BN * BM, 0.0), gt((size_t)A * BN), xt((size_t)A * BM);
+    for (int h = hs; h < he; ++h)
+        for (int u = 0; u < units; ++u)
+            for (int n = 0; n < g.N; ++n) {
+                const int w0 = w_first + u * RR;
+                for (int k = 0; k < BN; ++k) {
+                    double w[RR], o[A];
+                    for (int i = 0; i < RR; ++i) {
+                        const int kk = k0 + k, col = w0 + i;
+                        w[i] = (kk < g.K && col < g.Wo) ? dY[(((size_t)n * g.Ho + h) * g.Wo + col) * g.K + kk] : 0.0;
+                    }
+                    WT::ft(w, o);
+                    for (int x = 0; x < A; ++x) gt[(size_t)x * BN + k] = o[x];
+                }
+                const int xrow = h + cc.fh - g.pad;
+                for (int c = 0; c < BM; ++c) {
+                    double xv[A], o[A];
+                    for (int t = 0; t < A; ++t) {
+                        const int col = w0 + fw0 - g.pad + t, ccn = c0 + c;
+                        xv[t] = (col >= 0 && col < g.W && ccn < g.C && xrow >= 0 && xrow < g.H)
+                                    ? X[(((size_t)n * g.H + xrow) * g.W + col) * g.C + ccn] : 0.0;
+                    }
+                    WT::it(xv, o);
+                    for (int x = 0; x < A; ++x) xt[(size_t)x * BM + c] = o[x];
+                }
+                for (int x = 0; x < A; ++x)
+                    for (int k = 0; k < BN; ++k)
+                        for (int c = 0; c < BM; ++c)
+                            v[((size_t)x * BN + k) * BM + c] += gt[(size_t)x * BN + k] * xt[(size_t)x * BM + c];
+            }
+    for (int k = 0; k < BN; ++k)
+        for (int c = 0; c < BM; ++c) {
+            const int kg = k0 + k, cg = c0 + c;
+            if (kg >= g.K || cg >= g.C) continue;
+            double vv[A], y[NN];
+            for (int x = 0; x < A; ++x) vv[x] = v[((size_t)x * BN + k) * BM + c];
+            WT::ot(vv, y);
+            for (int j = 0; j < NN; ++j) {
+                double& dst = bucket[(((size_t)kg * g.R + cc.fh) * g.S + fw0 + j) * g.C + cg];
+                dst = accumulate ? dst + y[j] : y[j];
+            }
+        }
+}
+
+typedef void (*EmuFn)(const Geometry&, const double*, const double*, double*, const CtaCoord&, int, int, int,
+                      int, int, bool);
+
+EmuFn emu_fn(int a, int n, int r) {
+#define WINRS_EMU_CASE(A, N, R) if (a == A && n == N && r == R) return &emu_phase<A, N, R>;
+    WINRS_EMU_CASE(2, 2, 1) WINRS_EMU_CASE(4, 2, 3) WINRS_EMU_CASE(4, 3, 2)
+    WINRS_EMU_CASE(8, 3, 6) WINRS_EMU_CASE(8, 4, 5) WINRS_EMU_CASE(8, 5, 4) WINRS_EMU_CASE(8, 6, 3)
+    WINRS_EMU_CASE(8, 7, 2) WINRS_EMU_CASE(16, 5, 12) WINRS_EMU_CASE(16, 6, 11) WINRS_EMU_CASE(16, 7, 10)
+    WINRS_EMU_CASE(16, 8, 9) WINRS_EMU_CASE(16, 9, 8)
+#undef WINRS_EMU_CASE
+    return nullptr;
+}
+
+}  // namespace
+
+extern "C" {
+
+winrs_status_t winrs_debug_emulate(winrs_plan_t plan, const double* X, const double* dY, double* dW) {
+    if (!plan || !X || !dY || !dW) return WINRS_ERR_INVALID_ARG;
+    const Geometry& g = plan->pr.geom;
+    EmuFn f0 = emu_fn(g.a0, g.n0, g.r0);
+    EmuFn f1 = g.a1 ? emu_fn(g.a1, g.n1, g.r1) : nullptr;
+    if (!f0 || (g.a1 && !f1)) return WINRS_ERR_UNSUPPORTED;
+    std::vector<double> buckets((size_t)g.Z * g.dw_elems, 0.0);
+    const long long nct = num_ctas(g);
+    for (long long b = 0; b < nct; ++b) {
+        const CtaCoord cc = decode_cta(g, b);
+        const int seg = cc.band * g.seg_cols + cc.col;
+        double* bucket = buckets.data() + (size_t)seg * g.dw_elems;
+        int hs, he, wf, units;
+        band_rows(g, cc.band, cc.fh, &hs, &he);
+        seg_units(g, cc.col, &wf, &units);
+        const int fw0 = cc.ft * g.n0;
+        f0(g, X, dY, bucket, cc, hs, he, wf, units, fw0, false);
+        if (f1 && has_residual(g, cc.col))
+            for (int j = 0; j < g.n0 / g.n1; ++j)
+                f1(g, X, dY, bucket, cc, hs, he, g.res_col0, g.k1, fw0 + j * g.n1, true);
+    }
+    for (long long i = 0; i < g.dw_elems; ++i) {
+        double s = 0.0;
+        for (int z = 0; z < g.Z; ++z) s += buckets[(size_t)z * g.dw_elems + i];
+        dW[i] = s;
+    }
+    return WINRS_OK;
+}
+
+winrs_status_t winrs_debug_transform(int alpha, int n, int r, int which, const double* in, double* out) {
+    // which: 0 = ft (in[r] -> out[alpha]), 1 = it (in[alpha] -> out[alpha]), 2 = ot (in[alpha] -> out[n])
+    if (!in || !out) return WINRS_ERR_INVALID_ARG;
+#define WINRS_T_CASE(A, N, R)                                        \
+    if (alpha == A && n == N && r == R) {                            \
+        if (which == 0) { Wino<A, N, R>::ft(in, out); return WINRS_OK; }  \
+        if (which == 1) { Wino<A, N, R>::it(in, out); return WINRS_OK; }  \
+        if (which == 2) { Wino<A, N, R>::ot(in, out); return WINRS_OK; }  \
+        return WINRS_ERR_INVALID_ARG;                                \
+    }
+    WINRS_T_CASE(2, 2, 1) WINRS_T_CASE(4, 2, 3) WINRS_T_CASE(4, 3, 2)
+    WINRS_T_CASE(8, 3, 6) WINRS_T_CASE(8, 4, 5) WINRS_T_CASE(8, 5, 4) WINRS_T_CASE(8, 6, 3)
+    WINRS_T_CASE(8, 7, 2) WINRS_T_CASE(16, 5, 12) WINRS_T_CASE(16, 6, 11) WINRS_T_CASE(16, 7, 10)
+    WINRS_T_CASE(16, 8, 9) WINRS_T_CASE(16, 9, 8)
+#undef WINRS_T_CASE
+    return WINRS_ERR_UNSUPPORTED;
+}
+
+int winrs_debug_kernel_count(void) {
+    int n = 0;
+    kernel_entries(&n);
+    return n;
+}
+
+const char* winrs_debug_kernel_name(int i) {
+    int n = 0;
+    const KernelEntry* e = kernel_entries(&n);
+    return (i >= 0 && i < n) ? e[i].name : nullptr;
+}
+
+const char* winrs_debug_plan_kernel(winrs_plan_t plan) { return plan ? plan->pr.entry->name : nullptr; }
+
+}  // extern "C"

@@ -1,0 +1,93 @@
+// Internal plan layout and the index math shared by the CUDA kernels and the
+// host-side FP64 emulator (winrs_debug_emulate).  Not part of the public ABI.
+//
+// Geometry (§3 P@15252-17405, Figures 3/4; R6, R9, R10):
+//   * dY columns [0, k0*r0) form the Omega_a0 region, split into `bands` row
+//     bands (seg_h rows each, the last absorbs the remainder) and `seg_cols`
+//     column segments of seg_w columns (the last may be narrower).  Segment
+//     z = band*seg_cols + col writes dW bucket z (bucket 0 is dW itself).
+//   * dY columns [k0*r0, k0*r0 + k1*r1) are the residual region handled by
+//     Omega_a1 units; per band it is processed by the CTAs of the band's LAST
+//     column segment as a second phase that adds into the same bucket, so no
+//     extra workspace and no second launch is needed.  Columns >= Wo inside
+//     the last unit are zero-masked (R6).
+//   * CTA = (segment, fh, fw-tile, c-block, k-block); it computes the
+//     B_N x B_M x n0 tile dW_z[kb*B_N.., fh, ft*n0 .. ft*n0+n0, cb*B_M..].
+//   * Height clipping (P@32013-33698, Figure 7): a CTA only visits dY rows h
+//     whose X row h+fh-pad lies inside [0, H).
+#pragma once
+#include <stdint.h>
+#include <stddef.h>
+
+#if defined(__CUDACC__)
+#define WINRS_HD __host__ __device__ __forceinline__
+#else
+#define WINRS_HD inline
+#endif
+
+namespace winrs {
+
+struct KernelId {
+    int alpha, n, r;
+};
+
+// Everything a launch needs; passed by value to the kernels (< 4 KB).
+struct Geometry {
+    int N, C, H, W, K, R, S, pad, Ho, Wo;
+    // Omega_a0 region
+    int a0, n0, r0, k0;
+    int seg_h, bands, seg_w, seg_cols;
+    // residual region (a1 == 0: none)
+    int a1, n1, r1, k1;
+    int res_col0;               // = k0 * r0
+    // CTA tiling
+    int tile_k, tile_c;         // B_N (k), B_M (c)
+    int kblocks, cblocks, ftiles;   // ceil(K/B_N), ceil(C/B_M), S/n0
+    int Z;                      // buckets
+    long long dw_elems;         // K*R*S*C
+};
+
+struct CtaCoord {
+    int kb, cb, ft, fh, band, col;
+};
+
+WINRS_HD CtaCoord decode_cta(const Geometry& g, long long bid) {
+    CtaCoord c;
+    c.kb = (int)(bid % g.kblocks); bid /= g.kblocks;
+    c.cb = (int)(bid % g.cblocks); bid /= g.cblocks;
+    c.ft = (int)(bid % g.ftiles);  bid /= g.ftiles;
+    c.fh = (int)(bid % g.R);       bid /= g.R;
+    c.col = (int)(bid % g.seg_cols);
+    c.band = (int)(bid / g.seg_cols);
+    return c;
+}
+
+WINRS_HD long long num_ctas(const Geometry& g) {
+    return (long long)g.kblocks * g.cblocks * g.ftiles * g.R * g.seg_cols * g.bands;
+}
+
+// Valid (clipped) dY rows [hs, he) of a band for filter row fh.
+WINRS_HD void band_rows(const Geometry& g, int band, int fh, int* hs, int* he) {
+    const int h0 = band * g.seg_h;
+    const int h1 = (band == g.bands - 1) ? g.Ho : h0 + g.seg_h;
+    int a = g.pad - fh; if (a < h0) a = h0;
+    int b = g.H + g.pad - fh; if (b > h1) b = h1;
+    *hs = a;
+    *he = b > a ? b : a;
+}
+
+// Omega_a0 units of a column segment: first dY column and unit count.
+WINRS_HD void seg_units(const Geometry& g, int col, int* w_first, int* units) {
+    const int w0 = col * g.seg_w;
+    int w1 = w0 + g.seg_w;
+    const int lim = g.k0 * g.r0;
+    if (w1 > lim) w1 = lim;
+    *w_first = w0;
+    *units = (w1 - w0) / g.r0;
+}
+
+WINRS_HD bool has_residual(const Geometry& g, int col) {
+    return g.a1 != 0 && g.k1 > 0 && col == g.seg_cols - 1;
+}
+
+}  // namespace winrs

@@ -1,0 +1,44 @@
+"""The plan's full decomposition (segments, row clipping, unit split, masked
+tail, residual phase, buckets; §3 P@15252-17405, eq. (6) P@29449)
+evaluated in FP64 on the host by winrs_debug_emulate equals the FP64 oracle —
+the method reaches the plain definition exactly up to rounding."""
+import numpy as np
+import pytest
+
+import paper_conf_icpp_zhangc0zx0025_b200 as W
+from oracle import oracle as O
+
+CASES = [
+    # N, C, H, W, K, R, S, pad, env
+    (1, 4, 8, 8, 4, 3, 3, 1, {}),                                    # tiny BASELINE config
+    (2, 8, 16, 16, 8, 3, 3, 1, {"WINRS_FORCE_Z": "6"}),              # Figure 3-like: many segments
+    (2, 8, 7, 7, 8, 3, 3, 1, {}),                                    # Wo = 7: masked column
+    (2, 8, 9, 33, 4, 3, 3, 1, {"WINRS_FORCE_Z": "3"}),
+    (1, 4, 12, 12, 8, 2, 2, 1, {}),                                  # Omega_4(2,3)
+    (1, 4, 12, 11, 4, 4, 4, 2, {"WINRS_FORCE_Z": "2"}),              # Omega_8(4,5) + Omega_4(2,3), n1 | n0
+    (1, 4, 12, 14, 4, 5, 5, 2, {}),                                  # Omega_16(5,12) + Omega_8(5,4)
+    (1, 4, 10, 12, 4, 7, 7, 3, {}),                                  # Omega_16(7,10) + Omega_8(7,2)
+    (1, 4, 9, 10, 4, 9, 9, 4, {}),                                   # Omega_16(9,8)
+    (1, 4, 9, 9, 4, 6, 6, 2, {}),                                    # width 6
+    (1, 4, 9, 9, 4, 8, 8, 3, {}),                                    # width 8
+    (2, 4, 6, 6, 4, 3, 3, 0, {}),                                    # no padding
+    (1, 4, 5, 9, 4, 3, 3, 2, {"WINRS_FORCE_Z": "4"}),                # pad > needed, clipped rows
+    (3, 36, 6, 6, 40, 3, 3, 1, {"WINRS_FORCE_TILE": "32x32"}),       # channel tails over 2 tiles
+    (2, 8, 10, 10, 8, 3, 3, 1, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
+    (2, 8, 10, 10, 8, 3, 3, 1, {"WINRS_FORCE_PAIR": "8,3,6,0,0,0", "WINRS_FORCE_Z": "4"}),
+]
+
+
+@pytest.mark.parametrize("case", CASES)
+def test_emulated_plan_equals_oracle(case, monkeypatch):
+    N, C, H, Wd, K, R, S, pad, env = case
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    p = W.plan_for_device(N, C, H, Wd, K, R, S, pad, "f32")
+    Ho, Wo = p.info["Ho"], p.info["Wo"]
+    g = np.random.default_rng(sum(case[:8]))
+    X = g.uniform(-1, 1, (N, H, Wd, C))
+    dY = g.uniform(-1, 1, (N, Ho, Wo, K))
+    ref = O.bfc_c(X, dY, R, S, pad)
+    got = W.emulate(p, X, dY)
+    assert O.rel_max_err(got, ref) < 1e-12, (p, O.rel_max_err(got, ref))

@@ -1,0 +1,124 @@
+"""GPU parity: the CUDA path (through the C ABI, via the ctypes binding)
+against the FP64 CPU oracle on the same seeded inputs.
+
+Gate (BASELINE.json north_star): max|err| <= 1e-4 * max|ref| for FP32 inputs,
+<= 2e-2 * max|ref| for FP16 inputs (FP32 accumulation).  Inputs follow the
+paper's accuracy protocol (P@50685): U[0,1], dY x 1e-2 for FP16.
+"""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_icpp_zhangc0zx0025_b200 as W
+from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+from oracle import oracle as O
+
+pytestmark = pytest.mark.gpu
+
+TOL = {"f32": 1e-4, "f16": 2e-2}
+
+
+def _run(layer, X, dY, env=None, monkeypatch=None):
+    if env:
+        for k, v in env.items():
+            monkeypatch.setenv(k, v)
+    p = W.plan(layer.N, layer.C, layer.H, layer.W, layer.K, layer.R, layer.S, layer.pad, layer.dtype)
+    Xg = torch.from_numpy(X).cuda()
+    Gg = torch.from_numpy(dY).cuda()
+    dW = W.bfc(p, Xg, Gg)
+    torch.cuda.synchronize()
+    return p, dW.cpu().numpy().astype(np.float64)
+
+
+def _full_check(layer, dist="u01", env=None, monkeypatch=None, tol=None):
+    X, dY = wl.make_inputs(layer, dist)
+    p, got = _run(layer, X, dY, env, monkeypatch)
+    ref = O.bfc_c(X, dY, layer.R, layer.S, layer.pad)
+    err = O.rel_max_err(got, ref)
+    assert err <= (tol or TOL[layer.dtype]), (layer, p, err)
+    return p, err
+
+
+# ---- configs[0]: tiny, full oracle
+def test_tiny_f32():
+    _full_check(wl.LAYERS["tiny_f32"])
+
+
+# ---- reduced-size versions of every FP32 config: full oracle, several tiles + ragged tails
+REDUCED = [
+    wl.LAYERS["r50_c64_56_f32"].with_(N=2, name="r50_l1_n2"),
+    wl.LAYERS["r50_c128_28_f32"].with_(N=2, C=72, K=100, name="r50_l2_ragged"),
+    wl.LAYERS["r50_c256_14_f32"].with_(N=4, name="r50_l3_n4"),
+    wl.LAYERS["r50_c512_7_f32"].with_(N=2, C=136, K=200, name="r50_l4_ragged"),
+] + [l.with_(N=2, C=40, K=36, name=l.name + "_small") for l in wl.WIDE_F32]
+
+
+@pytest.mark.parametrize("layer", REDUCED, ids=lambda l: l.name)
+def test_reduced_f32(layer):
+    _full_check(layer)
+
+
+@pytest.mark.parametrize("layer", [l for l in REDUCED if l.R <= 4 or l.name.startswith("r50")], ids=lambda l: l.name)
+def test_reduced_f32_signed(layer):
+    """Signed U[-1,1) inputs, gated for alpha <= 8 plans (R17)."""
+    _full_check(layer, dist="signed")
+
+
+FORCED = [
+    {"WINRS_FORCE_Z": "1"}, {"WINRS_FORCE_Z": "5"}, {"WINRS_FORCE_Z": "12"},
+    {"WINRS_FORCE_TILE": "64x64"}, {"WINRS_FORCE_TILE": "32x32", "WINRS_FORCE_Z": "3"},
+    {"WINRS_FORCE_PAIR": "8,3,6,0,0,0"}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_Z": "7"},
+]
+
+
+@pytest.mark.parametrize("env", FORCED, ids=lambda e: ",".join(f"{k[12:]}={v}" for k, v in e.items()))
+def test_forced_plans(env, monkeypatch):
+    layer = wl.LAYERS["r50_c64_56_f32"].with_(N=2, H=30, W=29, C=68, K=44, name="forced")
+    _full_check(layer, env=env, monkeypatch=monkeypatch)
+
+
+def test_determinism():
+    layer = wl.LAYERS["r50_c64_56_f32"].with_(N=3, name="det")
+    X, dY = wl.make_inputs(layer)
+    _, a = _run(layer, X, dY)
+    _, b = _run(layer, X, dY)
+    assert np.array_equal(a, b)
+
+
+def test_zero_and_linearity():
+    layer = wl.LAYERS["r50_c128_28_f32"].with_(N=2, name="lin")
+    X, dY = wl.make_inputs(layer)
+    _, z = _run(layer, X, np.zeros_like(dY))
+    assert np.all(z == 0)
+    _, a = _run(layer, X, dY)
+    _, b = _run(layer, X, (2 * dY).astype(np.float32))
+    assert np.allclose(b, 2 * a, rtol=1e-6, atol=0)
+
+
+# ---- full BASELINE sizes: sampled outputs against the oracle element by element
+FULL_F32 = wl.RESNET50_F32 + wl.WIDE_F32
+
+
+@pytest.mark.parametrize("layer", FULL_F32, ids=lambda l: l.name)
+def test_full_size_sampled(layer):
+    X, dY = wl.make_inputs(layer)
+    p, got = _run(layer, X, dY)
+    idx = wl.sample_indices(layer, 384)
+    ref = O.bfc_c_sampled(X, dY, layer.R, layer.S, layer.pad, idx)
+    err = O.rel_max_err(got.ravel()[idx], ref)
+    assert err <= TOL[layer.dtype], (layer.name, p, err)
+    assert np.isfinite(got).all()
+
+
+def test_abi_errors():
+    import ctypes
+    from paper_conf_icpp_zhangc0zx0025_b200 import _lib
+    p = W.plan(8, 64, 56, 56, 64, 3, 3, 1, "f32")
+    X = torch.zeros(8, 56, 56, 64, device="cuda")
+    dY = torch.zeros(8, 56, 56, 64, device="cuda")
+    dW = torch.zeros(64, 3, 3, 64, device="cuda")
+    L = _lib.lib()
+    assert L.winrs_bfc(p.handle, X.data_ptr() + 4, dY.data_ptr(), dW.data_ptr(), None, None) == 1
+    assert L.winrs_bfc(None, X.data_ptr(), dY.data_ptr(), dW.data_ptr(), None, None) == 1
+    if p.workspace_bytes:
+        assert L.winrs_bfc(p.handle, X.data_ptr(), dY.data_ptr(), dW.data_ptr(), None, None) == 3

@@ -1,0 +1,144 @@
+"""Host-only tests of the planner (§4: kernel-pair selection §4.1
+P@20377, Algorithm 1 §4.2, Algorithm 2 §4.3) through winrs_plan_for_device,
+and of the C ABI surface (include/*.h)."""
+import os
+import re
+
+import pytest
+
+import paper_conf_icpp_zhangc0zx0025_b200 as W
+from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+from paper_conf_icpp_zhangc0zx0025_b200._lib import WinrsError
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_library_exports_every_declared_symbol():
+    import ctypes
+    L = ctypes.CDLL(os.path.join(ROOT, "paper_conf_icpp_zhangc0zx0025_b200", "libwinrs.so"))
+    names = []
+    for h in ("winrs.h", "winrs_debug.h"):
+        src = open(os.path.join(ROOT, "include", h)).read()
+        names += re.findall(r"WINRS_API\s+[\w\s\*]+?\b(winrs_\w+)\s*\(", src)
+    assert len(names) >= 15
+    for n in names:
+        assert hasattr(L, n), n
+    from paper_conf_icpp_zhangc0zx0025_b200._lib import SYMBOLS
+    assert sorted(names) == sorted(s[0] for s in SYMBOLS)
+
+
+def test_figure5_pair():
+    """Golden: F_W=3, O_W=16 -> Omega_8(3,6) on 12 columns + Omega_4(3,2) on 4 (P@21094)."""
+    for line in open(os.path.join(ROOT, "tests", "golden", "figure5_pairs.txt")):
+        if line.startswith("#") or not line.strip():
+            continue
+        FW, OW, a0, n0, r0, k0, a1, n1, r1, k1 = map(int, line.split())
+        # O_W = 16 with F_W = 3 and pad 1 -> W = 16
+        p = W.plan_for_device(8, 64, OW, OW, 64, FW, FW, 1, "f32")
+        i = p.info
+        assert (i["alpha0"], i["n0"], i["r0"], i["k0"]) == (a0, n0, r0, k0)
+        assert (i["alpha1"], i["n1"], i["r1"], i["k1"]) == (a1, n1, r1, k1)
+        assert i["masked_cols"] == 0
+
+
+@pytest.mark.parametrize("S,Wo,expect", [
+    (3, 56, (8, 3, 6, 9, 4, 3, 2, 1, 0)),      # 56 = 9*6 + 2
+    (3, 7, (8, 3, 6, 1, 4, 3, 2, 1, 1)),       # 7 = 6 + 2 - 1 masked (R6)
+    (3, 14, (8, 3, 6, 2, 4, 3, 2, 1, 0)),
+    (3, 28, (8, 3, 6, 4, 4, 3, 2, 2, 0)),
+    (5, 32, (16, 5, 12, 2, 8, 5, 4, 2, 0)),    # SURVEY R7 example
+    (7, 32, (16, 7, 10, 3, 8, 7, 2, 1, 0)),
+    (9, 32, (16, 9, 8, 4, 0, 0, 0, 0, 0)),
+    (2, 33, (4, 2, 3, 11, 0, 0, 0, 0, 0)),
+    (4, 33, (8, 4, 5, 6, 4, 2, 3, 1, 0)),
+])
+def test_pair_selection(S, Wo, expect):
+    pad = S // 2
+    Wd = Wo - 2 * pad + S - 1
+    p = W.plan_for_device(4, 32, 8, Wd, 32, S, S, pad, "f32")
+    i = p.info
+    assert i["Wo"] == Wo
+    got = (i["alpha0"], i["n0"], i["r0"], i["k0"], i["alpha1"], i["n1"], i["r1"], i["k1"], i["masked_cols"])
+    assert got == expect
+
+
+SHAPES = [(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype) for l in wl.LAYERS.values() if l.dtype == "f32"] + [
+    (3, 8, 17, 23, 12, 3, 3, 1, "f32"), (2, 4, 9, 40, 8, 5, 5, 0, "f32"), (1, 4, 30, 30, 4, 6, 6, 3, "f32"),
+    (2, 12, 11, 19, 16, 8, 8, 2, "f32"), (2, 4, 5, 5, 4, 2, 2, 0, "f32"), (1, 4, 3, 3, 4, 3, 3, 0, "f32"),
+]
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+def test_plan_invariants(shape):
+    N, C, H, Wd, K, R, S, pad, dt = shape
+    p = W.plan_for_device(N, C, H, Wd, K, R, S, pad, dt)
+    i = p.info
+    Ho, Wo = H + 2 * pad - R + 1, Wd + 2 * pad - S + 1
+    assert (i["Ho"], i["Wo"]) == (Ho, Wo)
+    # (1) n0, n1 divide F_W
+    assert S % i["n0"] == 0 and (i["alpha1"] == 0 or S % i["n1"] == 0)
+    assert i["alpha0"] == i["n0"] + i["r0"] - 1
+    # (2) units cover O_W; masked columns only inside the last unit
+    cover = i["k0"] * i["r0"] + i["k1"] * i["r1"]
+    assert cover - Wo == i["masked_cols"] >= 0
+    last_r = i["r1"] if i["k1"] else i["r0"]
+    assert i["masked_cols"] < last_r
+    # segments tile the Omega_a0 region: widths are multiples of r0
+    assert i["seg_w"] % i["r0"] == 0
+    assert i["seg_cols"] == -(-(i["k0"] * i["r0"]) // i["seg_w"])
+    assert 1 <= i["seg_h"] <= Ho and i["bands"] == max(1, Ho // i["seg_h"])
+    assert i["Z"] == i["bands"] * i["seg_cols"]
+    # workspace = (Z-1)|dW| fp32 and <= 4% of the data bytes (R11)
+    dw = K * R * S * C
+    assert i["workspace_bytes"] == (i["Z"] - 1) * 4 * dw
+    esz = 4 if dt == "f32" else 2
+    data = esz * (N * H * Wd * C + N * Ho * Wo * K)
+    assert i["workspace_bytes"] <= 0.04 * data + 1e-9
+    # Winograd work never exceeds direct work for alpha >= 4 kernels
+    assert i["ewm_flops"] > 0
+    # determinism
+    q = W.plan_for_device(N, C, H, Wd, K, R, S, pad, dt)
+    assert q.info == i and q.kernel_name == p.kernel_name
+
+
+def test_error_codes():
+    with pytest.raises(WinrsError) as e:
+        W.plan_for_device(0, 4, 8, 8, 4, 3, 3, 1)
+    assert e.value.status == 1
+    with pytest.raises(WinrsError) as e:
+        W.plan_for_device(1, 4, 2, 2, 4, 5, 5, 0)           # Ho < 1
+    assert e.value.status == 1
+    with pytest.raises(WinrsError) as e:
+        W.plan_for_device(1, 4, 8, 8, 4, 3, 3, -1)
+    assert e.value.status == 1
+    for S in (1, 11, 13):                                     # no kernel width divides S (P@28451)
+        with pytest.raises(WinrsError) as e:
+            W.plan_for_device(1, 4, 16, 16, 4, 3, S, 0)
+        assert e.value.status == 2
+    with pytest.raises(WinrsError) as e:
+        W.plan_for_device(1, 6, 8, 8, 4, 3, 3, 1)             # C % 4 != 0
+    assert e.value.status == 2
+    with pytest.raises(WinrsError) as e:
+        W.plan_for_device(1, 4, 8, 8, 4, 3, 3, 1, cc=(9, 0))  # not sm_100
+    assert e.value.status == 2
+
+
+def test_supported_widths():
+    """F_W in {n*k : 2 <= k <= 9} (P@28451): every S with a divisor in 2..9 plans."""
+    for S in range(2, 40):
+        ok = any(S % n == 0 for n in range(2, 10))
+        try:
+            W.plan_for_device(1, 4, S + 4, S + 4, 4, 2, S, 0)
+            assert ok, S
+        except WinrsError as e:
+            assert not ok and e.status == 2, S
+
+
+def test_forced_overrides(monkeypatch):
+    monkeypatch.setenv("WINRS_FORCE_Z", "6")
+    monkeypatch.setenv("WINRS_FORCE_TILE", "32x32")
+    p = W.plan_for_device(8, 64, 56, 56, 64, 3, 3, 1, "f32")
+    assert p.info["tile_k0"] == 32 and p.info["Z"] >= 2
+    monkeypatch.setenv("WINRS_FORCE_PAIR", "8,3,6,0,0,0")
+    p = W.plan_for_device(8, 64, 56, 56, 64, 3, 3, 1, "f32")
+    assert p.info["alpha1"] == 0 and p.info["k0"] == 10 and p.info["masked_cols"] == 4
