@@ -1,0 +1,53 @@
+#!/usr/bin/env python3
+"""Summarise an ncu --set full report (key roofline / pipe / stall metrics per
+kernel launch) as a markdown table.  Usage: ncu_summary.py report.ncu-rep [title]"""
+import csv
+import io
+import subprocess
+import sys
+
+METRICS = [
+    ("gpu__time_duration.sum", "duration"),
+    ("launch__grid_size", "grid"),
+    ("launch__registers_per_thread", "regs"),
+    ("sm__warps_active.avg.pct_of_peak_sustained_active", "warps active %"),
+    ("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active", "FMA pipe %"),
+    ("sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active", "FMA inst %"),
+    ("sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active", "ALU pipe %"),
+    ("sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active", "tensor pipe %"),
+    ("sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active", "LSU inst %"),
+    ("dram__bytes_read.sum", "DRAM read"),
+    ("dram__bytes_write.sum", "DRAM write"),
+    ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "DRAM %"),
+    ("lts__t_bytes.sum", "L2 bytes"),
+    ("l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum", "smem bank confl."),
+    ("smsp__inst_executed.sum", "warp inst"),
+    ("smsp__average_warps_issue_stalled_wait_per_issue_active.ratio", "stall wait"),
+    ("smsp__average_warps_issue_stalled_short_scoreboard_per_issue_active.ratio", "stall short_sb"),
+    ("smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio", "stall long_sb"),
+    ("smsp__average_warps_issue_stalled_barrier_per_issue_active.ratio", "stall barrier"),
+    ("smsp__average_warps_issue_stalled_math_pipe_throttle_per_issue_active.ratio", "stall math_throttle"),
+]
+
+
+def main():
+    rep = sys.argv[1]
+    title = sys.argv[2] if len(sys.argv) > 2 else rep
+    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    r = list(csv.reader(io.StringIO(raw)))
+    hdr, units, rows = r[0], r[1], r[2:]
+    col = {h: i for i, h in enumerate(hdr)}
+    kcol = col.get("Kernel Name")
+    print(f"### {title}\n")
+    print("| metric | " + " | ".join(f"#{i}" for i in range(len(rows))) + " |")
+    print("|---|" + "---|" * len(rows))
+    print("| kernel | " + " | ".join(row[kcol][:48].replace("|", "/") for row in rows) + " |")
+    for m, name in METRICS:
+        if m in col:
+            u = units[col[m]]
+            print(f"| {name} ({u}) | " + " | ".join(row[col[m]] for row in rows) + " |")
+    print()
+
+
+if __name__ == "__main__":
+    main()
