@@ -54,8 +54,11 @@ class Plan:
 
     def __del__(self):
         h, self._h = getattr(self, "_h", None), None
-        if h and _lib._lib is not None:
-            _lib._lib.winrs_plan_destroy(h)
+        try:
+            if h and _lib is not None and _lib._lib is not None:
+                _lib._lib.winrs_plan_destroy(h)
+        except Exception:   # interpreter shutdown
+            pass
 
     def __repr__(self):
         i = self.info

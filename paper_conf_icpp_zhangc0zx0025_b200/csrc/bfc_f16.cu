@@ -1,8 +1,96 @@
-// FP16 tensor-core kernels (tcgen05) — registered here.
+// FP16 tensor-core kernel instantiations, TMA tensor-map encoding and launch.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <mutex>
+#include "bfc_f16.cuh"
+#include "launch_util.cuh"
 #include "registry.h"
+
 namespace winrs {
-const KernelEntry* f16_entries(int* n) {
-    *n = 0;
-    return nullptr;
+namespace f16k {
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeTiledFn encode_fn() {
+    static EncodeTiledFn fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<EncodeTiledFn>(p);
+    });
+    return fn;
 }
+
+// 4-D NHWC fp16 tensor [N][H][W][Ch] as TMA dims {Ch, W, H, N}; box {bc, bw, 1, bn}.
+// Out-of-bounds elements are filled with zeros.
+static bool make_map(CUtensorMap* m, const void* base, int N, int H, int W, int Ch, int bc, int bw, int bn) {
+    EncodeTiledFn fn = encode_fn();
+    if (!fn) return false;
+    const cuuint64_t dims[4] = {(cuuint64_t)Ch, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
+    const cuuint64_t strides[3] = {(cuuint64_t)Ch * 2, (cuuint64_t)W * Ch * 2, (cuuint64_t)H * W * Ch * 2};
+    const cuuint32_t box[4] = {(cuuint32_t)bc, (cuuint32_t)bw, 1u, (cuuint32_t)bn};
+    const cuuint32_t es[4] = {1u, 1u, 1u, 1u};
+    return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+static int images_per_box(int N) {
+    for (int nb : {8, 4, 2})
+        if (N % nb == 0) return nb;
+    return 1;
+}
+
+template <int A0, int N0, int R0, int A1, int N1, int R1>
+cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
+    static std::atomic<unsigned long long> done{0};
+    auto k = bfc_f16_kernel<A0, N0, R0, A1, N1, R1>;
+    constexpr size_t sm = Smem<A0, R0>::bytes;
+    cudaError_t e = ensure_smem_attr(k, sm, done);
+    if (e != cudaSuccess) return e;
+    const long long grid = num_ctas(g);
+    if (grid <= 0) return cudaSuccess;
+    Args a;
+    a.g = g;
+    a.dW = dW;
+    a.ws = ws;
+    a.nb = images_per_box(g.N);
+    CUtensorMap mX0, mY0, mX1, mY1;
+    if (!make_map(&mX0, X, g.N, g.H, g.W, g.C, BM, A0, a.nb) ||
+        !make_map(&mY0, dY, g.N, g.Ho, g.Wo, g.K, BN, R0, a.nb))
+        return cudaErrorInvalidValue;
+    if (A1 != 0) {
+        if (!make_map(&mX1, X, g.N, g.H, g.W, g.C, BM, A1 ? A1 : A0, a.nb) ||
+            !make_map(&mY1, dY, g.N, g.Ho, g.Wo, g.K, BN, R1 ? R1 : R0, a.nb))
+            return cudaErrorInvalidValue;
+    } else {
+        mX1 = mX0;
+        mY1 = mY0;
+    }
+    k<<<(unsigned)grid, NTHREADS, sm, stream>>>(a, mX0, mY0, mX1, mY1);
+    return cudaGetLastError();
+}
+
+}  // namespace f16k
+
+#define WINRS_F16_ENTRY(A0, N0, R0, A1, N1, R1)                                                      \
+    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, ::winrs::f16k::BM, ::winrs::f16k::NTHREADS, 1,     \
+     ::winrs::f16k::Smem<A0, R0>::bytes, &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1>,             \
+     "f16tc_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x64"}
+
+const KernelEntry* f16_entries(int* n) {
+    static const KernelEntry e[] = {
+        WINRS_F16_ENTRY(8, 3, 6, 4, 3, 2),
+        WINRS_F16_ENTRY(8, 3, 6, 0, 0, 0),
+        WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0),
+    };
+    *n = sizeof(e) / sizeof(e[0]);
+    return e;
+}
+
 }  // namespace winrs

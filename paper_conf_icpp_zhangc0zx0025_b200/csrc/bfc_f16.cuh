@@ -1,0 +1,468 @@
+// FP16-in / FP32-accumulate tensor-core fused WinRS BFC kernel for sm_100a
+// (tcgen05 + TMEM + TMA + mbarrier, warp-specialised).
+//
+// PAPER.md §5 (P@28371-39921) ported FP16 kernels run the alpha-batched GEMM
+// on Tensor Cores with FT, IT and OT in FP32 (P@38729 "FT, IT, and OT are
+// temporarily computed in FP32 precision, and finally converted to FP16").
+// This is the B200 design of that kernel:
+//
+//   warp 0      TMA producer: per chunk of KC = 16 depth entries d = (h, u, n)
+//               it loads the raw dY units (box [B_N=128 k][r][1][NB images])
+//               and X windows (box [B_M=64 c][alpha][1][NB]) into a 2-stage
+//               raw ring; TMA out-of-bounds zero fill implements the width
+//               padding (P@33854), the masked tail unit (R6), the
+//               channel tails and the depth tail.
+//   warp 1      TMEM owner + MMA issuer: per chunk one
+//               tcgen05.mma.cta_group::1.kind::f16 (M=128 k, N=64 c, K=16 d)
+//               per Winograd point xi, accumulators D[xi] in TMEM columns
+//               [xi*64, xi*64+64) (eq. (6): everything stays in the Winograd
+//               domain for the whole main loop, P@29449).
+//   warps 2..7  transformers: FT G*w (dY) and IT D^T*x (X) in FP32 — packed
+//               f32x2 lanes (FFMA2) — then RN conversion to FP16 and 16-byte
+//               stores straight into the UMMA K-major (no-swizzle) operand
+//               layout of a 2-stage operand ring.  After the last chunk
+//               warps 2..5 (one per TMEM lane quarter) are the epilogue:
+//               tcgen05.ld -> OT A^T v in FP32 -> bucket (store or add).
+// The residual kernel Omega_a1 runs as further jobs of the same CTA (last
+// column segment only), adding into the same bucket (R10).
+#pragma once
+#include <cuda.h>
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include "winograd_generated.cuh"
+#include "winrs_internal.h"
+#include "winrs_vec.cuh"
+
+namespace winrs {
+namespace f16k {
+
+constexpr int BN = 128;          // k rows = UMMA M (TMEM lanes)
+constexpr int BM = 64;           // c columns = UMMA N
+constexpr int KC = 16;           // depth entries per chunk = UMMA K
+constexpr int NTHREADS = 256;    // 8 warps
+constexpr int TX_WARPS = 6;      // transformer warps (2..7)
+constexpr int S_RAW = 2, S_OP = 2;
+
+struct Args {
+    Geometry g;
+    float* dW;
+    float* ws;
+    int nb;          // images per TMA box (divides N and KC)
+};
+
+// ----------------------------------------------------------------------------- PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    const uint32_t a = smem_u32(bar);
+    asm volatile(
+        "{\n"
+        ".reg .pred P;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n"
+        "@!P bra WAIT_%=;\n"
+        "}\n" :: "r"(a), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tma_load_4d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                                            int c2, int c3) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];"
+        :: "r"(smem_u32(dst)), "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(c3),
+           "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void prefetch_tmap(const CUtensorMap* map) {
+    asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(map)) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// UMMA shared-memory descriptor, K-major, no swizzle: core matrices of 8 rows
+// x 16 bytes; LBO = byte distance between the two K-halves (8 elements each)
+// of a 16-deep slab, SBO = byte distance between 8-row groups.
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+           ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46);
+}
+// kind::f16 instruction descriptor: D f32, A/B f16, both K-major, M = 128, N = BM.
+constexpr uint32_t IDESC = (1u << 4) | ((uint32_t)(BM >> 3) << 17) | ((uint32_t)(BN >> 4) << 24);
+
+__device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accumulate) {
+    asm volatile(
+        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
+        :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(IDESC), "r"(accumulate));
+}
+__device__ __forceinline__ void umma_commit(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                 :: "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, float* v) {
+    uint32_t r[8];
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+                 : "r"(taddr));
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
+__device__ __forceinline__ uint32_t pack_h2(float lo, float hi) {
+    __half2 h = __floats2half2_rn(lo, hi);   // cvt.rn.f16x2.f32
+    return *reinterpret_cast<uint32_t*>(&h);
+}
+__device__ __forceinline__ F2 ld_h2(const __half* p) {
+    const __half2 h = *reinterpret_cast<const __half2*>(p);
+    const float2 f = __half22float2(h);
+    return F2{f.x, f.y};
+}
+
+// ----------------------------------------------------------------------------- shared memory plan
+template <int A0, int R0>
+struct Smem {
+    static constexpr int RAW_Y = KC * R0 * BN * 2;       // bytes per raw stage (dY)
+    static constexpr int RAW_X = KC * A0 * BM * 2;       // bytes per raw stage (X)
+    static constexpr int RAW = RAW_Y + RAW_X;
+    static constexpr int OPA = BN * KC * 2;              // one A_xi slab (4 KB)
+    static constexpr int OPB = BM * KC * 2;              // one B_xi slab (2 KB)
+    static constexpr int OP = A0 * (OPA + OPB);
+    static constexpr int raw_off = 0;
+    static constexpr int op_off = S_RAW * RAW;
+    static constexpr int bar_off = op_off + S_OP * OP;
+    static constexpr int bytes = bar_off + 256;
+};
+
+// Operand layout (K-major, no swizzle): element (row, kk) of a 16-deep slab at
+// byte (row/8)*256 + (kk/8)*128 + (row%8)*16 + (kk%8)*2.
+__device__ __forceinline__ uint32_t op_row_off(int row, int dgroup) {
+    return (uint32_t)((row >> 3) * 256 + dgroup * 128 + (row & 7) * 16);
+}
+
+struct Job {
+    int phase;          // 0: Omega_a0, 1: Omega_a1
+    int units, w_first, fw0;
+    bool accumulate;
+};
+
+struct Barriers {
+    uint64_t raw_full[S_RAW], raw_empty[S_RAW], op_full[S_OP], op_empty[S_OP], acc_full, acc_empty;
+    uint32_t tmem_base;
+};
+
+// Depth entry -> (n, h, u) for chunk-box issue.
+__device__ __forceinline__ void depth_coord(long long d, int N, int units, int hs, int* n, int* h, int* u) {
+    *n = (int)(d % N);
+    const long long t = d / N;
+    *u = (int)(t % units);
+    *h = hs + (int)(t / units);
+}
+
+// ---- transformer work for one chunk: FT units (k pair p, d-group g) and IT units.
+template <int A, int NN, int RR>
+__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tx_id) {
+    using WT = Wino<A, NN, RR>;
+    constexpr int RAW_Y = KC * RR * BN * 2;
+    const __half* rawY = reinterpret_cast<const __half*>(raw);            // [KC][RR][BN]
+    const __half* rawX = reinterpret_cast<const __half*>(raw + RAW_Y);    // [KC][A][BM]
+    constexpr int OPA = BN * KC * 2, OPB = BM * KC * 2;
+    if (tx_id < (BN / 2) * 2) {
+        // FT: rows k = 2p, 2p+1 of every A_xi, depth group g (8 entries)
+        const int p = tx_id % (BN / 2), g = tx_id / (BN / 2);
+        uint32_t pk[A][2][4];   // [xi][row k / k+1][4 x half2 along d]
+#pragma unroll
+        for (int j = 0; j < 8; j += 2) {
+            F2 o0[A], o1[A];
+            {
+                F2 w[RR];
+                const __half* src = rawY + ((g * 8 + j) * RR) * BN + 2 * p;
+#pragma unroll
+                for (int i = 0; i < RR; ++i) w[i] = ld_h2(src + i * BN);
+                WT::ft(w, o0);
+            }
+            {
+                F2 w[RR];
+                const __half* src = rawY + ((g * 8 + j + 1) * RR) * BN + 2 * p;
+#pragma unroll
+                for (int i = 0; i < RR; ++i) w[i] = ld_h2(src + i * BN);
+                WT::ft(w, o1);
+            }
+#pragma unroll
+            for (int x = 0; x < A; ++x) {
+                pk[x][0][j / 2] = pack_h2(o0[x].x, o1[x].x);
+                pk[x][1][j / 2] = pack_h2(o0[x].y, o1[x].y);
+            }
+        }
+#pragma unroll
+        for (int x = 0; x < A; ++x) {
+            uint8_t* a = op + x * OPA;
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+                uint4 v = make_uint4(pk[x][e][0], pk[x][e][1], pk[x][e][2], pk[x][e][3]);
+                *reinterpret_cast<uint4*>(a + op_row_off(2 * p + e, g)) = v;
+            }
+        }
+    } else if (tx_id < (BN / 2) * 2 + (BM / 2) * 2) {
+        // IT: rows c = 2q, 2q+1 of every B_xi, depth group g
+        const int t = tx_id - BN;
+        const int q = t % (BM / 2), g = t / (BM / 2);
+        uint32_t pk[A][2][4];
+#pragma unroll
+        for (int j = 0; j < 8; j += 2) {
+            F2 o0[A], o1[A];
+            {
+                F2 xv[A];
+                const __half* src = rawX + ((g * 8 + j) * A) * BM + 2 * q;
+#pragma unroll
+                for (int i = 0; i < A; ++i) xv[i] = ld_h2(src + i * BM);
+                WT::it(xv, o0);
+            }
+            {
+                F2 xv[A];
+                const __half* src = rawX + ((g * 8 + j + 1) * A) * BM + 2 * q;
+#pragma unroll
+                for (int i = 0; i < A; ++i) xv[i] = ld_h2(src + i * BM);
+                WT::it(xv, o1);
+            }
+#pragma unroll
+            for (int x = 0; x < A; ++x) {
+                pk[x][0][j / 2] = pack_h2(o0[x].x, o1[x].x);
+                pk[x][1][j / 2] = pack_h2(o0[x].y, o1[x].y);
+            }
+        }
+#pragma unroll
+        for (int x = 0; x < A; ++x) {
+            uint8_t* b = op + A * OPA + x * OPB;
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+                uint4 v = make_uint4(pk[x][e][0], pk[x][e][1], pk[x][e][2], pk[x][e][3]);
+                *reinterpret_cast<uint4*>(b + op_row_off(2 * q + e, g)) = v;
+            }
+        }
+    }
+}
+
+// ---- epilogue of one job: TMEM -> OT -> bucket.  Called by warps 2..5.
+template <int A, int NN, int RR>
+__device__ __forceinline__ void epilogue(const Geometry& g, float* bucket, const CtaCoord& cc, int fw0, bool accumulate,
+                                         bool empty, uint32_t tmem_base, int warp) {
+    using WT = Wino<A, NN, RR>;
+    const int quarter = warp & 3;
+    const int lane = threadIdx.x & 31;
+    const int kl = quarter * 32 + lane;
+    const int kg = cc.kb * BN + kl;
+    const bool krow_ok = kg < g.K;
+#pragma unroll 1
+    for (int c0 = 0; c0 < BM; c0 += 8) {
+        float v[A][8];
+        if (!empty) {
+#pragma unroll
+            for (int x = 0; x < A; ++x)
+                tmem_ld8(tmem_base + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(x * BM + c0), v[x]);
+            tmem_wait_ld();
+        } else {
+#pragma unroll
+            for (int x = 0; x < A; ++x)
+#pragma unroll
+                for (int i = 0; i < 8; ++i) v[x][i] = 0.f;
+        }
+        float y[NN][8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            float vv[A], yy[NN];
+#pragma unroll
+            for (int x = 0; x < A; ++x) vv[x] = v[x][i];
+            WT::ot(vv, yy);
+#pragma unroll
+            for (int j = 0; j < NN; ++j) y[j][i] = yy[j];
+        }
+        const int cg = cc.cb * BM + c0;
+        if (krow_ok && cg < g.C) {   // C % 8 == 0, so an 8-column group is all in or all out
+            float* dst = bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0) * g.C + cg;
+#pragma unroll
+            for (int j = 0; j < NN; ++j) {
+                float4* d4 = reinterpret_cast<float4*>(dst + (long long)j * g.C);
+                float4 a = make_float4(y[j][0], y[j][1], y[j][2], y[j][3]);
+                float4 b = make_float4(y[j][4], y[j][5], y[j][6], y[j][7]);
+                if (accumulate) {
+                    const float4 pa = d4[0], pb = d4[1];
+                    a.x += pa.x; a.y += pa.y; a.z += pa.z; a.w += pa.w;
+                    b.x += pb.x; b.y += pb.y; b.z += pb.z; b.w += pb.w;
+                }
+                d4[0] = a;
+                d4[1] = b;
+            }
+        }
+    }
+}
+
+template <int A0, int N0, int R0, int A1, int N1, int R1>
+__global__ void __launch_bounds__(NTHREADS, 1)
+bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX0,
+               const __grid_constant__ CUtensorMap tmY0, const __grid_constant__ CUtensorMap tmX1,
+               const __grid_constant__ CUtensorMap tmY1) {
+    using SM = Smem<A0, R0>;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    const Geometry& g = args.g;
+    Barriers* bars = reinterpret_cast<Barriers*>(smem + SM::bar_off);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+    const CtaCoord cc = decode_cta(g, blockIdx.x);
+    const int seg = cc.band * g.seg_cols + cc.col;
+    float* bucket = seg == 0 ? args.dW : args.ws + (long long)(seg - 1) * g.dw_elems;
+    int hs, he;
+    band_rows(g, cc.band, cc.fh, &hs, &he);
+    int w_first, units;
+    seg_units(g, cc.col, &w_first, &units);
+    const int rows = he - hs;
+
+    // Job list (identical in every role).
+    Job jobs[1 + 9];
+    int njobs = 0;
+    jobs[njobs++] = Job{0, units, w_first, cc.ft * N0, false};
+    if constexpr (A1 != 0) {
+        if (has_residual(g, cc.col))
+            for (int j = 0; j < N0 / N1; ++j) jobs[njobs++] = Job{1, g.k1, g.res_col0, cc.ft * N0 + j * N1, true};
+    }
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < S_RAW; ++s) { mbar_init(&bars->raw_full[s], 1); mbar_init(&bars->raw_empty[s], TX_WARPS); }
+        for (int s = 0; s < S_OP; ++s) { mbar_init(&bars->op_full[s], TX_WARPS); mbar_init(&bars->op_empty[s], 1); }
+        mbar_init(&bars->acc_full, 1);
+        mbar_init(&bars->acc_empty, 4);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 0 && lane == 0) {
+        prefetch_tmap(&tmX0); prefetch_tmap(&tmY0);
+        if (A1 != 0) { prefetch_tmap(&tmX1); prefetch_tmap(&tmY1); }
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;"
+                     :: "r"(smem_u32(&bars->tmem_base)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = bars->tmem_base;
+
+    if (warp == 0) {
+        // ===================== TMA producer =====================
+        if (lane == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            for (int jb = 0; jb < njobs; ++jb) {
+                const Job& J = jobs[jb];
+                const int RRj = J.phase == 0 ? R0 : R1;
+                const int Aj = J.phase == 0 ? A0 : A1;
+                const CUtensorMap* mX = J.phase == 0 ? &tmX0 : &tmX1;
+                const CUtensorMap* mY = J.phase == 0 ? &tmY0 : &tmY1;
+                const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
+                const int nch = (int)((depth + KC - 1) / KC);
+                const uint32_t bytes = (uint32_t)(KC * (RRj * BN + Aj * BM) * 2);
+                for (int ch = 0; ch < nch; ++ch) {
+                    mbar_wait(&bars->raw_empty[s], ph ^ 1);
+                    uint8_t* raw = smem + SM::raw_off + s * SM::RAW;
+                    uint8_t* rY = raw;
+                    uint8_t* rX = raw + KC * RRj * BN * 2;
+                    mbar_arrive_expect_tx(&bars->raw_full[s], bytes);
+                    for (int b = 0; b < KC; b += args.nb) {
+                        const long long d = (long long)ch * KC + b;
+                        int n = g.N, h = hs, u = 0;   // past-the-end image => zero fill
+                        if (d < depth) depth_coord(d, g.N, J.units, hs, &n, &h, &u);
+                        const int w0 = J.w_first + u * RRj;
+                        tma_load_4d(rY + b * RRj * BN * 2, mY, &bars->raw_full[s], cc.kb * BN, w0, h, n);
+                        tma_load_4d(rX + b * Aj * BM * 2, mX, &bars->raw_full[s], cc.cb * BM,
+                                    w0 + J.fw0 - g.pad, h + cc.fh - g.pad, n);
+                    }
+                    if (++s == S_RAW) { s = 0; ph ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ===================== MMA issuer =====================
+        if (lane == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            for (int jb = 0; jb < njobs; ++jb) {
+                const Job& J = jobs[jb];
+                const int Aj = J.phase == 0 ? A0 : A1;
+                const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
+                const int nch = (int)((depth + KC - 1) / KC);
+                if (jb > 0) {
+                    mbar_wait(&bars->acc_empty, (uint32_t)((jb - 1) & 1));
+                    tc_fence_after();
+                }
+                for (int ch = 0; ch < nch; ++ch) {
+                    mbar_wait(&bars->op_full[s], ph);
+                    tc_fence_after();
+                    const uint32_t base = smem_u32(smem + SM::op_off + s * SM::OP);
+                    for (int x = 0; x < Aj; ++x) {
+                        const uint64_t ad = umma_desc(base + x * SM::OPA, 128, 256);
+                        const uint64_t bd = umma_desc(base + Aj * SM::OPA + x * SM::OPB, 128, 256);
+                        umma_f16(tmem_base + (uint32_t)(x * BM), ad, bd, ch > 0 ? 1u : 0u);
+                    }
+                    umma_commit(&bars->op_empty[s]);
+                    if (++s == S_OP) { s = 0; ph ^= 1; }
+                }
+                umma_commit(&bars->acc_full);
+            }
+        }
+    } else {
+        // ===================== transformers (+ epilogue) =====================
+        const int tx_id = threadIdx.x - 64;
+        int sr = 0, so = 0;
+        uint32_t phr = 0, pho = 0;
+        for (int jb = 0; jb < njobs; ++jb) {
+            const Job& J = jobs[jb];
+            const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
+            const int nch = (int)((depth + KC - 1) / KC);
+            for (int ch = 0; ch < nch; ++ch) {
+                mbar_wait(&bars->raw_full[sr], phr);
+                mbar_wait(&bars->op_empty[so], pho ^ 1);
+                const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
+                uint8_t* op = smem + SM::op_off + so * SM::OP;
+                if (J.phase == 0) transform_chunk<A0, N0, R0>(raw, op, tx_id);
+                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1>(raw, op, tx_id);
+                fence_proxy_async();
+                __syncwarp();
+                if (lane == 0) {
+                    mbar_arrive(&bars->op_full[so]);
+                    mbar_arrive(&bars->raw_empty[sr]);
+                }
+                if (++sr == S_RAW) { sr = 0; phr ^= 1; }
+                if (++so == S_OP) { so = 0; pho ^= 1; }
+            }
+            if (warp < 6) {
+                mbar_wait(&bars->acc_full, (uint32_t)(jb & 1));
+                tc_fence_after();
+                if (J.phase == 0)
+                    epilogue<A0, N0, R0>(g, bucket, cc, J.fw0, J.accumulate, nch == 0, tmem_base, warp);
+                else if constexpr (A1 != 0)
+                    epilogue<A1, N1, R1>(g, bucket, cc, J.fw0, J.accumulate, nch == 0, tmem_base, warp);
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&bars->acc_empty);
+            }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 1) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem_base));
+    }
+}
+
+}  // namespace f16k
+}  // namespace winrs

@@ -122,3 +122,58 @@ def test_abi_errors():
     assert L.winrs_bfc(None, X.data_ptr(), dY.data_ptr(), dW.data_ptr(), None, None) == 1
     if p.workspace_bytes:
         assert L.winrs_bfc(p.handle, X.data_ptr(), dY.data_ptr(), dW.data_ptr(), None, None) == 3
+
+
+# ============================================================== FP16 tensor-core path
+REDUCED_F16 = [
+    wl.LAYERS["r50_c64_56_f16"].with_(N=2, name="r50f16_l1_n2"),
+    wl.LAYERS["r50_c128_28_f16"].with_(N=2, C=72, K=200, name="r50f16_l2_ragged"),
+    wl.LAYERS["r50_c256_14_f16"].with_(N=4, name="r50f16_l3_n4"),
+    wl.LAYERS["r50_c512_7_f16"].with_(N=3, C=136, K=264, name="r50f16_l4_ragged_n3"),
+    wl.LAYERS["vgg_64_64_224_f16"].with_(N=1, H=60, W=61, name="vgg_l1_crop"),
+    wl.LAYERS["r50_c64_56_f16"].with_(N=5, H=9, W=20, C=8, K=8, name="f16_tiny_channels_n5"),
+]
+
+
+@pytest.mark.parametrize("layer", REDUCED_F16, ids=lambda l: l.name)
+def test_reduced_f16(layer):
+    _full_check(layer)
+
+
+@pytest.mark.parametrize("layer", REDUCED_F16[:3], ids=lambda l: l.name)
+def test_reduced_f16_signed(layer):
+    _full_check(layer, dist="signed")
+
+
+FORCED_F16 = [
+    {"WINRS_FORCE_Z": "1"}, {"WINRS_FORCE_Z": "7"},
+    {"WINRS_FORCE_PAIR": "8,3,6,0,0,0"}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_Z": "3"},
+]
+
+
+@pytest.mark.parametrize("env", FORCED_F16, ids=lambda e: ",".join(f"{k[12:]}={v}" for k, v in e.items()))
+def test_forced_plans_f16(env, monkeypatch):
+    layer = wl.LAYERS["r50_c64_56_f16"].with_(N=2, H=30, W=29, C=72, K=136, name="forced16")
+    _full_check(layer, env=env, monkeypatch=monkeypatch)
+
+
+def test_determinism_f16():
+    layer = wl.LAYERS["r50_c128_28_f16"].with_(N=3, name="det16")
+    X, dY = wl.make_inputs(layer)
+    _, a = _run(layer, X, dY)
+    _, b = _run(layer, X, dY)
+    assert np.array_equal(a, b)
+
+
+FULL_F16 = wl.RESNET50_F16 + wl.VGG16_F16 + [wl.LAYERS["r50_l3_n512_f16"]]
+
+
+@pytest.mark.parametrize("layer", FULL_F16, ids=lambda l: l.name)
+def test_full_size_sampled_f16(layer):
+    X, dY = wl.make_inputs(layer)
+    p, got = _run(layer, X, dY)
+    idx = wl.sample_indices(layer, 256)
+    ref = O.bfc_c_sampled(X, dY, layer.R, layer.S, layer.pad, idx)
+    err = O.rel_max_err(got.ravel()[idx], ref)
+    assert err <= TOL[layer.dtype], (layer.name, p, err)
+    assert np.isfinite(got).all()

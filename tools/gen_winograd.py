@@ -138,20 +138,7 @@ def check_identity(alpha, n, r, A, G, DT):
 # ----------------------------------------------------------------------------- codegen
 
 def lit(v: Fr) -> str:
-    if v.denominator == 1:
-        return f"T({v.numerator})"
-    return f"(T({v.numerator}) / T({v.denominator}))"
-
-
-def term(coef: Fr, var: str):
-    """Returns (sign, expr) for coef*var; sign in {+1,-1}."""
-    if coef == 1:
-        return 1, var
-    if coef == -1:
-        return -1, var
-    if coef > 0:
-        return 1, f"{lit(coef)} * {var}"
-    return -1, f"{lit(-coef)} * {var}"
+    return f"wc<T>({v.numerator}, {v.denominator})"
 
 
 def _nmul(terms):
@@ -159,36 +146,47 @@ def _nmul(terms):
 
 
 def lin(terms):
-    """Sum of (coef, var) pairs as one expression ('T(0)' if empty).  A common
-    |coefficient| m is factored out, m * (sum (c/m) x), when that saves
-    multiplies (the eq. (7) row scaling makes many row entries equal)."""
+    """sum_i c_i x_i as nested explicit FMA calls (wmul / wfma / wadd / wsub /
+    wneg, see winrs_vec.cuh), 'wzero<T>()' if empty.  A common |coefficient| m
+    is factored out, m * (sum (c/m) x), when that saves multiplies (the eq. (7)
+    row scaling makes many row entries equal)."""
     terms = [(c, v) for c, v in terms if c != 0]
     best, best_n = None, _nmul(terms)
-    for m in {abs(c) for c, _ in terms if abs(c) != 1}:
+    for m in sorted({abs(c) for c, _ in terms if abs(c) != 1}):
         scaled = [(c / m, v) for c, v in terms]
         if 1 + _nmul(scaled) < best_n:
             best, best_n = m, 1 + _nmul(scaled)
     if best is not None:
-        return f"{lit(best)} * ({lin_plain([(c / best, v) for c, v in terms])})"
+        return f"wmul({lit(best)}, {lin_plain([(c / best, v) for c, v in terms])})"
     return lin_plain(terms)
 
 
 def lin_plain(terms):
-    parts = []
-    for coef, var in terms:
-        if coef == 0:
-            continue
-        s, e = term(coef, var)
-        if not parts:
-            parts.append(e if s > 0 else f"-{e}")
+    terms = [(c, v) for c, v in terms if c != 0]
+    if not terms:
+        return "wzero<T>()"
+    # start with a +/-1 term when there is one (saves a multiply)
+    terms.sort(key=lambda t: 0 if abs(t[0]) == 1 else 1)
+    c, v = terms[0]
+    if c == 1:
+        acc = v
+    elif c == -1:
+        acc = f"wneg({v})"
+    else:
+        acc = f"wmul({lit(c)}, {v})"
+    for c, v in terms[1:]:
+        if c == 1:
+            acc = f"wadd({acc}, {v})"
+        elif c == -1:
+            acc = f"wsub({acc}, {v})"
         else:
-            parts.append(f" + {e}" if s > 0 else f" - {e}")
-    return "".join(parts) if parts else "T(0)"
+            acc = f"wfma({lit(c)}, {v}, {acc})"
+    return acc
 
 
 def _cost(terms):
-    """Multiplies of lin(terms) after common-factor extraction."""
-    return lin(terms).count("*")
+    """Non-trivial multiplies of lin(terms) after common-factor extraction."""
+    return lin(terms).count("wc<T>")
 
 
 def row_pairing(M, rows):
@@ -217,9 +215,9 @@ def emit_apply(name, M, in_len, out_len, in_var="x", out_var="o"):
             nmul += _cost(ev) + _cost(od)
             lines.append(f"    {{ const T e = {lin(ev)}; const T d = {lin(od)};")
             if sgn > 0:
-                lines.append(f"      {out_var}[{xi}] = e + d; {out_var}[{xi + 1}] = e - d; }}")
+                lines.append(f"      {out_var}[{xi}] = wadd(e, d); {out_var}[{xi + 1}] = wsub(e, d); }}")
             else:
-                lines.append(f"      {out_var}[{xi}] = e + d; {out_var}[{xi + 1}] = d - e; }}")
+                lines.append(f"      {out_var}[{xi}] = wadd(e, d); {out_var}[{xi + 1}] = wsub(d, e); }}")
             xi += 2
         else:
             row = [(M[xi][i], f"{in_var}[{i}]") for i in range(in_len)]
@@ -241,7 +239,7 @@ def emit_ot(A, alpha, n):
         if xi + 1 < alpha and row_pairing(A, (xi, xi + 1)) != 0:
             sgn = row_pairing(A, (xi, xi + 1))
             s, d = f"s{xi}", f"d{xi}"
-            lines.append(f"    const T {s} = v[{xi}] + v[{xi + 1}]; const T {d} = v[{xi}] - v[{xi + 1}];")
+            lines.append(f"    const T {s} = wadd(v[{xi}], v[{xi + 1}]); const T {d} = wsub(v[{xi}], v[{xi + 1}]);")
             for j in range(n):
                 # even j: A[2k+1][j] = sgn*A[2k][j]; odd j: A[2k+1][j] = -sgn*A[2k][j]
                 same = (j % 2 == 0) == (sgn > 0)
@@ -265,6 +263,7 @@ def generate():
            "// eq. (7) row scaling P@39150 (unit L1 rows of G and D^T, A compensating).",
            "// ft: o[alpha] = G w[r]   it: o[alpha] = D^T x[alpha]   ot: y[n] = A^T v[alpha]",
            "#pragma once",
+           "#include \"winrs_vec.cuh\"",
            "",
            "namespace winrs {",
            "",
