@@ -258,6 +258,7 @@ def run_winrs(args):
             "config": {"workload": f"{args.workload}_{args.dtype}: " + ", ".join(x["layer"].name for x in items),
                        "global_batch": layers[0].N * world, "parallelism": f"dp{world}" if world > 1 else "single",
                        "l2": "flushed (256 MiB write) before every layer call; flush outside timed events",
+                       "workspace_cap": float(os.environ.get("WINRS_WS_CAP", "0.04")),
                        "layers": [{"name": x["layer"].name, "ms": per_layer_ms[j],
                                    "tflops": x["layer"].direct_flops / (per_layer_ms[j] * 1e-3) / 1e12,
                                    "workspace_bytes": x["plan"].workspace_bytes, "plan": repr(x["plan"]),
@@ -345,7 +346,11 @@ def main():
     ap.add_argument("--dtype", default=os.environ.get("WINRS_BENCH_DTYPE", "f32"), choices=["f32", "f16"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
+    ap.add_argument("--ws-cap", type=float, default=None,
+                    help="planner workspace cap as a fraction of X+dY bytes (default: the paper's 4%%)")
     args = ap.parse_args()
+    if args.ws_cap is not None:
+        os.environ["WINRS_WS_CAP"] = str(args.ws_cap)
     if args.warmup < 3:
         args.warmup = 3
     if args.workload in ("wide",):

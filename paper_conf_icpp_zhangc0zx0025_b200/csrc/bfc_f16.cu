@@ -46,11 +46,11 @@ static int images_per_box(int N) {
     return 1;
 }
 
-template <int A0, int N0, int R0, int A1, int N1, int R1>
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BM>
 cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
     static std::atomic<unsigned long long> done{0};
-    auto k = bfc_f16_kernel<A0, N0, R0, A1, N1, R1>;
-    constexpr size_t sm = Smem<A0, R0>::bytes;
+    auto k = bfc_f16_kernel<A0, N0, R0, A1, N1, R1, BM>;
+    constexpr size_t sm = Smem<A0, R0, BM>::bytes;
     cudaError_t e = ensure_smem_attr(k, sm, done);
     if (e != cudaSuccess) return e;
     const long long grid = num_ctas(g);
@@ -72,22 +72,31 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
         mX1 = mX0;
         mY1 = mY0;
     }
-    k<<<(unsigned)grid, NTHREADS, sm, stream>>>(a, mX0, mY0, mX1, mY1);
+    k<<<(unsigned)grid, nthreads<BM>(), sm, stream>>>(a, mX0, mY0, mX1, mY1);
     return cudaGetLastError();
 }
 
 }  // namespace f16k
 
-#define WINRS_F16_ENTRY(A0, N0, R0, A1, N1, R1)                                                      \
-    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, ::winrs::f16k::BM, ::winrs::f16k::NTHREADS, 1,     \
-     ::winrs::f16k::Smem<A0, R0>::bytes, &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1>,             \
-     "f16tc_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x64"}
+#define WINRS_F16_ENTRY(A0, N0, R0, A1, N1, R1, BM)                                                  \
+    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1,               \
+     ::winrs::f16k::Smem<A0, R0, BM>::bytes, &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1, BM>,     \
+     "f16tc_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x" #BM}
+
+#ifdef WINRS_TRACE
+extern "C" __attribute__((visibility("default"))) int winrs_trace_read(unsigned long long* out) {
+    return (int)cudaMemcpyFromSymbol(out, f16k::g_trace, sizeof(f16k::g_trace));
+}
+#endif
 
 const KernelEntry* f16_entries(int* n) {
     static const KernelEntry e[] = {
-        WINRS_F16_ENTRY(8, 3, 6, 4, 3, 2),
-        WINRS_F16_ENTRY(8, 3, 6, 0, 0, 0),
-        WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0),
+        WINRS_F16_ENTRY(8, 3, 6, 4, 3, 2, 64),
+        WINRS_F16_ENTRY(8, 3, 6, 4, 3, 2, 32),
+        WINRS_F16_ENTRY(8, 3, 6, 0, 0, 0, 64),
+        WINRS_F16_ENTRY(8, 3, 6, 0, 0, 0, 32),
+        WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 64),
+        WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 32),
     };
     *n = sizeof(e) / sizeof(e[0]);
     return e;

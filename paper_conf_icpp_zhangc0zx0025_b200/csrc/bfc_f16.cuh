@@ -38,11 +38,12 @@ namespace winrs {
 namespace f16k {
 
 constexpr int BN = 128;          // k rows = UMMA M (TMEM lanes)
-constexpr int BM = 64;           // c columns = UMMA N
 constexpr int KC = 16;           // depth entries per chunk = UMMA K
-constexpr int NTHREADS = 256;    // 8 warps
-constexpr int TX_WARPS = 6;      // transformer warps (2..7)
-constexpr int S_RAW = 2, S_OP = 2;
+constexpr int S_OP = 2;          // operand ring stages
+// transformer warps: one thread per (row pair, depth quad) unit of a chunk:
+// FT (BN/2 k pairs x 4 quads) + IT (BM/2 c pairs x 4 quads)
+template <int BM> __host__ __device__ constexpr int tx_warps() { return ((BN / 2) * 2 + (BM / 2) * 2) / 32; }
+template <int BM> __host__ __device__ constexpr int nthreads() { return 64 + 32 * tx_warps<BM>(); }
 
 struct Args {
     Geometry g;
@@ -96,13 +97,15 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
            ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46);
 }
 // kind::f16 instruction descriptor: D f32, A/B f16, both K-major, M = 128, N = BM.
-constexpr uint32_t IDESC = (1u << 4) | ((uint32_t)(BM >> 3) << 17) | ((uint32_t)(BN >> 4) << 24);
+template <int BM>
+__host__ __device__ constexpr uint32_t idesc() { return (1u << 4) | ((uint32_t)(BM >> 3) << 17) | ((uint32_t)(BN >> 4) << 24); }
 
+template <int BM>
 __device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accumulate) {
     asm volatile(
         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
-        :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(IDESC), "r"(accumulate));
+        :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(idesc<BM>()), "r"(accumulate));
 }
 __device__ __forceinline__ void umma_commit(uint64_t* bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
@@ -129,14 +132,18 @@ __device__ __forceinline__ F2 ld_h2(const __half* p) {
 }
 
 // ----------------------------------------------------------------------------- shared memory plan
-template <int A0, int R0>
+template <int A0, int R0, int BM>
 struct Smem {
     static constexpr int RAW_Y = KC * R0 * BN * 2;       // bytes per raw stage (dY)
     static constexpr int RAW_X = KC * A0 * BM * 2;       // bytes per raw stage (X)
     static constexpr int RAW = RAW_Y + RAW_X;
     static constexpr int OPA = BN * KC * 2;              // one A_xi slab (4 KB)
-    static constexpr int OPB = BM * KC * 2;              // one B_xi slab (2 KB)
+    static constexpr int OPB = BM * KC * 2;              // one B_xi slab
     static constexpr int OP = A0 * (OPA + OPB);
+    static constexpr int LIMIT = 227 * 1024 - 256;
+    // as many raw (TMA) stages as fit: the raw ring is the latency-hiding depth
+    static constexpr int S_RAW = (LIMIT - S_OP * OP) / RAW > 4 ? 4 : (LIMIT - S_OP * OP) / RAW;
+    static_assert(S_RAW >= 2, "shared memory too small for a 2-stage raw ring");
     static constexpr int raw_off = 0;
     static constexpr int op_off = S_RAW * RAW;
     static constexpr int bar_off = op_off + S_OP * OP;
@@ -149,6 +156,19 @@ __device__ __forceinline__ uint32_t op_row_off(int row, int dgroup) {
     return (uint32_t)((row >> 3) * 256 + dgroup * 128 + (row & 7) * 16);
 }
 
+#ifdef WINRS_TRACE
+// Debug-build timeline of CTA 0 (globaltimer ns): [role][chunk][event].
+__device__ unsigned long long g_trace[3][256][4];
+__device__ __forceinline__ unsigned long long gtime() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#define TRACE(role, ch, ev) do { if (blockIdx.x == 0 && (ch) < 256) g_trace[role][ch][ev] = gtime(); } while (0)
+#else
+#define TRACE(role, ch, ev) do { } while (0)
+#endif
+
 struct Job {
     int phase;          // 0: Omega_a0, 1: Omega_a1
     int units, w_first, fw0;
@@ -156,7 +176,7 @@ struct Job {
 };
 
 struct Barriers {
-    uint64_t raw_full[S_RAW], raw_empty[S_RAW], op_full[S_OP], op_empty[S_OP], acc_full, acc_empty;
+    uint64_t raw_full[4], raw_empty[4], op_full[S_OP], op_empty[S_OP], acc_full, acc_empty;
     uint32_t tmem_base;
 };
 
@@ -168,92 +188,72 @@ __device__ __forceinline__ void depth_coord(long long d, int N, int units, int h
     *h = hs + (int)(t / units);
 }
 
-// ---- transformer work for one chunk: FT units (k pair p, d-group g) and IT units.
-template <int A, int NN, int RR>
-__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tx_id) {
+// ---- transformer work for one chunk.  A unit is (row pair, 8 consecutive
+// depth entries): FT units cover the B_N/2 k pairs of every A_xi, IT units
+// the B_M/2 c pairs of every B_xi; 2 depth octets per KC = 16 chunk.  Each
+// unit computes 8 transforms per row in packed f32x2 (rows 2p, 2p+1), rounds
+// to FP16 and writes one 16-byte core-matrix row per (xi, row).
+constexpr int DQ = 8;                    // depth entries per unit
+constexpr int NQ = KC / DQ;              // depth octets per chunk
+template <int BM> __host__ __device__ constexpr int ft_units() { return (BN / 2) * NQ; }
+template <int BM> __host__ __device__ constexpr int it_units() { return (BM / 2) * NQ; }
+
+template <int WT_FN, int A, int NN, int RR, int NIN>
+__device__ __forceinline__ void unit_transform(const __half* src, int row_stride, int depth_stride, uint8_t* dst0,
+                                               int slab_bytes, int p, int g) {
     using WT = Wino<A, NN, RR>;
+    uint32_t pk[A][2][4];   // [xi][row 2p / 2p+1][4 x half2 along d]
+#pragma unroll
+    for (int j = 0; j < DQ; j += 2) {
+        F2 o0[A], o1[A];
+        {
+            F2 in[NIN];
+            const __half* s0 = src + (g * DQ + j) * depth_stride + 2 * p;
+#pragma unroll
+            for (int i = 0; i < NIN; ++i) in[i] = ld_h2(s0 + i * row_stride);
+            if (WT_FN == 0) WT::ft(in, o0); else WT::it(in, o0);
+        }
+        {
+            F2 in[NIN];
+            const __half* s1 = src + (g * DQ + j + 1) * depth_stride + 2 * p;
+#pragma unroll
+            for (int i = 0; i < NIN; ++i) in[i] = ld_h2(s1 + i * row_stride);
+            if (WT_FN == 0) WT::ft(in, o1); else WT::it(in, o1);
+        }
+#pragma unroll
+        for (int x = 0; x < A; ++x) {
+            pk[x][0][j / 2] = pack_h2(o0[x].x, o1[x].x);
+            pk[x][1][j / 2] = pack_h2(o0[x].y, o1[x].y);
+        }
+    }
+#pragma unroll
+    for (int x = 0; x < A; ++x) {
+        uint8_t* base = dst0 + x * slab_bytes;
+#pragma unroll
+        for (int e = 0; e < 2; ++e)
+            *reinterpret_cast<uint4*>(base + op_row_off(2 * p + e, g)) =
+                make_uint4(pk[x][e][0], pk[x][e][1], pk[x][e][2], pk[x][e][3]);
+    }
+}
+
+template <int A, int NN, int RR, int BM>
+__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tx_id) {
     constexpr int RAW_Y = KC * RR * BN * 2;
     const __half* rawY = reinterpret_cast<const __half*>(raw);            // [KC][RR][BN]
     const __half* rawX = reinterpret_cast<const __half*>(raw + RAW_Y);    // [KC][A][BM]
     constexpr int OPA = BN * KC * 2, OPB = BM * KC * 2;
-    if (tx_id < (BN / 2) * 2) {
-        // FT: rows k = 2p, 2p+1 of every A_xi, depth group g (8 entries)
+    if (tx_id < ft_units<BM>()) {
         const int p = tx_id % (BN / 2), g = tx_id / (BN / 2);
-        uint32_t pk[A][2][4];   // [xi][row k / k+1][4 x half2 along d]
-#pragma unroll
-        for (int j = 0; j < 8; j += 2) {
-            F2 o0[A], o1[A];
-            {
-                F2 w[RR];
-                const __half* src = rawY + ((g * 8 + j) * RR) * BN + 2 * p;
-#pragma unroll
-                for (int i = 0; i < RR; ++i) w[i] = ld_h2(src + i * BN);
-                WT::ft(w, o0);
-            }
-            {
-                F2 w[RR];
-                const __half* src = rawY + ((g * 8 + j + 1) * RR) * BN + 2 * p;
-#pragma unroll
-                for (int i = 0; i < RR; ++i) w[i] = ld_h2(src + i * BN);
-                WT::ft(w, o1);
-            }
-#pragma unroll
-            for (int x = 0; x < A; ++x) {
-                pk[x][0][j / 2] = pack_h2(o0[x].x, o1[x].x);
-                pk[x][1][j / 2] = pack_h2(o0[x].y, o1[x].y);
-            }
-        }
-#pragma unroll
-        for (int x = 0; x < A; ++x) {
-            uint8_t* a = op + x * OPA;
-#pragma unroll
-            for (int e = 0; e < 2; ++e) {
-                uint4 v = make_uint4(pk[x][e][0], pk[x][e][1], pk[x][e][2], pk[x][e][3]);
-                *reinterpret_cast<uint4*>(a + op_row_off(2 * p + e, g)) = v;
-            }
-        }
-    } else if (tx_id < (BN / 2) * 2 + (BM / 2) * 2) {
-        // IT: rows c = 2q, 2q+1 of every B_xi, depth group g
-        const int t = tx_id - BN;
+        unit_transform<0, A, NN, RR, RR>(rawY, BN, RR * BN, op, OPA, p, g);
+    } else if (tx_id < ft_units<BM>() + it_units<BM>()) {
+        const int t = tx_id - ft_units<BM>();
         const int q = t % (BM / 2), g = t / (BM / 2);
-        uint32_t pk[A][2][4];
-#pragma unroll
-        for (int j = 0; j < 8; j += 2) {
-            F2 o0[A], o1[A];
-            {
-                F2 xv[A];
-                const __half* src = rawX + ((g * 8 + j) * A) * BM + 2 * q;
-#pragma unroll
-                for (int i = 0; i < A; ++i) xv[i] = ld_h2(src + i * BM);
-                WT::it(xv, o0);
-            }
-            {
-                F2 xv[A];
-                const __half* src = rawX + ((g * 8 + j + 1) * A) * BM + 2 * q;
-#pragma unroll
-                for (int i = 0; i < A; ++i) xv[i] = ld_h2(src + i * BM);
-                WT::it(xv, o1);
-            }
-#pragma unroll
-            for (int x = 0; x < A; ++x) {
-                pk[x][0][j / 2] = pack_h2(o0[x].x, o1[x].x);
-                pk[x][1][j / 2] = pack_h2(o0[x].y, o1[x].y);
-            }
-        }
-#pragma unroll
-        for (int x = 0; x < A; ++x) {
-            uint8_t* b = op + A * OPA + x * OPB;
-#pragma unroll
-            for (int e = 0; e < 2; ++e) {
-                uint4 v = make_uint4(pk[x][e][0], pk[x][e][1], pk[x][e][2], pk[x][e][3]);
-                *reinterpret_cast<uint4*>(b + op_row_off(2 * q + e, g)) = v;
-            }
-        }
+        unit_transform<1, A, NN, RR, A>(rawX, BM, A * BM, op + A * OPA, OPB, q, g);
     }
 }
 
 // ---- epilogue of one job: TMEM -> OT -> bucket.  Called by warps 2..5.
-template <int A, int NN, int RR>
+template <int A, int NN, int RR, int BM>
 __device__ __forceinline__ void epilogue(const Geometry& g, float* bucket, const CtaCoord& cc, int fw0, bool accumulate,
                                          bool empty, uint32_t tmem_base, int warp) {
     using WT = Wino<A, NN, RR>;
@@ -306,12 +306,14 @@ __device__ __forceinline__ void epilogue(const Geometry& g, float* bucket, const
     }
 }
 
-template <int A0, int N0, int R0, int A1, int N1, int R1>
-__global__ void __launch_bounds__(NTHREADS, 1)
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BM>
+__global__ void __launch_bounds__(nthreads<BM>(), 1)
 bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX0,
                const __grid_constant__ CUtensorMap tmY0, const __grid_constant__ CUtensorMap tmX1,
                const __grid_constant__ CUtensorMap tmY1) {
-    using SM = Smem<A0, R0>;
+    using SM = Smem<A0, R0, BM>;
+    constexpr int S_RAW = SM::S_RAW;
+    constexpr int TX_WARPS = tx_warps<BM>();
     extern __shared__ __align__(1024) uint8_t smem[];
     const Geometry& g = args.g;
     Barriers* bars = reinterpret_cast<Barriers*>(smem + SM::bar_off);
@@ -371,7 +373,9 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 const int nch = (int)((depth + KC - 1) / KC);
                 const uint32_t bytes = (uint32_t)(KC * (RRj * BN + Aj * BM) * 2);
                 for (int ch = 0; ch < nch; ++ch) {
+                    TRACE(0, ch + jb * 64, 0);
                     mbar_wait(&bars->raw_empty[s], ph ^ 1);
+                    TRACE(0, ch + jb * 64, 1);
                     uint8_t* raw = smem + SM::raw_off + s * SM::RAW;
                     uint8_t* rY = raw;
                     uint8_t* rX = raw + KC * RRj * BN * 2;
@@ -405,14 +409,16 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 }
                 for (int ch = 0; ch < nch; ++ch) {
                     mbar_wait(&bars->op_full[s], ph);
+                    TRACE(1, ch + jb * 64, 0);
                     tc_fence_after();
                     const uint32_t base = smem_u32(smem + SM::op_off + s * SM::OP);
                     for (int x = 0; x < Aj; ++x) {
                         const uint64_t ad = umma_desc(base + x * SM::OPA, 128, 256);
                         const uint64_t bd = umma_desc(base + Aj * SM::OPA + x * SM::OPB, 128, 256);
-                        umma_f16(tmem_base + (uint32_t)(x * BM), ad, bd, ch > 0 ? 1u : 0u);
+                        umma_f16<BM>(tmem_base + (uint32_t)(x * BM), ad, bd, ch > 0 ? 1u : 0u);
                     }
                     umma_commit(&bars->op_empty[s]);
+                    TRACE(1, ch + jb * 64, 1);
                     if (++s == S_OP) { s = 0; ph ^= 1; }
                 }
                 umma_commit(&bars->acc_full);
@@ -428,14 +434,18 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
             const int nch = (int)((depth + KC - 1) / KC);
             for (int ch = 0; ch < nch; ++ch) {
+                if (threadIdx.x == 64) TRACE(2, ch + jb * 64, 0);
                 mbar_wait(&bars->raw_full[sr], phr);
+                if (threadIdx.x == 64) TRACE(2, ch + jb * 64, 1);
                 mbar_wait(&bars->op_empty[so], pho ^ 1);
+                if (threadIdx.x == 64) TRACE(2, ch + jb * 64, 2);
                 const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
                 uint8_t* op = smem + SM::op_off + so * SM::OP;
-                if (J.phase == 0) transform_chunk<A0, N0, R0>(raw, op, tx_id);
-                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1>(raw, op, tx_id);
+                if (J.phase == 0) transform_chunk<A0, N0, R0, BM>(raw, op, tx_id);
+                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM>(raw, op, tx_id);
                 fence_proxy_async();
                 __syncwarp();
+                if (threadIdx.x == 64) TRACE(2, ch + jb * 64, 3);
                 if (lane == 0) {
                     mbar_arrive(&bars->op_full[so]);
                     mbar_arrive(&bars->raw_empty[sr]);
@@ -447,9 +457,9 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 mbar_wait(&bars->acc_full, (uint32_t)(jb & 1));
                 tc_fence_after();
                 if (J.phase == 0)
-                    epilogue<A0, N0, R0>(g, bucket, cc, J.fw0, J.accumulate, nch == 0, tmem_base, warp);
+                    epilogue<A0, N0, R0, BM>(g, bucket, cc, J.fw0, J.accumulate, nch == 0, tmem_base, warp);
                 else if constexpr (A1 != 0)
-                    epilogue<A1, N1, R1>(g, bucket, cc, J.fw0, J.accumulate, nch == 0, tmem_base, warp);
+                    epilogue<A1, N1, R1, BM>(g, bucket, cc, J.fw0, J.accumulate, nch == 0, tmem_base, warp);
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&bars->acc_empty);

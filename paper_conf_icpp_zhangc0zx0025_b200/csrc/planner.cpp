@@ -12,7 +12,8 @@
 //      eq. (5); readings R9, R10).
 //
 // Debug overrides (tests only): WINRS_FORCE_Z=<z>, WINRS_FORCE_TILE=<bn>x<bm>,
-// WINRS_FORCE_PAIR=a0,n0,r0,a1,n1,r1.
+// WINRS_FORCE_PAIR=a0,n0,r0,a1,n1,r1.  Policy: WINRS_WS_CAP=<fraction> replaces the
+// 4% workspace cap (R11).
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
@@ -106,7 +107,12 @@ static int alg1(const Problem& p, const KernelEntry& e, int num_sms, int* zmax_o
     const double esz = p.dtype == 0 ? 4.0 : 2.0;
     const double data = esz * ((double)p.N * p.H * p.W * p.C + (double)p.N * p.Ho * p.Wo * p.K);
     const double dw_bytes = 4.0 * (double)p.K * p.R * p.S * p.C;
-    const int zmax = 1 + (int)std::floor(0.04 * data / dw_bytes);
+    double cap = 0.04;                                   // R11: workspace <= 4% of X+dY bytes
+    if (const char* c = getenv("WINRS_WS_CAP")) {       // policy knob (fraction of X+dY bytes)
+        const double v = atof(c);
+        if (v > 0) cap = v;
+    }
+    const int zmax = 1 + (int)std::floor(cap * data / dw_bytes);
     *zmax_out = zmax;
     if (zh < 2.0 && b2 >= bhat2) return 1;                                          // line 3
     const long long z1 = cdiv(2LL * e.occ * num_sms, b2);                          // line 4

@@ -51,7 +51,12 @@ def _compile(src: str, force: bool, hdr_m: float) -> str:
     return o
 
 
-def build(force: bool = False, jobs: int = 0) -> str:
+def build(force: bool = False, jobs: int = 0, trace: bool = False) -> str:
+    global OBJ, LIB, FLAGS
+    if trace:   # debug build with the CTA-0 timeline (csrc/bfc_f16.cuh TRACE)
+        OBJ = os.path.join(ROOT, "build", "obj_trace")
+        LIB = os.path.join(PKG, "libwinrs_trace.so")
+        FLAGS = FLAGS + ["-DWINRS_TRACE"]
     os.makedirs(OBJ, exist_ok=True)
     if not os.path.exists(GEN_OUT) or os.path.getmtime(GEN_OUT) < os.path.getmtime(GEN):
         subprocess.check_call([sys.executable, GEN])
@@ -71,5 +76,6 @@ if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--force", action="store_true")
     ap.add_argument("-j", type=int, default=0)
+    ap.add_argument("--trace", action="store_true")
     a = ap.parse_args()
-    print(build(a.force, a.j))
+    print(build(a.force, a.j, a.trace))
