@@ -115,10 +115,17 @@ def run_winrs(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    torch.cuda.set_device(local % ndev)
+    dev = torch.device("cuda", local % ndev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        # NCCL over NVLink/NVSwitch; WINRS_DIST_BACKEND=gloo only to exercise the
+        # multi-rank path on a single-GPU box (ranks sharing one device).
+        backend = os.environ.get("WINRS_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     layers = _workload(args.workload, args.dtype)
     tdt = torch.float32 if args.dtype == "f32" else torch.float16
 

@@ -19,7 +19,7 @@ from dataclasses import dataclass
 from . import _lib
 from ._lib import WinrsError, DTYPES
 
-__all__ = ["Plan", "plan", "plan_for_device", "bfc", "bfc_host", "as_kcrs", "bfc_data_parallel",
+__all__ = ["Plan", "plan", "plan_for_device", "bfc", "bfc_host", "as_kcrs", "bfc_data_parallel", "shard_range",
            "WinrsError", "version", "emulate", "transform", "kernel_names"]
 
 
@@ -143,6 +143,14 @@ def bfc_host(p: Plan, X_host, dY_host, dW_host, dev_X, dev_dY, dev_dW, workspace
 def as_kcrs(dW):
     """KRSC storage -> logical [K,C,R,S] view (channels_last strides), no copy."""
     return dW.permute(0, 3, 1, 2)
+
+
+def shard_range(N: int, world: int, rank: int):
+    """Contiguous batch slice [start, end) of rank `rank` (NHWC => the slice of
+    X and dY is contiguous in memory); the first N % world ranks get one more."""
+    base, extra = divmod(N, world)
+    start = rank * base + min(rank, extra)
+    return start, start + base + (1 if rank < extra else 0)
 
 
 def bfc_data_parallel(X_shard, dY_shard, R: int, S: int, pad: int, dtype: str = "f32", group=None,
