@@ -93,6 +93,7 @@ typedef struct {
     int tile_k0, tile_c0;          /* CTA tile B_N x B_M of the bulk kernel               */
     int tile_k1, tile_c1;          /* CTA tile of the residual kernel                     */
     long long ctas_main, ctas_resid, ctas_reduce;
+    int csplit;                    /* CTAs per tile: thread-block cluster depth split   */
     size_t workspace_bytes;        /* (Z-1) * 4 * K*R*S*C, 0 when Z == 1                  */
     double direct_flops;           /* 2*N*C*K*Ho*Wo*R*S (P@43462)                         */
     double ewm_flops;              /* Winograd-domain EWM flops actually issued           */

@@ -65,7 +65,8 @@ class Plan:
         s = (f"Plan(Omega_{i['alpha0']}({i['n0']},{i['r0']})x{i['k0']}")
         if i["alpha1"]:
             s += f" + Omega_{i['alpha1']}({i['n1']},{i['r1']})x{i['k1']}"
-        return s + (f", Z={i['Z']}, tile={i['tile_k0']}x{i['tile_c0']}, ws={i['workspace_bytes']}B)")
+        return s + (f", Z={i['Z']}, tile={i['tile_k0']}x{i['tile_c0']}, csplit={i['csplit']}, "
+                    f"ws={i['workspace_bytes']}B)")
 
 
 def plan(N, C, H, W, K, R, S, pad, dtype: str = "f32") -> Plan:

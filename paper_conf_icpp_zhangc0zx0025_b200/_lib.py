@@ -35,7 +35,7 @@ class PlanInfoT(ctypes.Structure):
                  "z_hat", "Z", "seg_h", "seg_w", "bands", "seg_cols",
                  "tile_k0", "tile_c0", "tile_k1", "tile_c1")] + [
         ("ctas_main", ctypes.c_longlong), ("ctas_resid", ctypes.c_longlong),
-        ("ctas_reduce", ctypes.c_longlong), ("workspace_bytes", ctypes.c_size_t),
+        ("ctas_reduce", ctypes.c_longlong), ("csplit", ctypes.c_int), ("workspace_bytes", ctypes.c_size_t),
         ("direct_flops", ctypes.c_double), ("ewm_flops", ctypes.c_double)]
 
 

@@ -79,7 +79,7 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
 }  // namespace f16k
 
 #define WINRS_F16_ENTRY(A0, N0, R0, A1, N1, R1, BM)                                                  \
-    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1,               \
+    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1, 0,            \
      ::winrs::f16k::Smem<A0, R0, BM>::bytes, &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1, BM>,     \
      "f16tc_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x" #BM}
 

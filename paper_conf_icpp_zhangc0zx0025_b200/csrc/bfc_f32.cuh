@@ -26,9 +26,29 @@
 #include <stdint.h>
 #include "winrs_internal.h"
 #include "winograd_generated.cuh"
+#include "winrs_vec.cuh"
 
 namespace winrs {
 namespace f32k {
+
+// Packed FP32 pair helpers: ptxas folds pk2(a, a) into the scalar-broadcast
+// operand form of FFMA2, so the outer product acc[i][j..j+1] += a_i * b[j..j+1]
+// issues one FFMA2 per two FMAs with no extra moves.
+__device__ __forceinline__ uint64_t pk2(float lo, float hi) {
+    uint64_t r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+    return r;
+}
+__device__ __forceinline__ float2 up2(uint64_t r) {
+    float2 f;
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(f.x), "=f"(f.y) : "l"(r));
+    return f;
+}
+__device__ __forceinline__ uint64_t ffma2(uint64_t a, uint64_t b, uint64_t c) {
+    uint64_t d;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+    return d;
+}
 
 constexpr int NT = 256;   // threads per CTA (8 warps)
 constexpr int BD = 8;     // depth entries per chunk
@@ -74,14 +94,19 @@ struct PhaseSmem {
     static constexpr int floats = pipe > ot ? pipe : ot;
 };
 
-// One phase: the main loop over `units` units of width RR starting at dY
-// column w_first, for dW columns [fw0, fw0 + NN), then the OT and the bucket
-// write (store, or add when `accumulate`).
+// Output staging tile in shared memory: [n0][B_N][B_M + 4] floats (row pad
+// keeps the float4 staging stores conflict-free).
+template <int BM> __host__ __device__ constexpr int out_ld() { return BM + 4; }
+
+// One phase: the main loop over this CTA's chunk range of the depth of
+// `units` units of width RR starting at dY column w_first, for dW columns
+// [fw0, fw0 + NN), then the OT into the output staging tile at column offset
+// j_off (store, or add when `accumulate`).
 template <int ALPHA, int NN, int RR, int BN, int BM>
 __device__ __forceinline__ void run_phase(const Geometry& g, const float* __restrict__ X,
-                                          const float* __restrict__ dY, float* __restrict__ bucket,
+                                          const float* __restrict__ dY, float* __restrict__ Out,
                                           const CtaCoord& cc, int hs, int he, int w_first, int units,
-                                          int fw0, bool accumulate, float* smem) {
+                                          int fw0, int j_off, bool accumulate, int rank, float* smem) {
     using WT = Wino<ALPHA, NN, RR>;
     using L = GemmLayout<ALPHA, BN, BM>;
     using SM = PhaseSmem<ALPHA, RR, BN, BM>;
@@ -94,13 +119,15 @@ __device__ __forceinline__ void run_phase(const Geometry& g, const float* __rest
     const int k_base = cc.kb * BN, c_base = cc.cb * BM;
     const int rows = he - hs;
     const long long depth = (long long)(rows > 0 ? rows : 0) * units * g.N;
-    const int nchunks = (int)((depth + BD - 1) / BD);
+    int c_lo, c_hi;   // this cluster rank's share of the chunks
+    split_chunks((int)((depth + BD - 1) / BD), rank, g.csplit, &c_lo, &c_hi);
+    const int nchunks = c_hi - c_lo;
 
     // ---- loader: 32 threads per depth entry of a chunk
     constexpr int TPD = NT / BD;
     const int ld_d = tid / TPD, ld_l = tid % TPD;
     auto issue = [&](int chunk, int buf) {
-        const long long d = (long long)chunk * BD + ld_d;
+        const long long d = (long long)(c_lo + chunk) * BD + ld_d;
         const bool dv = d < depth;
         int n = 0, h = hs, u = 0;
         if (dv) {
@@ -133,12 +160,12 @@ __device__ __forceinline__ void run_phase(const Geometry& g, const float* __rest
         }
     };
 
-    // ---- accumulators
-    float v[L::TM][L::TN];
+    // ---- accumulators: pairs along c, FFMA2
+    uint64_t v2[L::TM][L::TN / 2];
 #pragma unroll
     for (int i = 0; i < L::TM; ++i)
 #pragma unroll
-        for (int j = 0; j < L::TN; ++j) v[i][j] = 0.f;
+        for (int j = 0; j < L::TN / 2; ++j) v2[i][j] = 0ull;
     const int xi = tid / L::TPX;
     const int tl = tid % L::TPX;
     const int tk = tl / L::TPC, tc = tl % L::TPC;
@@ -157,27 +184,35 @@ __device__ __forceinline__ void run_phase(const Geometry& g, const float* __rest
             cp_async_wait<0>();
         }
         __syncthreads();
-        // ---- transforms (FP32), raw[buf] -> Gt / Xt
+        // ---- transforms (FP32, packed f32x2 over channel pairs), raw[buf] -> Gt / Xt
         {
             const float* rg = rawG + buf * BD * RR * BN;
-            for (int p = tid; p < BD * BN; p += NT) {
-                const int d = p / BN, k = p % BN;
-                float w[RR], o[ALPHA];
+            for (int p = tid; p < BD * (BN / 2); p += NT) {
+                const int d = p / (BN / 2), k = 2 * (p % (BN / 2));
+                F2 w[RR], o[ALPHA];
 #pragma unroll
-                for (int i = 0; i < RR; ++i) w[i] = rg[(d * RR + i) * BN + k];
+                for (int i = 0; i < RR; ++i) {
+                    const float2 t = *reinterpret_cast<const float2*>(rg + (d * RR + i) * BN + k);
+                    w[i] = F2{t.x, t.y};
+                }
                 WT::ft(w, o);
 #pragma unroll
-                for (int x = 0; x < ALPHA; ++x) Gt[(x * BD + d) * BN + k] = o[x];
+                for (int x = 0; x < ALPHA; ++x)
+                    *reinterpret_cast<float2*>(Gt + (x * BD + d) * BN + k) = make_float2(o[x].x, o[x].y);
             }
             const float* rx = rawX + buf * BD * ALPHA * BM;
-            for (int p = tid; p < BD * BM; p += NT) {
-                const int d = p / BM, c = p % BM;
-                float xv[ALPHA], o[ALPHA];
+            for (int p = tid; p < BD * (BM / 2); p += NT) {
+                const int d = p / (BM / 2), c = 2 * (p % (BM / 2));
+                F2 xv[ALPHA], o[ALPHA];
 #pragma unroll
-                for (int t = 0; t < ALPHA; ++t) xv[t] = rx[(d * ALPHA + t) * BM + c];
+                for (int t = 0; t < ALPHA; ++t) {
+                    const float2 q = *reinterpret_cast<const float2*>(rx + (d * ALPHA + t) * BM + c);
+                    xv[t] = F2{q.x, q.y};
+                }
                 WT::it(xv, o);
 #pragma unroll
-                for (int x = 0; x < ALPHA; ++x) Xt[(x * BD + d) * BM + c] = o[x];
+                for (int x = 0; x < ALPHA; ++x)
+                    *reinterpret_cast<float2*>(Xt + (x * BD + d) * BM + c) = make_float2(o[x].x, o[x].y);
             }
         }
         __syncthreads();
@@ -187,7 +222,8 @@ __device__ __forceinline__ void run_phase(const Geometry& g, const float* __rest
             const float* xb = Xt + xi * BD * BM;
 #pragma unroll
             for (int d = 0; d < BD; ++d) {
-                float a[L::TM], b[L::TN];
+                float a[L::TM];
+                uint64_t b2[L::TN / 2];
 #pragma unroll
                 for (int gm = 0; gm < L::GM; ++gm) {
                     const float4 t = *reinterpret_cast<const float4*>(ga + d * BN + (gm * L::TPK + tk) * 4);
@@ -196,12 +232,15 @@ __device__ __forceinline__ void run_phase(const Geometry& g, const float* __rest
 #pragma unroll
                 for (int gn = 0; gn < L::GN; ++gn) {
                     const float4 t = *reinterpret_cast<const float4*>(xb + d * BM + (gn * L::TPC + tc) * 4);
-                    b[gn * 4 + 0] = t.x; b[gn * 4 + 1] = t.y; b[gn * 4 + 2] = t.z; b[gn * 4 + 3] = t.w;
+                    b2[gn * 2 + 0] = pk2(t.x, t.y);
+                    b2[gn * 2 + 1] = pk2(t.z, t.w);
                 }
 #pragma unroll
-                for (int i = 0; i < L::TM; ++i)
+                for (int i = 0; i < L::TM; ++i) {
+                    const uint64_t aa = pk2(a[i], a[i]);
 #pragma unroll
-                    for (int j = 0; j < L::TN; ++j) v[i][j] = fmaf(a[i], b[j], v[i][j]);
+                    for (int j = 0; j < L::TN / 2; ++j) v2[i][j] = ffma2(aa, b2[j], v2[i][j]);
+                }
             }
         }
     }
@@ -217,9 +256,9 @@ __device__ __forceinline__ void run_phase(const Geometry& g, const float* __rest
         for (int e = 0; e < 4; ++e)
 #pragma unroll
             for (int gn = 0; gn < L::GN; ++gn) {
+                const float2 lo = up2(v2[gm * 4 + e][gn * 2 + 0]), hi = up2(v2[gm * 4 + e][gn * 2 + 1]);
                 float4 t;
-                t.x = v[gm * 4 + e][gn * 4 + 0]; t.y = v[gm * 4 + e][gn * 4 + 1];
-                t.z = v[gm * 4 + e][gn * 4 + 2]; t.w = v[gm * 4 + e][gn * 4 + 3];
+                t.x = lo.x; t.y = lo.y; t.z = hi.x; t.w = hi.y;
                 *reinterpret_cast<float4*>(As + (xi * KR + tk * 4 + e) * BM + (gn * L::TPC + tc) * 4) = t;
             }
         __syncthreads();
@@ -230,27 +269,85 @@ __device__ __forceinline__ void run_phase(const Geometry& g, const float* __rest
 #pragma unroll
             for (int x = 0; x < ALPHA; ++x) vv[x] = As[(x * KR + kl) * BM + c];
             WT::ot(vv, y);
-            if (kg < g.K && cg < g.C) {
-                float* dst = bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0) * g.C + cg;
+            float* o = Out + ((long long)j_off * BN + gm * KR + kl) * out_ld<BM>() + c;
 #pragma unroll
-                for (int j = 0; j < NN; ++j) {
-                    if (accumulate) dst[(long long)j * g.C] += y[j];
-                    else dst[(long long)j * g.C] = y[j];
-                }
+            for (int j = 0; j < NN; ++j) {
+                float* dst = o + (long long)j * BN * out_ld<BM>();
+                *dst = accumulate ? *dst + y[j] : y[j];
             }
         }
         __syncthreads();
     }
 }
 
+// Writes the staged output tile [n0][B_N][B_M] to the bucket.  With a cluster
+// split, rank r first waits for every rank's partial tile, sums the rows
+// [r*rows/cs, (r+1)*rows/cs) over ranks 0..cs-1 in order through distributed
+// shared memory (deterministic), and writes them.
+template <int N0, int BN, int BM>
+__device__ __forceinline__ void write_out(const Geometry& g, float* __restrict__ bucket, const CtaCoord& cc,
+                                          int fw0, int rank, const float* Out) {
+    const int k_base = cc.kb * BN, c_base = cc.cb * BM;
+    constexpr int C4 = BM / 4;
+    constexpr int ROWS = N0 * BN;
+    int r_lo = 0, r_hi = ROWS;
+    if (g.csplit > 1) {
+        asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+        r_lo = ROWS * rank / g.csplit;
+        r_hi = ROWS * (rank + 1) / g.csplit;
+    }
+    const uint32_t out_s = static_cast<uint32_t>(__cvta_generic_to_shared(Out));
+    for (int p = r_lo * C4 + threadIdx.x; p < r_hi * C4; p += NT) {
+        const int row = p / C4, c4 = p % C4;
+        const int j = row / BN, kl = row % BN;
+        const int kg = k_base + kl, cg = c_base + c4 * 4;
+        const uint32_t off = (uint32_t)(((row) * out_ld<BM>() + c4 * 4) * 4);
+        float4 acc;
+        if (g.csplit > 1) {
+            acc = make_float4(0.f, 0.f, 0.f, 0.f);
+            for (int q = 0; q < g.csplit; ++q) {
+                uint32_t remote;
+                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(out_s + off), "r"(q));
+                float4 v;
+                asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+                             : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(remote) : "memory");
+                acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+            }
+        } else {
+            acc = *reinterpret_cast<const float4*>(Out + row * out_ld<BM>() + c4 * 4);
+        }
+        if (kg < g.K && cg < g.C)
+            *reinterpret_cast<float4*>(bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0 + j) * g.C + cg) = acc;
+    }
+    if (g.csplit > 1)   // peers may still be reading this CTA's tile
+        asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 // The fused launch: every CTA runs the Omega_a0 phase over its segment, and
 // CTAs of a band's last column segment also run the residual Omega_a1 phase.
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BN, int BM>
+constexpr size_t pipe_floats() {
+    size_t a = PhaseSmem<A0, R0, BN, BM>::floats;
+    size_t b = A1 ? PhaseSmem<(A1 ? A1 : A0), (R1 ? R1 : R0), BN, BM>::floats : 0;
+    return a > b ? a : b;
+}
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BN, int BM>
+constexpr size_t smem_bytes() {
+    return 4 * (pipe_floats<A0, N0, R0, A1, N1, R1, BN, BM>() + (size_t)N0 * BN * out_ld<BM>());
+}
+
+// The fused launch: every CTA runs the Omega_a0 phase over its segment (its
+// cluster rank's share of the depth), CTAs of a band's last column segment
+// also run the residual Omega_a1 phase into the same staged tile, then the
+// tile (summed over the cluster) is written to the segment's bucket.
 template <int A0, int N0, int R0, int A1, int N1, int R1, int BN, int BM>
 __global__ void __launch_bounds__(NT, 1)
 bfc_f32_kernel(const Geometry g, const float* __restrict__ X, const float* __restrict__ dY,
                float* __restrict__ dW, float* __restrict__ ws) {
     extern __shared__ __align__(16) float smem[];
-    const CtaCoord cc = decode_cta(g, blockIdx.x);
+    float* Out = smem + pipe_floats<A0, N0, R0, A1, N1, R1, BN, BM>();
+    const int rank = (int)(blockIdx.x % g.csplit);
+    const CtaCoord cc = decode_cta(g, blockIdx.x / g.csplit);
     const int seg = cc.band * g.seg_cols + cc.col;
     float* bucket = seg == 0 ? dW : ws + (long long)(seg - 1) * g.dw_elems;
     int hs, he;
@@ -258,23 +355,18 @@ bfc_f32_kernel(const Geometry g, const float* __restrict__ X, const float* __res
     int w_first, units;
     seg_units(g, cc.col, &w_first, &units);
     const int fw0 = cc.ft * N0;
-    run_phase<A0, N0, R0, BN, BM>(g, X, dY, bucket, cc, hs, he, w_first, units, fw0, false, smem);
+    run_phase<A0, N0, R0, BN, BM>(g, X, dY, Out, cc, hs, he, w_first, units, fw0, 0, false, rank, smem);
     if constexpr (A1 != 0) {
         if (has_residual(g, cc.col)) {
             static_assert(N0 % N1 == 0, "residual n1 must divide n0");
 #pragma unroll 1
             for (int j = 0; j < N0 / N1; ++j)
-                run_phase<A1, N1, R1, BN, BM>(g, X, dY, bucket, cc, hs, he, g.res_col0, g.k1,
-                                              fw0 + j * N1, true, smem);
+                run_phase<A1, N1, R1, BN, BM>(g, X, dY, Out, cc, hs, he, g.res_col0, g.k1, fw0 + j * N1, j * N1,
+                                              true, rank, smem);
         }
     }
-}
-
-template <int A0, int N0, int R0, int A1, int N1, int R1, int BN, int BM>
-constexpr size_t smem_bytes() {
-    size_t a = PhaseSmem<A0, R0, BN, BM>::floats;
-    size_t b = A1 ? PhaseSmem<(A1 ? A1 : A0), (R1 ? R1 : R0), BN, BM>::floats : 0;
-    return 4 * (a > b ? a : b);
+    __syncthreads();
+    write_out<N0, BN, BM>(g, bucket, cc, fw0, rank, Out);
 }
 
 }  // namespace f32k

@@ -11,7 +11,7 @@
 //   3. Segment shape S^_H x S^_W and the final segment count (§4.3 Algorithm 2,
 //      eq. (5); readings R9, R10).
 //
-// Debug overrides (tests only): WINRS_FORCE_Z=<z>, WINRS_FORCE_TILE=<bn>x<bm>,
+// Debug overrides (tests only): WINRS_FORCE_Z=<z>, WINRS_FORCE_TILE=<bn>x<bm>, WINRS_FORCE_CSPLIT=<1|2|4|8>,
 // WINRS_FORCE_PAIR=a0,n0,r0,a1,n1,r1.  Policy: WINRS_WS_CAP=<fraction> replaces the
 // 4% workspace cap (R11).
 #include <algorithm>
@@ -176,7 +176,44 @@ static void fill_geometry(const Problem& p, const KernelEntry& e, const PairChoi
     g->cblocks = (int)cdiv(p.C, e.bm);
     g->ftiles = p.S / e.n0;
     g->Z = g->bands * g->seg_cols;
+    g->csplit = 1;
+    g->chunk = p.dtype == 0 ? 8 : 16;
     g->dw_elems = (long long)p.K * p.R * p.S * p.C;
+}
+
+// Fewest chunks any tile of the Omega_a0 phase walks (its segment's clipped
+// rows x units x N / chunk).
+static long long min_tile_chunks(const Geometry& g) {
+    long long best = -1;
+    for (int band = 0; band < g.bands; ++band)
+        for (int fh = 0; fh < g.R; ++fh) {
+            int hs, he;
+            band_rows(g, band, fh, &hs, &he);
+            for (int col = 0; col < g.seg_cols; ++col) {
+                int wf, units;
+                seg_units(g, col, &wf, &units);
+                const long long d = (long long)(he - hs) * units * g.N;
+                const long long c = (d + g.chunk - 1) / g.chunk;
+                if (c > 0 && (best < 0 || c < best)) best = c;
+            }
+        }
+    return best < 0 ? 0 : best;
+}
+
+// B200 cluster split: when the tile grid cannot fill the SMs,
+// split each tile's depth over a cluster of 2/4/8 CTAs (partial tiles summed
+// through DSMEM), keeping >= 4 chunks per CTA.
+static int choose_csplit(const Geometry& g, int occ, int num_sms) {
+    if (const char* f = getenv("WINRS_FORCE_CSPLIT")) {
+        const int v = atoi(f);
+        if (v == 1 || v == 2 || v == 4 || v == 8) return v;
+    }
+    const long long tiles = num_tiles(g);
+    const long long target = (long long)occ * num_sms;
+    const long long mc = min_tile_chunks(g);
+    int cs = 1;
+    while (cs < 8 && tiles * cs < target && mc / (cs * 2) >= 4) cs *= 2;
+    return cs;
 }
 
 // Winograd-domain EWM flops the kernels issue (clipped rows, masked columns
@@ -211,6 +248,7 @@ static void plan_with_tile(const Problem& p, const KernelEntry& e, const PairCho
         if (g.Z <= zmax || z <= 1) break;     // enforce the workspace cap (R11)
         z = std::min(z_used, z) - 1;
     }
+    g.csplit = e.csplit_ok ? choose_csplit(g, e.occ, num_sms) : 1;
     out->geom = g;
     out->entry = &e;
     out->z_hat = z_used;
@@ -248,7 +286,7 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
         plan_with_tile(p, *e, pc, num_sms, &r);
         const long long ctas = num_ctas(r.geom);
         if (!have || ctas > best_ctas) { best = r; best_ctas = ctas; have = true; }
-        if (ctas >= (long long)e->occ * num_sms) { best = r; have = true; break; }
+        if (4 * ctas >= 3LL * e->occ * num_sms) { best = r; have = true; break; }
     }
     if (!have) return WINRS_ERR_UNSUPPORTED;
     best.ewm_flops = ewm_flops(best.geom);

@@ -18,6 +18,7 @@ struct KernelEntry {
     int bn, bm;                // CTA tile B_N (k) x B_M (c)
     int threads;
     int occ;                   // planner's CTAs/SM hint
+    int csplit_ok;             // kernel supports the thread-block-cluster depth split
     size_t smem;               // dynamic shared memory bytes
     LaunchFn launch;
     const char* name;

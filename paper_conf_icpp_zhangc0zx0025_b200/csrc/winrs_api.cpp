@@ -3,6 +3,7 @@
 // (2) Kernel Execution — one fused launch over all segments (both kernels of
 // the pair), (3) Reduction — the bucket reduction kernel when Z > 1.
 #include <cuda_runtime.h>
+#include <algorithm>
 #include <cstdlib>
 #include <cstring>
 #include <new>
@@ -55,6 +56,7 @@ static winrs_status_t build_plan(int N, int C, int H, int W, int K, int R, int S
     in.tile_k0 = g.tile_k; in.tile_c0 = g.tile_c;
     in.tile_k1 = g.a1 ? g.tile_k : 0; in.tile_c1 = g.a1 ? g.tile_c : 0;
     in.ctas_main = num_ctas(g);
+    in.csplit = g.csplit;
     in.ctas_resid = 0;   // the residual phase runs inside the main launch's last-column CTAs
     in.ctas_reduce = g.Z > 1 ? 1 : 0;
     in.workspace_bytes = g.Z > 1 ? (size_t)(g.Z - 1) * 4u * (size_t)g.dw_elems : 0;
@@ -174,14 +176,19 @@ namespace {
 
 template <int A, int NN, int RR>
 void emu_phase(const Geometry& g, const double* X, const double* dY, double* bucket, const CtaCoord& cc,
-               int hs, int he, int w_first, int units, int fw0, bool accumulate) {
+               int hs, int he, int w_first, int units, int fw0, bool accumulate, int rank) {
     using WT = Wino<A, NN, RR>;
     const int BN = g.tile_k, BM = g.tile_c;
     const int k0 = cc.kb * BN, c0 = cc.cb * BM;
     std::vector<double> v((size_t)A * BN * BM, 0.0), gt((size_t)A * BN), xt((size_t)A * BM);
-    for (int h = hs; h < he; ++h)
-        for (int u = 0; u < units; ++u)
-            for (int n = 0; n < g.N; ++n) {
+    const long long depth = (long long)(he > hs ? he - hs : 0) * units * g.N;
+    int c_lo, c_hi;
+    split_chunks((int)((depth + g.chunk - 1) / g.chunk), rank, g.csplit, &c_lo, &c_hi);
+    const long long d_hi = std::min<long long>(depth, (long long)c_hi * g.chunk);
+    for (long long d = (long long)c_lo * g.chunk; d < d_hi; ++d) {
+                const int n = (int)(d % g.N);
+                const int u = (int)((d / g.N) % units);
+                const int h = hs + (int)(d / g.N / units);
                 const int w0 = w_first + u * RR;
                 for (int k = 0; k < BN; ++k) {
                     double w[RR], o[A];
@@ -207,7 +214,7 @@ void emu_phase(const Geometry& g, const double* X, const double* dY, double* buc
                     for (int k = 0; k < BN; ++k)
                         for (int c = 0; c < BM; ++c)
                             v[((size_t)x * BN + k) * BM + c] += gt[(size_t)x * BN + k] * xt[(size_t)x * BM + c];
-            }
+    }
     for (int k = 0; k < BN; ++k)
         for (int c = 0; c < BM; ++c) {
             const int kg = k0 + k, cg = c0 + c;
@@ -223,7 +230,7 @@ void emu_phase(const Geometry& g, const double* X, const double* dY, double* buc
 }
 
 typedef void (*EmuFn)(const Geometry&, const double*, const double*, double*, const CtaCoord&, int, int, int,
-                      int, int, bool);
+                      int, int, bool, int);
 
 EmuFn emu_fn(int a, int n, int r) {
 #define WINRS_EMU_CASE(A, N, R) if (a == A && n == N && r == R) return &emu_phase<A, N, R>;
@@ -246,8 +253,9 @@ winrs_status_t winrs_debug_emulate(winrs_plan_t plan, const double* X, const dou
     EmuFn f1 = g.a1 ? emu_fn(g.a1, g.n1, g.r1) : nullptr;
     if (!f0 || (g.a1 && !f1)) return WINRS_ERR_UNSUPPORTED;
     std::vector<double> buckets((size_t)g.Z * g.dw_elems, 0.0);
-    const long long nct = num_ctas(g);
-    for (long long b = 0; b < nct; ++b) {
+    std::vector<double> part((size_t)g.dw_elems);
+    const long long nt = num_tiles(g);
+    for (long long b = 0; b < nt; ++b) {
         const CtaCoord cc = decode_cta(g, b);
         const int seg = cc.band * g.seg_cols + cc.col;
         double* bucket = buckets.data() + (size_t)seg * g.dw_elems;
@@ -255,10 +263,15 @@ winrs_status_t winrs_debug_emulate(winrs_plan_t plan, const double* X, const dou
         band_rows(g, cc.band, cc.fh, &hs, &he);
         seg_units(g, cc.col, &wf, &units);
         const int fw0 = cc.ft * g.n0;
-        f0(g, X, dY, bucket, cc, hs, he, wf, units, fw0, false);
-        if (f1 && has_residual(g, cc.col))
-            for (int j = 0; j < g.n0 / g.n1; ++j)
-                f1(g, X, dY, bucket, cc, hs, he, g.res_col0, g.k1, fw0 + j * g.n1, true);
+        // cluster ranks each compute a partial tile; the tile is their sum
+        for (int rank = 0; rank < g.csplit; ++rank) {
+            std::fill(part.begin(), part.end(), 0.0);
+            f0(g, X, dY, part.data(), cc, hs, he, wf, units, fw0, false, rank);
+            if (f1 && has_residual(g, cc.col))
+                for (int j = 0; j < g.n0 / g.n1; ++j)
+                    f1(g, X, dY, part.data(), cc, hs, he, g.res_col0, g.k1, fw0 + j * g.n1, true, rank);
+            for (long long i = 0; i < g.dw_elems; ++i) bucket[i] += part[i];
+        }
     }
     for (long long i = 0; i < g.dw_elems; ++i) {
         double s = 0.0;

@@ -15,6 +15,11 @@
 //     B_N x B_M x n0 tile dW_z[kb*B_N.., fh, ft*n0 .. ft*n0+n0, cb*B_M..].
 //   * Height clipping (P@32013-33698, Figure 7): a CTA only visits dY rows h
 //     whose X row h+fh-pad lies inside [0, H).
+//   * Cluster split (B200 addition): the depth of one tile can
+//     be split over `csplit` CTAs of a thread-block cluster; each computes a
+//     partial output tile in shared memory and the cluster sums them through
+//     distributed shared memory in fixed rank order (deterministic, no
+//     workspace).  CTA = (cluster of csplit ranks) x (tile coordinate).
 #pragma once
 #include <stdint.h>
 #include <stddef.h>
@@ -44,6 +49,8 @@ struct Geometry {
     int tile_k, tile_c;         // B_N (k), B_M (c)
     int kblocks, cblocks, ftiles;   // ceil(K/B_N), ceil(C/B_M), S/n0
     int Z;                      // buckets
+    int csplit;                 // CTAs per tile (thread-block cluster size), >= 1
+    int chunk;                  // depth entries per main-loop chunk (8 FP32, 16 FP16)
     long long dw_elems;         // K*R*S*C
 };
 
@@ -51,6 +58,7 @@ struct CtaCoord {
     int kb, cb, ft, fh, band, col;
 };
 
+// bid: tile index (blockIdx.x / csplit).
 WINRS_HD CtaCoord decode_cta(const Geometry& g, long long bid) {
     CtaCoord c;
     c.kb = (int)(bid % g.kblocks); bid /= g.kblocks;
@@ -62,8 +70,15 @@ WINRS_HD CtaCoord decode_cta(const Geometry& g, long long bid) {
     return c;
 }
 
-WINRS_HD long long num_ctas(const Geometry& g) {
+WINRS_HD long long num_tiles(const Geometry& g) {
     return (long long)g.kblocks * g.cblocks * g.ftiles * g.R * g.seg_cols * g.bands;
+}
+WINRS_HD long long num_ctas(const Geometry& g) { return num_tiles(g) * g.csplit; }
+
+// Chunk range [lo, hi) of cluster rank `rank` out of `nchunks` chunks.
+WINRS_HD void split_chunks(int nchunks, int rank, int csplit, int* lo, int* hi) {
+    *lo = (int)((long long)nchunks * rank / csplit);
+    *hi = (int)((long long)nchunks * (rank + 1) / csplit);
 }
 
 // Valid (clipped) dY rows [hs, he) of a band for filter row fh.

@@ -26,6 +26,9 @@ CASES = [
     (3, 36, 6, 6, 40, 3, 3, 1, {"WINRS_FORCE_TILE": "32x32"}),       # channel tails over 2 tiles
     (2, 8, 10, 10, 8, 3, 3, 1, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
     (2, 8, 10, 10, 8, 3, 3, 1, {"WINRS_FORCE_PAIR": "8,3,6,0,0,0", "WINRS_FORCE_Z": "4"}),
+    (3, 8, 12, 12, 8, 3, 3, 1, {"WINRS_FORCE_CSPLIT": "4"}),                  # cluster depth split
+    (2, 4, 9, 12, 8, 4, 4, 2, {"WINRS_FORCE_CSPLIT": "8", "WINRS_FORCE_Z": "2"}),
+    (2, 4, 7, 7, 4, 3, 3, 1, {"WINRS_FORCE_CSPLIT": "8"}),                  # more ranks than chunks
 ]
 
 

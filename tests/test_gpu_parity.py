@@ -68,6 +68,8 @@ FORCED = [
     {"WINRS_FORCE_Z": "1"}, {"WINRS_FORCE_Z": "5"}, {"WINRS_FORCE_Z": "12"},
     {"WINRS_FORCE_TILE": "64x64"}, {"WINRS_FORCE_TILE": "32x32", "WINRS_FORCE_Z": "3"},
     {"WINRS_FORCE_PAIR": "8,3,6,0,0,0"}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_Z": "7"},
+    {"WINRS_FORCE_CSPLIT": "1"}, {"WINRS_FORCE_CSPLIT": "2"}, {"WINRS_FORCE_CSPLIT": "8", "WINRS_FORCE_Z": "3"},
+    {"WINRS_FORCE_CSPLIT": "4", "WINRS_FORCE_TILE": "32x32"},
 ]
 
 
