@@ -350,7 +350,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="winrs", choices=["winrs", "reference"])
     ap.add_argument("--workload", default="r50", choices=["r50", "vgg", "wide", "r50l3"])
-    ap.add_argument("--dtype", default=os.environ.get("WINRS_BENCH_DTYPE", "f32"), choices=["f32", "f16"])
+    ap.add_argument("--dtype", default=os.environ.get("WINRS_BENCH_DTYPE", "f16"), choices=["f32", "f16"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
     ap.add_argument("--ws-cap", type=float, default=None,

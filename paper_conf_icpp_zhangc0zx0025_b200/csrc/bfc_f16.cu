@@ -72,14 +72,17 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
         mX1 = mX0;
         mY1 = mY0;
     }
-    k<<<(unsigned)grid, nthreads<BM>(), sm, stream>>>(a, mX0, mY0, mX1, mY1);
-    return cudaGetLastError();
+    if (g.csplit <= 1) {
+        k<<<(unsigned)grid, nthreads<BM>(), sm, stream>>>(a, mX0, mY0, mX1, mY1);
+        return cudaGetLastError();
+    }
+    return launch_cluster(k, (unsigned)grid, (unsigned)nthreads<BM>(), sm, stream, g.csplit, a, mX0, mY0, mX1, mY1);
 }
 
 }  // namespace f16k
 
 #define WINRS_F16_ENTRY(A0, N0, R0, A1, N1, R1, BM)                                                  \
-    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1, 0,            \
+    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1, 1,            \
      ::winrs::f16k::Smem<A0, R0, BM>::bytes, &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1, BM>,     \
      "f16tc_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x" #BM}
 

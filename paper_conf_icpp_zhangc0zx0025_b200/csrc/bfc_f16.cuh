@@ -252,23 +252,33 @@ __device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op,
     }
 }
 
-// ---- epilogue of one job: TMEM -> OT -> bucket.  Called by warps 2..5.
-template <int A, int NN, int RR, int BM>
-__device__ __forceinline__ void epilogue(const Geometry& g, float* bucket, const CtaCoord& cc, int fw0, bool accumulate,
-                                         bool empty, uint32_t tmem_base, int warp) {
+__device__ __forceinline__ void tmem_st8(uint32_t taddr, const float* v) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};"
+                 :: "r"(taddr), "r"(__float_as_uint(v[0])), "r"(__float_as_uint(v[1])), "r"(__float_as_uint(v[2])),
+                    "r"(__float_as_uint(v[3])), "r"(__float_as_uint(v[4])), "r"(__float_as_uint(v[5])),
+                    "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7])) : "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
+// TMEM column where the n0 x BM output tile is staged between jobs (top of
+// the 512 columns; the residual job's accumulators live below it).
+template <int N0, int BM> __host__ __device__ constexpr int stash_col() { return 512 - N0 * BM; }
+
+// ---- epilogue of one job (warps 2..5, one TMEM lane quarter each):
+// accumulators -> OT (FP32) -> output columns [j_off, j_off + NN) of the
+// TMEM-staged tile (store for the first job, add for the residual jobs).
+// Reading the 8 columns c0.. of every xi before writing the stash columns
+// c0.. keeps the in-place overlap with the first job's accumulators safe.
+template <int A, int NN, int RR, int N0, int BM>
+__device__ __forceinline__ void epilogue(int j_off, bool first, bool empty, uint32_t tmem_base, int warp) {
     using WT = Wino<A, NN, RR>;
-    const int quarter = warp & 3;
-    const int lane = threadIdx.x & 31;
-    const int kl = quarter * 32 + lane;
-    const int kg = cc.kb * BN + kl;
-    const bool krow_ok = kg < g.K;
+    const uint32_t lane_base = tmem_base + ((uint32_t)((warp & 3) * 32) << 16);
 #pragma unroll 1
     for (int c0 = 0; c0 < BM; c0 += 8) {
         float v[A][8];
         if (!empty) {
 #pragma unroll
-            for (int x = 0; x < A; ++x)
-                tmem_ld8(tmem_base + ((uint32_t)(quarter * 32) << 16) + (uint32_t)(x * BM + c0), v[x]);
+            for (int x = 0; x < A; ++x) tmem_ld8(lane_base + (uint32_t)(x * BM + c0), v[x]);
             tmem_wait_ld();
         } else {
 #pragma unroll
@@ -286,24 +296,86 @@ __device__ __forceinline__ void epilogue(const Geometry& g, float* bucket, const
 #pragma unroll
             for (int j = 0; j < NN; ++j) y[j][i] = yy[j];
         }
-        const int cg = cc.cb * BM + c0;
-        if (krow_ok && cg < g.C) {   // C % 8 == 0, so an 8-column group is all in or all out
-            float* dst = bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0) * g.C + cg;
+        if (!first) {
 #pragma unroll
             for (int j = 0; j < NN; ++j) {
-                float4* d4 = reinterpret_cast<float4*>(dst + (long long)j * g.C);
-                float4 a = make_float4(y[j][0], y[j][1], y[j][2], y[j][3]);
-                float4 b = make_float4(y[j][4], y[j][5], y[j][6], y[j][7]);
-                if (accumulate) {
-                    const float4 pa = d4[0], pb = d4[1];
-                    a.x += pa.x; a.y += pa.y; a.z += pa.z; a.w += pa.w;
-                    b.x += pb.x; b.y += pb.y; b.z += pb.z; b.w += pb.w;
+                float prev[8];
+                tmem_ld8(lane_base + (uint32_t)(stash_col<N0, BM>() + (j_off + j) * BM + c0), prev);
+                tmem_wait_ld();
+#pragma unroll
+                for (int i = 0; i < 8; ++i) y[j][i] += prev[i];
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < NN; ++j) tmem_st8(lane_base + (uint32_t)(stash_col<N0, BM>() + (j_off + j) * BM + c0), y[j]);
+        tmem_wait_st();
+    }
+}
+
+// Output staging tile in shared memory for the cluster reduction: [n0][BN][BM+4].
+template <int BM> __host__ __device__ constexpr int out_ld() { return BM + 4; }
+
+// ---- final pass (warps 2..5): staged tile -> bucket (no cluster split) or ->
+// the shared-memory staging tile (cluster split).
+template <int N0, int BM>
+__device__ __forceinline__ void final_out(const Geometry& g, float* bucket, const CtaCoord& cc, int fw0, uint32_t tmem_base,
+                                          int warp, float* Out) {
+    const int quarter = warp & 3, lane = threadIdx.x & 31;
+    const int kl = quarter * 32 + lane;
+    const int kg = cc.kb * BN + kl;
+    const uint32_t lane_base = tmem_base + ((uint32_t)(quarter * 32) << 16);
+#pragma unroll 1
+    for (int c0 = 0; c0 < BM; c0 += 8) {
+#pragma unroll
+        for (int j = 0; j < N0; ++j) {
+            float y[8];
+            tmem_ld8(lane_base + (uint32_t)(stash_col<N0, BM>() + j * BM + c0), y);
+            tmem_wait_ld();
+            const float4 a = make_float4(y[0], y[1], y[2], y[3]), b = make_float4(y[4], y[5], y[6], y[7]);
+            if (g.csplit > 1) {
+                float4* o = reinterpret_cast<float4*>(Out + ((long long)j * BN + kl) * out_ld<BM>() + c0);
+                o[0] = a;
+                o[1] = b;
+            } else {
+                const int cg = cc.cb * BM + c0;
+                if (kg < g.K && cg < g.C) {   // C % 8 == 0: an 8-column group is all in or all out
+                    float4* d4 = reinterpret_cast<float4*>(bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0 + j) * g.C + cg);
+                    d4[0] = a;
+                    d4[1] = b;
                 }
-                d4[0] = a;
-                d4[1] = b;
             }
         }
     }
+}
+
+// ---- cluster reduction (all threads): rank r sums rows [r*rows/cs, ...) of
+// the staged tiles of ranks 0..cs-1 in order through DSMEM and writes them.
+template <int N0, int BM>
+__device__ __forceinline__ void cluster_reduce(const Geometry& g, float* bucket, const CtaCoord& cc, int fw0, int rank,
+                                               const float* Out, int nthreads_) {
+    constexpr int C4 = BM / 4;
+    constexpr int ROWS = N0 * BN;
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    const int r_lo = ROWS * rank / g.csplit, r_hi = ROWS * (rank + 1) / g.csplit;
+    const uint32_t out_s = smem_u32(Out);
+    for (int p = r_lo * C4 + (int)threadIdx.x; p < r_hi * C4; p += nthreads_) {
+        const int row = p / C4, c4 = p % C4;
+        const int j = row / BN, kl = row % BN;
+        const uint32_t off = (uint32_t)((row * out_ld<BM>() + c4 * 4) * 4);
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int q = 0; q < g.csplit; ++q) {
+            uint32_t remote;
+            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(out_s + off), "r"(q));
+            float4 v;
+            asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+                         : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(remote) : "memory");
+            acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+        }
+        const int kg = cc.kb * BN + kl, cg = cc.cb * BM + c4 * 4;
+        if (kg < g.K && cg < g.C)
+            *reinterpret_cast<float4*>(bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0 + j) * g.C + cg) = acc;
+    }
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
 template <int A0, int N0, int R0, int A1, int N1, int R1, int BM>
@@ -314,12 +386,15 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     using SM = Smem<A0, R0, BM>;
     constexpr int S_RAW = SM::S_RAW;
     constexpr int TX_WARPS = tx_warps<BM>();
+    static_assert(A1 * BM <= stash_col<N0, BM>(), "residual accumulators overlap the TMEM output stash");
+    static_assert(N0 * BN * out_ld<BM>() * 4 <= SM::bar_off, "cluster staging tile must fit in the rings");
     extern __shared__ __align__(1024) uint8_t smem[];
     const Geometry& g = args.g;
     Barriers* bars = reinterpret_cast<Barriers*>(smem + SM::bar_off);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
-    const CtaCoord cc = decode_cta(g, blockIdx.x);
+    const int rank = (int)(blockIdx.x % g.csplit);
+    const CtaCoord cc = decode_cta(g, blockIdx.x / g.csplit);
     const int seg = cc.band * g.seg_cols + cc.col;
     float* bucket = seg == 0 ? args.dW : args.ws + (long long)(seg - 1) * g.dw_elems;
     int hs, he;
@@ -327,15 +402,22 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     int w_first, units;
     seg_units(g, cc.col, &w_first, &units);
     const int rows = he - hs;
+    const int fw0 = cc.ft * N0;
 
-    // Job list (identical in every role).
+    // Job list (identical in every role): (phase, units, first dY column,
+    // first output column, output column offset in the tile).
     Job jobs[1 + 9];
     int njobs = 0;
-    jobs[njobs++] = Job{0, units, w_first, cc.ft * N0, false};
+    jobs[njobs++] = Job{0, units, w_first, fw0, false};
     if constexpr (A1 != 0) {
         if (has_residual(g, cc.col))
-            for (int j = 0; j < N0 / N1; ++j) jobs[njobs++] = Job{1, g.k1, g.res_col0, cc.ft * N0 + j * N1, true};
+            for (int j = 0; j < N0 / N1; ++j) jobs[njobs++] = Job{1, g.k1, g.res_col0, fw0 + j * N1, true};
     }
+    // this cluster rank's chunk range of a job
+    auto chunk_range = [&](const Job& J, int* lo, int* hi) {
+        const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
+        split_chunks((int)((depth + KC - 1) / KC), rank, g.csplit, lo, hi);
+    };
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S_RAW; ++s) { mbar_init(&bars->raw_full[s], 1); mbar_init(&bars->raw_empty[s], TX_WARPS); }
@@ -370,12 +452,13 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 const CUtensorMap* mX = J.phase == 0 ? &tmX0 : &tmX1;
                 const CUtensorMap* mY = J.phase == 0 ? &tmY0 : &tmY1;
                 const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
-                const int nch = (int)((depth + KC - 1) / KC);
+                int c_lo, c_hi;
+                chunk_range(J, &c_lo, &c_hi);
                 const uint32_t bytes = (uint32_t)(KC * (RRj * BN + Aj * BM) * 2);
-                for (int ch = 0; ch < nch; ++ch) {
-                    TRACE(0, ch + jb * 64, 0);
+                for (int ch = c_lo; ch < c_hi; ++ch) {
+                    TRACE(0, ch - c_lo + jb * 64, 0);
                     mbar_wait(&bars->raw_empty[s], ph ^ 1);
-                    TRACE(0, ch + jb * 64, 1);
+                    TRACE(0, ch - c_lo + jb * 64, 1);
                     uint8_t* raw = smem + SM::raw_off + s * SM::RAW;
                     uint8_t* rY = raw;
                     uint8_t* rX = raw + KC * RRj * BN * 2;
@@ -401,24 +484,24 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             for (int jb = 0; jb < njobs; ++jb) {
                 const Job& J = jobs[jb];
                 const int Aj = J.phase == 0 ? A0 : A1;
-                const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
-                const int nch = (int)((depth + KC - 1) / KC);
+                int c_lo, c_hi;
+                chunk_range(J, &c_lo, &c_hi);
                 if (jb > 0) {
                     mbar_wait(&bars->acc_empty, (uint32_t)((jb - 1) & 1));
                     tc_fence_after();
                 }
-                for (int ch = 0; ch < nch; ++ch) {
+                for (int ch = c_lo; ch < c_hi; ++ch) {
                     mbar_wait(&bars->op_full[s], ph);
-                    TRACE(1, ch + jb * 64, 0);
+                    TRACE(1, ch - c_lo + jb * 64, 0);
                     tc_fence_after();
                     const uint32_t base = smem_u32(smem + SM::op_off + s * SM::OP);
                     for (int x = 0; x < Aj; ++x) {
                         const uint64_t ad = umma_desc(base + x * SM::OPA, 128, 256);
                         const uint64_t bd = umma_desc(base + Aj * SM::OPA + x * SM::OPB, 128, 256);
-                        umma_f16<BM>(tmem_base + (uint32_t)(x * BM), ad, bd, ch > 0 ? 1u : 0u);
+                        umma_f16<BM>(tmem_base + (uint32_t)(x * BM), ad, bd, ch > c_lo ? 1u : 0u);
                     }
                     umma_commit(&bars->op_empty[s]);
-                    TRACE(1, ch + jb * 64, 1);
+                    TRACE(1, ch - c_lo + jb * 64, 1);
                     if (++s == S_OP) { s = 0; ph ^= 1; }
                 }
                 umma_commit(&bars->acc_full);
@@ -431,21 +514,21 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         uint32_t phr = 0, pho = 0;
         for (int jb = 0; jb < njobs; ++jb) {
             const Job& J = jobs[jb];
-            const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
-            const int nch = (int)((depth + KC - 1) / KC);
-            for (int ch = 0; ch < nch; ++ch) {
-                if (threadIdx.x == 64) TRACE(2, ch + jb * 64, 0);
+            int c_lo, c_hi;
+            chunk_range(J, &c_lo, &c_hi);
+            for (int ch = c_lo; ch < c_hi; ++ch) {
+                if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 0);
                 mbar_wait(&bars->raw_full[sr], phr);
-                if (threadIdx.x == 64) TRACE(2, ch + jb * 64, 1);
+                if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 1);
                 mbar_wait(&bars->op_empty[so], pho ^ 1);
-                if (threadIdx.x == 64) TRACE(2, ch + jb * 64, 2);
+                if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 2);
                 const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
                 uint8_t* op = smem + SM::op_off + so * SM::OP;
                 if (J.phase == 0) transform_chunk<A0, N0, R0, BM>(raw, op, tx_id);
                 else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM>(raw, op, tx_id);
                 fence_proxy_async();
                 __syncwarp();
-                if (threadIdx.x == 64) TRACE(2, ch + jb * 64, 3);
+                if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 3);
                 if (lane == 0) {
                     mbar_arrive(&bars->op_full[so]);
                     mbar_arrive(&bars->raw_empty[sr]);
@@ -456,18 +539,25 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             if (warp < 6) {
                 mbar_wait(&bars->acc_full, (uint32_t)(jb & 1));
                 tc_fence_after();
+                const bool empty = c_hi <= c_lo;
                 if (J.phase == 0)
-                    epilogue<A0, N0, R0, BM>(g, bucket, cc, J.fw0, J.accumulate, nch == 0, tmem_base, warp);
+                    epilogue<A0, N0, R0, N0, BM>(0, true, empty, tmem_base, warp);
                 else if constexpr (A1 != 0)
-                    epilogue<A1, N1, R1, BM>(g, bucket, cc, J.fw0, J.accumulate, nch == 0, tmem_base, warp);
+                    epilogue<A1, N1, R1, N0, BM>(J.fw0 - fw0, false, empty, tmem_base, warp);
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&bars->acc_empty);
             }
         }
+        if (warp < 6) {
+            // every job's epilogue is done (this warp's own, in program order)
+            final_out<N0, BM>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
+        }
     }
     tc_fence_before();
     __syncthreads();
+    if (g.csplit > 1)
+        cluster_reduce<N0, BM>(g, bucket, cc, fw0, rank, reinterpret_cast<const float*>(smem), nthreads<BM>());
     if (warp == 1) {
         tc_fence_after();
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem_base));

@@ -150,6 +150,9 @@ def test_reduced_f16_signed(layer):
 FORCED_F16 = [
     {"WINRS_FORCE_Z": "1"}, {"WINRS_FORCE_Z": "7"},
     {"WINRS_FORCE_PAIR": "8,3,6,0,0,0"}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_Z": "3"},
+    {"WINRS_FORCE_CSPLIT": "1"}, {"WINRS_FORCE_CSPLIT": "2"}, {"WINRS_FORCE_CSPLIT": "8"},
+    {"WINRS_FORCE_CSPLIT": "4", "WINRS_FORCE_TILE": "128x32", "WINRS_FORCE_Z": "2"},
+    {"WINRS_FORCE_CSPLIT": "4", "WINRS_FORCE_PAIR": "8,3,6,0,0,0"},
 ]
 
 
