@@ -200,20 +200,30 @@ static long long min_tile_chunks(const Geometry& g) {
     return best < 0 ? 0 : best;
 }
 
-// B200 cluster split: when the tile grid cannot fill the SMs,
-// split each tile's depth over a cluster of 2/4/8 CTAs (partial tiles summed
-// through DSMEM), keeping >= 4 chunks per CTA.
+// B200 cluster split: split each tile's depth over a cluster
+// of cs in {1, 2, 4, 8} CTAs (partial tiles summed through DSMEM), choosing
+// the cs that minimises the wave-quantised time  ceil(tiles*cs / slots(cs)) / cs
+// (each CTA does 1/cs of a tile's work), keeping >= 4 chunks per CTA.  Cluster
+// placement strands SMs for cs >= 4 (B300/B200 measurement: 132 of 148 SMs
+// usable at cs = 4, 128 at cs = 8).
 static int choose_csplit(const Geometry& g, int occ, int num_sms) {
     if (const char* f = getenv("WINRS_FORCE_CSPLIT")) {
         const int v = atoi(f);
         if (v == 1 || v == 2 || v == 4 || v == 8) return v;
     }
     const long long tiles = num_tiles(g);
-    const long long target = (long long)occ * num_sms;
     const long long mc = min_tile_chunks(g);
-    int cs = 1;
-    while (cs < 8 && tiles * cs < target && mc / (cs * 2) >= 4) cs *= 2;
-    return cs;
+    int best = 1;
+    double best_t = 1e30;
+    for (int cs = 1; cs <= 8; cs *= 2) {
+        if (cs > 1 && mc / cs < 4) break;
+        const double frac = cs <= 2 ? 1.0 : (cs == 4 ? 132.0 / 148.0 : 128.0 / 148.0);
+        const long long slots = std::max(1LL, (long long)(occ * num_sms * frac));
+        const long long waves = (tiles * cs + slots - 1) / slots;
+        const double t = (double)waves / cs * (1.0 + 0.02 * (cs > 1));   // small DSMEM-reduction cost
+        if (t < best_t - 1e-9) { best_t = t; best = cs; }
+    }
+    return best;
 }
 
 // Winograd-domain EWM flops the kernels issue (clipped rows, masked columns
@@ -266,8 +276,12 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
     const KernelEntry* es = kernel_entries(&ne);
     PairChoice pc;
     if (!choose_pair(p, es, ne, &pc)) return WINRS_ERR_UNSUPPORTED;
-    // Step 1b (B200): CTA tile.  Largest tile that still fills one wave of
-    // the SMs at its occupancy, else the variant giving the most CTAs.
+    // Step 1b (B200): CTA tile.  Each compiled tile variant is planned (Z,
+    // segments, cluster split) and scored by the wave-quantised time model
+    //   t ~ waves(ctas) / (csplit * tiles * eff(tile))
+    // where eff is the relative per-CTA efficiency of the tile (larger tiles
+    // amortise the transforms and operand traffic better: 1.0 for the largest
+    // variant, 0.55 for the half-size one — calibrated on B200).
     std::vector<const KernelEntry*> tiles;
     for (int i = 0; i < ne; ++i)
         if (same_pair(es[i], *pc.proto)) tiles.push_back(&es[i]);
@@ -279,14 +293,19 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
     const bool force_tile = parse_force_tile(&fbn, &fbm);
     PlanResult best;
     bool have = false;
-    long long best_ctas = -1;
+    double best_t = 1e30;
+    const int big = tiles.empty() ? 1 : tiles.front()->bn * tiles.front()->bm;
     for (const KernelEntry* e : tiles) {
         if (force_tile && (e->bn != fbn || e->bm != fbm)) continue;
         PlanResult r;
         plan_with_tile(p, *e, pc, num_sms, &r);
-        const long long ctas = num_ctas(r.geom);
-        if (!have || ctas > best_ctas) { best = r; best_ctas = ctas; have = true; }
-        if (4 * ctas >= 3LL * e->occ * num_sms) { best = r; have = true; break; }
+        const Geometry& g = r.geom;
+        const double eff = e->bn * e->bm >= big ? 1.0 : 0.55;
+        const double frac = g.csplit <= 2 ? 1.0 : (g.csplit == 4 ? 132.0 / 148.0 : 128.0 / 148.0);
+        const long long slots = std::max(1LL, (long long)(e->occ * num_sms * frac));
+        const long long waves = (num_ctas(g) + slots - 1) / slots;
+        const double t = (double)waves / ((double)g.csplit * (double)num_tiles(g) * eff);
+        if (!have || t < best_t - 1e-12) { best = r; best_t = t; have = true; }
     }
     if (!have) return WINRS_ERR_UNSUPPORTED;
     best.ewm_flops = ewm_flops(best.geom);
