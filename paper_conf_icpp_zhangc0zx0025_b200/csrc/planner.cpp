@@ -200,28 +200,49 @@ static long long min_tile_chunks(const Geometry& g) {
     return best < 0 ? 0 : best;
 }
 
-// B200 cluster split: split each tile's depth over a cluster
-// of cs in {1, 2, 4, 8} CTAs (partial tiles summed through DSMEM), choosing
-// the cs that minimises the wave-quantised time  ceil(tiles*cs / slots(cs)) / cs
-// (each CTA does 1/cs of a tile's work), keeping >= 4 chunks per CTA.  Cluster
-// placement strands SMs for cs >= 4 (B300/B200 measurement: 132 of 148 SMs
-// usable at cs = 4, 128 at cs = 8).
-static int choose_csplit(const Geometry& g, int occ, int num_sms) {
+// B200 time model used to pick the CTA tile and the cluster split (DESIGN.md
+// §7), calibrated with tools/sweep.py on B200:
+//   t = waves(ctas, slots) * (F + tile_ewm_flops / csplit / rate_cta)
+// rate_cta = per-SM Winograd-domain rate of the tile / CTAs per SM; F = fixed
+// per-CTA cost (prologue, pipeline fill, epilogue, cluster reduction).
+// Cluster placement strands SMs for cs >= 4 (132 of 148 usable at cs = 4,
+// 128 at cs = 8).
+struct TimeModel {
+    double rate_sm;    // EWM FLOP/s per SM for this tile
+    double fixed_s;    // per-CTA fixed cost (s)
+};
+
+static TimeModel time_model(int dtype, int bn, int bm) {
+    if (dtype == 1) return {bm >= 64 ? 1.15e12 : 0.75e12, 4e-6};
+    const int area = bn * bm;
+    return {area >= 4096 ? 0.20e12 : (area >= 2048 ? 0.16e12 : 0.11e12), 8e-6};
+}
+
+static double slots_frac(int cs) { return cs <= 2 ? 1.0 : (cs == 4 ? 132.0 / 148.0 : 128.0 / 148.0); }
+
+static double model_time(const Geometry& g, const KernelEntry& e, int num_sms, double ewm) {
+    const TimeModel m = time_model(e.dtype, e.bn, e.bm);
+    const long long slots = std::max(1LL, (long long)(e.occ * num_sms * slots_frac(g.csplit)));
+    const long long waves = (num_ctas(g) + slots - 1) / slots;
+    const double per_cta = ewm / (double)num_tiles(g) / g.csplit / (m.rate_sm / e.occ);
+    return waves * (m.fixed_s + per_cta);
+}
+
+// Cluster split: cs in {1, 2, 4, 8} minimising the model time, keeping >= 4
+// chunks per CTA.
+static int choose_csplit(Geometry g, const KernelEntry& e, int num_sms, double ewm) {
     if (const char* f = getenv("WINRS_FORCE_CSPLIT")) {
         const int v = atoi(f);
         if (v == 1 || v == 2 || v == 4 || v == 8) return v;
     }
-    const long long tiles = num_tiles(g);
     const long long mc = min_tile_chunks(g);
     int best = 1;
     double best_t = 1e30;
     for (int cs = 1; cs <= 8; cs *= 2) {
         if (cs > 1 && mc / cs < 4) break;
-        const double frac = cs <= 2 ? 1.0 : (cs == 4 ? 132.0 / 148.0 : 128.0 / 148.0);
-        const long long slots = std::max(1LL, (long long)(occ * num_sms * frac));
-        const long long waves = (tiles * cs + slots - 1) / slots;
-        const double t = (double)waves / cs * (1.0 + 0.02 * (cs > 1));   // small DSMEM-reduction cost
-        if (t < best_t - 1e-9) { best_t = t; best = cs; }
+        g.csplit = cs;
+        const double t = model_time(g, e, num_sms, ewm);
+        if (t < best_t * (1.0 - 1e-9)) { best_t = t; best = cs; }
     }
     return best;
 }
@@ -258,7 +279,7 @@ static void plan_with_tile(const Problem& p, const KernelEntry& e, const PairCho
         if (g.Z <= zmax || z <= 1) break;     // enforce the workspace cap (R11)
         z = std::min(z_used, z) - 1;
     }
-    g.csplit = e.csplit_ok ? choose_csplit(g, e.occ, num_sms) : 1;
+    g.csplit = e.csplit_ok ? choose_csplit(g, e, num_sms, ewm_flops(g)) : 1;
     out->geom = g;
     out->entry = &e;
     out->z_hat = z_used;
@@ -277,11 +298,7 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
     PairChoice pc;
     if (!choose_pair(p, es, ne, &pc)) return WINRS_ERR_UNSUPPORTED;
     // Step 1b (B200): CTA tile.  Each compiled tile variant is planned (Z,
-    // segments, cluster split) and scored by the wave-quantised time model
-    //   t ~ waves(ctas) / (csplit * tiles * eff(tile))
-    // where eff is the relative per-CTA efficiency of the tile (larger tiles
-    // amortise the transforms and operand traffic better: 1.0 for the largest
-    // variant, 0.55 for the half-size one — calibrated on B200).
+    // segments, cluster split) and scored by the B200 time model above.
     std::vector<const KernelEntry*> tiles;
     for (int i = 0; i < ne; ++i)
         if (same_pair(es[i], *pc.proto)) tiles.push_back(&es[i]);
@@ -294,17 +311,11 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
     PlanResult best;
     bool have = false;
     double best_t = 1e30;
-    const int big = tiles.empty() ? 1 : tiles.front()->bn * tiles.front()->bm;
     for (const KernelEntry* e : tiles) {
         if (force_tile && (e->bn != fbn || e->bm != fbm)) continue;
         PlanResult r;
         plan_with_tile(p, *e, pc, num_sms, &r);
-        const Geometry& g = r.geom;
-        const double eff = e->bn * e->bm >= big ? 1.0 : 0.55;
-        const double frac = g.csplit <= 2 ? 1.0 : (g.csplit == 4 ? 132.0 / 148.0 : 128.0 / 148.0);
-        const long long slots = std::max(1LL, (long long)(e->occ * num_sms * frac));
-        const long long waves = (num_ctas(g) + slots - 1) / slots;
-        const double t = (double)waves / ((double)g.csplit * (double)num_tiles(g) * eff);
+        const double t = model_time(r.geom, *e, num_sms, ewm_flops(r.geom));
         if (!have || t < best_t - 1e-12) { best = r; best_t = t; have = true; }
     }
     if (!have) return WINRS_ERR_UNSUPPORTED;
