@@ -50,7 +50,7 @@ template <int A0, int N0, int R0, int A1, int N1, int R1, int BM>
 cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
     static std::atomic<unsigned long long> done{0};
     auto k = bfc_f16_kernel<A0, N0, R0, A1, N1, R1, BM>;
-    constexpr size_t sm = Smem<A0, R0, BM>::bytes;
+    constexpr size_t sm = smem_total<A0, N0, R0, BM>();
     cudaError_t e = ensure_smem_attr(k, sm, done);
     if (e != cudaSuccess) return e;
     const long long grid = num_ctas(g);
@@ -83,7 +83,7 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
 
 #define WINRS_F16_ENTRY(A0, N0, R0, A1, N1, R1, BM)                                                  \
     {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1, 1,            \
-     ::winrs::f16k::Smem<A0, R0, BM>::bytes, &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1, BM>,     \
+     ::winrs::f16k::smem_total<A0, N0, R0, BM>(), &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1, BM>, \
      "f16tc_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x" #BM}
 
 #ifdef WINRS_TRACE
@@ -98,6 +98,7 @@ const KernelEntry* f16_entries(int* n) {
         WINRS_F16_ENTRY(8, 3, 6, 4, 3, 2, 32),
         WINRS_F16_ENTRY(8, 3, 6, 0, 0, 0, 64),
         WINRS_F16_ENTRY(8, 3, 6, 0, 0, 0, 32),
+        WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 128),
         WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 64),
         WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 32),
     };

@@ -42,7 +42,7 @@ constexpr int KC = 16;           // depth entries per chunk = UMMA K
 constexpr int S_OP = 2;          // operand ring stages
 // transformer warps: one thread per (row pair, depth quad) unit of a chunk:
 // FT (BN/2 k pairs x 4 quads) + IT (BM/2 c pairs x 4 quads)
-template <int BM> __host__ __device__ constexpr int tx_warps() { return ((BN / 2) * 2 + (BM / 2) * 2) / 32; }
+template <int BM> __host__ __device__ constexpr int tx_warps() { return (BN / 32) * 2 + (BM / 32) * 2; }
 template <int BM> __host__ __device__ constexpr int nthreads() { return 64 + 32 * tx_warps<BM>(); }
 
 struct Args {
@@ -152,13 +152,14 @@ struct Smem {
 
 // Operand layout (K-major, no swizzle): element (row, kk) of a 16-deep slab at
 // byte (row/8)*256 + (kk/8)*128 + (row%8)*16 + (kk%8)*2.
+
 __device__ __forceinline__ uint32_t op_row_off(int row, int dgroup) {
     return (uint32_t)((row >> 3) * 256 + dgroup * 128 + (row & 7) * 16);
 }
 
 #ifdef WINRS_TRACE
 // Debug-build timeline of CTA 0 (globaltimer ns): [role][chunk][event].
-__device__ unsigned long long g_trace[3][256][4];
+__device__ unsigned long long g_trace[4][256][4];
 __device__ __forceinline__ unsigned long long gtime() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
@@ -188,67 +189,74 @@ __device__ __forceinline__ void depth_coord(long long d, int N, int units, int h
     *h = hs + (int)(t / units);
 }
 
-// ---- transformer work for one chunk.  A unit is (row pair, 8 consecutive
-// depth entries): FT units cover the B_N/2 k pairs of every A_xi, IT units
-// the B_M/2 c pairs of every B_xi; 2 depth octets per KC = 16 chunk.  Each
-// unit computes 8 transforms per row in packed f32x2 (rows 2p, 2p+1), rounds
-// to FP16 and writes one 16-byte core-matrix row per (xi, row).
+// ---- transformer work for one chunk.  A unit is (one row, 8 consecutive
+// depth entries = a depth octet): FT units cover the B_N rows (k) of every
+// A_xi, IT units the B_M rows (c) of every B_xi; 2 octets per KC = 16 chunk.
+// A thread computes its 8 transforms two depth entries at a time in packed
+// f32x2 (lanes = depth d, d+1), so each FP16 pack is already a K-adjacent
+// half2 and the 8 results of a row form one 16-byte core-matrix row: one
+// STS.128 per xi.  A warp holds 32 consecutive rows of one octet, so its raw
+// loads (consecutive channels) and its operand stores (8 distinct rows per
+// quarter-warp) are bank-conflict free.  FT and IT warps are interleaved so
+// every SM sub-partition (warp % 4) gets the same mix.
 constexpr int DQ = 8;                    // depth entries per unit
 constexpr int NQ = KC / DQ;              // depth octets per chunk
-template <int BM> __host__ __device__ constexpr int ft_units() { return (BN / 2) * NQ; }
-template <int BM> __host__ __device__ constexpr int it_units() { return (BM / 2) * NQ; }
+template <int BM> __host__ __device__ constexpr int ft_warps() { return (BN / 32) * NQ; }
+template <int BM> __host__ __device__ constexpr int it_warps() { return (BM / 32) * NQ; }
 
 template <int WT_FN, int A, int NN, int RR, int NIN>
-__device__ __forceinline__ void unit_transform(const __half* src, int row_stride, int depth_stride, uint8_t* dst0,
-                                               int slab_bytes, int p, int g) {
+__device__ __forceinline__ void unit_transform(const __half* src, int tap_stride, int depth_stride, uint8_t* dst0,
+                                               int slab_bytes, int row, int oct) {
     using WT = Wino<A, NN, RR>;
-    uint32_t pk[A][2][4];   // [xi][row 2p / 2p+1][4 x half2 along d]
+    uint32_t pk[A][4];   // [xi][half2 of depth (2j, 2j+1)]
 #pragma unroll
-    for (int j = 0; j < DQ; j += 2) {
-        F2 o0[A], o1[A];
-        {
-            F2 in[NIN];
-            const __half* s0 = src + (g * DQ + j) * depth_stride + 2 * p;
+    for (int j = 0; j < DQ / 2; ++j) {
+        F2 in[NIN], o[A];
+        const __half* s0 = src + (oct * DQ + 2 * j) * depth_stride + row;
 #pragma unroll
-            for (int i = 0; i < NIN; ++i) in[i] = ld_h2(s0 + i * row_stride);
-            if (WT_FN == 0) WT::ft(in, o0); else WT::it(in, o0);
-        }
-        {
-            F2 in[NIN];
-            const __half* s1 = src + (g * DQ + j + 1) * depth_stride + 2 * p;
+        for (int i = 0; i < NIN; ++i)
+            in[i] = F2{__half2float(s0[i * tap_stride]), __half2float(s0[depth_stride + i * tap_stride])};
+        if (WT_FN == 0) WT::ft(in, o); else WT::it(in, o);
 #pragma unroll
-            for (int i = 0; i < NIN; ++i) in[i] = ld_h2(s1 + i * row_stride);
-            if (WT_FN == 0) WT::ft(in, o1); else WT::it(in, o1);
-        }
-#pragma unroll
-        for (int x = 0; x < A; ++x) {
-            pk[x][0][j / 2] = pack_h2(o0[x].x, o1[x].x);
-            pk[x][1][j / 2] = pack_h2(o0[x].y, o1[x].y);
-        }
+        for (int x = 0; x < A; ++x) pk[x][j] = pack_h2(o[x].x, o[x].y);
     }
 #pragma unroll
-    for (int x = 0; x < A; ++x) {
-        uint8_t* base = dst0 + x * slab_bytes;
-#pragma unroll
-        for (int e = 0; e < 2; ++e)
-            *reinterpret_cast<uint4*>(base + op_row_off(2 * p + e, g)) =
-                make_uint4(pk[x][e][0], pk[x][e][1], pk[x][e][2], pk[x][e][3]);
-    }
+    for (int x = 0; x < A; ++x)
+        *reinterpret_cast<uint4*>(dst0 + x * slab_bytes + op_row_off(row, oct)) =
+            make_uint4(pk[x][0], pk[x][1], pk[x][2], pk[x][3]);
+}
+
+// tx warp tw (0 .. tx_warps-1) -> IT warp index (>= 0) or FT warp index
+// (-1 - idx).  IT units cost more than FT units, so IT warps are spread so
+// that each SM sub-partition ((tw + 2) % 4) gets the same number of them.
+template <int BM>
+__host__ __device__ __forceinline__ bool tx_is_it(int tw) {
+    constexpr int T = tx_warps<BM>(), I = it_warps<BM>();
+    if (T == 3 * I) return tw % 3 == 2;                            // e.g. B_M = 64: 12 warps, 4 IT
+    if (T == 2 * I) return ((tw & 1) ^ ((tw >> 2) & 1)) != 0;      // e.g. B_M = 128: 16 warps, 8 IT
+    return (tw + 1) * I / T > tw * I / T;                          // generic even spread
+}
+template <int BM>
+__device__ __forceinline__ int tx_role(int tw) {
+    int before = 0;
+#pragma unroll 1
+    for (int t = 0; t < tw; ++t) before += tx_is_it<BM>(t) ? 1 : 0;
+    return tx_is_it<BM>(tw) ? before : -1 - (tw - before);
 }
 
 template <int A, int NN, int RR, int BM>
-__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tx_id) {
+__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tw, int lane) {
     constexpr int RAW_Y = KC * RR * BN * 2;
     const __half* rawY = reinterpret_cast<const __half*>(raw);            // [KC][RR][BN]
     const __half* rawX = reinterpret_cast<const __half*>(raw + RAW_Y);    // [KC][A][BM]
     constexpr int OPA = BN * KC * 2, OPB = BM * KC * 2;
-    if (tx_id < ft_units<BM>()) {
-        const int p = tx_id % (BN / 2), g = tx_id / (BN / 2);
-        unit_transform<0, A, NN, RR, RR>(rawY, BN, RR * BN, op, OPA, p, g);
-    } else if (tx_id < ft_units<BM>() + it_units<BM>()) {
-        const int t = tx_id - ft_units<BM>();
-        const int q = t % (BM / 2), g = t / (BM / 2);
-        unit_transform<1, A, NN, RR, A>(rawX, BM, A * BM, op + A * OPA, OPB, q, g);
+    const int role = tx_role<BM>(tw);
+    if (role < 0) {
+        const int f = -1 - role;
+        unit_transform<0, A, NN, RR, RR>(rawY, BN, RR * BN, op, OPA, (f % (BN / 32)) * 32 + lane, f / (BN / 32));
+    } else {
+        unit_transform<1, A, NN, RR, A>(rawX, BM, A * BM, op + A * OPA, OPB, (role % (BM / 32)) * 32 + lane,
+                                        role / (BM / 32));
     }
 }
 
@@ -313,7 +321,13 @@ __device__ __forceinline__ void epilogue(int j_off, bool first, bool empty, uint
 }
 
 // Output staging tile in shared memory for the cluster reduction: [n0][BN][BM+4].
+// It overlays the rings (and, when larger, the mbarriers): it is only written
+// after the last job, when all of them are idle.
 template <int BM> __host__ __device__ constexpr int out_ld() { return BM + 4; }
+template <int A0, int N0, int R0, int BM> __host__ __device__ constexpr size_t smem_total() {
+    return Smem<A0, R0, BM>::bytes > (size_t)N0 * BN * out_ld<BM>() * 4 ? Smem<A0, R0, BM>::bytes
+                                                                           : (size_t)N0 * BN * out_ld<BM>() * 4;
+}
 
 // ---- final pass (warps 2..5): staged tile -> bucket (no cluster split) or ->
 // the shared-memory staging tile (cluster split).
@@ -387,7 +401,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     constexpr int S_RAW = SM::S_RAW;
     constexpr int TX_WARPS = tx_warps<BM>();
     static_assert(A1 * BM <= stash_col<N0, BM>(), "residual accumulators overlap the TMEM output stash");
-    static_assert(N0 * BN * out_ld<BM>() * 4 <= SM::bar_off, "cluster staging tile must fit in the rings");
+    static_assert(N0 * BN * out_ld<BM>() * 4 <= 227 * 1024, "cluster staging tile must fit in shared memory");
     extern __shared__ __align__(1024) uint8_t smem[];
     const Geometry& g = args.g;
     Barriers* bars = reinterpret_cast<Barriers*>(smem + SM::bar_off);
@@ -441,39 +455,43 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     const uint32_t tmem_base = bars->tmem_base;
 
     if (warp == 0) {
-        // ===================== TMA producer =====================
-        if (lane == 0) {
-            int s = 0;
-            uint32_t ph = 0;
-            for (int jb = 0; jb < njobs; ++jb) {
-                const Job& J = jobs[jb];
-                const int RRj = J.phase == 0 ? R0 : R1;
-                const int Aj = J.phase == 0 ? A0 : A1;
-                const CUtensorMap* mX = J.phase == 0 ? &tmX0 : &tmX1;
-                const CUtensorMap* mY = J.phase == 0 ? &tmY0 : &tmY1;
-                const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
-                int c_lo, c_hi;
-                chunk_range(J, &c_lo, &c_hi);
-                const uint32_t bytes = (uint32_t)(KC * (RRj * BN + Aj * BM) * 2);
-                for (int ch = c_lo; ch < c_hi; ++ch) {
-                    TRACE(0, ch - c_lo + jb * 64, 0);
-                    mbar_wait(&bars->raw_empty[s], ph ^ 1);
-                    TRACE(0, ch - c_lo + jb * 64, 1);
-                    uint8_t* raw = smem + SM::raw_off + s * SM::RAW;
-                    uint8_t* rY = raw;
-                    uint8_t* rX = raw + KC * RRj * BN * 2;
-                    mbar_arrive_expect_tx(&bars->raw_full[s], bytes);
-                    for (int b = 0; b < KC; b += args.nb) {
-                        const long long d = (long long)ch * KC + b;
-                        int n = g.N, h = hs, u = 0;   // past-the-end image => zero fill
-                        if (d < depth) depth_coord(d, g.N, J.units, hs, &n, &h, &u);
-                        const int w0 = J.w_first + u * RRj;
-                        tma_load_4d(rY + b * RRj * BN * 2, mY, &bars->raw_full[s], cc.kb * BN, w0, h, n);
-                        tma_load_4d(rX + b * Aj * BM * 2, mX, &bars->raw_full[s], cc.cb * BM,
+        // ===================== TMA producer (whole warp) =====================
+        // Lane 0 arms the stage's mbarrier; lanes 0 .. 2*KC/nb-1 then each issue
+        // one box (even lanes dY, odd lanes X) so the boxes of a chunk are in
+        // flight together instead of being issued back to back by one thread.
+        int s = 0;
+        uint32_t ph = 0;
+        const int nbox = 2 * (KC / args.nb);
+        for (int jb = 0; jb < njobs; ++jb) {
+            const Job& J = jobs[jb];
+            const int RRj = J.phase == 0 ? R0 : R1;
+            const int Aj = J.phase == 0 ? A0 : A1;
+            const CUtensorMap* mX = J.phase == 0 ? &tmX0 : &tmX1;
+            const CUtensorMap* mY = J.phase == 0 ? &tmY0 : &tmY1;
+            const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
+            int c_lo, c_hi;
+            chunk_range(J, &c_lo, &c_hi);
+            const uint32_t bytes = (uint32_t)(KC * (RRj * BN + Aj * BM) * 2);
+            for (int ch = c_lo; ch < c_hi; ++ch) {
+                if (lane == 0) TRACE(0, ch - c_lo + jb * 64, 0);
+                mbar_wait(&bars->raw_empty[s], ph ^ 1);
+                if (lane == 0) TRACE(0, ch - c_lo + jb * 64, 1);
+                uint8_t* raw = smem + SM::raw_off + s * SM::RAW;
+                if (lane == 0) mbar_arrive_expect_tx(&bars->raw_full[s], bytes);
+                __syncwarp();
+                if (lane < nbox) {
+                    const int b = (lane >> 1) * args.nb;
+                    const long long d = (long long)ch * KC + b;
+                    int n = g.N, h = hs, u = 0;   // past-the-end image => zero fill
+                    if (d < depth) depth_coord(d, g.N, J.units, hs, &n, &h, &u);
+                    const int w0 = J.w_first + u * RRj;
+                    if ((lane & 1) == 0)
+                        tma_load_4d(raw + b * RRj * BN * 2, mY, &bars->raw_full[s], cc.kb * BN, w0, h, n);
+                    else
+                        tma_load_4d(raw + KC * RRj * BN * 2 + b * Aj * BM * 2, mX, &bars->raw_full[s], cc.cb * BM,
                                     w0 + J.fw0 - g.pad, h + cc.fh - g.pad, n);
-                    }
-                    if (++s == S_RAW) { s = 0; ph ^= 1; }
                 }
+                if (++s == S_RAW) { s = 0; ph ^= 1; }
             }
         }
     } else if (warp == 1) {
@@ -498,7 +516,11 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     for (int x = 0; x < Aj; ++x) {
                         const uint64_t ad = umma_desc(base + x * SM::OPA, 128, 256);
                         const uint64_t bd = umma_desc(base + Aj * SM::OPA + x * SM::OPB, 128, 256);
+#ifndef WINRS_NO_MMA
                         umma_f16<BM>(tmem_base + (uint32_t)(x * BM), ad, bd, ch > c_lo ? 1u : 0u);
+#else
+                        (void)ad; (void)bd;
+#endif
                     }
                     umma_commit(&bars->op_empty[s]);
                     TRACE(1, ch - c_lo + jb * 64, 1);
@@ -509,7 +531,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         }
     } else {
         // ===================== transformers (+ epilogue) =====================
-        const int tx_id = threadIdx.x - 64;
+        const int tw = warp - 2;
         int sr = 0, so = 0;
         uint32_t phr = 0, pho = 0;
         for (int jb = 0; jb < njobs; ++jb) {
@@ -524,9 +546,12 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 2);
                 const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
                 uint8_t* op = smem + SM::op_off + so * SM::OP;
-                if (J.phase == 0) transform_chunk<A0, N0, R0, BM>(raw, op, tx_id);
-                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM>(raw, op, tx_id);
+                if (J.phase == 0) transform_chunk<A0, N0, R0, BM>(raw, op, tw, lane);
+                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM>(raw, op, tw, lane);
+                if (threadIdx.x == 64) TRACE(3, ch - c_lo + jb * 64, 0);
+                if (threadIdx.x == 64 + 32 * 2) TRACE(3, ch - c_lo + jb * 64, 1);   // an IT warp
                 fence_proxy_async();
+                if (threadIdx.x == 64) TRACE(3, ch - c_lo + jb * 64, 2);
                 __syncwarp();
                 if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 3);
                 if (lane == 0) {

@@ -51,12 +51,12 @@ def _compile(src: str, force: bool, hdr_m: float) -> str:
     return o
 
 
-def build(force: bool = False, jobs: int = 0, trace: bool = False) -> str:
+def build(force: bool = False, jobs: int = 0, trace: bool = False, extra=()) -> str:
     global OBJ, LIB, FLAGS
     if trace:   # debug build with the CTA-0 timeline (csrc/bfc_f16.cuh TRACE)
-        OBJ = os.path.join(ROOT, "build", "obj_trace")
-        LIB = os.path.join(PKG, "libwinrs_trace.so")
-        FLAGS = FLAGS + ["-DWINRS_TRACE"]
+        OBJ = os.path.join(ROOT, "build", "obj_trace" + "".join(extra))
+        LIB = os.path.join(PKG, "libwinrs_trace%s.so" % "".join(extra))
+        FLAGS = FLAGS + ["-DWINRS_TRACE"] + ["-D" + e for e in extra]
     os.makedirs(OBJ, exist_ok=True)
     if not os.path.exists(GEN_OUT) or os.path.getmtime(GEN_OUT) < os.path.getmtime(GEN):
         subprocess.check_call([sys.executable, GEN])
@@ -77,5 +77,6 @@ if __name__ == "__main__":
     ap.add_argument("--force", action="store_true")
     ap.add_argument("-j", type=int, default=0)
     ap.add_argument("--trace", action="store_true")
+    ap.add_argument("--define", action="append", default=[])
     a = ap.parse_args()
-    print(build(a.force, a.j, a.trace))
+    print(build(a.force, a.j, a.trace, tuple(a.define)))

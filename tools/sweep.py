@@ -14,15 +14,21 @@ from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl  # noqa: E402
 
 layers = [wl.LAYERS[n] for n in sys.argv[1].split(",")] if len(sys.argv) > 1 else \
     wl.RESNET50_F32 + wl.RESNET50_F16 + wl.WIDE_F32
-tiles = {"f32": ["64x64", "32x32", "64x32"], "f16": ["128x64", "128x32"]}
+tiles = {"f32": ["64x64", "32x32", "64x32"], "f16": ["128x128", "128x64", "128x32"]}
+pairs = {"f32": [None], "f16": [None, "4,3,2,0,0,0"]}
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 for l in layers:
     X, dY = wl.make_inputs(l)
     Xg, Gg = torch.from_numpy(X).cuda(), torch.from_numpy(dY).cuda()
-    for t in tiles[l.dtype]:
+    for pair in pairs[l.dtype]:
+      for t in tiles[l.dtype]:
         for cs in (1, 2, 4, 8):
             os.environ["WINRS_FORCE_TILE"] = t
             os.environ["WINRS_FORCE_CSPLIT"] = str(cs)
+            if pair:
+                os.environ["WINRS_FORCE_PAIR"] = pair
+            else:
+                os.environ.pop("WINRS_FORCE_PAIR", None)
             try:
                 p = W.plan(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype)
             except Exception:
@@ -42,7 +48,7 @@ for l in layers:
                 if i >= 2:
                     ts.append(a.elapsed_time(b))
             ms = statistics.median(ts)
-            print(json.dumps({"layer": l.name, "tile": t, "csplit": p.info["csplit"], "Z": p.info["Z"],
+            print(json.dumps({"layer": l.name, "pair": p.kernel_name, "tile": t, "csplit": p.info["csplit"], "Z": p.info["Z"],
                               "ctas": p.info["ctas_main"], "us": round(ms * 1e3, 1),
                               "tflops": round(l.direct_flops / ms / 1e9, 1)}), flush=True)
 os.environ.pop("WINRS_FORCE_TILE", None)
