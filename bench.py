@@ -44,6 +44,23 @@ def _peaks():
     return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0, "sm_max_mhz": 1965.0}, "fallback"
 
 
+def _ncu_traffic(dtype: str, layer_name: str):
+    """DRAM bytes (read + write) per launch of the dominant kernel from the
+    latest committed ncu --set full capture (profiles/r*/traffic.json)."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*", "traffic.json")))
+    if not files:
+        return None, None
+    with open(files[-1]) as f:
+        t = json.load(f)
+    base = layer_name.rsplit("_", 1)[0]
+    if dtype in t and base in t.get("layers", []):
+        i = t["layers"].index(base)
+        if i < len(t[dtype]):
+            return t[dtype][i]["dram_bytes"], os.path.relpath(files[-1], ROOT) + " (ncu --set full)"
+    return None, None
+
+
 def _workload(name: str, dtype: str):
     from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
     if name == "r50":
@@ -242,7 +259,7 @@ def run_winrs(args):
                         "peak": peaks["bf16_tflops"], "unit": "TFLOP/s", "peak_source": src + " (fp16 = bf16 rate)"}
             roof.update(kernel=p.kernel_name, layer=l.name)
         roof["frac"] = roof["achieved"] / roof["peak"]
-        roof["traffic"] = None
+        roof["traffic"], roof["traffic_source"] = _ncu_traffic(args.dtype, l.name)
         roof["alg_bytes"] = alg_bytes
         roof["ewm_flops"] = info["ewm_flops"]
         roof["kernel_ms"] = dom_ms
