@@ -90,6 +90,9 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
 extern "C" __attribute__((visibility("default"))) int winrs_trace_read(unsigned long long* out) {
     return (int)cudaMemcpyFromSymbol(out, f16k::g_trace, sizeof(f16k::g_trace));
 }
+extern "C" __attribute__((visibility("default"))) int winrs_trace_read_w(unsigned long long* out) {
+    return (int)cudaMemcpyFromSymbol(out, f16k::g_trace_w, sizeof(f16k::g_trace_w));
+}
 #endif
 
 const KernelEntry* f16_entries(int* n) {

@@ -42,7 +42,7 @@ constexpr int KC = 16;           // depth entries per chunk = UMMA K
 constexpr int S_OP = 2;          // operand ring stages
 // transformer warps: one thread per (row pair, depth quad) unit of a chunk:
 // FT (BN/2 k pairs x 4 quads) + IT (BM/2 c pairs x 4 quads)
-template <int BM> __host__ __device__ constexpr int tx_warps() { return (BN / 32) * 2 + (BM / 32) * 2; }
+template <int BM> __host__ __device__ constexpr int tx_warps() { return (BN / 2) * 2 / 32 + (BM / 2) * 2 / 32; }
 template <int BM> __host__ __device__ constexpr int nthreads() { return 64 + 32 * tx_warps<BM>(); }
 
 struct Args {
@@ -65,15 +65,19 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
+// Wait for the phase with the given parity.  The suspend-time hint lets the
+// waiting warp sleep in hardware until the phase completes instead of
+// re-polling, so idle producer / MMA warps do not steal issue slots from the
+// transformer warps sharing their SM sub-partition.
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     const uint32_t a = smem_u32(bar);
     asm volatile(
         "{\n"
         ".reg .pred P;\n"
         "WAIT_%=:\n"
-        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1, %2;\n"
         "@!P bra WAIT_%=;\n"
-        "}\n" :: "r"(a), "r"(parity) : "memory");
+        "}\n" :: "r"(a), "r"(parity), "r"(1000000) : "memory");
 }
 __device__ __forceinline__ void tma_load_4d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
                                             int c2, int c3) {
@@ -152,6 +156,16 @@ struct Smem {
 
 // Operand layout (K-major, no swizzle): element (row, kk) of a 16-deep slab at
 // byte (row/8)*256 + (kk/8)*128 + (row%8)*16 + (kk%8)*2.
+//
+// Rows are stored permuted within blocks of 16: logical row r -> physical
+// perm16(r) = 16*(r/16) + 8*(r%2) + (r%16)/2.  A transformer thread owns the
+// logical row pair (2p, 2p+1); with the permutation the 8 lanes of a
+// quarter-warp store 8 distinct physical row%8 values, so the 16-byte operand
+// stores are bank-conflict free.  The MMA is row-order agnostic: the
+// permutation reappears as a TMEM lane (k) / column (c) permutation that the
+// final output pass undoes.
+__host__ __device__ __forceinline__ int perm16(int r) { return (r & ~15) | ((r & 1) << 3) | ((r >> 1) & 7); }
+__host__ __device__ __forceinline__ int iperm16(int l) { return (l & ~15) | ((l & 7) << 1) | ((l >> 3) & 1); }
 
 __device__ __forceinline__ uint32_t op_row_off(int row, int dgroup) {
     return (uint32_t)((row >> 3) * 256 + dgroup * 128 + (row & 7) * 16);
@@ -160,6 +174,7 @@ __device__ __forceinline__ uint32_t op_row_off(int row, int dgroup) {
 #ifdef WINRS_TRACE
 // Debug-build timeline of CTA 0 (globaltimer ns): [role][chunk][event].
 __device__ unsigned long long g_trace[4][256][4];
+__device__ unsigned long long g_trace_w[256][16];   // per-warp "chunk done" times
 __device__ __forceinline__ unsigned long long gtime() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
@@ -189,52 +204,70 @@ __device__ __forceinline__ void depth_coord(long long d, int N, int units, int h
     *h = hs + (int)(t / units);
 }
 
-// ---- transformer work for one chunk.  A unit is (one row, 8 consecutive
-// depth entries = a depth octet): FT units cover the B_N rows (k) of every
-// A_xi, IT units the B_M rows (c) of every B_xi; 2 octets per KC = 16 chunk.
-// A thread computes its 8 transforms two depth entries at a time in packed
-// f32x2 (lanes = depth d, d+1), so each FP16 pack is already a K-adjacent
-// half2 and the 8 results of a row form one 16-byte core-matrix row: one
-// STS.128 per xi.  A warp holds 32 consecutive rows of one octet, so its raw
-// loads (consecutive channels) and its operand stores (8 distinct rows per
-// quarter-warp) are bank-conflict free.  FT and IT warps are interleaved so
-// every SM sub-partition (warp % 4) gets the same mix.
-constexpr int DQ = 8;                    // depth entries per unit
-constexpr int NQ = KC / DQ;              // depth octets per chunk
-template <int BM> __host__ __device__ constexpr int ft_warps() { return (BN / 32) * NQ; }
-template <int BM> __host__ __device__ constexpr int it_warps() { return (BM / 32) * NQ; }
+// ---- transformer work for one chunk.  A unit is (row pair 2p/2p+1, 8
+// consecutive depth entries = a depth octet for FT, 4 = a quad for IT, whose
+// units cost more): FT units cover the B_N/2 k pairs of every A_xi, IT units
+// the B_M/2 c pairs of every B_xi.  Each raw load is a half2 of the row pair at one depth (one
+// 128-byte wavefront per warp); a thread computes its transforms two depth
+// entries at a time in packed f32x2 (lanes = depth d, d+1) separately for
+// each row, so each FP16 pack is already a K-adjacent half2 and the 8 results
+// of a row form one 16-byte core-matrix row: two STS.128 per xi, conflict
+// free through perm16.  FT and IT warps are interleaved so every SM
+// sub-partition (warp % 4) gets the same mix.
+constexpr int DQ_FT = 8;                 // depth entries per FT unit (an octet)
+constexpr int DQ_IT = 8;                 // depth entries per IT unit (an octet)
+template <int BM> __host__ __device__ constexpr int ft_warps() { return (BN / 2) * (KC / DQ_FT) / 32; }
+template <int BM> __host__ __device__ constexpr int it_warps() { return (BM / 2) * (KC / DQ_IT) / 32; }
 
-template <int WT_FN, int A, int NN, int RR, int NIN>
+template <int WT_FN, int A, int NN, int RR, int NIN, int DQ>
 __device__ __forceinline__ void unit_transform(const __half* src, int tap_stride, int depth_stride, uint8_t* dst0,
-                                               int slab_bytes, int row, int oct) {
+                                               int slab_bytes, int p, int grp) {
     using WT = Wino<A, NN, RR>;
-    uint32_t pk[A][4];   // [xi][half2 of depth (2j, 2j+1)]
+    const int oct = grp;     // depth group index (DQ entries each)
+    uint32_t pk[A][2][DQ / 2];   // [xi][row 2p / 2p+1][half2 of depth (2j, 2j+1)]
 #pragma unroll
     for (int j = 0; j < DQ / 2; ++j) {
-        F2 in[NIN], o[A];
-        const __half* s0 = src + (oct * DQ + 2 * j) * depth_stride + row;
+        F2 in0[NIN], in1[NIN], o[A];
+        const __half* s0 = src + (oct * DQ + 2 * j) * depth_stride + 2 * p;
 #pragma unroll
-        for (int i = 0; i < NIN; ++i)
-            in[i] = F2{__half2float(s0[i * tap_stride]), __half2float(s0[depth_stride + i * tap_stride])};
-        if (WT_FN == 0) WT::ft(in, o); else WT::it(in, o);
+        for (int i = 0; i < NIN; ++i) {
+            const float2 a = __half22float2(*reinterpret_cast<const __half2*>(s0 + i * tap_stride));
+            const float2 b = __half22float2(*reinterpret_cast<const __half2*>(s0 + depth_stride + i * tap_stride));
+            in0[i] = F2{a.x, b.x};    // row 2p,   depth 2j, 2j+1
+            in1[i] = F2{a.y, b.y};    // row 2p+1, depth 2j, 2j+1
+        }
+        if (WT_FN == 0) WT::ft(in0, o); else WT::it(in0, o);
 #pragma unroll
-        for (int x = 0; x < A; ++x) pk[x][j] = pack_h2(o[x].x, o[x].y);
+        for (int x = 0; x < A; ++x) pk[x][0][j] = pack_h2(o[x].x, o[x].y);
+        if (WT_FN == 0) WT::ft(in1, o); else WT::it(in1, o);
+#pragma unroll
+        for (int x = 0; x < A; ++x) pk[x][1][j] = pack_h2(o[x].x, o[x].y);
     }
+    // depth group -> K position kk0 = grp*DQ: K half kk0/8, byte offset (kk0%8)*2 in the 16-byte row
+    const int kk0 = grp * DQ;
 #pragma unroll
     for (int x = 0; x < A; ++x)
-        *reinterpret_cast<uint4*>(dst0 + x * slab_bytes + op_row_off(row, oct)) =
-            make_uint4(pk[x][0], pk[x][1], pk[x][2], pk[x][3]);
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+            uint8_t* d = dst0 + x * slab_bytes + op_row_off(perm16(2 * p + e), kk0 >> 3) + (kk0 & 7) * 2;
+            if constexpr (DQ == 8)
+                *reinterpret_cast<uint4*>(d) = make_uint4(pk[x][e][0], pk[x][e][1], pk[x][e][2], pk[x][e][3]);
+            else
+                *reinterpret_cast<uint2*>(d) = make_uint2(pk[x][e][0], pk[x][e][1]);
+        }
 }
 
 // tx warp tw (0 .. tx_warps-1) -> IT warp index (>= 0) or FT warp index
-// (-1 - idx).  IT units cost more than FT units, so IT warps are spread so
-// that each SM sub-partition ((tw + 2) % 4) gets the same number of them.
+// (-1 - idx).  IT units cost ~1.3x FT units; the IT warps are spread over
+// the SM sub-partitions (warp w runs on w % 4).  Measured on B200: the
+// per-chunk time is bounded by shared-memory / LSU throughput, so more or
+// smaller units do not help.
 template <int BM>
 __host__ __device__ __forceinline__ bool tx_is_it(int tw) {
     constexpr int T = tx_warps<BM>(), I = it_warps<BM>();
-    if (T == 3 * I) return tw % 3 == 2;                            // e.g. B_M = 64: 12 warps, 4 IT
-    if (T == 2 * I) return ((tw & 1) ^ ((tw >> 2) & 1)) != 0;      // e.g. B_M = 128: 16 warps, 8 IT
-    return (tw + 1) * I / T > tw * I / T;                          // generic even spread
+    if (T == 3 * I) return tw % 3 == 2;
+    if (T == 2 * I) return ((tw & 1) ^ ((tw >> 2) & 1)) != 0;
+    return (tw + 1) * I / T > tw * I / T;
 }
 template <int BM>
 __device__ __forceinline__ int tx_role(int tw) {
@@ -252,11 +285,14 @@ __device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op,
     constexpr int OPA = BN * KC * 2, OPB = BM * KC * 2;
     const int role = tx_role<BM>(tw);
     if (role < 0) {
-        const int f = -1 - role;
-        unit_transform<0, A, NN, RR, RR>(rawY, BN, RR * BN, op, OPA, (f % (BN / 32)) * 32 + lane, f / (BN / 32));
-    } else {
-        unit_transform<1, A, NN, RR, A>(rawX, BM, A * BM, op + A * OPA, OPB, (role % (BM / 32)) * 32 + lane,
-                                        role / (BM / 32));
+        const int f = -1 - role;   // FT warp: 32 k pairs x one octet
+        unit_transform<0, A, NN, RR, RR, DQ_FT>(rawY, BN, RR * BN, op, OPA, (f % (BN / 64)) * 32 + lane,
+                                                f / (BN / 64));
+    } else {                       // IT warp: 32 c pairs (or BM/2 pairs x 32/(BM/2) quads) x quads
+        constexpr int PW = BM / 2 < 32 ? BM / 2 : 32;
+        const int q = (role % ((BM / 2) / PW)) * PW + (lane % PW);
+        const int quad = role / ((BM / 2) / PW) * (32 / PW) + lane / PW;
+        unit_transform<1, A, NN, RR, A, DQ_IT>(rawX, BM, A * BM, op + A * OPA, OPB, q, quad);
     }
 }
 
@@ -330,32 +366,41 @@ template <int A0, int N0, int R0, int BM> __host__ __device__ constexpr size_t s
 }
 
 // ---- final pass (warps 2..5): staged tile -> bucket (no cluster split) or ->
-// the shared-memory staging tile (cluster split).
+// the shared-memory staging tile (cluster split).  Undoes the operand row
+// permutation: TMEM lane L holds k = iperm16(L); physical columns
+// [16b, 16b+16) hold logical c = 16b + 2i (first 8) and 16b + 2i + 1 (last 8).
 template <int N0, int BM>
 __device__ __forceinline__ void final_out(const Geometry& g, float* bucket, const CtaCoord& cc, int fw0, uint32_t tmem_base,
                                           int warp, float* Out) {
     const int quarter = warp & 3, lane = threadIdx.x & 31;
-    const int kl = quarter * 32 + lane;
+    const int kl = iperm16(quarter * 32 + lane);
     const int kg = cc.kb * BN + kl;
     const uint32_t lane_base = tmem_base + ((uint32_t)(quarter * 32) << 16);
 #pragma unroll 1
-    for (int c0 = 0; c0 < BM; c0 += 8) {
-#pragma unroll
+    for (int c0 = 0; c0 < BM; c0 += 16) {
+#pragma unroll 1
         for (int j = 0; j < N0; ++j) {
-            float y[8];
-            tmem_ld8(lane_base + (uint32_t)(stash_col<N0, BM>() + j * BM + c0), y);
+            float ph[16], y[16];
+            tmem_ld8(lane_base + (uint32_t)(stash_col<N0, BM>() + j * BM + c0), ph);
+            tmem_ld8(lane_base + (uint32_t)(stash_col<N0, BM>() + j * BM + c0 + 8), ph + 8);
             tmem_wait_ld();
-            const float4 a = make_float4(y[0], y[1], y[2], y[3]), b = make_float4(y[4], y[5], y[6], y[7]);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                y[2 * i] = ph[i];
+                y[2 * i + 1] = ph[8 + i];
+            }
             if (g.csplit > 1) {
                 float4* o = reinterpret_cast<float4*>(Out + ((long long)j * BN + kl) * out_ld<BM>() + c0);
-                o[0] = a;
-                o[1] = b;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) o[q] = make_float4(y[4 * q], y[4 * q + 1], y[4 * q + 2], y[4 * q + 3]);
             } else {
                 const int cg = cc.cb * BM + c0;
-                if (kg < g.K && cg < g.C) {   // C % 8 == 0: an 8-column group is all in or all out
+                if (kg < g.K && cg < g.C) {   // C % 8 == 0: 8-column groups are all in or all out
                     float4* d4 = reinterpret_cast<float4*>(bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0 + j) * g.C + cg);
-                    d4[0] = a;
-                    d4[1] = b;
+                    const int nq = cg + 16 <= g.C ? 4 : 2;
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        if (q < nq) d4[q] = make_float4(y[4 * q], y[4 * q + 1], y[4 * q + 2], y[4 * q + 3]);
                 }
             }
         }
@@ -554,6 +599,9 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 if (threadIdx.x == 64) TRACE(3, ch - c_lo + jb * 64, 2);
                 __syncwarp();
                 if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 3);
+#ifdef WINRS_TRACE
+                if (lane == 0 && blockIdx.x == 0 && ch - c_lo + jb * 64 < 256) g_trace_w[ch - c_lo + jb * 64][warp] = gtime();
+#endif
                 if (lane == 0) {
                     mbar_arrive(&bars->op_full[so]);
                     mbar_arrive(&bars->raw_empty[sr]);

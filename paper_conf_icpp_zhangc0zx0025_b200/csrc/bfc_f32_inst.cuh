@@ -30,7 +30,7 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
 }  // namespace winrs
 
 #define WINRS_F32_ENTRY(A0, N0, R0, A1, N1, R1, BN, BM)                                         \
-    {0, A0, N0, R0, A1, N1, R1, BN, BM, ::winrs::f32k::NT, ((BN) * (BM) >= 2048 ? 1 : 2), 1,                                  \
+    {0, A0, N0, R0, A1, N1, R1, BN, BM, ::winrs::f32k::NT, ((BN) * (BM) >= 4096 ? 1 : 2), 1,                                  \
      ::winrs::f32k::smem_bytes<A0, N0, R0, A1, N1, R1, BN, BM>(),                                \
      &::winrs::f32k::launch<A0, N0, R0, A1, N1, R1, BN, BM>,                                     \
      "f32_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_" #BN "x" #BM}

@@ -26,3 +26,11 @@ for c in list(range(0, 40)) + list(range(64, 90)):
     if b[2, c, 0] < 0 and b[0, c, 0] < 0:
         continue
     print(c, "|", b[0, c, 0], b[0, c, 1], "|", b[2, c, 0], b[2, c, 1], b[2, c, 2], b[2, c, 3], "|", b[1, c, 0], b[1, c, 1], "|", b[3, c, 0], b[3, c, 1], b[3, c, 2])
+
+bw = np.zeros((256, 16), dtype=np.uint64)
+L.winrs_trace_read_w.argtypes = [ctypes.c_void_p]
+L.winrs_trace_read_w(bw.ctypes.data)
+print("per-warp chunk-done times (ns from t0), warps 2..")
+for c in range(0, 12):
+    row = [int(v) - int(t0) if v > 0 else -1 for v in bw[c]]
+    print(c, row[2:14])
