@@ -39,7 +39,10 @@ namespace f16k {
 
 constexpr int BN = 128;          // k rows = UMMA M (TMEM lanes)
 constexpr int KC = 16;           // depth entries per chunk = UMMA K
-constexpr int S_OP = 2;          // operand ring stages
+#ifndef WINRS_F16_SOP
+#define WINRS_F16_SOP 2
+#endif
+constexpr int S_OP = WINRS_F16_SOP;   // operand ring stages
 // transformer warps: one thread per (row pair, depth quad) unit of a chunk:
 // FT (BN/2 k pairs x 4 quads) + IT (BM/2 c pairs x 4 quads)
 template <int BM> __host__ __device__ constexpr int tx_warps() { return (BN / 2) * 2 / 32 + (BM / 2) * 2 / 32; }
@@ -192,7 +195,7 @@ struct Job {
 };
 
 struct Barriers {
-    uint64_t raw_full[4], raw_empty[4], op_full[S_OP], op_empty[S_OP], acc_full, acc_empty;
+    uint64_t raw_full[4], raw_empty[4], op_full[4], op_empty[4], acc_full, acc_empty;
     uint32_t tmem_base;
 };
 
