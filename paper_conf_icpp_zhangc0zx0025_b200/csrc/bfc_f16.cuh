@@ -625,6 +625,10 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 if (lane == 0) mbar_arrive(&bars->acc_empty);
             }
         }
+        // All transformer warps are past their last raw-ring read before the
+        // staging tile (which overlays the rings) is written.  (Already implied
+        // by acc_full -> all MMAs -> all op_full arrivals; made explicit.)
+        asm volatile("bar.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
         if (warp < 6) {
             // every job's epilogue is done (this warp's own, in program order)
             final_out<N0, BM>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
