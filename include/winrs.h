@@ -129,6 +129,15 @@ WINRS_API size_t winrs_workspace_bytes(winrs_plan_t plan);
 WINRS_API winrs_status_t winrs_bfc(winrs_plan_t plan, const void* X, const void* dY, float* dW,
                          void* workspace, void* stream);
 
+/* Same as winrs_bfc for a dY whose pixels are `ldy` elements apart (ldy >= K,
+ * ldy % 4 == 0 for FP32, % 8 for FP16): dY points at channel k0 of a wider
+ * NHWC tensor, so a rank can compute dW for the channel slice [k0, k0+K) of a
+ * K-sharded layer without copying (BASELINE.json's K-sharding alternative,
+ * DESIGN.md §8).  dW is the [K][R][S][C] slice (contiguous in KRSC).  Returns
+ * INVALID_ARG for a bad ldy. */
+WINRS_API winrs_status_t winrs_bfc_strided(winrs_plan_t plan, const void* X, const void* dY, long long ldy,
+                                           float* dW, void* workspace, void* stream);
+
 /* Same computation with HOST buffers: copies X and dY host->device into
  * caller-provided device staging buffers, runs winrs_bfc and copies dW back to
  * host_dW, all on `stream`, then synchronises that stream.  Used for the

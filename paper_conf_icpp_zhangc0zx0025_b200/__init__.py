@@ -20,6 +20,7 @@ from . import _lib
 from ._lib import WinrsError, DTYPES
 
 __all__ = ["Plan", "plan", "plan_for_device", "bfc", "bfc_host", "as_kcrs", "bfc_data_parallel", "shard_range",
+           "bfc_k_sharded",
            "WinrsError", "version", "emulate", "transform", "kernel_names"]
 
 
@@ -122,6 +123,33 @@ def bfc(p: Plan, X, dY, dW=None, workspace=None, stream=None):
     _lib.check(_lib.lib().winrs_bfc(p.handle, Xn.data_ptr(), Gn.data_ptr(), dW.data_ptr(),
                                     workspace.data_ptr() if wsb else None, sp), "winrs_bfc")
     return dW
+
+
+def bfc_k_sharded(X, dY, R: int, S: int, pad: int, dtype: str, rank: int, world: int):
+    """K-sharded BFC (BASELINE.json's communication-free alternative, DESIGN.md
+    §8): rank `rank` computes dW[k0:k1] for its slice of the output channels
+    over the FULL batch, reading its channel slice of dY in place
+    (winrs_bfc_strided, ldy = K).  Returns (dW_slice [k1-k0, R, S, C], k0, k1);
+    the slices of all ranks concatenated along K are the full dW."""
+    import torch
+    N, H, W, C = X.shape
+    K = dY.shape[-1]
+    align = 4 if dtype == "f32" else 8
+    if K % align:
+        raise ValueError("K must be a multiple of %d" % align)
+    a, b = shard_range(K // align, world, rank)
+    k0, k1 = a * align, b * align
+    p = plan(N, C, H, W, k1 - k0, R, S, pad, dtype)
+    if not (dY.is_contiguous() and X.is_contiguous()):
+        raise ValueError("X and dY must be contiguous NHWC")
+    dW = torch.empty((k1 - k0, R, S, C), dtype=torch.float32, device=X.device)
+    wsb = p.workspace_bytes
+    ws = torch.empty(wsb, dtype=torch.uint8, device=X.device) if wsb else None
+    sp = torch.cuda.current_stream(X.device).cuda_stream
+    _lib.check(_lib.lib().winrs_bfc_strided(p.handle, X.data_ptr(), dY.data_ptr() + k0 * dY.element_size(), K,
+                                            dW.data_ptr(), ws.data_ptr() if wsb else None, sp),
+               "winrs_bfc_strided")
+    return dW, k0, k1
 
 
 def bfc_host(p: Plan, X_host, dY_host, dW_host, dev_X, dev_dY, dev_dW, workspace=None, stream=None):

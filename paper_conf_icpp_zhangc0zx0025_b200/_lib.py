@@ -47,6 +47,7 @@ SYMBOLS = [
     ("winrs_plan_info", _i, [_p, ctypes.POINTER(PlanInfoT)]),
     ("winrs_workspace_bytes", _s, [_p]),
     ("winrs_bfc", _i, [_p, _p, _p, _p, _p, _p]),
+    ("winrs_bfc_strided", _i, [_p, _p, _p, ctypes.c_longlong, _p, _p, _p]),
     ("winrs_bfc_host", _i, [_p, _p, _p, _p, _p, _p, _p, _p, _p]),
     ("winrs_plan_destroy", None, [_p]),
     ("winrs_status_string", ctypes.c_char_p, [_i]),

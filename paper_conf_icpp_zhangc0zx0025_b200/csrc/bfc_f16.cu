@@ -26,13 +26,15 @@ static EncodeTiledFn encode_fn() {
     return fn;
 }
 
-// 4-D NHWC fp16 tensor [N][H][W][Ch] as TMA dims {Ch, W, H, N}; box {bc, bw, 1, bn}.
-// Out-of-bounds elements are filled with zeros.
-static bool make_map(CUtensorMap* m, const void* base, int N, int H, int W, int Ch, int bc, int bw, int bn) {
+// 4-D NHWC fp16 tensor [N][H][W][Ch] (pixel stride ld >= Ch elements) as TMA
+// dims {Ch, W, H, N}; box {bc, bw, 1, bn}.  Out-of-bounds elements are zero.
+static bool make_map(CUtensorMap* m, const void* base, int N, int H, int W, int Ch, int bc, int bw, int bn,
+                     int ld = 0) {
     EncodeTiledFn fn = encode_fn();
     if (!fn) return false;
+    if (ld <= 0) ld = Ch;
     const cuuint64_t dims[4] = {(cuuint64_t)Ch, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
-    const cuuint64_t strides[3] = {(cuuint64_t)Ch * 2, (cuuint64_t)W * Ch * 2, (cuuint64_t)H * W * Ch * 2};
+    const cuuint64_t strides[3] = {(cuuint64_t)ld * 2, (cuuint64_t)W * ld * 2, (cuuint64_t)H * W * ld * 2};
     const cuuint32_t box[4] = {(cuuint32_t)bc, (cuuint32_t)bw, 1u, (cuuint32_t)bn};
     const cuuint32_t es[4] = {1u, 1u, 1u, 1u};
     return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
@@ -62,11 +64,11 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
     a.nb = images_per_box(g.N);
     CUtensorMap mX0, mY0, mX1, mY1;
     if (!make_map(&mX0, X, g.N, g.H, g.W, g.C, BM, A0, a.nb) ||
-        !make_map(&mY0, dY, g.N, g.Ho, g.Wo, g.K, BN, R0, a.nb))
+        !make_map(&mY0, dY, g.N, g.Ho, g.Wo, g.K, BN, R0, a.nb, g.ldy))
         return cudaErrorInvalidValue;
     if (A1 != 0) {
         if (!make_map(&mX1, X, g.N, g.H, g.W, g.C, BM, A1 ? A1 : A0, a.nb) ||
-            !make_map(&mY1, dY, g.N, g.Ho, g.Wo, g.K, BN, R1 ? R1 : R0, a.nb))
+            !make_map(&mY1, dY, g.N, g.Ho, g.Wo, g.K, BN, R1 ? R1 : R0, a.nb, g.ldy))
             return cudaErrorInvalidValue;
     } else {
         mX1 = mX0;

@@ -137,7 +137,7 @@ __device__ __forceinline__ void run_phase(const Geometry& g, const float* __rest
             h = hs + (int)(t / units);
         }
         const int w0 = w_first + u * RR;
-        const float* gsrc = dY + (((long long)n * g.Ho + h) * g.Wo + w0) * g.K + k_base;
+        const float* gsrc = dY + (((long long)n * g.Ho + h) * g.Wo + w0) * g.ldy + k_base;
         const int xrow = h + cc.fh - g.pad;
         const int xcol0 = w0 + fw0 - g.pad;
         const float* xsrc = X + (((long long)n * g.H + xrow) * g.W) * g.C + c_base;
@@ -148,7 +148,7 @@ __device__ __forceinline__ void run_phase(const Geometry& g, const float* __rest
             const int i = q / (BN / 4), v4 = q % (BN / 4);
             const int kk = k_base + v4 * 4;
             const bool ok = dv && (w0 + i < g.Wo) && (kk < g.K);
-            cp_async16(gdst + i * BN + v4 * 4, ok ? (const void*)(gsrc + (long long)i * g.K + v4 * 4) : (const void*)dY, ok);
+            cp_async16(gdst + i * BN + v4 * 4, ok ? (const void*)(gsrc + (long long)i * g.ldy + v4 * 4) : (const void*)dY, ok);
         }
         constexpr int XV = ALPHA * (BM / 4);
         for (int q = ld_l; q < XV; q += TPD) {

@@ -164,6 +164,7 @@ static void fill_geometry(const Problem& p, const KernelEntry& e, const PairChoi
     memset(g, 0, sizeof(*g));
     g->N = p.N; g->C = p.C; g->H = p.H; g->W = p.W; g->K = p.K; g->R = p.R; g->S = p.S; g->pad = p.pad;
     g->Ho = p.Ho; g->Wo = p.Wo;
+    g->ldy = p.K;
     g->a0 = e.a0; g->n0 = e.n0; g->r0 = e.r0; g->k0 = pc.k0;
     g->seg_h = seg_h;
     g->bands = std::max(1, p.Ho / seg_h);

@@ -105,9 +105,18 @@ static bool misaligned(const void* p) { return (reinterpret_cast<uintptr_t>(p) &
 
 winrs_status_t winrs_bfc(winrs_plan_t plan, const void* X, const void* dY, float* dW, void* workspace,
                          void* stream) {
+    if (!plan) return WINRS_ERR_INVALID_ARG;
+    return winrs_bfc_strided(plan, X, dY, (long long)plan->info.K, dW, workspace, stream);
+}
+
+winrs_status_t winrs_bfc_strided(winrs_plan_t plan, const void* X, const void* dY, long long ldy, float* dW,
+                                 void* workspace, void* stream) {
     if (!plan || !X || !dY || !dW) return WINRS_ERR_INVALID_ARG;
     if (misaligned(X) || misaligned(dY) || misaligned(dW)) return WINRS_ERR_INVALID_ARG;
-    const Geometry& g = plan->pr.geom;
+    const int align = plan->info.dtype == WINRS_F32 ? 4 : 8;
+    if (ldy < plan->info.K || ldy % align != 0 || ldy > (1LL << 30)) return WINRS_ERR_INVALID_ARG;
+    Geometry g = plan->pr.geom;
+    g.ldy = (int)ldy;
     if (plan->info.workspace_bytes > 0) {
         if (!workspace) return WINRS_ERR_WORKSPACE;
         if (misaligned(workspace)) return WINRS_ERR_INVALID_ARG;
@@ -194,7 +203,7 @@ void emu_phase(const Geometry& g, const double* X, const double* dY, double* buc
                     double w[RR], o[A];
                     for (int i = 0; i < RR; ++i) {
                         const int kk = k0 + k, col = w0 + i;
-                        w[i] = (kk < g.K && col < g.Wo) ? dY[(((size_t)n * g.Ho + h) * g.Wo + col) * g.K + kk] : 0.0;
+                        w[i] = (kk < g.K && col < g.Wo) ? dY[(((size_t)n * g.Ho + h) * g.Wo + col) * g.ldy + kk] : 0.0;
                     }
                     WT::ft(w, o);
                     for (int x = 0; x < A; ++x) gt[(size_t)x * BN + k] = o[x];

@@ -39,6 +39,7 @@ struct KernelId {
 // Everything a launch needs; passed by value to the kernels (< 4 KB).
 struct Geometry {
     int N, C, H, W, K, R, S, pad, Ho, Wo;
+    int ldy;                    // dY pixel stride in elements (>= K; K-sharding passes a channel slice)
     // Omega_a0 region
     int a0, n0, r0, k0;
     int seg_h, bands, seg_w, seg_cols;

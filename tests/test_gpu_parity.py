@@ -182,3 +182,24 @@ def test_full_size_sampled_f16(layer):
     err = O.rel_max_err(got.ravel()[idx], ref)
     assert err <= TOL[layer.dtype], (layer.name, p, err)
     assert np.isfinite(got).all()
+
+
+# ============================================================== K-sharding (strided dY)
+@pytest.mark.parametrize("layer", [wl.LAYERS["r50_c128_28_f32"].with_(N=2, K=136, name="ks32"),
+                                   wl.LAYERS["r50_c128_28_f16"].with_(N=2, K=200, name="ks16")],
+                         ids=lambda l: l.name)
+@pytest.mark.parametrize("world", [2, 3])
+def test_k_sharded_slices_concatenate_to_oracle(layer, world):
+    """Each rank's dW slice (channel slice of dY read in place, ldy = K) —
+    concatenated along K — equals the full-batch oracle; no communication."""
+    X, dY = wl.make_inputs(layer)
+    Xg, Gg = torch.from_numpy(X).cuda(), torch.from_numpy(dY).cuda()
+    parts = []
+    for r in range(world):
+        dW, k0, k1 = W.bfc_k_sharded(Xg, Gg, layer.R, layer.S, layer.pad, layer.dtype, r, world)
+        parts.append((k0, dW))
+    torch.cuda.synchronize()
+    assert [k0 for k0, _ in parts] == sorted(k0 for k0, _ in parts)
+    got = torch.cat([d for _, d in parts], dim=0).cpu().numpy()
+    ref = O.bfc_c(X, dY, layer.R, layer.S, layer.pad)
+    assert O.rel_max_err(got, ref) <= TOL[layer.dtype]

@@ -142,3 +142,15 @@ def test_forced_overrides(monkeypatch):
     monkeypatch.setenv("WINRS_FORCE_PAIR", "8,3,6,0,0,0")
     p = W.plan_for_device(8, 64, 56, 56, 64, 3, 3, 1, "f32")
     assert p.info["alpha1"] == 0 and p.info["k0"] == 10 and p.info["masked_cols"] == 4
+
+
+def test_strided_entry_validates_ldy():
+    """winrs_bfc_strided rejects ldy < K or misaligned ldy before any launch."""
+    from paper_conf_icpp_zhangc0zx0025_b200 import _lib
+    p = W.plan_for_device(2, 16, 8, 8, 16, 3, 3, 1, "f32")
+    L = _lib.lib()
+    fake = 1 << 20   # 16-byte aligned dummy addresses: rejected before use
+    assert L.winrs_bfc_strided(p.handle, fake, fake, 8, fake, None, None) == 1     # ldy < K
+    assert L.winrs_bfc_strided(p.handle, fake, fake, 18, fake, None, None) == 1    # ldy % 4
+    p16 = W.plan_for_device(2, 16, 8, 8, 16, 3, 3, 1, "f16")
+    assert L.winrs_bfc_strided(p16.handle, fake, fake, 20, fake, None, None) == 1  # ldy % 8
