@@ -146,17 +146,40 @@ def run_winrs(args):
     layers = _workload(args.workload, args.dtype)
     tdt = torch.float32 if args.dtype == "f32" else torch.float16
 
-    # Inputs resident in HBM (seeded, per-rank shard offset), plans prebuilt.
+    # Inputs resident in HBM, plans prebuilt.  dp: each rank has its own
+    # seeded batch shard (weak scaling); kshard: every rank holds the full
+    # batch and computes its slice of the output channels (strong scaling, no
+    # communication: BASELINE's K-sharding alternative).
+    kshard = args.parallel == "kshard" and world > 1
     items = []
     for l in layers:
-        X, dY = wl.make_inputs(l, seed_offset=1000 * rank)
-        p = W.plan(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype)
+        X, dY = wl.make_inputs(l, seed_offset=0 if kshard else 1000 * rank)
+        align = 4 if l.dtype == "f32" else 8
+        if kshard:
+            a, b = W.shard_range(l.K // align, world, rank)
+            k0, k1 = a * align, b * align
+        else:
+            k0, k1 = 0, l.K
+        p = W.plan(l.N, l.C, l.H, l.W, k1 - k0, l.R, l.S, l.pad, l.dtype)
         Xg = torch.from_numpy(X).to(dev)
         Gg = torch.from_numpy(dY).to(dev)
-        dW = torch.empty((l.K, l.R, l.S, l.C), dtype=torch.float32, device=dev)
+        dW = torch.empty((k1 - k0, l.R, l.S, l.C), dtype=torch.float32, device=dev)
         ws = torch.empty(max(p.workspace_bytes, 16), dtype=torch.uint8, device=dev)
         items.append(dict(layer=l, plan=p, X=Xg, dY=Gg, dW=dW, ws=ws, Xh=torch.from_numpy(X).pin_memory(),
-                          Gh=torch.from_numpy(dY).pin_memory(), dWh=torch.empty(dW.shape).pin_memory()))
+                          Gh=torch.from_numpy(dY).pin_memory(), dWh=torch.empty(dW.shape).pin_memory(),
+                          k0=k0, k1=k1, flops=l.direct_flops * (k1 - k0) / l.K))
+
+    def run_bfc(it, stream):
+        if kshard:   # channel slice of dY read in place (ldy = K), no communication
+            from paper_conf_icpp_zhangc0zx0025_b200 import _lib
+            _lib.check(_lib.lib().winrs_bfc_strided(it["plan"].handle, it["X"].data_ptr(),
+                                                    it["dY"].data_ptr() + it["k0"] * it["dY"].element_size(),
+                                                    it["layer"].K, it["dW"].data_ptr(), it["ws"].data_ptr(),
+                                                    stream.cuda_stream), "winrs_bfc_strided")
+        else:
+            W.bfc(it["plan"], it["X"], it["dY"], it["dW"], it["ws"], stream)
+            if world > 1:
+                dist.all_reduce(it["dW"])
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream(dev)
 
@@ -165,9 +188,7 @@ def run_winrs(args):
             flush.fill_(j & 0xFF)                                  # evict L2 (outside the events)
             if timed_events is not None:
                 timed_events[j][0].record(stream)
-            W.bfc(it["plan"], it["X"], it["dY"], it["dW"], it["ws"], stream)
-            if world > 1:
-                dist.all_reduce(it["dW"])
+            run_bfc(it, stream)
             if timed_events is not None:
                 timed_events[j][1].record(stream)
 
@@ -209,7 +230,10 @@ def run_winrs(args):
     for _ in range(max(3, args.steps)):
         flush.fill_(1)
         e0.record(stream)
-        W.bfc(p, it["X"], it["dY"], it["dW"], it["ws"], stream)
+        if kshard:
+            run_bfc(it, stream)
+        else:
+            W.bfc(p, it["X"], it["dY"], it["dW"], it["ws"], stream)
         e1.record(stream)
         torch.cuda.synchronize()
         kt.append(e0.elapsed_time(e1))
@@ -224,7 +248,15 @@ def run_winrs(args):
             dX = torch.empty_like(it2["X"])
             dG = torch.empty_like(it2["dY"])
             a.record(stream)
-            W.bfc_host(it2["plan"], it2["Xh"], it2["Gh"], it2["dWh"], dX, dG, it2["dW"], it2["ws"], stream)
+            if kshard or world > 1:   # H2D, the BFC (+ all_reduce for dp), D2H of (this rank's) dW
+                dX.copy_(it2["Xh"], non_blocking=True)
+                dG.copy_(it2["Gh"], non_blocking=True)
+                it3 = dict(it2, X=dX, dY=dG)
+                run_bfc(it3, stream)
+                it2["dWh"].copy_(it2["dW"], non_blocking=True)
+                stream.synchronize()
+            else:
+                W.bfc_host(it2["plan"], it2["Xh"], it2["Gh"], it2["dWh"], dX, dG, it2["dW"], it2["ws"], stream)
             b.record(stream)
             torch.cuda.synchronize()
             tot += a.elapsed_time(b)
@@ -236,7 +268,7 @@ def run_winrs(args):
         e2e = float(t.item())
 
     if rank == 0:
-        flops = sum(it["layer"].direct_flops for it in items) * world
+        flops = sum(it["layer"].direct_flops for it in items) * (1 if kshard else world)
         value = flops / (step_ms * 1e-3) / 1e12
         peaks, src = _peaks()
         esz = 4 if args.dtype == "f32" else 2
@@ -265,7 +297,7 @@ def run_winrs(args):
         roof["kernel_ms"] = dom_ms
         h2d = sum(it2["X"].numel() * it2["X"].element_size() + it2["dY"].numel() * it2["dY"].element_size()
                   for it2 in items)
-        d2h = sum(it2["dW"].numel() * 4 for it2 in items)
+        d2h = sum(it2["dW"].numel() * 4 for it2 in items)   # this rank's dW (slice under kshard)
         out = {
             "metric": METRIC,
             "value": value,
@@ -275,12 +307,13 @@ def run_winrs(args):
             "warmup": args.warmup,
             "ms_per_step": step_ms,
             "higher_is_better": True,
-            "scaling": "weak",
+            "scaling": "strong" if kshard else "weak",
             "vs_baseline": None,
             "dtype": args.dtype,
             "data": "synthetic (seeded U[0,1), dY x 1e-2 for f16; PAPER.md P@50685)",
             "config": {"workload": f"{args.workload}_{args.dtype}: " + ", ".join(x["layer"].name for x in items),
-                       "global_batch": layers[0].N * world, "parallelism": f"dp{world}" if world > 1 else "single",
+                       "global_batch": layers[0].N * (1 if kshard else world),
+                       "parallelism": (f"kshard{world}" if kshard else f"dp{world}") if world > 1 else "single",
                        "l2": "flushed (256 MiB write) before every layer call; flush outside timed events",
                        "workspace_cap": float(os.environ.get("WINRS_WS_CAP", "0.04")),
                        "layers": [{"name": x["layer"].name, "ms": per_layer_ms[j],
@@ -370,6 +403,9 @@ def main():
     ap.add_argument("--dtype", default=os.environ.get("WINRS_BENCH_DTYPE", "f16"), choices=["f32", "f16"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
+    ap.add_argument("--parallel", default="dp", choices=["dp", "kshard"],
+                    help="N>1: dp = batch shards + one all_reduce of dW (weak); kshard = output-channel "
+                         "shards of the full batch, no communication (strong)")
     ap.add_argument("--ws-cap", type=float, default=None,
                     help="planner workspace cap as a fraction of X+dY bytes (default: the paper's 4%%)")
     args = ap.parse_args()
