@@ -84,7 +84,8 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
 }  // namespace f16k
 
 #define WINRS_F16_ENTRY(A0, N0, R0, A1, N1, R1, BM)                                                  \
-    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1, 1,            \
+    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1,               \
+     ::winrs::f16k::csplit_fits<N0, BM>() ? 1 : 0,                                                     \
      ::winrs::f16k::smem_total<A0, N0, R0, BM>(), &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1, BM>, \
      "f16tc_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x" #BM}
 
@@ -106,6 +107,13 @@ const KernelEntry* f16_entries(int* n) {
         WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 128),
         WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 64),
         WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 32),
+        // wider widths: F_W multiple of 5, 7, 4, 2
+        WINRS_F16_ENTRY(8, 5, 4, 0, 0, 0, 64),
+        WINRS_F16_ENTRY(8, 7, 2, 0, 0, 0, 64),
+        WINRS_F16_ENTRY(8, 4, 5, 4, 2, 3, 64),
+        WINRS_F16_ENTRY(8, 4, 5, 0, 0, 0, 64),
+        WINRS_F16_ENTRY(4, 2, 3, 0, 0, 0, 128),
+        WINRS_F16_ENTRY(4, 2, 3, 0, 0, 0, 64),
     };
     *n = sizeof(e) / sizeof(e[0]);
     return e;

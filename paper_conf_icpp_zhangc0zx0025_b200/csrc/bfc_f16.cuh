@@ -363,9 +363,13 @@ __device__ __forceinline__ void epilogue(int j_off, bool first, bool empty, uint
 // It overlays the rings (and, when larger, the mbarriers): it is only written
 // after the last job, when all of them are idle.
 template <int BM> __host__ __device__ constexpr int out_ld() { return BM + 4; }
+// The cluster split needs the whole staged output tile in shared memory.
+template <int N0, int BM> __host__ __device__ constexpr bool csplit_fits() {
+    return (size_t)N0 * BN * out_ld<BM>() * 4 <= 227u * 1024u;
+}
 template <int A0, int N0, int R0, int BM> __host__ __device__ constexpr size_t smem_total() {
-    return Smem<A0, R0, BM>::bytes > (size_t)N0 * BN * out_ld<BM>() * 4 ? Smem<A0, R0, BM>::bytes
-                                                                           : (size_t)N0 * BN * out_ld<BM>() * 4;
+    const size_t out = csplit_fits<N0, BM>() ? (size_t)N0 * BN * out_ld<BM>() * 4 : 0;
+    return Smem<A0, R0, BM>::bytes > out ? Smem<A0, R0, BM>::bytes : out;
 }
 
 // ---- final pass (warps 2..5): staged tile -> bucket (no cluster split) or ->
@@ -449,7 +453,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     constexpr int S_RAW = SM::S_RAW;
     constexpr int TX_WARPS = tx_warps<BM>();
     static_assert(A1 * BM <= stash_col<N0, BM>(), "residual accumulators overlap the TMEM output stash");
-    static_assert(N0 * BN * out_ld<BM>() * 4 <= 227 * 1024, "cluster staging tile must fit in shared memory");
+    constexpr bool kCluster = csplit_fits<N0, BM>();
     extern __shared__ __align__(1024) uint8_t smem[];
     const Geometry& g = args.g;
     Barriers* bars = reinterpret_cast<Barriers*>(smem + SM::bar_off);
@@ -636,8 +640,10 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     }
     tc_fence_before();
     __syncthreads();
-    if (g.csplit > 1)
-        cluster_reduce<N0, BM>(g, bucket, cc, fw0, rank, reinterpret_cast<const float*>(smem), nthreads<BM>());
+    if constexpr (kCluster) {
+        if (g.csplit > 1)
+            cluster_reduce<N0, BM>(g, bucket, cc, fw0, rank, reinterpret_cast<const float*>(smem), nthreads<BM>());
+    }
     if (warp == 1) {
         tc_fence_after();
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem_base));

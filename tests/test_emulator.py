@@ -45,3 +45,15 @@ def test_emulated_plan_equals_oracle(case, monkeypatch):
     ref = O.bfc_c(X, dY, R, S, pad)
     got = W.emulate(p, X, dY)
     assert O.rel_max_err(got, ref) < 1e-12, (p, O.rel_max_err(got, ref))
+
+
+@pytest.mark.parametrize("S", [2, 3, 4, 5, 7, 8, 9])
+def test_emulated_f16_plans_equal_oracle(S, monkeypatch):
+    """FP16 plans (tile 128 x B_M, 16-deep chunks, cluster split) emulated in FP64."""
+    monkeypatch.setenv("WINRS_FORCE_CSPLIT", "2")
+    N, C, H, Wd, K, pad = 2, 16, 9, 13, 24, S // 2
+    p = W.plan_for_device(N, C, H, Wd, K, S, S, pad, "f16")
+    g = np.random.default_rng(S)
+    X = g.uniform(-1, 1, (N, H, Wd, C))
+    dY = g.uniform(-1, 1, (N, p.info["Ho"], p.info["Wo"], K))
+    assert O.rel_max_err(W.emulate(p, X, dY), O.bfc_c(X, dY, S, S, pad)) < 1e-12

@@ -203,3 +203,11 @@ def test_k_sharded_slices_concatenate_to_oracle(layer, world):
     got = torch.cat([d for _, d in parts], dim=0).cpu().numpy()
     ref = O.bfc_c(X, dY, layer.R, layer.S, layer.pad)
     assert O.rel_max_err(got, ref) <= TOL[layer.dtype]
+
+
+# ============================================================== FP16 widths 2..9
+@pytest.mark.parametrize("S", [2, 4, 5, 6, 7, 8, 9])
+def test_f16_all_widths(S):
+    layer = wl.LAYERS["wide_r5_f32"].with_(N=2, C=48, K=72, H=20, W=23, R=S, S=S, pad=S // 2, dtype="f16",
+                                           name=f"f16_w{S}")
+    _full_check(layer)
