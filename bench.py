@@ -64,6 +64,8 @@ def _ncu_traffic(dtype: str, layer_name: str):
 def _workload(name: str, dtype: str):
     from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
     if name == "r50":
+        if dtype == "bf16":
+            return [l.with_(dtype="bf16", name=l.name.replace("f16", "bf16")) for l in wl.RESNET50_F16]
         return wl.RESNET50_F32 if dtype == "f32" else wl.RESNET50_F16
     if name == "vgg":
         return wl.VGG16_F16
@@ -161,12 +163,15 @@ def run_winrs(args):
         else:
             k0, k1 = 0, l.K
         p = W.plan(l.N, l.C, l.H, l.W, k1 - k0, l.R, l.S, l.pad, l.dtype)
-        Xg = torch.from_numpy(X).to(dev)
-        Gg = torch.from_numpy(dY).to(dev)
+        Xt, Gt = torch.from_numpy(X), torch.from_numpy(dY)
+        if l.dtype == "bf16":   # workloads carries bf16 values in float32
+            Xt, Gt = Xt.to(torch.bfloat16), Gt.to(torch.bfloat16)
+        Xg = Xt.to(dev)
+        Gg = Gt.to(dev)
         dW = torch.empty((k1 - k0, l.R, l.S, l.C), dtype=torch.float32, device=dev)
         ws = torch.empty(max(p.workspace_bytes, 16), dtype=torch.uint8, device=dev)
-        items.append(dict(layer=l, plan=p, X=Xg, dY=Gg, dW=dW, ws=ws, Xh=torch.from_numpy(X).pin_memory(),
-                          Gh=torch.from_numpy(dY).pin_memory(), dWh=torch.empty(dW.shape).pin_memory(),
+        items.append(dict(layer=l, plan=p, X=Xg, dY=Gg, dW=dW, ws=ws, Xh=Xt.pin_memory(),
+                          Gh=Gt.pin_memory(), dWh=torch.empty(dW.shape).pin_memory(),
                           k0=k0, k1=k1, flops=l.direct_flops * (k1 - k0) / l.K))
 
     def run_bfc(it, stream):
@@ -271,7 +276,7 @@ def run_winrs(args):
         flops = sum(it["layer"].direct_flops for it in items) * (1 if kshard else world)
         value = flops / (step_ms * 1e-3) / 1e12
         peaks, src = _peaks()
-        esz = 4 if args.dtype == "f32" else 2
+        esz = 4 if args.dtype == "f32" else 2   # f16 / bf16
         l = it["layer"]
         alg_bytes = esz * (l.N * l.H * l.W * l.C + l.N * l.Ho * l.Wo * l.K) + 4 * l.K * l.R * l.S * l.C * (
             1 if info["Z"] == 1 else 2 * info["Z"] + 1)
@@ -400,7 +405,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="winrs", choices=["winrs", "reference"])
     ap.add_argument("--workload", default="r50", choices=["r50", "vgg", "wide", "r50l3"])
-    ap.add_argument("--dtype", default=os.environ.get("WINRS_BENCH_DTYPE", "f16"), choices=["f32", "f16"])
+    ap.add_argument("--dtype", default=os.environ.get("WINRS_BENCH_DTYPE", "f16"), choices=["f32", "f16", "bf16"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
     ap.add_argument("--parallel", default="dp", choices=["dp", "kshard"],

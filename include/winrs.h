@@ -15,7 +15,8 @@
  *
  * Layouts (Table 1): X is NHWC [N][H][W][C]; dY is NHWC [N][Ho][Wo][K]; dW is
  * KRSC [K][R][S][C] and is ALWAYS float32.  X and dY are both float32
- * (WINRS_F32) or both IEEE binary16 (WINRS_F16).  These are exactly the
+ * (WINRS_F32), both IEEE binary16 (WINRS_F16) or both bfloat16 (WINRS_BF16;
+ * the BF16 variant named in the paper's conclusion, P@56336).  These are exactly the
  * physical orders of PyTorch channels_last activations and channels_last
  * 4-D weights.
  *
@@ -55,7 +56,7 @@
 extern "C" {
 #endif
 
-typedef enum { WINRS_F32 = 0, WINRS_F16 = 1 } winrs_dtype_t;
+typedef enum { WINRS_F32 = 0, WINRS_F16 = 1, WINRS_BF16 = 2 } winrs_dtype_t;
 
 typedef enum {
     WINRS_OK = 0,
@@ -104,7 +105,7 @@ typedef struct {
  * Returns INVALID_ARG for a dimension <= 0, pad < 0, Ho < 1, Wo < 1 or a null
  * `out`; UNSUPPORTED when S has no divisor n in {2..9} of the kernel set
  * (§5 P@28451: F_W in {n*k : 2 <= k <= 9}), when C % 4 or K % 4 != 0
- * (FP32) / C % 8 or K % 8 != 0 (FP16), or when the device is not sm_100.
+ * (FP32) / C % 8 or K % 8 != 0 (FP16, BF16), or when the device is not sm_100.
  * On success *out owns a new plan (free with winrs_plan_destroy). */
 WINRS_API winrs_status_t winrs_plan(int N, int C, int H, int W, int K, int R, int S, int pad,
                           winrs_dtype_t dtype, winrs_plan_t* out);

@@ -51,7 +51,7 @@ class Plan:
 
     @property
     def dtype(self) -> str:
-        return "f32" if self.info["dtype"] == 0 else "f16"
+        return {0: "f32", 1: "f16", 2: "bf16"}[self.info["dtype"]]
 
     def __del__(self):
         h, self._h = getattr(self, "_h", None), None
@@ -103,7 +103,7 @@ def bfc(p: Plan, X, dY, dW=None, workspace=None, stream=None):
     """winrs_bfc on torch CUDA tensors; returns dW [K,R,S,C] float32."""
     import torch
     i = p.info
-    tdt = torch.float32 if p.dtype == "f32" else torch.float16
+    tdt = {"f32": torch.float32, "f16": torch.float16, "bf16": torch.bfloat16}[p.dtype]
     Xn = _as_nhwc(X, i["N"], i["H"], i["W"], i["C"], "X")
     Gn = _as_nhwc(dY, i["N"], i["Ho"], i["Wo"], i["K"], "dY")
     if Xn.dtype != tdt or Gn.dtype != tdt:

@@ -15,7 +15,7 @@ LIB_PATH = os.path.join(_HERE, "libwinrs.so")
 WINRS_OK = 0
 STATUS = {0: "WINRS_OK", 1: "WINRS_ERR_INVALID_ARG", 2: "WINRS_ERR_UNSUPPORTED",
           3: "WINRS_ERR_WORKSPACE", 4: "WINRS_ERR_CUDA", 5: "WINRS_ERR_HOST_ALLOC"}
-DTYPES = {"f32": 0, "f16": 1}
+DTYPES = {"f32": 0, "f16": 1, "bf16": 2}
 
 
 class WinrsError(RuntimeError):

@@ -29,7 +29,7 @@ static EncodeTiledFn encode_fn() {
 // 4-D NHWC fp16 tensor [N][H][W][Ch] (pixel stride ld >= Ch elements) as TMA
 // dims {Ch, W, H, N}; box {bc, bw, 1, bn}.  Out-of-bounds elements are zero.
 static bool make_map(CUtensorMap* m, const void* base, int N, int H, int W, int Ch, int bc, int bw, int bn,
-                     int ld = 0) {
+                     int ld, bool bf) {
     EncodeTiledFn fn = encode_fn();
     if (!fn) return false;
     if (ld <= 0) ld = Ch;
@@ -37,7 +37,7 @@ static bool make_map(CUtensorMap* m, const void* base, int N, int H, int W, int 
     const cuuint64_t strides[3] = {(cuuint64_t)ld * 2, (cuuint64_t)W * ld * 2, (cuuint64_t)H * W * ld * 2};
     const cuuint32_t box[4] = {(cuuint32_t)bc, (cuuint32_t)bw, 1u, (cuuint32_t)bn};
     const cuuint32_t es[4] = {1u, 1u, 1u, 1u};
-    return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
+    return fn(m, bf ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
@@ -48,10 +48,10 @@ static int images_per_box(int N) {
     return 1;
 }
 
-template <int A0, int N0, int R0, int A1, int N1, int R1, int BM>
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BM, bool BF>
 cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
     static std::atomic<unsigned long long> done{0};
-    auto k = bfc_f16_kernel<A0, N0, R0, A1, N1, R1, BM>;
+    auto k = bfc_f16_kernel<A0, N0, R0, A1, N1, R1, BM, BF>;
     constexpr size_t sm = smem_total<A0, N0, R0, BM>();
     cudaError_t e = ensure_smem_attr(k, sm, done);
     if (e != cudaSuccess) return e;
@@ -63,12 +63,12 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
     a.ws = ws;
     a.nb = images_per_box(g.N);
     CUtensorMap mX0, mY0, mX1, mY1;
-    if (!make_map(&mX0, X, g.N, g.H, g.W, g.C, BM, A0, a.nb) ||
-        !make_map(&mY0, dY, g.N, g.Ho, g.Wo, g.K, BN, R0, a.nb, g.ldy))
+    if (!make_map(&mX0, X, g.N, g.H, g.W, g.C, BM, A0, a.nb, 0, BF) ||
+        !make_map(&mY0, dY, g.N, g.Ho, g.Wo, g.K, BN, R0, a.nb, g.ldy, BF))
         return cudaErrorInvalidValue;
     if (A1 != 0) {
-        if (!make_map(&mX1, X, g.N, g.H, g.W, g.C, BM, A1 ? A1 : A0, a.nb) ||
-            !make_map(&mY1, dY, g.N, g.Ho, g.Wo, g.K, BN, R1 ? R1 : R0, a.nb, g.ldy))
+        if (!make_map(&mX1, X, g.N, g.H, g.W, g.C, BM, A1 ? A1 : A0, a.nb, 0, BF) ||
+            !make_map(&mY1, dY, g.N, g.Ho, g.Wo, g.K, BN, R1 ? R1 : R0, a.nb, g.ldy, BF))
             return cudaErrorInvalidValue;
     } else {
         mX1 = mX0;
@@ -83,11 +83,13 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
 
 }  // namespace f16k
 
-#define WINRS_F16_ENTRY(A0, N0, R0, A1, N1, R1, BM)                                                  \
-    {1, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1,               \
-     ::winrs::f16k::csplit_fits<N0, BM>() ? 1 : 0,                                                     \
-     ::winrs::f16k::smem_total<A0, N0, R0, BM>(), &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1, BM>, \
-     "f16tc_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x" #BM}
+#define WINRS_TC_ENTRY(DT, BF, PFX, A0, N0, R0, A1, N1, R1, BM)                                     \
+    {DT, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1,              \
+     ::winrs::f16k::csplit_fits<N0, BM>() ? 1 : 0, ::winrs::f16k::smem_total<A0, N0, R0, BM>(),       \
+     &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1, BM, BF>,                                          \
+     PFX "_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x" #BM}
+#define WINRS_F16_ENTRY(...) WINRS_TC_ENTRY(1, false, "f16tc", __VA_ARGS__)
+#define WINRS_BF16_ENTRY(...) WINRS_TC_ENTRY(2, true, "bf16tc", __VA_ARGS__)
 
 #ifdef WINRS_TRACE
 extern "C" __attribute__((visibility("default"))) int winrs_trace_read(unsigned long long* out) {
@@ -114,6 +116,16 @@ const KernelEntry* f16_entries(int* n) {
         WINRS_F16_ENTRY(8, 4, 5, 0, 0, 0, 64),
         WINRS_F16_ENTRY(4, 2, 3, 0, 0, 0, 128),
         WINRS_F16_ENTRY(4, 2, 3, 0, 0, 0, 64),
+        // BF16 inputs: the same kernels with bf16 operands
+        WINRS_BF16_ENTRY(8, 3, 6, 4, 3, 2, 64),
+        WINRS_BF16_ENTRY(8, 3, 6, 4, 3, 2, 32),
+        WINRS_BF16_ENTRY(8, 3, 6, 0, 0, 0, 64),
+        WINRS_BF16_ENTRY(4, 3, 2, 0, 0, 0, 128),
+        WINRS_BF16_ENTRY(4, 3, 2, 0, 0, 0, 64),
+        WINRS_BF16_ENTRY(8, 5, 4, 0, 0, 0, 64),
+        WINRS_BF16_ENTRY(8, 7, 2, 0, 0, 0, 64),
+        WINRS_BF16_ENTRY(8, 4, 5, 4, 2, 3, 64),
+        WINRS_BF16_ENTRY(4, 2, 3, 0, 0, 0, 128),
     };
     *n = sizeof(e) / sizeof(e[0]);
     return e;

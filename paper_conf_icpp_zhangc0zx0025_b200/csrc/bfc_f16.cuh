@@ -1,4 +1,4 @@
-// FP16-in / FP32-accumulate tensor-core fused WinRS BFC kernel for sm_100a
+// FP16- (or BF16-) in / FP32-accumulate tensor-core fused WinRS BFC kernel for sm_100a
 // (tcgen05 + TMEM + TMA + mbarrier, warp-specialised).
 //
 // PAPER.md §5 (P@28371-39921) ported FP16 kernels run the alpha-batched GEMM
@@ -27,6 +27,7 @@
 // column segment only), adding into the same bucket (R10).
 #pragma once
 #include <cuda.h>
+#include <cuda_bf16.h>
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -104,15 +105,19 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
            ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46);
 }
 // kind::f16 instruction descriptor: D f32, A/B f16, both K-major, M = 128, N = BM.
-template <int BM>
-__host__ __device__ constexpr uint32_t idesc() { return (1u << 4) | ((uint32_t)(BM >> 3) << 17) | ((uint32_t)(BN >> 4) << 24); }
+// A/B format field (bits 7-9, 10-12): 0 = F16, 1 = BF16.
+template <int BM, bool BF>
+__host__ __device__ constexpr uint32_t idesc() {
+    return (1u << 4) | ((BF ? 1u : 0u) << 7) | ((BF ? 1u : 0u) << 10) | ((uint32_t)(BM >> 3) << 17) |
+           ((uint32_t)(BN >> 4) << 24);
+}
 
-template <int BM>
+template <int BM, bool BF>
 __device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accumulate) {
     asm volatile(
         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
-        :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(idesc<BM>()), "r"(accumulate));
+        :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(idesc<BM, BF>()), "r"(accumulate));
 }
 __device__ __forceinline__ void umma_commit(uint64_t* bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
@@ -128,10 +133,28 @@ __device__ __forceinline__ void tmem_ld8(uint32_t taddr, float* v) {
 }
 __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 
-__device__ __forceinline__ uint32_t pack_h2(float lo, float hi) {
-    __half2 h = __floats2half2_rn(lo, hi);   // cvt.rn.f16x2.f32
-    return *reinterpret_cast<uint32_t*>(&h);
-}
+// 16-bit element traits: FP16 (IEEE binary16) or BF16 inputs / operands.
+template <bool BF> struct Elem;
+template <> struct Elem<false> {
+    __device__ static __forceinline__ float2 unpack(uint32_t w) {
+        return __half22float2(*reinterpret_cast<const __half2*>(&w));
+    }
+    __device__ static __forceinline__ uint32_t pack(float lo, float hi) {   // cvt.rn.f16x2.f32
+        __half2 h = __floats2half2_rn(lo, hi);
+        return *reinterpret_cast<uint32_t*>(&h);
+    }
+};
+template <> struct Elem<true> {
+    __device__ static __forceinline__ float2 unpack(uint32_t w) {
+        return __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&w));
+    }
+    __device__ static __forceinline__ uint32_t pack(float lo, float hi) {   // cvt.rn.bf16x2.f32
+        __nv_bfloat162 h = __floats2bfloat162_rn(lo, hi);
+        return *reinterpret_cast<uint32_t*>(&h);
+    }
+};
+
+__device__ __forceinline__ uint32_t pack_h2(float lo, float hi) { return Elem<false>::pack(lo, hi); }
 __device__ __forceinline__ F2 ld_h2(const __half* p) {
     const __half2 h = *reinterpret_cast<const __half2*>(p);
     const float2 f = __half22float2(h);
@@ -222,8 +245,8 @@ constexpr int DQ_IT = 8;                 // depth entries per IT unit (an octet)
 template <int BM> __host__ __device__ constexpr int ft_warps() { return (BN / 2) * (KC / DQ_FT) / 32; }
 template <int BM> __host__ __device__ constexpr int it_warps() { return (BM / 2) * (KC / DQ_IT) / 32; }
 
-template <int WT_FN, int A, int NN, int RR, int NIN, int DQ>
-__device__ __forceinline__ void unit_transform(const __half* src, int tap_stride, int depth_stride, uint8_t* dst0,
+template <int WT_FN, int A, int NN, int RR, int NIN, int DQ, bool BF>
+__device__ __forceinline__ void unit_transform(const uint16_t* src, int tap_stride, int depth_stride, uint8_t* dst0,
                                                int slab_bytes, int p, int grp) {
     using WT = Wino<A, NN, RR>;
     const int oct = grp;     // depth group index (DQ entries each)
@@ -231,20 +254,20 @@ __device__ __forceinline__ void unit_transform(const __half* src, int tap_stride
 #pragma unroll
     for (int j = 0; j < DQ / 2; ++j) {
         F2 in0[NIN], in1[NIN], o[A];
-        const __half* s0 = src + (oct * DQ + 2 * j) * depth_stride + 2 * p;
+        const uint16_t* s0 = src + (oct * DQ + 2 * j) * depth_stride + 2 * p;
 #pragma unroll
         for (int i = 0; i < NIN; ++i) {
-            const float2 a = __half22float2(*reinterpret_cast<const __half2*>(s0 + i * tap_stride));
-            const float2 b = __half22float2(*reinterpret_cast<const __half2*>(s0 + depth_stride + i * tap_stride));
+            const float2 a = Elem<BF>::unpack(*reinterpret_cast<const uint32_t*>(s0 + i * tap_stride));
+            const float2 b = Elem<BF>::unpack(*reinterpret_cast<const uint32_t*>(s0 + depth_stride + i * tap_stride));
             in0[i] = F2{a.x, b.x};    // row 2p,   depth 2j, 2j+1
             in1[i] = F2{a.y, b.y};    // row 2p+1, depth 2j, 2j+1
         }
         if (WT_FN == 0) WT::ft(in0, o); else WT::it(in0, o);
 #pragma unroll
-        for (int x = 0; x < A; ++x) pk[x][0][j] = pack_h2(o[x].x, o[x].y);
+        for (int x = 0; x < A; ++x) pk[x][0][j] = Elem<BF>::pack(o[x].x, o[x].y);
         if (WT_FN == 0) WT::ft(in1, o); else WT::it(in1, o);
 #pragma unroll
-        for (int x = 0; x < A; ++x) pk[x][1][j] = pack_h2(o[x].x, o[x].y);
+        for (int x = 0; x < A; ++x) pk[x][1][j] = Elem<BF>::pack(o[x].x, o[x].y);
     }
     // depth group -> K position kk0 = grp*DQ: K half kk0/8, byte offset (kk0%8)*2 in the 16-byte row
     const int kk0 = grp * DQ;
@@ -280,22 +303,22 @@ __device__ __forceinline__ int tx_role(int tw) {
     return tx_is_it<BM>(tw) ? before : -1 - (tw - before);
 }
 
-template <int A, int NN, int RR, int BM>
+template <int A, int NN, int RR, int BM, bool BF>
 __device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tw, int lane) {
     constexpr int RAW_Y = KC * RR * BN * 2;
-    const __half* rawY = reinterpret_cast<const __half*>(raw);            // [KC][RR][BN]
-    const __half* rawX = reinterpret_cast<const __half*>(raw + RAW_Y);    // [KC][A][BM]
+    const uint16_t* rawY = reinterpret_cast<const uint16_t*>(raw);            // [KC][RR][BN]
+    const uint16_t* rawX = reinterpret_cast<const uint16_t*>(raw + RAW_Y);    // [KC][A][BM]
     constexpr int OPA = BN * KC * 2, OPB = BM * KC * 2;
     const int role = tx_role<BM>(tw);
     if (role < 0) {
         const int f = -1 - role;   // FT warp: 32 k pairs x one octet
-        unit_transform<0, A, NN, RR, RR, DQ_FT>(rawY, BN, RR * BN, op, OPA, (f % (BN / 64)) * 32 + lane,
+        unit_transform<0, A, NN, RR, RR, DQ_FT, BF>(rawY, BN, RR * BN, op, OPA, (f % (BN / 64)) * 32 + lane,
                                                 f / (BN / 64));
     } else {                       // IT warp: 32 c pairs (or BM/2 pairs x 32/(BM/2) quads) x quads
         constexpr int PW = BM / 2 < 32 ? BM / 2 : 32;
         const int q = (role % ((BM / 2) / PW)) * PW + (lane % PW);
         const int quad = role / ((BM / 2) / PW) * (32 / PW) + lane / PW;
-        unit_transform<1, A, NN, RR, A, DQ_IT>(rawX, BM, A * BM, op + A * OPA, OPB, q, quad);
+        unit_transform<1, A, NN, RR, A, DQ_IT, BF>(rawX, BM, A * BM, op + A * OPA, OPB, q, quad);
     }
 }
 
@@ -444,7 +467,7 @@ __device__ __forceinline__ void cluster_reduce(const Geometry& g, float* bucket,
     asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
-template <int A0, int N0, int R0, int A1, int N1, int R1, int BM>
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BM, bool BF>
 __global__ void __launch_bounds__(nthreads<BM>(), 1)
 bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX0,
                const __grid_constant__ CUtensorMap tmY0, const __grid_constant__ CUtensorMap tmX1,
@@ -569,7 +592,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                         const uint64_t ad = umma_desc(base + x * SM::OPA, 128, 256);
                         const uint64_t bd = umma_desc(base + Aj * SM::OPA + x * SM::OPB, 128, 256);
 #ifndef WINRS_NO_MMA
-                        umma_f16<BM>(tmem_base + (uint32_t)(x * BM), ad, bd, ch > c_lo ? 1u : 0u);
+                        umma_f16<BM, BF>(tmem_base + (uint32_t)(x * BM), ad, bd, ch > c_lo ? 1u : 0u);
 #else
                         (void)ad; (void)bd;
 #endif
@@ -598,8 +621,8 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 2);
                 const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
                 uint8_t* op = smem + SM::op_off + so * SM::OP;
-                if (J.phase == 0) transform_chunk<A0, N0, R0, BM>(raw, op, tw, lane);
-                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM>(raw, op, tw, lane);
+                if (J.phase == 0) transform_chunk<A0, N0, R0, BM, BF>(raw, op, tw, lane);
+                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM, BF>(raw, op, tw, lane);
                 if (threadIdx.x == 64) TRACE(3, ch - c_lo + jb * 64, 0);
                 if (threadIdx.x == 64 + 32 * 2) TRACE(3, ch - c_lo + jb * 64, 1);   // an IT warp
                 fence_proxy_async();

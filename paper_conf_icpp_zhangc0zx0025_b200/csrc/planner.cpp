@@ -214,7 +214,7 @@ struct TimeModel {
 };
 
 static TimeModel time_model(int dtype, int bn, int bm) {
-    if (dtype == 1) return {bm >= 128 ? 1.2e12 : (bm >= 64 ? 1.4e12 : 0.8e12), 4e-6};
+    if (dtype != 0) return {bm >= 128 ? 1.2e12 : (bm >= 64 ? 1.4e12 : 0.8e12), 4e-6};
     const int area = bn * bm;
     return {area >= 4096 ? 0.20e12 : (area >= 2048 ? 0.16e12 : 0.11e12), 8e-6};
 }

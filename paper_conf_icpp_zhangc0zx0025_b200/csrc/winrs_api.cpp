@@ -27,7 +27,7 @@ static winrs_status_t build_plan(int N, int C, int H, int W, int K, int R, int S
     *out = nullptr;
     if (N <= 0 || C <= 0 || H <= 0 || W <= 0 || K <= 0 || R <= 0 || S <= 0 || pad < 0)
         return WINRS_ERR_INVALID_ARG;
-    if (dtype != WINRS_F32 && dtype != WINRS_F16) return WINRS_ERR_INVALID_ARG;
+    if (dtype != WINRS_F32 && dtype != WINRS_F16 && dtype != WINRS_BF16) return WINRS_ERR_INVALID_ARG;
     const int Ho = H + 2 * pad - R + 1, Wo = W + 2 * pad - S + 1;
     if (Ho < 1 || Wo < 1) return WINRS_ERR_INVALID_ARG;
     if (!dev || dev->num_sms <= 0) return WINRS_ERR_INVALID_ARG;

@@ -24,7 +24,7 @@ class Layer:
     R: int
     S: int
     pad: int
-    dtype: str          # "f32" or "f16": dtype of X and dY (dW is always f32)
+    dtype: str          # "f32", "f16" or "bf16": dtype of X and dY (dW is always f32)
     index: int          # stable config index: seeds are 1000003+index / 2000003+index
 
     @property
@@ -81,7 +81,15 @@ WIDE_F32 = [l for n, l in LAYERS.items() if n.startswith("wide_")]
 
 
 def np_dtype(dtype: str):
-    return {"f32": np.float32, "f16": np.float16}[dtype]
+    """numpy storage dtype of the inputs (bf16 values are carried in float32)."""
+    return {"f32": np.float32, "f16": np.float16, "bf16": np.float32}[dtype]
+
+
+def round_to_bf16(x: np.ndarray) -> np.ndarray:
+    """float32 -> nearest bfloat16 value (round to nearest even), kept in float32."""
+    b = np.ascontiguousarray(x, dtype=np.float32).view(np.uint32)
+    b = (b + np.uint32(0x7FFF) + ((b >> np.uint32(16)) & np.uint32(1))) & np.uint32(0xFFFF0000)
+    return b.view(np.float32)
 
 
 def make_inputs(layer: Layer, dist: str = "u01", seed_offset: int = 0):
@@ -100,8 +108,10 @@ def make_inputs(layer: Layer, dist: str = "u01", seed_offset: int = 0):
         dY = dY * 2 - 1
     elif dist != "u01":
         raise ValueError(dist)
-    if layer.dtype == "f16":
+    if layer.dtype in ("f16", "bf16"):
         dY = dY * np.float32(1e-2)
+    if layer.dtype == "bf16":
+        return round_to_bf16(X), round_to_bf16(dY)
     dt = np_dtype(layer.dtype)
     return X.astype(dt), dY.astype(dt)
 

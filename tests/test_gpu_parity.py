@@ -15,7 +15,12 @@ from oracle import oracle as O
 
 pytestmark = pytest.mark.gpu
 
-TOL = {"f32": 1e-4, "f16": 2e-2}
+TOL = {"f32": 1e-4, "f16": 2e-2, "bf16": 2e-2}
+
+
+def _dev(a, dtype):
+    t = torch.from_numpy(a).cuda()
+    return t.to(torch.bfloat16) if dtype == "bf16" else t
 
 
 def _run(layer, X, dY, env=None, monkeypatch=None):
@@ -23,8 +28,8 @@ def _run(layer, X, dY, env=None, monkeypatch=None):
         for k, v in env.items():
             monkeypatch.setenv(k, v)
     p = W.plan(layer.N, layer.C, layer.H, layer.W, layer.K, layer.R, layer.S, layer.pad, layer.dtype)
-    Xg = torch.from_numpy(X).cuda()
-    Gg = torch.from_numpy(dY).cuda()
+    Xg = _dev(X, layer.dtype)
+    Gg = _dev(dY, layer.dtype)
     dW = W.bfc(p, Xg, Gg)
     torch.cuda.synchronize()
     return p, dW.cpu().numpy().astype(np.float64)
@@ -211,3 +216,28 @@ def test_f16_all_widths(S):
     layer = wl.LAYERS["wide_r5_f32"].with_(N=2, C=48, K=72, H=20, W=23, R=S, S=S, pad=S // 2, dtype="f16",
                                            name=f"f16_w{S}")
     _full_check(layer)
+
+
+# ============================================================== BF16 tensor-core variant
+REDUCED_BF16 = [l.with_(dtype="bf16", name=l.name.replace("f16", "bf16")) for l in REDUCED_F16[:4]]
+
+
+@pytest.mark.parametrize("layer", REDUCED_BF16, ids=lambda l: l.name)
+def test_reduced_bf16(layer):
+    _full_check(layer)
+
+
+@pytest.mark.parametrize("S", [2, 5, 7])
+def test_bf16_widths(S):
+    layer = wl.LAYERS["wide_r5_f32"].with_(N=2, C=48, K=72, H=20, W=23, R=S, S=S, pad=S // 2, dtype="bf16",
+                                           name=f"bf16_w{S}")
+    _full_check(layer)
+
+
+def test_bf16_full_size_sampled():
+    layer = wl.LAYERS["r50_c256_14_f16"].with_(dtype="bf16", name="r50_c256_14_bf16")
+    X, dY = wl.make_inputs(layer)
+    p, got = _run(layer, X, dY)
+    idx = wl.sample_indices(layer, 256)
+    ref = O.bfc_c_sampled(X, dY, layer.R, layer.S, layer.pad, idx)
+    assert O.rel_max_err(got.ravel()[idx], ref) <= TOL["bf16"]
