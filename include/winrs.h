@@ -62,7 +62,8 @@ typedef enum {
     WINRS_OK = 0,
     WINRS_ERR_INVALID_ARG = 1,   /* bad dimension, null/unaligned pointer      */
     WINRS_ERR_UNSUPPORTED = 2,   /* no kernel for S/dtype, channel alignment,
-                                    or the device is not sm_100                */
+                                    N*Ho*Wo >= 2^31, or the device is not
+                                    sm_100                                     */
     WINRS_ERR_WORKSPACE = 3,     /* workspace == NULL but workspace_bytes > 0  */
     WINRS_ERR_CUDA = 4,          /* a CUDA launch/runtime error                */
     WINRS_ERR_HOST_ALLOC = 5     /* host allocation of the plan failed         */

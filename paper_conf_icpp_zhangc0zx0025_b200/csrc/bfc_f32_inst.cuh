@@ -19,10 +19,10 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
     const long long grid = num_ctas(g);
     if (grid <= 0) return cudaSuccess;
     if (g.csplit <= 1) {
-        k<<<(unsigned)grid, NT, sm, stream>>>(g, static_cast<const float*>(X), static_cast<const float*>(dY), dW, ws);
+        k<<<(unsigned)grid, NTOT, sm, stream>>>(g, static_cast<const float*>(X), static_cast<const float*>(dY), dW, ws);
         return cudaGetLastError();
     }
-    return launch_cluster(k, (unsigned)grid, NT, sm, stream, g.csplit, g, static_cast<const float*>(X),
+    return launch_cluster(k, (unsigned)grid, NTOT, sm, stream, g.csplit, g, static_cast<const float*>(X),
                           static_cast<const float*>(dY), dW, ws);
 }
 
@@ -30,7 +30,7 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
 }  // namespace winrs
 
 #define WINRS_F32_ENTRY(A0, N0, R0, A1, N1, R1, BN, BM)                                         \
-    {0, A0, N0, R0, A1, N1, R1, BN, BM, ::winrs::f32k::NT, ((BN) * (BM) >= 4096 ? 1 : 2), 1,                                  \
+    {0, A0, N0, R0, A1, N1, R1, BN, BM, ::winrs::f32k::NTOT, 1, 1,                                  \
      ::winrs::f32k::smem_bytes<A0, N0, R0, A1, N1, R1, BN, BM>(),                                \
      &::winrs::f32k::launch<A0, N0, R0, A1, N1, R1, BN, BM>,                                     \
      "f32_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_" #BN "x" #BM}

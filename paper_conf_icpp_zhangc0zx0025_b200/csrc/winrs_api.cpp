@@ -34,6 +34,7 @@ static winrs_status_t build_plan(int N, int C, int H, int W, int K, int R, int S
     if (dev->cc_major != 10 || dev->cc_minor != 0) return WINRS_ERR_UNSUPPORTED;   // sm_100a build
     const int align = dtype == WINRS_F32 ? 4 : 8;                                  // 16-byte vectors
     if (C % align || K % align) return WINRS_ERR_UNSUPPORTED;
+    if ((long long)N * Ho * Wo >= (1LL << 31)) return WINRS_ERR_UNSUPPORTED;   // 32-bit depth index
     Problem p{N, C, H, W, K, R, S, pad, Ho, Wo, (int)dtype};
     PlanResult pr;
     const winrs_status_t st = make_plan(p, dev->num_sms, &pr);

@@ -12,8 +12,10 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_icpp_zhangc0zx0025_b200 as W  # noqa: E402
 from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl  # noqa: E402
 
-layers = [wl.LAYERS[n] for n in sys.argv[1].split(",")] if len(sys.argv) > 1 else \
+layers = [wl.LAYERS[n] for n in sys.argv[1].split(",")] if len(sys.argv) > 1 and sys.argv[1] != "all" else \
     wl.RESNET50_F32 + wl.RESNET50_F16 + wl.WIDE_F32
+# optional second argument: comma-separated forced segment counts Z (default: the planner's)
+zs = [int(z) for z in sys.argv[2].split(",")] if len(sys.argv) > 2 else [None]
 tiles = {"f32": ["64x64", "32x32", "64x32"], "f16": ["128x128", "128x64", "128x32"]}
 pairs = {"f32": [None], "f16": [None, "4,3,2,0,0,0"]}
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
@@ -22,7 +24,12 @@ for l in layers:
     Xg, Gg = torch.from_numpy(X).cuda(), torch.from_numpy(dY).cuda()
     for pair in pairs[l.dtype]:
       for t in tiles[l.dtype]:
+       for z in zs:
         for cs in (1, 2, 4, 8):
+            if z is None:
+                os.environ.pop("WINRS_FORCE_Z", None)
+            else:
+                os.environ["WINRS_FORCE_Z"] = str(z)
             os.environ["WINRS_FORCE_TILE"] = t
             os.environ["WINRS_FORCE_CSPLIT"] = str(cs)
             if pair:
@@ -49,7 +56,8 @@ for l in layers:
                     ts.append(a.elapsed_time(b))
             ms = statistics.median(ts)
             print(json.dumps({"layer": l.name, "pair": p.kernel_name, "tile": t, "csplit": p.info["csplit"], "Z": p.info["Z"],
-                              "ctas": p.info["ctas_main"], "us": round(ms * 1e3, 1),
+                              "ctas": p.info["ctas_main"], "ewm": p.info["ewm_flops"], "us": round(ms * 1e3, 1),
                               "tflops": round(l.direct_flops / ms / 1e9, 1)}), flush=True)
 os.environ.pop("WINRS_FORCE_TILE", None)
 os.environ.pop("WINRS_FORCE_CSPLIT", None)
+os.environ.pop("WINRS_FORCE_Z", None)
