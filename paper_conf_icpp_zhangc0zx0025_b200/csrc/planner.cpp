@@ -47,8 +47,21 @@ static bool parse_force_pair(int out[6]) {
     return sscanf(s, "%d,%d,%d,%d,%d,%d", &out[0], &out[1], &out[2], &out[3], &out[4], &out[5]) == 6;
 }
 
-// Step 1: kernel-pair selection.
-static bool choose_pair(const Problem& p, const KernelEntry* es, int ne, PairChoice* best) {
+// The paper's ordering of pair candidates: least cost, then fewest masked
+// columns, more bulk units, larger alpha0, smaller alpha1.
+static bool pair_better(const PairChoice& cur, bool have, double c, int masked, int k0, const KernelEntry& e) {
+    if (!have) return true;
+    if (c != cur.cost) return c < cur.cost;
+    if (masked != cur.masked) return masked < cur.masked;
+    if (k0 != cur.k0) return k0 > cur.k0;
+    if (e.a0 != cur.proto->a0) return e.a0 > cur.proto->a0;
+    return e.a1 < cur.proto->a1;
+}
+
+// Step 1: kernel-pair selection.  `best` receives the paper's choice; `all`
+// (optional) every valid pair with its own best (k0, k1) split.
+static bool choose_pair(const Problem& p, const KernelEntry* es, int ne, PairChoice* best,
+                        std::vector<PairChoice>* all = nullptr) {
     int forced[6];
     const bool force = parse_force_pair(forced);
     bool found = false;
@@ -64,21 +77,15 @@ static bool choose_pair(const Problem& p, const KernelEntry* es, int ne, PairCho
             continue;
         if (p.S % e.n0 != 0) continue;                       // criterion (1)
         if (e.a1 && (p.S % e.n1 != 0 || e.n0 % e.n1 != 0)) continue;
+        PairChoice local;
+        bool lfound = false;
         auto consider = [&](int k0, int k1, int masked) {
             const double c = k0 * (double)e.a0 * (p.S / e.n0) / tau(e.a0, e.n0, e.r0) +
                              (e.a1 ? k1 * (double)e.a1 * (p.S / e.n1) / tau(e.a1, e.n1, e.r1) : 0.0);
-            bool better = !found;
-            if (!better) {
-                if (c != best->cost) better = c < best->cost;
-                else if (masked != best->masked) better = masked < best->masked;
-                else if (k0 != best->k0) better = k0 > best->k0;
-                else if (e.a0 != best->proto->a0) better = e.a0 > best->proto->a0;
-                else better = e.a1 < best->proto->a1;
-            }
-            if (better) {
-                best->proto = &e;
-                best->k0 = k0; best->k1 = k1; best->masked = masked; best->cost = c;
-                found = true;
+            if (pair_better(local, lfound, c, masked, k0, e)) {
+                local.proto = &e;
+                local.k0 = k0; local.k1 = k1; local.masked = masked; local.cost = c;
+                lfound = true;
             }
         };
         if (e.a1 == 0) {
@@ -92,6 +99,12 @@ static bool choose_pair(const Problem& p, const KernelEntry* es, int ne, PairCho
                 const int masked = k1 * e.r1 - rem;
                 consider(k0, k1, masked);
             }
+        }
+        if (!lfound) continue;
+        if (all) all->push_back(local);
+        if (pair_better(*best, found, local.cost, local.masked, local.k0, e)) {
+            *best = local;
+            found = true;
         }
     }
     return found;
@@ -201,51 +214,109 @@ static long long min_tile_chunks(const Geometry& g) {
     return best < 0 ? 0 : best;
 }
 
-// B200 time model used to pick the CTA tile and the cluster split (DESIGN.md
-// §7), calibrated with tools/sweep.py on B200:
-//   t = waves(ctas, slots) * (F + tile_ewm_flops / csplit / rate_cta)
-// rate_cta = per-SM Winograd-domain rate of the tile / CTAs per SM; F = fixed
-// per-CTA cost (prologue, pipeline fill, epilogue, cluster reduction).
-// Cluster placement strands SMs for cs >= 4 (132 of 148 usable at cs = 4,
-// 128 at cs = 8).
+// B200 time model used to pick the CTA tile, the segment count Z and the
+// cluster split, fitted by tools/fit_model.py to a
+// tools/sweep.py calibration run on B200 (profiles/r01/planner_fit.md).  It
+// simulates the block scheduler: a CTA (cluster) costs
+//   D[cs > 1] + max over ranks (F + chunks0 * T0 + jobs * (J + chunks1 * T1)),
+// T_a = a * chunk * BN * BM * 2 / rate (its Winograd-domain EWM flops at the
+// tile's sustained per-SM rate), and clusters are list-scheduled in launch
+// order onto the free slots (cs = 4 / 8 clusters: the measured resident
+// cluster counts).  Z > 1 adds the bucket reduction launch.
 struct TimeModel {
-    double rate_sm;    // EWM FLOP/s per SM for this tile
-    double fixed_s;    // per-CTA fixed cost (s)
+    double fixed_s;    // F: per-CTA prologue, pipeline fill, OT, epilogue
+    double rate_sm;    // EWM FLOP/s of one CTA (one CTA per SM)
+};
+struct SharedModel {
+    double job_s;       // J: per residual job (OT + job boundary)
+    double cluster_s;   // D: per-cluster DSMEM reduction / barriers
+    double reduce_s;    // fixed cost of the bucket-reduce launch
+    double reduce_bw;   // its bytes/s over (2Z) * |dW| fp32
+    double slots4, slots8;   // resident 4- / 8-CTA clusters on 148 SMs
 };
 
 static TimeModel time_model(int dtype, int bn, int bm) {
-    if (dtype != 0) return {bm >= 128 ? 1.2e12 : (bm >= 64 ? 1.4e12 : 0.8e12), 4e-6};
-    const int area = bn * bm;
-    return {area >= 4096 ? 0.20e12 : (area >= 2048 ? 0.16e12 : 0.11e12), 8e-6};
+    if (dtype != 0) {
+        if (bm >= 128) return {11.02e-6, 3.095e12};
+        if (bm >= 64) return {6.19e-6, 1.545e12};
+        return {3.80e-6, 0.812e12};
+    }
+    if (bn * bm >= 4096) return {7.12e-6, 3.49e11};
+    if (bn * bm >= 2048) return {5.61e-6, 2.59e11};
+    return {4.02e-6, 1.95e11};
+}
+static SharedModel shared_model(int dtype) {
+    if (dtype != 0) return {2.02e-6, 2.13e-6, 10.8e-6, 7.86e12, 33.1, 14.0};
+    return {0.0, 2.01e-6, 20.8e-6, 2.0e13, 34.8, 15.6};
 }
 
-static double slots_frac(int cs) { return cs <= 2 ? 1.0 : (cs == 4 ? 132.0 / 148.0 : 128.0 / 148.0); }
+// Resident cluster slots for a cluster size on num_sms SMs.
+static long long cluster_slots(int cs, int occ, int num_sms, const SharedModel& sm) {
+    const double f = (double)num_sms / 148.0;
+    long long s;
+    if (cs == 1) s = (long long)occ * num_sms;
+    else if (cs == 2) s = (long long)occ * num_sms / 2;
+    else if (cs == 4) s = (long long)(occ * sm.slots4 * f);
+    else s = (long long)(occ * sm.slots8 * f);
+    return std::max(1LL, s);
+}
 
-static double model_time(const Geometry& g, const KernelEntry& e, int num_sms, double ewm) {
+static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
     const TimeModel m = time_model(e.dtype, e.bn, e.bm);
-    const long long slots = std::max(1LL, (long long)(e.occ * num_sms * slots_frac(g.csplit)));
-    const long long waves = (num_ctas(g) + slots - 1) / slots;
-    const double per_cta = ewm / (double)num_tiles(g) / g.csplit / (m.rate_sm / e.occ);
-    return waves * (m.fixed_s + per_cta);
+    const SharedModel sh = shared_model(e.dtype);
+    const double per_chunk = (double)g.chunk * e.bn * e.bm * 2.0 / m.rate_sm;
+    const double t0 = g.a0 * per_chunk, t1 = (g.a1 ? g.a1 : 1) * per_chunk;
+    const long long mult = (long long)g.kblocks * g.cblocks * g.ftiles;
+    const int jobs_res = g.a1 ? g.n0 / g.n1 : 0;
+    const long long slots = cluster_slots(g.csplit, e.occ, num_sms, sh);
+    // min-heap of slot free times (list scheduling in launch order: band, col, fh outer; kb fastest)
+    std::vector<double> heap((size_t)slots, 0.0);
+    auto push_root = [&](double v) {   // replace the minimum (root) by v and sift down
+        size_t k = 0;
+        const size_t n = heap.size();
+        for (;;) {
+            size_t l = 2 * k + 1, r = l + 1, s = k;
+            double sv = v;
+            if (l < n && heap[l] < sv) { s = l; sv = heap[l]; }
+            if (r < n && heap[r] < sv) { s = r; sv = heap[r]; }
+            if (s == k) break;
+            heap[k] = heap[s];
+            k = s;
+        }
+        heap[k] = v;
+    };
+    for (int band = 0; band < g.bands; ++band)
+        for (int col = 0; col < g.seg_cols; ++col)
+            for (int fh = 0; fh < g.R; ++fh) {
+                int hs, he, wf, units;
+                band_rows(g, band, fh, &hs, &he);
+                seg_units(g, col, &wf, &units);
+                const long long rows = he - hs;
+                const long long cm = (rows * units * g.N + g.chunk - 1) / g.chunk;
+                const bool res = has_residual(g, col);
+                const long long cr = res ? (rows * g.k1 * g.N + g.chunk - 1) / g.chunk : 0;
+                double t = 0;
+                for (int r = 0; r < g.csplit; ++r) {
+                    const long long a = cm * (r + 1) / g.csplit - cm * r / g.csplit;
+                    const long long b = cr * (r + 1) / g.csplit - cr * r / g.csplit;
+                    const double tr = m.fixed_s + a * t0 + (res ? jobs_res * (sh.job_s + b * t1) : 0.0);
+                    t = std::max(t, tr);
+                }
+                if (g.csplit > 1) t += sh.cluster_s;
+                for (long long q = 0; q < mult; ++q) push_root(heap[0] + t);
+            }
+    double mk = 0;
+    for (double v : heap) mk = std::max(mk, v);
+    if (g.Z > 1) mk += sh.reduce_s + 2.0 * g.Z * (double)g.dw_elems * 4.0 / sh.reduce_bw;
+    return mk;
 }
 
-// Cluster split: cs in {1, 2, 4, 8} minimising the model time, keeping >= 4
-// chunks per CTA.
-static int choose_csplit(Geometry g, const KernelEntry& e, int num_sms, double ewm) {
+static int forced_csplit() {
     if (const char* f = getenv("WINRS_FORCE_CSPLIT")) {
         const int v = atoi(f);
         if (v == 1 || v == 2 || v == 4 || v == 8) return v;
     }
-    const long long mc = min_tile_chunks(g);
-    int best = 1;
-    double best_t = 1e30;
-    for (int cs = 1; cs <= 8; cs *= 2) {
-        if (cs > 1 && mc / cs < 4) break;
-        g.csplit = cs;
-        const double t = model_time(g, e, num_sms, ewm);
-        if (t < best_t * (1.0 - 1e-9)) { best_t = t; best = cs; }
-    }
-    return best;
+    return 0;
 }
 
 // Winograd-domain EWM flops the kernels issue (clipped rows, masked columns
@@ -264,27 +335,62 @@ static double ewm_flops(const Geometry& g) {
     return 2.0 * g.K * g.C * (double)g.N * tot;
 }
 
-static void plan_with_tile(const Problem& p, const KernelEntry& e, const PairChoice& pc, int num_sms,
-                           PlanResult* out) {
+// Steps 2-3 for one CTA tile.  Algorithm 1 gives Z^ (reported as z_hat);
+// on B200 the planner then evaluates every segment count Z <= Z_max (the
+// workspace cap, R11) through Algorithm 2 and every cluster split, and keeps
+// the (Z, cs) of least model time (R19).  WINRS_PLANNER=paper keeps
+// Algorithm 1's Z^ (only cs is searched).
+static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairChoice& pc, int num_sms,
+                             PlanResult* out) {
     int zmax = 1;
-    int z = alg1(p, e, num_sms, &zmax);
+    const int z_alg1 = alg1(p, e, num_sms, &zmax);
+    int z_lo = 1, z_hi = zmax;
+    const char* mode = getenv("WINRS_PLANNER");
+    if (mode && strcmp(mode, "paper") == 0) z_lo = z_hi = std::min(z_alg1, zmax);
     if (const char* fz = getenv("WINRS_FORCE_Z")) {
         const int v = atoi(fz);
-        if (v >= 1) { z = v; zmax = 1 << 30; }
+        if (v >= 1) { z_lo = z_hi = v; zmax = 1 << 30; }
     }
-    int z_used = 1, seg_h = p.Ho, seg_w = pc.k0 * e.r0;
-    Geometry g;
-    for (;;) {
+    int zhat_used = 1, sh0 = p.Ho, sw0 = pc.k0 * e.r0;
+    alg2(p, e.r0, pc.k0, std::min(z_alg1, zmax), &zhat_used, &sh0, &sw0);
+    const int fcs = forced_csplit();
+    const long long zlimit = (long long)std::max(1, p.pad > 0 ? p.Ho / p.pad : p.Ho) * pc.k0;   // alg2 line 1
+    if (z_hi > zlimit) z_hi = (int)std::max<long long>(z_lo, zlimit);
+    double best_t = 1e30;
+    bool have = false;
+    int last_bands = -1, last_cols = -1, last_sh = -1, last_sw = -1;
+    for (int z = z_lo; z <= z_hi; ++z) {
+        int z_used = 1, seg_h = p.Ho, seg_w = pc.k0 * e.r0;
         alg2(p, e.r0, pc.k0, z, &z_used, &seg_h, &seg_w);
+        Geometry g;
         fill_geometry(p, e, pc, seg_h, seg_w, &g);
-        if (g.Z <= zmax || z <= 1) break;     // enforce the workspace cap (R11)
-        z = std::min(z_used, z) - 1;
+        if (g.Z > zmax && z > 1) continue;   // workspace cap (R11)
+        if (z > z_lo && num_tiles(g) > 32LL * e.occ * num_sms) break;   // > 32 waves: per-CTA cost dominates
+        if (g.bands == last_bands && g.seg_cols == last_cols && seg_h == last_sh && seg_w == last_sw) continue;
+        last_bands = g.bands; last_cols = g.seg_cols; last_sh = seg_h; last_sw = seg_w;
+        const long long mc = min_tile_chunks(g);
+        for (int cs = 1; cs <= 8; cs *= 2) {
+            if (fcs ? cs != fcs : (cs > 1 && (!e.csplit_ok || mc < cs))) continue;
+            g.csplit = cs;
+            const double t = model_time(g, e, num_sms);
+            if (!have || t < best_t * (1.0 - 1e-9)) {
+                best_t = t;
+                have = true;
+                out->geom = g;
+            }
+        }
     }
-    g.csplit = e.csplit_ok ? choose_csplit(g, e, num_sms, ewm_flops(g)) : 1;
-    out->geom = g;
+    if (!have) {   // forced values that the loop filtered: plan Z^ with cs = 1 (or forced)
+        int z_used = 1, seg_h = p.Ho, seg_w = pc.k0 * e.r0;
+        alg2(p, e.r0, pc.k0, z_lo, &z_used, &seg_h, &seg_w);
+        fill_geometry(p, e, pc, seg_h, seg_w, &out->geom);
+        out->geom.csplit = fcs ? fcs : 1;
+        best_t = model_time(out->geom, e, num_sms);
+    }
     out->entry = &e;
-    out->z_hat = z_used;
+    out->z_hat = zhat_used;
     out->masked = pc.masked;
+    return best_t;
 }
 
 static int parse_force_tile(int* bn, int* bm) {
@@ -297,27 +403,34 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
     int ne = 0;
     const KernelEntry* es = kernel_entries(&ne);
     PairChoice pc;
-    if (!choose_pair(p, es, ne, &pc)) return WINRS_ERR_UNSUPPORTED;
-    // Step 1b (B200): CTA tile.  Each compiled tile variant is planned (Z,
-    // segments, cluster split) and scored by the B200 time model above.
-    std::vector<const KernelEntry*> tiles;
-    for (int i = 0; i < ne; ++i)
-        if (same_pair(es[i], *pc.proto)) tiles.push_back(&es[i]);
-    std::sort(tiles.begin(), tiles.end(), [](const KernelEntry* a, const KernelEntry* b) {
-        if (a->bn * a->bm != b->bn * b->bm) return a->bn * a->bm > b->bn * b->bm;
-        return a->bn > b->bn;
-    });
+    std::vector<PairChoice> pairs;
+    if (!choose_pair(p, es, ne, &pc, &pairs)) return WINRS_ERR_UNSUPPORTED;
+    // Step 1 with measured throughput (B200, R19): the paper's cost divides by
+    // kernel-specific throughput coefficients tau (P@20823); here every valid
+    // pair x compiled CTA tile is planned (Z, segments, cluster split) and
+    // scored by the B200 time model, whose per-tile rates play tau's role.
+    // WINRS_PLANNER=paper keeps the pure alpha-count pair choice.
+    const char* mode = getenv("WINRS_PLANNER");
+    if (mode && strcmp(mode, "paper") == 0) pairs.assign(1, pc);
     int fbn = 0, fbm = 0;
     const bool force_tile = parse_force_tile(&fbn, &fbm);
     PlanResult best;
     bool have = false;
     double best_t = 1e30;
-    for (const KernelEntry* e : tiles) {
-        if (force_tile && (e->bn != fbn || e->bm != fbm)) continue;
-        PlanResult r;
-        plan_with_tile(p, *e, pc, num_sms, &r);
-        const double t = model_time(r.geom, *e, num_sms, ewm_flops(r.geom));
-        if (!have || t < best_t - 1e-12) { best = r; best_t = t; have = true; }
+    for (const PairChoice& cand : pairs) {
+        std::vector<const KernelEntry*> tiles;
+        for (int i = 0; i < ne; ++i)
+            if (same_pair(es[i], *cand.proto)) tiles.push_back(&es[i]);
+        std::sort(tiles.begin(), tiles.end(), [](const KernelEntry* a, const KernelEntry* b) {
+            if (a->bn * a->bm != b->bn * b->bm) return a->bn * a->bm > b->bn * b->bm;
+            return a->bn > b->bn;
+        });
+        for (const KernelEntry* e : tiles) {
+            if (force_tile && (e->bn != fbn || e->bm != fbm)) continue;
+            PlanResult r;
+            const double t = plan_with_tile(p, *e, cand, num_sms, &r);
+            if (!have || t < best_t * (1.0 - 1e-9)) { best = r; best_t = t; have = true; }
+        }
     }
     if (!have) return WINRS_ERR_UNSUPPORTED;
     best.ewm_flops = ewm_flops(best.geom);

@@ -52,7 +52,10 @@ def test_figure5_pair():
     (2, 33, (4, 2, 3, 11, 0, 0, 0, 0, 0)),
     (4, 33, (8, 4, 5, 6, 4, 2, 3, 1, 0)),
 ])
-def test_pair_selection(S, Wo, expect):
+def test_pair_selection(S, Wo, expect, monkeypatch):
+    # the paper's step 1 (alpha-count cost); the default planner also scores
+    # every valid pair with the B200 time model (R19)
+    monkeypatch.setenv("WINRS_PLANNER", "paper")
     pad = S // 2
     Wd = Wo - 2 * pad + S - 1
     p = W.plan_for_device(4, 32, 8, Wd, 32, S, S, pad, "f32")
