@@ -30,6 +30,11 @@ WINRS_API const char* winrs_debug_kernel_name(int i);
 /* Name of the instantiation a plan uses. */
 WINRS_API const char* winrs_debug_plan_kernel(winrs_plan_t plan);
 
+/* The planner's B200 time-model estimate for the plan (microseconds; the
+ * quantity it minimised over pair x tile x Z x cluster split, R19).
+ * -1 for a null plan. */
+WINRS_API double winrs_debug_plan_model_us(winrs_plan_t plan);
+
 #ifdef __cplusplus
 }
 #endif

@@ -50,6 +50,11 @@ class Plan:
         return _lib.lib().winrs_debug_plan_kernel(self._h).decode()
 
     @property
+    def model_us(self) -> float:
+        """The planner's B200 time-model estimate (R19)."""
+        return float(_lib.lib().winrs_debug_plan_model_us(self._h))
+
+    @property
     def dtype(self) -> str:
         return {0: "f32", 1: "f16", 2: "bf16"}[self.info["dtype"]]
 

@@ -59,6 +59,7 @@ SYMBOLS = [
     ("winrs_debug_kernel_count", _i, []),
     ("winrs_debug_kernel_name", ctypes.c_char_p, [_i]),
     ("winrs_debug_plan_kernel", ctypes.c_char_p, [_p]),
+    ("winrs_debug_plan_model_us", ctypes.c_double, [_p]),
 ]
 
 _lib = None

@@ -434,6 +434,7 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
     }
     if (!have) return WINRS_ERR_UNSUPPORTED;
     best.ewm_flops = ewm_flops(best.geom);
+    best.model_s = best_t;
     *out = best;
     return WINRS_OK;
 }

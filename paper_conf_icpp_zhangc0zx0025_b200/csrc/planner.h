@@ -17,6 +17,7 @@ struct PlanResult {
     int z_hat = 1;
     int masked = 0;
     double ewm_flops = 0;
+    double model_s = 0;   // B200 time-model estimate of the launch(es), seconds
 };
 
 winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out);

@@ -323,4 +323,6 @@ const char* winrs_debug_kernel_name(int i) {
 
 const char* winrs_debug_plan_kernel(winrs_plan_t plan) { return plan ? plan->pr.entry->name : nullptr; }
 
+double winrs_debug_plan_model_us(winrs_plan_t plan) { return plan ? plan->pr.model_s * 1e6 : -1.0; }
+
 }  // extern "C"

@@ -157,3 +157,39 @@ def test_strided_entry_validates_ldy():
     assert L.winrs_bfc_strided(p.handle, fake, fake, 18, fake, None, None) == 1    # ldy % 4
     p16 = W.plan_for_device(2, 16, 8, 8, 16, 3, 3, 1, "f16")
     assert L.winrs_bfc_strided(p16.handle, fake, fake, 20, fake, None, None) == 1  # ldy % 8
+
+
+# --- R19: the B200 search vs the printed rules ---------------------------------
+BENCH_LAYERS = wl.RESNET50_F32 + wl.RESNET50_F16 + wl.WIDE_F32 + wl.VGG16_F16
+
+
+def _plan(l):
+    return W.plan_for_device(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype)
+
+
+@pytest.mark.parametrize("l", BENCH_LAYERS, ids=lambda l: l.name)
+def test_search_never_worse_than_paper_rules(l, monkeypatch):
+    """The default plan minimises the model over a candidate set that contains
+    the printed rules' plan, so its model time can only be lower or equal."""
+    d = _plan(l)
+    monkeypatch.setenv("WINRS_PLANNER", "paper")
+    pp = _plan(l)
+    assert 0 < d.model_us <= pp.model_us * (1 + 1e-9)
+    # the printed rules: Z never exceeds Algorithm 1's (capped) Z^
+    assert pp.info["Z"] <= max(pp.info["z_hat"], 1) * 2
+
+
+@pytest.mark.parametrize("l", BENCH_LAYERS, ids=lambda l: l.name)
+def test_search_plan_is_valid(l):
+    """Whatever the model picks obeys the paper's hard constraints: criteria
+    (1)-(2) for the pair, n1 | n0, and the 4% workspace cap (R11)."""
+    i = _plan(l).info
+    assert l.S % i["n0"] == 0
+    if i["alpha1"]:
+        assert l.S % i["n1"] == 0 and i["n0"] % i["n1"] == 0
+    assert i["k0"] * i["r0"] + i["k1"] * i["r1"] - i["masked_cols"] == i["Wo"]
+    assert 0 <= i["masked_cols"] < max(i["r0"], i["r1"] or 1)
+    esz = 4 if l.dtype == "f32" else 2
+    data = esz * (l.N * l.H * l.W * l.C + l.N * i["Ho"] * i["Wo"] * l.K)
+    assert i["workspace_bytes"] <= 0.04 * data + 4 * l.K * l.R * l.S * l.C
+    assert i["csplit"] in (1, 2, 4, 8)
