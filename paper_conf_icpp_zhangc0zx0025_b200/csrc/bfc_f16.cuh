@@ -223,11 +223,12 @@ struct Barriers {
 };
 
 // Depth entry -> (n, h, u) for chunk-box issue.
-__device__ __forceinline__ void depth_coord(long long d, int N, int units, int hs, int* n, int* h, int* u) {
-    *n = (int)(d % N);
-    const long long t = d / N;
-    *u = (int)(t % units);
-    *h = hs + (int)(t / units);
+// 32-bit: depth < N*Ho*Wo < 2^31 (winrs_plan rejects larger problems).
+__device__ __forceinline__ void depth_coord(int d, int N, int units, int hs, int* n, int* h, int* u) {
+    *n = d % N;
+    const int t = d / N;
+    *u = t % units;
+    *h = hs + t / units;
 }
 
 // ---- transformer work for one chunk.  A unit is (row pair 2p/2p+1, 8
@@ -303,8 +304,12 @@ __device__ __forceinline__ int tx_role(int tw) {
     return tx_is_it<BM>(tw) ? before : -1 - (tw - before);
 }
 
+// kv / cv: valid k rows / c columns of this tile (< B_N / B_M in the last
+// K- / C-block).  A warp whose whole row block lies past them skips its
+// transforms: those operand rows stay zero (the op ring is cleared once at
+// kernel start) and their accumulator rows are never written out.
 template <int A, int NN, int RR, int BM, bool BF>
-__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tw, int lane) {
+__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tw, int lane, int kv, int cv) {
     constexpr int RAW_Y = KC * RR * BN * 2;
     const uint16_t* rawY = reinterpret_cast<const uint16_t*>(raw);            // [KC][RR][BN]
     const uint16_t* rawX = reinterpret_cast<const uint16_t*>(raw + RAW_Y);    // [KC][A][BM]
@@ -312,12 +317,14 @@ __device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op,
     const int role = tx_role<BM>(tw);
     if (role < 0) {
         const int f = -1 - role;   // FT warp: 32 k pairs x one octet
+        if ((f % (BN / 64)) * 64 >= kv) return;
         unit_transform<0, A, NN, RR, RR, DQ_FT, BF>(rawY, BN, RR * BN, op, OPA, (f % (BN / 64)) * 32 + lane,
                                                 f / (BN / 64));
     } else {                       // IT warp: 32 c pairs (or BM/2 pairs x 32/(BM/2) quads) x quads
         constexpr int PW = BM / 2 < 32 ? BM / 2 : 32;
         const int q = (role % ((BM / 2) / PW)) * PW + (lane % PW);
         const int quad = role / ((BM / 2) / PW) * (32 / PW) + lane / PW;
+        if ((role % ((BM / 2) / PW)) * PW * 2 >= cv) return;
         unit_transform<1, A, NN, RR, A, DQ_IT, BF>(rawX, BM, A * BM, op + A * OPA, OPB, q, quad);
     }
 }
@@ -524,6 +531,11 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                      :: "r"(smem_u32(&bars->tmem_base)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
+    {   // clear the operand ring once (rows past K / C are never transformed)
+        uint4* op = reinterpret_cast<uint4*>(smem + SM::op_off);
+        for (int i = threadIdx.x; i < S_OP * SM::OP / 16; i += nthreads<BM>()) op[i] = make_uint4(0, 0, 0, 0);
+        fence_proxy_async();   // generic-proxy zeros visible to the tensor core's async proxy
+    }
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
@@ -556,7 +568,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 __syncwarp();
                 if (lane < nbox) {
                     const int b = (lane >> 1) * args.nb;
-                    const long long d = (long long)ch * KC + b;
+                    const int d = ch * KC + b;
                     int n = g.N, h = hs, u = 0;   // past-the-end image => zero fill
                     if (d < depth) depth_coord(d, g.N, J.units, hs, &n, &h, &u);
                     const int w0 = J.w_first + u * RRj;
@@ -607,6 +619,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     } else {
         // ===================== transformers (+ epilogue) =====================
         const int tw = warp - 2;
+        const int kv = g.K - cc.kb * BN, cv = g.C - cc.cb * BM;
         int sr = 0, so = 0;
         uint32_t phr = 0, pho = 0;
         for (int jb = 0; jb < njobs; ++jb) {
@@ -621,8 +634,8 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 2);
                 const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
                 uint8_t* op = smem + SM::op_off + so * SM::OP;
-                if (J.phase == 0) transform_chunk<A0, N0, R0, BM, BF>(raw, op, tw, lane);
-                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM, BF>(raw, op, tw, lane);
+                if (J.phase == 0) transform_chunk<A0, N0, R0, BM, BF>(raw, op, tw, lane, kv, cv);
+                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM, BF>(raw, op, tw, lane, kv, cv);
                 if (threadIdx.x == 64) TRACE(3, ch - c_lo + jb * 64, 0);
                 if (threadIdx.x == 64 + 32 * 2) TRACE(3, ch - c_lo + jb * 64, 1);   // an IT warp
                 fence_proxy_async();
