@@ -10,7 +10,9 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libwinrs.so")
+# WINRS_LIB selects another in-tree build of the same library (an A/B kernel
+# variant from `tools/build.py --variant TAG`, e.g. libwinrs_TAG.so).
+LIB_PATH = os.path.join(_HERE, os.environ.get("WINRS_LIB", "libwinrs.so"))
 
 WINRS_OK = 0
 STATUS = {0: "WINRS_OK", 1: "WINRS_ERR_INVALID_ARG", 2: "WINRS_ERR_UNSUPPORTED",

@@ -98,6 +98,12 @@ extern "C" __attribute__((visibility("default"))) int winrs_trace_read(unsigned 
 extern "C" __attribute__((visibility("default"))) int winrs_trace_read_w(unsigned long long* out) {
     return (int)cudaMemcpyFromSymbol(out, f16k::g_trace_w, sizeof(f16k::g_trace_w));
 }
+extern "C" __attribute__((visibility("default"))) int winrs_trace_read_cta(unsigned long long* out) {
+    return (int)cudaMemcpyFromSymbol(out, f16k::g_cta_time, sizeof(f16k::g_cta_time));
+}
+extern "C" __attribute__((visibility("default"))) int winrs_trace_read_slots(unsigned int* out) {
+    return (int)cudaMemcpyFromSymbol(out, f16k::g_warpslot, sizeof(f16k::g_warpslot));
+}
 #endif
 
 const KernelEntry* f16_entries(int* n) {

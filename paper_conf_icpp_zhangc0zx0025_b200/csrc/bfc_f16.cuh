@@ -31,6 +31,7 @@
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include "dsmem.cuh"
 #include "winograd_generated.cuh"
 #include "winrs_internal.h"
 #include "winrs_vec.cuh"
@@ -41,12 +42,34 @@ namespace f16k {
 constexpr int BN = 128;          // k rows = UMMA M (TMEM lanes)
 constexpr int KC = 16;           // depth entries per chunk = UMMA K
 #ifndef WINRS_F16_SOP
-#define WINRS_F16_SOP 2
+#define WINRS_F16_SOP 0          // 0: as many operand stages (<= 4) as leave 3 raw stages
 #endif
-constexpr int S_OP = WINRS_F16_SOP;   // operand ring stages
-// transformer warps: one thread per (row pair, depth quad) unit of a chunk:
-// FT (BN/2 k pairs x 4 quads) + IT (BM/2 c pairs x 4 quads)
-template <int BM> __host__ __device__ constexpr int tx_warps() { return (BN / 2) * 2 / 32 + (BM / 2) * 2 / 32; }
+#ifndef WINRS_F16_DQ
+#define WINRS_F16_DQ 8           // depth entries per transformer unit (8: octet; 4 measured slower)
+#endif
+// transformer warps: one thread per (row pair, depth group of DQ) unit of a
+// chunk: FT (BN/2 k pairs x KC/DQ groups) + IT (BM/2 c pairs x KC/DQ groups)
+constexpr int DQ_FT = WINRS_F16_DQ;      // depth entries per FT unit
+constexpr int DQ_IT = WINRS_F16_DQ;      // depth entries per IT unit
+#ifndef WINRS_F16_DYN
+#define WINRS_F16_DYN 1          // 1: transformer warps grab work units dynamically (else a fixed role per warp)
+#endif
+#ifndef WINRS_F16_TXW
+#define WINRS_F16_TXW 0          // transformer warps (0: one per unit of a chunk)
+#endif
+// A chunk's transform work is split into warp-sized units: FT units (32 k
+// pairs x one depth group) and IT units (32 c pairs, or BM/2 pairs x several
+// groups, x depth groups).
+template <int BM> __host__ __device__ constexpr int ft_warps() { return (BN / 2) * (KC / DQ_FT) / 32; }
+template <int BM> __host__ __device__ constexpr int it_warps() { return (BM / 2) * (KC / DQ_IT) / 32; }
+template <int BM> __host__ __device__ constexpr int n_units() { return ft_warps<BM>() + it_warps<BM>(); }
+// More warps than units per chunk let several chunks be in flight, which
+// hides the shared-memory latency of the transforms; measured best on B200
+// (A/B of 8..16 warps over the ResNet-50 / VGG-16 layers): 10 warps for the
+// 128x64 / 128x32 tiles, 14 for 128x128.
+template <int BM> __host__ __device__ constexpr int tx_warps() {
+    return !WINRS_F16_DYN ? n_units<BM>() : WINRS_F16_TXW > 0 ? WINRS_F16_TXW : BM >= 128 ? 14 : 10;
+}
 template <int BM> __host__ __device__ constexpr int nthreads() { return 64 + 32 * tx_warps<BM>(); }
 
 struct Args {
@@ -171,6 +194,10 @@ struct Smem {
     static constexpr int OPB = BM * KC * 2;              // one B_xi slab
     static constexpr int OP = A0 * (OPA + OPB);
     static constexpr int LIMIT = 227 * 1024 - 256;
+    // operand stages: the deeper the ring, the less the transformers wait for
+    // the MMAs of the chunk S_OP back; keep >= 3 raw stages for TMA latency.
+    static constexpr int S_OP = WINRS_F16_SOP > 0 ? WINRS_F16_SOP
+                              : (LIMIT - 4 * OP) / RAW >= 3 ? 4 : (LIMIT - 3 * OP) / RAW >= 3 ? 3 : 2;
     // as many raw (TMA) stages as fit: the raw ring is the latency-hiding depth
     static constexpr int S_RAW = (LIMIT - S_OP * OP) / RAW > 4 ? 4 : (LIMIT - S_OP * OP) / RAW;
     static_assert(S_RAW >= 2, "shared memory too small for a 2-stage raw ring");
@@ -200,14 +227,19 @@ __device__ __forceinline__ uint32_t op_row_off(int row, int dgroup) {
 #ifdef WINRS_TRACE
 // Debug-build timeline of CTA 0 (globaltimer ns): [role][chunk][event].
 __device__ unsigned long long g_trace[4][256][4];
-__device__ unsigned long long g_trace_w[256][16];   // per-warp "chunk done" times
+__device__ unsigned long long g_trace_w[256][24][3];   // per-warp (raw ok, op ok, chunk done) times
+__device__ unsigned int g_warpslot[24];                 // %warpid of each warp (SM sub-partition = %4)
 __device__ __forceinline__ unsigned long long gtime() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
     return t;
 }
 #define TRACE(role, ch, ev) do { if (blockIdx.x == 0 && (ch) < 256) g_trace[role][ch][ev] = gtime(); } while (0)
+__device__ unsigned long long g_cta_time[2048][8];      // per-CTA phase times (all CTAs)
+#define PTRACE(i) do { if (blockIdx.x == 0) g_trace[0][240 + (i)][0] = gtime(); \
+                       if (blockIdx.x < 2048) g_cta_time[blockIdx.x][i] = gtime(); } while (0)
 #else
+#define PTRACE(i) do { } while (0)
 #define TRACE(role, ch, ev) do { } while (0)
 #endif
 
@@ -220,6 +252,7 @@ struct Job {
 struct Barriers {
     uint64_t raw_full[4], raw_empty[4], op_full[4], op_empty[4], acc_full, acc_empty;
     uint32_t tmem_base;
+    int unit_ctr;       // next transform unit (dynamic scheduling)
 };
 
 // Depth entry -> (n, h, u) for chunk-box issue.
@@ -241,10 +274,6 @@ __device__ __forceinline__ void depth_coord(int d, int N, int units, int hs, int
 // of a row form one 16-byte core-matrix row: two STS.128 per xi, conflict
 // free through perm16.  FT and IT warps are interleaved so every SM
 // sub-partition (warp % 4) gets the same mix.
-constexpr int DQ_FT = 8;                 // depth entries per FT unit (an octet)
-constexpr int DQ_IT = 8;                 // depth entries per IT unit (an octet)
-template <int BM> __host__ __device__ constexpr int ft_warps() { return (BN / 2) * (KC / DQ_FT) / 32; }
-template <int BM> __host__ __device__ constexpr int it_warps() { return (BM / 2) * (KC / DQ_IT) / 32; }
 
 template <int WT_FN, int A, int NN, int RR, int NIN, int DQ, bool BF>
 __device__ __forceinline__ void unit_transform(const uint16_t* src, int tap_stride, int depth_stride, uint8_t* dst0,
@@ -308,13 +337,13 @@ __device__ __forceinline__ int tx_role(int tw) {
 // K- / C-block).  A warp whose whole row block lies past them skips its
 // transforms: those operand rows stay zero (the op ring is cleared once at
 // kernel start) and their accumulator rows are never written out.
+// role >= 0: IT unit `role`; role < 0: FT unit -1 - role.
 template <int A, int NN, int RR, int BM, bool BF>
-__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tw, int lane, int kv, int cv) {
+__device__ __forceinline__ void transform_role(const uint8_t* raw, uint8_t* op, int role, int lane, int kv, int cv) {
     constexpr int RAW_Y = KC * RR * BN * 2;
     const uint16_t* rawY = reinterpret_cast<const uint16_t*>(raw);            // [KC][RR][BN]
     const uint16_t* rawX = reinterpret_cast<const uint16_t*>(raw + RAW_Y);    // [KC][A][BM]
     constexpr int OPA = BN * KC * 2, OPB = BM * KC * 2;
-    const int role = tx_role<BM>(tw);
     if (role < 0) {
         const int f = -1 - role;   // FT warp: 32 k pairs x one octet
         if ((f % (BN / 64)) * 64 >= kv) return;
@@ -327,6 +356,16 @@ __device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op,
         if ((role % ((BM / 2) / PW)) * PW * 2 >= cv) return;
         unit_transform<1, A, NN, RR, A, DQ_IT, BF>(rawX, BM, A * BM, op + A * OPA, OPB, q, quad);
     }
+}
+// Static schedule: transformer warp tw always runs the same unit.
+template <int A, int NN, int RR, int BM, bool BF>
+__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tw, int lane, int kv, int cv) {
+    transform_role<A, NN, RR, BM, BF>(raw, op, tx_role<BM>(tw), lane, kv, cv);
+}
+// Dynamic schedule: unit u of a chunk, the (costlier) IT units first.
+template <int A, int NN, int RR, int BM, bool BF>
+__device__ __forceinline__ void transform_unit(const uint8_t* raw, uint8_t* op, int u, int lane, int kv, int cv) {
+    transform_role<A, NN, RR, BM, BF>(raw, op, u < it_warps<BM>() ? u : -1 - (u - it_warps<BM>()), lane, kv, cv);
 }
 
 __device__ __forceinline__ void tmem_st8(uint32_t taddr, const float* v) {
@@ -458,15 +497,7 @@ __device__ __forceinline__ void cluster_reduce(const Geometry& g, float* bucket,
         const int row = p / C4, c4 = p % C4;
         const int j = row / BN, kl = row % BN;
         const uint32_t off = (uint32_t)((row * out_ld<BM>() + c4 * 4) * 4);
-        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-        for (int q = 0; q < g.csplit; ++q) {
-            uint32_t remote;
-            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(out_s + off), "r"(q));
-            float4 v;
-            asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
-                         : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(remote) : "memory");
-            acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
-        }
+        const float4 acc = dsmem_sum4(out_s + off, g.csplit);
         const int kg = cc.kb * BN + kl, cg = cc.cb * BM + c4 * 4;
         if (kg < g.K && cg < g.C)
             *reinterpret_cast<float4*>(bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0 + j) * g.C + cg) = acc;
@@ -488,6 +519,14 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     const Geometry& g = args.g;
     Barriers* bars = reinterpret_cast<Barriers*>(smem + SM::bar_off);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) PTRACE(0);
+#ifdef WINRS_TRACE
+    if (threadIdx.x == 0 && blockIdx.x < 2048) {
+        unsigned int smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        g_cta_time[blockIdx.x][7] = smid;
+    }
+#endif
 
     const int rank = (int)(blockIdx.x % g.csplit);
     const CtaCoord cc = decode_cta(g, blockIdx.x / g.csplit);
@@ -516,8 +555,10 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     };
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < S_RAW; ++s) { mbar_init(&bars->raw_full[s], 1); mbar_init(&bars->raw_empty[s], TX_WARPS); }
-        for (int s = 0; s < S_OP; ++s) { mbar_init(&bars->op_full[s], TX_WARPS); mbar_init(&bars->op_empty[s], 1); }
+        constexpr int NU = n_units<BM>();
+        for (int s = 0; s < S_RAW; ++s) { mbar_init(&bars->raw_full[s], 1); mbar_init(&bars->raw_empty[s], NU); }
+        for (int s = 0; s < SM::S_OP; ++s) { mbar_init(&bars->op_full[s], NU); mbar_init(&bars->op_empty[s], 1); }
+        bars->unit_ctr = 0;
         mbar_init(&bars->acc_full, 1);
         mbar_init(&bars->acc_empty, 4);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -533,13 +574,21 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     }
     {   // clear the operand ring once (rows past K / C are never transformed)
         uint4* op = reinterpret_cast<uint4*>(smem + SM::op_off);
-        for (int i = threadIdx.x; i < S_OP * SM::OP / 16; i += nthreads<BM>()) op[i] = make_uint4(0, 0, 0, 0);
+        for (int i = threadIdx.x; i < SM::S_OP * SM::OP / 16; i += nthreads<BM>()) op[i] = make_uint4(0, 0, 0, 0);
         fence_proxy_async();   // generic-proxy zeros visible to the tensor core's async proxy
     }
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = bars->tmem_base;
+    if (threadIdx.x == 0) PTRACE(1);
+#ifdef WINRS_TRACE
+    if (blockIdx.x == 0 && lane == 0) {
+        unsigned int wid;
+        asm volatile("mov.u32 %0, %%warpid;" : "=r"(wid));
+        g_warpslot[warp] = wid;
+    }
+#endif
 
     if (warp == 0) {
         // ===================== TMA producer (whole warp) =====================
@@ -611,10 +660,82 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     }
                     umma_commit(&bars->op_empty[s]);
                     TRACE(1, ch - c_lo + jb * 64, 1);
-                    if (++s == S_OP) { s = 0; ph ^= 1; }
+                    if (++s == SM::S_OP) { s = 0; ph ^= 1; }
                 }
                 umma_commit(&bars->acc_full);
             }
+            PTRACE(2);
+        }
+    } else if (WINRS_F16_DYN) {
+        // ============ transformers (+ epilogue), dynamic unit schedule ============
+        // Every chunk of every job is n_units() warp-sized units; warps grab
+        // units in global order (job, chunk, unit) from a shared counter, so a
+        // warp that ran a cheap unit (FT) or sits on a lightly loaded SM
+        // sub-partition takes more: the chunk rate follows the average unit
+        // cost instead of the slowest fixed role.  Ring stage / parity follow
+        // from the global chunk index, as in the producer and MMA loops.
+        constexpr int NU = n_units<BM>();
+        const int kv = g.K - cc.kb * BN, cv = g.C - cc.cb * BM;
+        int jlo[1 + 9], jhi[1 + 9];
+        for (int jb = 0; jb < njobs; ++jb) chunk_range(jobs[jb], &jlo[jb], &jhi[jb]);
+        int jb = 0, unit_base = 0, gch_base = 0, epi = 0;
+        auto run_epilogue = [&](int e) {
+            const Job& J = jobs[e];
+            mbar_wait(&bars->acc_full, (uint32_t)(e & 1));
+            tc_fence_after();
+            const bool empty = jhi[e] <= jlo[e];
+            if (J.phase == 0)
+                epilogue<A0, N0, R0, N0, BM>(0, true, empty, tmem_base, warp);
+            else if constexpr (A1 != 0)
+                epilogue<A1, N1, R1, N0, BM>(J.fw0 - fw0, false, empty, tmem_base, warp);
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&bars->acc_empty);
+        };
+        for (;;) {
+            int gi = 0;
+            if (lane == 0) gi = atomicAdd(&bars->unit_ctr, 1);
+            gi = __shfl_sync(0xffffffffu, gi, 0);
+            while (jb < njobs && gi >= unit_base + (jhi[jb] - jlo[jb]) * NU) {
+                unit_base += (jhi[jb] - jlo[jb]) * NU;
+                gch_base += jhi[jb] - jlo[jb];
+                ++jb;
+            }
+            // epilogues of the jobs whose units are all handed out (warps 2..5:
+            // one TMEM lane quarter each)
+            if (warp < 6)
+                while (epi < jb) run_epilogue(epi++);
+            if (jb >= njobs) break;
+            const int rel = gi - unit_base;
+            const int u = rel % NU, gch = gch_base + rel / NU;
+            const int sr = gch % S_RAW, so = gch % SM::S_OP;
+            mbar_wait(&bars->raw_full[sr], (uint32_t)((gch / S_RAW) & 1));
+#ifdef WINRS_TRACE
+            if (lane == 0 && blockIdx.x == 0 && gch < 256) g_trace_w[gch][warp][0] = gtime();
+#endif
+            mbar_wait(&bars->op_empty[so], (uint32_t)(((gch / SM::S_OP) & 1) ^ 1));
+#ifdef WINRS_TRACE
+            if (lane == 0 && blockIdx.x == 0 && gch < 256) g_trace_w[gch][warp][1] = gtime();
+#endif
+            const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
+            uint8_t* op = smem + SM::op_off + so * SM::OP;
+            if (jobs[jb].phase == 0) transform_unit<A0, N0, R0, BM, BF>(raw, op, u, lane, kv, cv);
+            else if constexpr (A1 != 0) transform_unit<A1, N1, R1, BM, BF>(raw, op, u, lane, kv, cv);
+            fence_proxy_async();
+            __syncwarp();
+#ifdef WINRS_TRACE
+            if (lane == 0 && blockIdx.x == 0 && gch < 256) g_trace_w[gch][warp][2] = gtime();
+#endif
+            if (lane == 0) {
+                mbar_arrive(&bars->op_full[so]);
+                mbar_arrive(&bars->raw_empty[sr]);
+            }
+        }
+        if (threadIdx.x == 64) PTRACE(3);
+        asm volatile("bar.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
+        if (warp < 6) {
+            final_out<N0, BM>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
+            if (threadIdx.x == 64) PTRACE(4);
         }
     } else {
         // ===================== transformers (+ epilogue) =====================
@@ -630,8 +751,14 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 0);
                 mbar_wait(&bars->raw_full[sr], phr);
                 if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 1);
+#ifdef WINRS_TRACE
+                if (lane == 0 && blockIdx.x == 0 && ch - c_lo + jb * 64 < 256) g_trace_w[ch - c_lo + jb * 64][warp][0] = gtime();
+#endif
                 mbar_wait(&bars->op_empty[so], pho ^ 1);
                 if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 2);
+#ifdef WINRS_TRACE
+                if (lane == 0 && blockIdx.x == 0 && ch - c_lo + jb * 64 < 256) g_trace_w[ch - c_lo + jb * 64][warp][1] = gtime();
+#endif
                 const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
                 uint8_t* op = smem + SM::op_off + so * SM::OP;
                 if (J.phase == 0) transform_chunk<A0, N0, R0, BM, BF>(raw, op, tw, lane, kv, cv);
@@ -643,14 +770,14 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 __syncwarp();
                 if (threadIdx.x == 64) TRACE(2, ch - c_lo + jb * 64, 3);
 #ifdef WINRS_TRACE
-                if (lane == 0 && blockIdx.x == 0 && ch - c_lo + jb * 64 < 256) g_trace_w[ch - c_lo + jb * 64][warp] = gtime();
+                if (lane == 0 && blockIdx.x == 0 && ch - c_lo + jb * 64 < 256) g_trace_w[ch - c_lo + jb * 64][warp][2] = gtime();
 #endif
                 if (lane == 0) {
                     mbar_arrive(&bars->op_full[so]);
                     mbar_arrive(&bars->raw_empty[sr]);
                 }
                 if (++sr == S_RAW) { sr = 0; phr ^= 1; }
-                if (++so == S_OP) { so = 0; pho ^= 1; }
+                if (++so == SM::S_OP) { so = 0; pho ^= 1; }
             }
             if (warp < 6) {
                 mbar_wait(&bars->acc_full, (uint32_t)(jb & 1));
@@ -668,18 +795,22 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         // All transformer warps are past their last raw-ring read before the
         // staging tile (which overlays the rings) is written.  (Already implied
         // by acc_full -> all MMAs -> all op_full arrivals; made explicit.)
+        if (threadIdx.x == 64) PTRACE(3);
         asm volatile("bar.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
         if (warp < 6) {
             // every job's epilogue is done (this warp's own, in program order)
             final_out<N0, BM>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
+            if (threadIdx.x == 64) PTRACE(4);
         }
     }
     tc_fence_before();
     __syncthreads();
+    if (threadIdx.x == 0) PTRACE(5);
     if constexpr (kCluster) {
         if (g.csplit > 1)
             cluster_reduce<N0, BM>(g, bucket, cc, fw0, rank, reinterpret_cast<const float*>(smem), nthreads<BM>());
     }
+    if (threadIdx.x == 0) PTRACE(6);
     if (warp == 1) {
         tc_fence_after();
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem_base));

@@ -28,6 +28,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include "dsmem.cuh"
 #include "winrs_internal.h"
 #include "winograd_generated.cuh"
 #include "winrs_vec.cuh"
@@ -386,15 +387,7 @@ __device__ __forceinline__ void write_out(const Geometry& g, float* __restrict__
         const uint32_t off = (uint32_t)(((row) * out_ld<BM>() + c4 * 4) * 4);
         float4 acc;
         if (g.csplit > 1) {
-            acc = make_float4(0.f, 0.f, 0.f, 0.f);
-            for (int q = 0; q < g.csplit; ++q) {
-                uint32_t remote;
-                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(out_s + off), "r"(q));
-                float4 v;
-                asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
-                             : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(remote) : "memory");
-                acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
-            }
+            acc = dsmem_sum4(out_s + off, g.csplit);
         } else {
             acc = *reinterpret_cast<const float4*>(Out + row * out_ld<BM>() + c4 * 4);
         }

@@ -51,9 +51,13 @@ def _compile(src: str, force: bool, hdr_m: float) -> str:
     return o
 
 
-def build(force: bool = False, jobs: int = 0, trace: bool = False, extra=()) -> str:
+def build(force: bool = False, jobs: int = 0, trace: bool = False, extra=(), variant: str = "") -> str:
     global OBJ, LIB, FLAGS
-    if trace:   # debug build with the CTA-0 timeline (csrc/bfc_f16.cuh TRACE)
+    if variant:   # A/B build with extra -D knobs: libwinrs_<variant>.so (select with WINRS_LIB)
+        OBJ = os.path.join(ROOT, "build", "obj_" + variant)
+        LIB = os.path.join(PKG, "libwinrs_%s.so" % variant)
+        FLAGS = FLAGS + ["-D" + e for e in extra]
+    elif trace:   # debug build with the CTA-0 timeline (csrc/bfc_f16.cuh TRACE)
         OBJ = os.path.join(ROOT, "build", "obj_trace" + "".join(extra))
         LIB = os.path.join(PKG, "libwinrs_trace%s.so" % "".join(extra))
         FLAGS = FLAGS + ["-DWINRS_TRACE"] + ["-D" + e for e in extra]
@@ -78,5 +82,6 @@ if __name__ == "__main__":
     ap.add_argument("-j", type=int, default=0)
     ap.add_argument("--trace", action="store_true")
     ap.add_argument("--define", action="append", default=[])
+    ap.add_argument("--variant", default="")
     a = ap.parse_args()
-    print(build(a.force, a.j, a.trace, tuple(a.define)))
+    print(build(a.force, a.j, a.trace, tuple(a.define), a.variant))

@@ -18,7 +18,7 @@ buf = np.zeros((4, 256, 4), dtype=np.uint64)
 L = _lib.lib()
 L.winrs_trace_read.argtypes = [ctypes.c_void_p]
 print("rc", L.winrs_trace_read(buf.ctypes.data))
-t0 = min(v for v in buf.ravel() if v > 0)
+t0 = int(buf[0, 240, 0]) if buf[0, 240, 0] > 0 else min(v for v in buf.ravel() if v > 0)
 b = np.where(buf > 0, buf.astype(np.int64) - int(t0), -1)
 print(p)
 print("chunk | prod: before_wait after_wait | tx: start raw_ok op_ok done | mma: opfull issued | ft_computed it_computed ft_fenced")
@@ -27,10 +27,35 @@ for c in list(range(0, 40)) + list(range(64, 90)):
         continue
     print(c, "|", b[0, c, 0], b[0, c, 1], "|", b[2, c, 0], b[2, c, 1], b[2, c, 2], b[2, c, 3], "|", b[1, c, 0], b[1, c, 1], "|", b[3, c, 0], b[3, c, 1], b[3, c, 2])
 
-bw = np.zeros((256, 16), dtype=np.uint64)
+names = ["entry", "setup done", "last MMA commit", "tx jobs+epilogues done", "final_out done", "post-sync", "cluster reduce done"]
+print("phases (ns from t0):", {n: int(buf[0, 240 + i, 0]) - int(t0) for i, n in enumerate(names) if buf[0, 240 + i, 0] > 0})
+bw = np.zeros((256, 24, 3), dtype=np.uint64)
 L.winrs_trace_read_w.argtypes = [ctypes.c_void_p]
 L.winrs_trace_read_w(bw.ctypes.data)
-print("per-warp chunk-done times (ns from t0), warps 2..")
-for c in range(0, 12):
-    row = [int(v) - int(t0) if v > 0 else -1 for v in bw[c]]
-    print(c, row[2:14])
+slots = np.zeros(24, dtype=np.uint32)
+L.winrs_trace_read_slots.argtypes = [ctypes.c_void_p]
+L.winrs_trace_read_slots(slots.ctypes.data)
+print("warp -> %warpid:", list(slots))
+print("per-warp (raw_ok, op_ok, done) ns from t0, tx warps")
+for c in range(0, 16):
+    row = []
+    for w in range(2, 24):
+        if bw[c, w, 2] == 0:
+            continue
+        row.append("w%d:%d/%d/%d" % (w, int(bw[c, w, 0]) - int(t0), int(bw[c, w, 1]) - int(t0), int(bw[c, w, 2]) - int(t0)))
+    print(c, " ".join(row))
+
+ct = np.zeros((2048, 8), dtype=np.uint64)
+L.winrs_trace_read_cta.argtypes = [ctypes.c_void_p]
+L.winrs_trace_read_cta(ct.ctypes.data)
+n = int(p.info["ctas_main"]) if "ctas_main" in p.info else 0
+n = n or int((ct[:, 0] > 0).sum())
+c = ct[:n].astype(np.int64)
+T0 = c[:, 0].min()
+cs = p.info.get("csplit", 1)
+print("per-CTA (us from first entry): entry, setup, lastMMA, txdone, finalout, end | smid")
+for i in range(n):
+    print(i, " ".join("%.1f" % ((c[i, j] - T0) / 1e3) if c[i, j] > 0 else "-" for j in (0, 1, 2, 3, 4, 6)), "| sm", int(ct[i, 7]))
+ent, lm, end = (c[:, 0] - T0) / 1e3, (c[:, 2] - T0) / 1e3, (c[:, 6] - T0) / 1e3
+print("entry spread %.1f us; main-loop (setup->lastMMA) min %.1f max %.1f mean %.1f; end max %.1f" % (
+    ent.max(), ((c[:, 2] - c[:, 1]) / 1e3).min(), ((c[:, 2] - c[:, 1]) / 1e3).max(), ((c[:, 2] - c[:, 1]) / 1e3).mean(), end.max()))
