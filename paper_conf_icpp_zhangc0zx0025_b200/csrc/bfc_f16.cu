@@ -1,6 +1,7 @@
 // FP16 tensor-core kernel instantiations, TMA tensor-map encoding and launch.
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <cstdlib>
 #include <mutex>
 #include "bfc_f16.cuh"
 #include "launch_util.cuh"
@@ -43,8 +44,10 @@ static bool make_map(CUtensorMap* m, const void* base, int N, int H, int W, int 
 }
 
 static int images_per_box(int N) {
-    for (int nb : {8, 4, 2})
-        if (N % nb == 0) return nb;
+    // 16 (= KC: one box per tensor per chunk) measured fastest; WINRS_F16_NB caps it (A/B)
+    static const int cap = [] { const char* e = getenv("WINRS_F16_NB"); return e && *e ? atoi(e) : 16; }();
+    for (int nb : {16, 8, 4, 2})
+        if (nb <= cap && N % nb == 0) return nb;
     return 1;
 }
 

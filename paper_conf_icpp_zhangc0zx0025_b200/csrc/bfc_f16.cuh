@@ -44,6 +44,12 @@ constexpr int KC = 16;           // depth entries per chunk = UMMA K
 #ifndef WINRS_F16_SOP
 #define WINRS_F16_SOP 0          // 0: as many operand stages (<= 4) as leave 3 raw stages
 #endif
+#ifndef WINRS_F16_NATIVE
+#define WINRS_F16_NATIVE 0       // 1: Omega_4(3,2) in 16-bit arithmetic, MN-major SW128 operands (measured 6% slower on B200)
+#endif
+#ifndef WINRS_F16_RAWMAX
+#define WINRS_F16_RAWMAX 4       // cap on raw (TMA) ring stages
+#endif
 #ifndef WINRS_F16_DQ
 #define WINRS_F16_DQ 8           // depth entries per transformer unit (8: octet; 4 measured slower)
 #endif
@@ -67,6 +73,28 @@ template <int BM> __host__ __device__ constexpr int n_units() { return ft_warps<
 // hides the shared-memory latency of the transforms; measured best on B200
 // (A/B of 8..16 warps over the ResNet-50 / VGG-16 layers): 10 warps for the
 // 128x64 / 128x32 tiles, 14 for 128x128.
+// ---- native path (Omega_4(3,2), B_M a multiple of 64).  Every output of
+// this kernel's FT (G w) and IT (D^T x) is one add or subtract of two inputs
+// followed by an exact halving, so computing it in the input's own 16-bit
+// arithmetic (one fused rounding, HFMA2) gives the correctly rounded FP16 /
+// BF16 operand — what P@38729's "computed in FP32, then converted" produces,
+// without the FP32 unpack / repack.  Operands are then stored MN-major (k or
+// c contiguous, the raw TMA order) in the 128-byte-swizzled canonical UMMA
+// layout, so a thread moves 8 channels per 16-byte load and store.
+template <int A0, int N0, int R0, int A1, int BM>
+__host__ __device__ constexpr bool native_path() {
+    return WINRS_F16_NATIVE && A0 == 4 && N0 == 3 && R0 == 2 && A1 == 0 && BM % 64 == 0 && WINRS_F16_DYN;
+}
+#ifndef WINRS_NAT_IPT
+#define WINRS_NAT_IPT 4
+#endif
+constexpr int NAT_IPT = WINRS_NAT_IPT;   // (channel octet, depth) items per thread per unit
+template <int BM> __host__ __device__ constexpr int nat_ft_units() { return (BN / 8) * KC / (32 * NAT_IPT); }
+template <int BM> __host__ __device__ constexpr int nat_it_units() { return (BM / 8) * KC / (32 * NAT_IPT); }
+template <int BM, bool NAT> __host__ __device__ constexpr int units_per_chunk() {
+    return NAT ? nat_ft_units<BM>() + nat_it_units<BM>() : n_units<BM>();
+}
+
 template <int BM> __host__ __device__ constexpr int tx_warps() {
     return !WINRS_F16_DYN ? n_units<BM>() : WINRS_F16_TXW > 0 ? WINRS_F16_TXW : BM >= 128 ? 14 : 10;
 }
@@ -96,15 +124,28 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
 // waiting warp sleep in hardware until the phase completes instead of
 // re-polling, so idle producer / MMA warps do not steal issue slots from the
 // transformer warps sharing their SM sub-partition.
+#ifndef WINRS_WAIT_HINT
+#define WINRS_WAIT_HINT 1000000
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     const uint32_t a = smem_u32(bar);
+#if WINRS_WAIT_HINT > 0
     asm volatile(
         "{\n"
         ".reg .pred P;\n"
         "WAIT_%=:\n"
         "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1, %2;\n"
         "@!P bra WAIT_%=;\n"
-        "}\n" :: "r"(a), "r"(parity), "r"(1000000) : "memory");
+        "}\n" :: "r"(a), "r"(parity), "r"(WINRS_WAIT_HINT) : "memory");
+#else
+    asm volatile(
+        "{\n"
+        ".reg .pred P;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n"
+        "@!P bra WAIT_%=;\n"
+        "}\n" :: "r"(a), "r"(parity) : "memory");
+#endif
 }
 __device__ __forceinline__ void tma_load_4d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
                                             int c2, int c3) {
@@ -129,18 +170,26 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint
 }
 // kind::f16 instruction descriptor: D f32, A/B f16, both K-major, M = 128, N = BM.
 // A/B format field (bits 7-9, 10-12): 0 = F16, 1 = BF16.
-template <int BM, bool BF>
+// Bits 15 / 16: A / B MN-major (the native path).
+template <int BM, bool BF, bool MN = false>
 __host__ __device__ constexpr uint32_t idesc() {
-    return (1u << 4) | ((BF ? 1u : 0u) << 7) | ((BF ? 1u : 0u) << 10) | ((uint32_t)(BM >> 3) << 17) |
-           ((uint32_t)(BN >> 4) << 24);
+    return (1u << 4) | ((BF ? 1u : 0u) << 7) | ((BF ? 1u : 0u) << 10) | ((MN ? 1u : 0u) << 15) | ((MN ? 1u : 0u) << 16) |
+           ((uint32_t)(BM >> 3) << 17) | ((uint32_t)(BN >> 4) << 24);
+}
+// MN-major, 128-byte swizzle (layout type 2): atoms of 64 MN elements x 8 K
+// rows (1 KB); LBO = byte stride between MN atoms, SBO = between K atoms
+// (probed on B200: tools/microbench/umma_mn.cu).  Atom bases 1 KB aligned.
+__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+           ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46) | (2ull << 61);
 }
 
-template <int BM, bool BF>
+template <int BM, bool BF, bool MN = false>
 __device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t accumulate) {
     asm volatile(
         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
-        :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(idesc<BM, BF>()), "r"(accumulate));
+        :: "r"(tmem_d), "l"(adesc), "l"(bdesc), "r"(idesc<BM, BF, MN>()), "r"(accumulate));
 }
 __device__ __forceinline__ void umma_commit(uint64_t* bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
@@ -199,8 +248,8 @@ struct Smem {
     static constexpr int S_OP = WINRS_F16_SOP > 0 ? WINRS_F16_SOP
                               : (LIMIT - 4 * OP) / RAW >= 3 ? 4 : (LIMIT - 3 * OP) / RAW >= 3 ? 3 : 2;
     // as many raw (TMA) stages as fit: the raw ring is the latency-hiding depth
-    static constexpr int S_RAW = (LIMIT - S_OP * OP) / RAW > 4 ? 4 : (LIMIT - S_OP * OP) / RAW;
-    static_assert(S_RAW >= 2, "shared memory too small for a 2-stage raw ring");
+    static constexpr int S_RAW = (LIMIT - S_OP * OP) / RAW > WINRS_F16_RAWMAX ? WINRS_F16_RAWMAX : (LIMIT - S_OP * OP) / RAW;
+    static_assert(S_RAW >= 2 && S_RAW <= 8, "raw ring: 2..8 stages");
     static constexpr int raw_off = 0;
     static constexpr int op_off = S_RAW * RAW;
     static constexpr int bar_off = op_off + S_OP * OP;
@@ -250,7 +299,7 @@ struct Job {
 };
 
 struct Barriers {
-    uint64_t raw_full[4], raw_empty[4], op_full[4], op_empty[4], acc_full, acc_empty;
+    uint64_t raw_full[8], raw_empty[8], op_full[4], op_empty[4], acc_full, acc_empty;
     uint32_t tmem_base;
     int unit_ctr;       // next transform unit (dynamic scheduling)
 };
@@ -275,9 +324,15 @@ __device__ __forceinline__ void depth_coord(int d, int N, int units, int hs, int
 // free through perm16.  FT and IT warps are interleaved so every SM
 // sub-partition (warp % 4) gets the same mix.
 
-template <int WT_FN, int A, int NN, int RR, int NIN, int DQ, bool BF>
+// `mid()` runs between the transform (raw ring -> registers) and the operand
+// stores: the caller releases the raw stage there and waits for the operand
+// stage to be free, so the transform math of chunk c+S_OP overlaps the MMAs
+// of chunk c instead of waiting for them.
+struct NoMid { __device__ __forceinline__ void operator()() const {} };
+
+template <int WT_FN, int A, int NN, int RR, int NIN, int DQ, bool BF, class Mid>
 __device__ __forceinline__ void unit_transform(const uint16_t* src, int tap_stride, int depth_stride, uint8_t* dst0,
-                                               int slab_bytes, int p, int grp) {
+                                               int slab_bytes, int p, int grp, const Mid& mid) {
     using WT = Wino<A, NN, RR>;
     const int oct = grp;     // depth group index (DQ entries each)
     uint32_t pk[A][2][DQ / 2];   // [xi][row 2p / 2p+1][half2 of depth (2j, 2j+1)]
@@ -299,6 +354,7 @@ __device__ __forceinline__ void unit_transform(const uint16_t* src, int tap_stri
 #pragma unroll
         for (int x = 0; x < A; ++x) pk[x][1][j] = Elem<BF>::pack(o[x].x, o[x].y);
     }
+    mid();
     // depth group -> K position kk0 = grp*DQ: K half kk0/8, byte offset (kk0%8)*2 in the 16-byte row
     const int kk0 = grp * DQ;
 #pragma unroll
@@ -338,23 +394,24 @@ __device__ __forceinline__ int tx_role(int tw) {
 // transforms: those operand rows stay zero (the op ring is cleared once at
 // kernel start) and their accumulator rows are never written out.
 // role >= 0: IT unit `role`; role < 0: FT unit -1 - role.
-template <int A, int NN, int RR, int BM, bool BF>
-__device__ __forceinline__ void transform_role(const uint8_t* raw, uint8_t* op, int role, int lane, int kv, int cv) {
+template <int A, int NN, int RR, int BM, bool BF, class Mid = NoMid>
+__device__ __forceinline__ void transform_role(const uint8_t* raw, uint8_t* op, int role, int lane, int kv, int cv,
+                                               const Mid& mid = Mid()) {
     constexpr int RAW_Y = KC * RR * BN * 2;
     const uint16_t* rawY = reinterpret_cast<const uint16_t*>(raw);            // [KC][RR][BN]
     const uint16_t* rawX = reinterpret_cast<const uint16_t*>(raw + RAW_Y);    // [KC][A][BM]
     constexpr int OPA = BN * KC * 2, OPB = BM * KC * 2;
     if (role < 0) {
         const int f = -1 - role;   // FT warp: 32 k pairs x one octet
-        if ((f % (BN / 64)) * 64 >= kv) return;
+        if ((f % (BN / 64)) * 64 >= kv) { mid(); return; }
         unit_transform<0, A, NN, RR, RR, DQ_FT, BF>(rawY, BN, RR * BN, op, OPA, (f % (BN / 64)) * 32 + lane,
-                                                f / (BN / 64));
+                                                f / (BN / 64), mid);
     } else {                       // IT warp: 32 c pairs (or BM/2 pairs x 32/(BM/2) quads) x quads
         constexpr int PW = BM / 2 < 32 ? BM / 2 : 32;
         const int q = (role % ((BM / 2) / PW)) * PW + (lane % PW);
         const int quad = role / ((BM / 2) / PW) * (32 / PW) + lane / PW;
-        if ((role % ((BM / 2) / PW)) * PW * 2 >= cv) return;
-        unit_transform<1, A, NN, RR, A, DQ_IT, BF>(rawX, BM, A * BM, op + A * OPA, OPB, q, quad);
+        if ((role % ((BM / 2) / PW)) * PW * 2 >= cv) { mid(); return; }
+        unit_transform<1, A, NN, RR, A, DQ_IT, BF>(rawX, BM, A * BM, op + A * OPA, OPB, q, quad, mid);
     }
 }
 // Static schedule: transformer warp tw always runs the same unit.
@@ -363,9 +420,132 @@ __device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op,
     transform_role<A, NN, RR, BM, BF>(raw, op, tx_role<BM>(tw), lane, kv, cv);
 }
 // Dynamic schedule: unit u of a chunk, the (costlier) IT units first.
-template <int A, int NN, int RR, int BM, bool BF>
-__device__ __forceinline__ void transform_unit(const uint8_t* raw, uint8_t* op, int u, int lane, int kv, int cv) {
-    transform_role<A, NN, RR, BM, BF>(raw, op, u < it_warps<BM>() ? u : -1 - (u - it_warps<BM>()), lane, kv, cv);
+template <int A, int NN, int RR, int BM, bool BF, class Mid>
+__device__ __forceinline__ void transform_unit(const uint8_t* raw, uint8_t* op, int u, int lane, int kv, int cv,
+                                               const Mid& mid) {
+    transform_role<A, NN, RR, BM, BF>(raw, op, u < it_warps<BM>() ? u : -1 - (u - it_warps<BM>()), lane, kv, cv, mid);
+}
+
+// 16-bit pair arithmetic for the native path.
+template <bool BF> struct H2;
+template <> struct H2<false> {
+    typedef __half2 T;
+    __device__ static __forceinline__ T c(float v) { return __float2half2_rn(v); }
+};
+template <> struct H2<true> {
+    typedef __nv_bfloat162 T;
+    __device__ static __forceinline__ T c(float v) { return __float2bfloat162_rn(v); }
+};
+template <bool BF>
+__device__ __forceinline__ uint4 h2_scale(uint4 a, typename H2<BF>::T k) {
+    typedef typename H2<BF>::T T;
+    uint4 r;
+    T* ra = reinterpret_cast<T*>(&r);
+    const T* aa = reinterpret_cast<const T*>(&a);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) ra[i] = __hmul2(aa[i], k);
+    return r;
+}
+template <bool BF>   // a * k + b, one rounding per element
+__device__ __forceinline__ uint4 h2_fma(uint4 a, typename H2<BF>::T k, uint4 b) {
+    typedef typename H2<BF>::T T;
+    uint4 r;
+    T* ra = reinterpret_cast<T*>(&r);
+    const T* aa = reinterpret_cast<const T*>(&a);
+    const T* bb = reinterpret_cast<const T*>(&b);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) ra[i] = __hfma2(aa[i], k, bb[i]);
+    return r;
+}
+template <bool BF>
+__device__ __forceinline__ uint4 h2_neg(uint4 a) {
+    typedef typename H2<BF>::T T;
+    uint4 r;
+    T* ra = reinterpret_cast<T*>(&r);
+    const T* aa = reinterpret_cast<const T*>(&a);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) ra[i] = __hneg2(aa[i]);
+    return r;
+}
+
+// Byte offset of the 16-byte (8-channel) group g at depth d in an MN-major
+// SW128 operand slab whose MN extent is `mn` channels (K = KC = 16).
+template <int MNEXT>
+__device__ __forceinline__ uint32_t nat_off(int g, int d) {
+    return (uint32_t)((g >> 3) * 1024 + (d >> 3) * (MNEXT / 64) * 1024 + (d & 7) * 128 + (((g & 7) ^ (d & 7)) << 4));
+}
+
+// One native unit: NAT_IPT (channel octet, depth) items per lane.  IT units
+// (X, B operand) come first, then FT units (dY, A operand).  A quarter-warp
+// covers 8 consecutive octets at one depth: 128 contiguous raw bytes per
+// load, 8 distinct swizzled 16-byte chunks per store (conflict free).
+template <int BM, bool BF, class Mid>
+__device__ __forceinline__ void native_unit(const uint8_t* raw, uint8_t* op, int u, int lane, int kv, int cv,
+                                            const Mid& mid) {
+    constexpr int A = 4, RR = 2;
+    constexpr int RAW_Y = KC * RR * BN * 2;
+    constexpr int OPA = BN * KC * 2, OPB = BM * KC * 2;
+    typedef typename H2<BF>::T T;
+    const T half = H2<BF>::c(0.5f), mhalf = H2<BF>::c(-0.5f);
+    if (u < nat_it_units<BM>()) {
+        // IT, Omega_4(3,2): o0 = (x2+x1)/2, o1 = (x2-x1)/2, o2 = (x0-x2)/2, o3 = (x3-x1)/2
+        constexpr int G = BM / 8;
+        uint4 o[NAT_IPT][A];
+        int gg[NAT_IPT], dd[NAT_IPT];
+#pragma unroll
+        for (int i = 0; i < NAT_IPT; ++i) {
+            const int idx = (u * NAT_IPT + i) * 32 + lane;
+            gg[i] = idx % G;
+            dd[i] = idx / G;
+            if (gg[i] * 8 < cv) {
+                const uint4* x = reinterpret_cast<const uint4*>(raw + RAW_Y + ((dd[i] * A) * BM + gg[i] * 8) * 2);
+                const uint4 x0 = x[0], x1 = x[BM / 8], x2 = x[2 * (BM / 8)], x3 = x[3 * (BM / 8)];
+                const uint4 x2h = h2_scale<BF>(x2, half), x1h = h2_scale<BF>(x1, half);
+                o[i][0] = h2_fma<BF>(x1, half, x2h);
+                o[i][1] = h2_fma<BF>(x1, mhalf, x2h);
+                o[i][2] = h2_fma<BF>(x0, half, h2_neg<BF>(x2h));
+                o[i][3] = h2_fma<BF>(x3, half, h2_neg<BF>(x1h));
+            }
+        }
+        mid();
+#pragma unroll
+        for (int i = 0; i < NAT_IPT; ++i)
+            if (gg[i] * 8 < cv) {
+                uint8_t* b = op + A * OPA + nat_off<BM>(gg[i], dd[i]);
+#pragma unroll
+                for (int x = 0; x < A; ++x) *reinterpret_cast<uint4*>(b + x * OPB) = o[i][x];
+            }
+    } else {
+        // FT, Omega_4(3,2): o0 = (w0+w1)/2, o1 = (w0-w1)/2, o2 = w0, o3 = w1
+        constexpr int G = BN / 8;
+        const int f = u - nat_it_units<BM>();
+        uint4 o[NAT_IPT][2], w0s[NAT_IPT], w1s[NAT_IPT];
+        int gg[NAT_IPT], dd[NAT_IPT];
+#pragma unroll
+        for (int i = 0; i < NAT_IPT; ++i) {
+            const int idx = (f * NAT_IPT + i) * 32 + lane;
+            gg[i] = idx % G;
+            dd[i] = idx / G;
+            if (gg[i] * 8 < kv) {
+                const uint4* w = reinterpret_cast<const uint4*>(raw + ((dd[i] * RR) * BN + gg[i] * 8) * 2);
+                w0s[i] = w[0];
+                w1s[i] = w[BN / 8];
+                const uint4 e = h2_scale<BF>(w0s[i], half);
+                o[i][0] = h2_fma<BF>(w1s[i], half, e);
+                o[i][1] = h2_fma<BF>(w1s[i], mhalf, e);
+            }
+        }
+        mid();
+#pragma unroll
+        for (int i = 0; i < NAT_IPT; ++i)
+            if (gg[i] * 8 < kv) {
+                uint8_t* b = op + nat_off<BN>(gg[i], dd[i]);
+                *reinterpret_cast<uint4*>(b) = o[i][0];
+                *reinterpret_cast<uint4*>(b + OPA) = o[i][1];
+                *reinterpret_cast<uint4*>(b + 2 * OPA) = w0s[i];
+                *reinterpret_cast<uint4*>(b + 3 * OPA) = w1s[i];
+            }
+    }
 }
 
 __device__ __forceinline__ void tmem_st8(uint32_t taddr, const float* v) {
@@ -445,11 +625,11 @@ template <int A0, int N0, int R0, int BM> __host__ __device__ constexpr size_t s
 // the shared-memory staging tile (cluster split).  Undoes the operand row
 // permutation: TMEM lane L holds k = iperm16(L); physical columns
 // [16b, 16b+16) hold logical c = 16b + 2i (first 8) and 16b + 2i + 1 (last 8).
-template <int N0, int BM>
+template <int N0, int BM, bool NAT = false>
 __device__ __forceinline__ void final_out(const Geometry& g, float* bucket, const CtaCoord& cc, int fw0, uint32_t tmem_base,
                                           int warp, float* Out) {
     const int quarter = warp & 3, lane = threadIdx.x & 31;
-    const int kl = iperm16(quarter * 32 + lane);
+    const int kl = NAT ? quarter * 32 + lane : iperm16(quarter * 32 + lane);
     const int kg = cc.kb * BN + kl;
     const uint32_t lane_base = tmem_base + ((uint32_t)(quarter * 32) << 16);
 #pragma unroll 1
@@ -462,8 +642,8 @@ __device__ __forceinline__ void final_out(const Geometry& g, float* bucket, cons
             tmem_wait_ld();
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
-                y[2 * i] = ph[i];
-                y[2 * i + 1] = ph[8 + i];
+                y[NAT ? i : 2 * i] = ph[i];
+                y[NAT ? 8 + i : 2 * i + 1] = ph[8 + i];
             }
             if (g.csplit > 1) {
                 float4* o = reinterpret_cast<float4*>(Out + ((long long)j * BN + kl) * out_ld<BM>() + c0);
@@ -515,6 +695,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     constexpr int TX_WARPS = tx_warps<BM>();
     static_assert(A1 * BM <= stash_col<N0, BM>(), "residual accumulators overlap the TMEM output stash");
     constexpr bool kCluster = csplit_fits<N0, BM>();
+    constexpr bool NAT = native_path<A0, N0, R0, A1, BM>();
     extern __shared__ __align__(1024) uint8_t smem[];
     const Geometry& g = args.g;
     Barriers* bars = reinterpret_cast<Barriers*>(smem + SM::bar_off);
@@ -555,7 +736,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     };
 
     if (threadIdx.x == 0) {
-        constexpr int NU = n_units<BM>();
+        constexpr int NU = units_per_chunk<BM, NAT>();
         for (int s = 0; s < S_RAW; ++s) { mbar_init(&bars->raw_full[s], 1); mbar_init(&bars->raw_empty[s], NU); }
         for (int s = 0; s < SM::S_OP; ++s) { mbar_init(&bars->op_full[s], NU); mbar_init(&bars->op_empty[s], 1); }
         bars->unit_ctr = 0;
@@ -608,24 +789,42 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             int c_lo, c_hi;
             chunk_range(J, &c_lo, &c_hi);
             const uint32_t bytes = (uint32_t)(KC * (RRj * BN + Aj * BM) * 2);
+            // This lane's box start d = ch*KC + b and its (n, h, u), advanced
+            // incrementally (one division per job, not per chunk: the
+            // producer shares its SM sub-partition with transformer warps).
+            const int b = (lane >> 1) * args.nb;
+            int d = c_lo * KC + b, n = 0, h = hs, u = 0;
+            if (d < depth) depth_coord(d, g.N, J.units, hs, &n, &h, &u);
             for (int ch = c_lo; ch < c_hi; ++ch) {
                 if (lane == 0) TRACE(0, ch - c_lo + jb * 64, 0);
                 mbar_wait(&bars->raw_empty[s], ph ^ 1);
                 if (lane == 0) TRACE(0, ch - c_lo + jb * 64, 1);
                 uint8_t* raw = smem + SM::raw_off + s * SM::RAW;
+#ifdef WINRS_NO_TMA   // debug: the raw ring carries no data (pipeline-only timing)
+                if (lane == 0) mbar_arrive(&bars->raw_full[s]);
+                (void)bytes; (void)raw; (void)mX; (void)mY;
+                if (false) {
+#else
                 if (lane == 0) mbar_arrive_expect_tx(&bars->raw_full[s], bytes);
                 __syncwarp();
                 if (lane < nbox) {
-                    const int b = (lane >> 1) * args.nb;
-                    const int d = ch * KC + b;
-                    int n = g.N, h = hs, u = 0;   // past-the-end image => zero fill
-                    if (d < depth) depth_coord(d, g.N, J.units, hs, &n, &h, &u);
-                    const int w0 = J.w_first + u * RRj;
+#endif
+                    const bool in = d < depth;     // past-the-end image => zero fill
+                    const int nn = in ? n : g.N, hh = in ? h : hs;
+                    const int w0 = J.w_first + (in ? u : 0) * RRj;
                     if ((lane & 1) == 0)
-                        tma_load_4d(raw + b * RRj * BN * 2, mY, &bars->raw_full[s], cc.kb * BN, w0, h, n);
+                        tma_load_4d(raw + b * RRj * BN * 2, mY, &bars->raw_full[s], cc.kb * BN, w0, hh, nn);
                     else
                         tma_load_4d(raw + KC * RRj * BN * 2 + b * Aj * BM * 2, mX, &bars->raw_full[s], cc.cb * BM,
-                                    w0 + J.fw0 - g.pad, h + cc.fh - g.pad, n);
+                                    w0 + J.fw0 - g.pad, hh + cc.fh - g.pad, nn);
+                    if (lane == 0) TRACE(0, ch - c_lo + jb * 64, 2);
+                    if (lane == 1) TRACE(0, ch - c_lo + jb * 64, 3);
+                }
+                d += KC;
+                n += KC;
+                while (n >= g.N) {
+                    n -= g.N;
+                    if (++u == J.units) { u = 0; ++h; }
                 }
                 if (++s == S_RAW) { s = 0; ph ^= 1; }
             }
@@ -635,6 +834,12 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         if (lane == 0) {
             int s = 0;
             uint32_t ph = 0;
+            // descriptors differ only in the start-address field (16-byte units,
+            // 14 bits: no carry for addresses < 256 KB)
+            const uint64_t desc0 = NAT ? umma_desc_sw128(smem_u32(smem + SM::op_off), 1024, 2048)
+                                       : umma_desc(smem_u32(smem + SM::op_off), 128, 256);
+            // B slabs: SBO (K-atom stride) = (BM / 64) KB instead of 2 KB
+            const uint64_t bsbo_fix = NAT ? ((uint64_t)(((BM / 64) * 1024) >> 4) << 32) - ((uint64_t)(2048 >> 4) << 32) : 0;
             for (int jb = 0; jb < njobs; ++jb) {
                 const Job& J = jobs[jb];
                 const int Aj = J.phase == 0 ? A0 : A1;
@@ -648,17 +853,21 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     mbar_wait(&bars->op_full[s], ph);
                     TRACE(1, ch - c_lo + jb * 64, 0);
                     tc_fence_after();
-                    const uint32_t base = smem_u32(smem + SM::op_off + s * SM::OP);
+                    const uint64_t dstage = desc0 + (uint64_t)((s * SM::OP) >> 4);
                     for (int x = 0; x < Aj; ++x) {
-                        const uint64_t ad = umma_desc(base + x * SM::OPA, 128, 256);
-                        const uint64_t bd = umma_desc(base + Aj * SM::OPA + x * SM::OPB, 128, 256);
+                        const uint64_t ad = dstage + (uint64_t)((x * SM::OPA) >> 4);
+                        const uint64_t bd = dstage + (uint64_t)((Aj * SM::OPA + x * SM::OPB) >> 4) + bsbo_fix;
 #ifndef WINRS_NO_MMA
-                        umma_f16<BM, BF>(tmem_base + (uint32_t)(x * BM), ad, bd, ch > c_lo ? 1u : 0u);
+                        umma_f16<BM, BF, NAT>(tmem_base + (uint32_t)(x * BM), ad, bd, ch > c_lo ? 1u : 0u);
 #else
                         (void)ad; (void)bd;
 #endif
                     }
+#ifdef WINRS_NO_COMMIT   // debug (with WINRS_NO_MMA only): release the stage without the tensor-core round trip
+                    mbar_arrive(&bars->op_empty[s]);
+#else
                     umma_commit(&bars->op_empty[s]);
+#endif
                     TRACE(1, ch - c_lo + jb * 64, 1);
                     if (++s == SM::S_OP) { s = 0; ph ^= 1; }
                 }
@@ -674,7 +883,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         // sub-partition takes more: the chunk rate follows the average unit
         // cost instead of the slowest fixed role.  Ring stage / parity follow
         // from the global chunk index, as in the producer and MMA loops.
-        constexpr int NU = n_units<BM>();
+        constexpr int NU = units_per_chunk<BM, NAT>();
         const int kv = g.K - cc.kb * BN, cv = g.C - cc.cb * BM;
         int jlo[1 + 9], jhi[1 + 9];
         for (int jb = 0; jb < njobs; ++jb) chunk_range(jobs[jb], &jlo[jb], &jhi[jb]);
@@ -713,28 +922,41 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
 #ifdef WINRS_TRACE
             if (lane == 0 && blockIdx.x == 0 && gch < 256) g_trace_w[gch][warp][0] = gtime();
 #endif
-            mbar_wait(&bars->op_empty[so], (uint32_t)(((gch / SM::S_OP) & 1) ^ 1));
-#ifdef WINRS_TRACE
-            if (lane == 0 && blockIdx.x == 0 && gch < 256) g_trace_w[gch][warp][1] = gtime();
-#endif
             const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
             uint8_t* op = smem + SM::op_off + so * SM::OP;
-            if (jobs[jb].phase == 0) transform_unit<A0, N0, R0, BM, BF>(raw, op, u, lane, kv, cv);
-            else if constexpr (A1 != 0) transform_unit<A1, N1, R1, BM, BF>(raw, op, u, lane, kv, cv);
+            // between transform and stores: every lane's raw reads are done
+            // (their values are in registers) -> release the raw stage; then
+            // wait for the MMAs of the chunk that last used this operand stage.
+            // A skipped unit also waits, so its op_full arrival cannot land in
+            // the previous phase of the stage.
+            const auto mid = [&]() {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&bars->raw_empty[sr]);
+                mbar_wait(&bars->op_empty[so], (uint32_t)(((gch / SM::S_OP) & 1) ^ 1));
+#ifdef WINRS_TRACE
+                if (lane == 0 && blockIdx.x == 0 && gch < 256) g_trace_w[gch][warp][1] = gtime();
+#endif
+            };
+#ifdef WINRS_NO_TX     // debug: transformer units keep only the barrier protocol
+            if (true) mid();
+            else
+#endif
+            if constexpr (NAT) native_unit<BM, BF>(raw, op, u, lane, kv, cv, mid);
+            else if (jobs[jb].phase == 0) transform_unit<A0, N0, R0, BM, BF>(raw, op, u, lane, kv, cv, mid);
+            else if constexpr (A1 != 0) transform_unit<A1, N1, R1, BM, BF>(raw, op, u, lane, kv, cv, mid);
+#ifndef WINRS_NO_FENCE
             fence_proxy_async();
+#endif
             __syncwarp();
 #ifdef WINRS_TRACE
             if (lane == 0 && blockIdx.x == 0 && gch < 256) g_trace_w[gch][warp][2] = gtime();
 #endif
-            if (lane == 0) {
-                mbar_arrive(&bars->op_full[so]);
-                mbar_arrive(&bars->raw_empty[sr]);
-            }
+            if (lane == 0) mbar_arrive(&bars->op_full[so]);
         }
         if (threadIdx.x == 64) PTRACE(3);
         asm volatile("bar.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
         if (warp < 6) {
-            final_out<N0, BM>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
+            final_out<N0, BM, NAT>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
             if (threadIdx.x == 64) PTRACE(4);
         }
     } else {

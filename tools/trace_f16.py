@@ -25,7 +25,7 @@ print("chunk | prod: before_wait after_wait | tx: start raw_ok op_ok done | mma:
 for c in list(range(0, 40)) + list(range(64, 90)):
     if b[2, c, 0] < 0 and b[0, c, 0] < 0:
         continue
-    print(c, "|", b[0, c, 0], b[0, c, 1], "|", b[2, c, 0], b[2, c, 1], b[2, c, 2], b[2, c, 3], "|", b[1, c, 0], b[1, c, 1], "|", b[3, c, 0], b[3, c, 1], b[3, c, 2])
+    print(c, "|", b[0, c, 0], b[0, c, 1], b[0, c, 2], b[0, c, 3], "|", b[2, c, 0], b[2, c, 1], b[2, c, 2], b[2, c, 3], "|", b[1, c, 0], b[1, c, 1], "|", b[3, c, 0], b[3, c, 1], b[3, c, 2])
 
 names = ["entry", "setup done", "last MMA commit", "tx jobs+epilogues done", "final_out done", "post-sync", "cluster reduce done"]
 print("phases (ns from t0):", {n: int(buf[0, 240 + i, 0]) - int(t0) for i, n in enumerate(names) if buf[0, 240 + i, 0] > 0})
