@@ -47,6 +47,13 @@ constexpr int KC = 16;           // depth entries per chunk = UMMA K
 #ifndef WINRS_F16_NATIVE
 #define WINRS_F16_NATIVE 0       // 1: Omega_4(3,2) in 16-bit arithmetic, MN-major SW128 operands (measured 6% slower on B200)
 #endif
+#ifndef WINRS_F16_PUSH
+#define WINRS_F16_PUSH 0         // 1: fused epilogue + one-way DSMEM push reduction for cluster-split single-job tiles (measured: no gain, DSMEM-bandwidth bound either way)
+#endif
+#ifndef WINRS_F16_RR
+#define WINRS_F16_RR 2           // 1: static round-robin unit assignment instead of the shared counter; 2: for alpha = 4 only
+                                 // (measured on B200: round-robin 6-12% faster for alpha = 4, 15% slower for alpha = 8)
+#endif
 #ifndef WINRS_F16_RAWMAX
 #define WINRS_F16_RAWMAX 4       // cap on raw (TMA) ring stages
 #endif
@@ -685,6 +692,101 @@ __device__ __forceinline__ void cluster_reduce(const Geometry& g, float* bucket,
     asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
+// ---- fused epilogue + cluster reduction (single-job tiles with a cluster
+// depth split).  After barrier B1 (every rank is past its main loop, so every
+// rank's rings are free), 12 transformer warps — three per TMEM lane quarter,
+// each a third of the column groups — read the accumulators, run the OT
+// (FP32) and store each output row straight into the receive buffer of the
+// rank that owns that row: rank s owns physical rows [s*ROWS/cs, (s+1)*ROWS/cs)
+// (row = j*B_N + TMEM lane) and receives them as [source rank][row][column].
+// The stores are one-way DSMEM traffic (no staging tile, no round-trip
+// loads).  After barrier B2 each rank sums its rows over the source ranks in
+// the fixed order 0..cs-1 (the same order as cluster_reduce: bitwise equal)
+// and writes them to the bucket, undoing the operand row / column
+// permutation of the K-major path.
+template <int BM> __host__ __device__ constexpr int push_warps() { return tx_warps<BM>() >= 12 ? 12 : 8; }
+template <int A, int NN, int RR, int N0, int BM, bool NAT>
+__device__ __forceinline__ void cluster_push_reduce(const Geometry& g, float* bucket, const CtaCoord& cc, int fw0,
+                                                    int rank, uint32_t tmem_base, bool empty, float* Rcv, int nthreads_) {
+    using WT = Wino<A, NN, RR>;
+    constexpr int ROWS = N0 * BN, LD = out_ld<BM>();
+    const int cs = g.csplit, slice = ROWS / cs;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");   // B1
+    tc_fence_after();
+    constexpr int PUSH_WARPS = push_warps<BM>();
+    if (warp >= 2 && warp < 2 + PUSH_WARPS) {
+        const int q = warp & 3, part = (warp - 2) >> 2;
+        const uint32_t lane_base = tmem_base + ((uint32_t)(q * 32) << 16);
+        const uint32_t rcv = smem_u32(Rcv);
+#pragma unroll 1
+        for (int cg = part; cg < BM / 8; cg += PUSH_WARPS / 4) {
+            float v[A][8];
+            if (!empty) {
+#pragma unroll
+                for (int x = 0; x < A; ++x) tmem_ld8(lane_base + (uint32_t)(x * BM + cg * 8), v[x]);
+                tmem_wait_ld();
+            } else {
+#pragma unroll
+                for (int x = 0; x < A; ++x)
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) v[x][i] = 0.f;
+            }
+            float y[NN][8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                float vv[A], yy[NN];
+#pragma unroll
+                for (int x = 0; x < A; ++x) vv[x] = v[x][i];
+                WT::ot(vv, yy);
+#pragma unroll
+                for (int j = 0; j < NN; ++j) y[j][i] = yy[j];
+            }
+#pragma unroll
+            for (int j = 0; j < NN; ++j) {
+                const int prow = j * BN + q * 32 + lane;
+                const int owner = prow / slice;
+                const uint32_t off = (uint32_t)((((rank * slice) + (prow - owner * slice)) * LD + cg * 8) * 4);
+                uint32_t remote;
+                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(rcv + off), "r"(owner));
+                asm volatile("st.shared::cluster.v4.f32 [%0], {%1, %2, %3, %4};"
+                             :: "r"(remote), "f"(y[j][0]), "f"(y[j][1]), "f"(y[j][2]), "f"(y[j][3]) : "memory");
+                asm volatile("st.shared::cluster.v4.f32 [%0], {%1, %2, %3, %4};"
+                             :: "r"(remote + 16), "f"(y[j][4]), "f"(y[j][5]), "f"(y[j][6]), "f"(y[j][7]) : "memory");
+            }
+        }
+    }
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");   // B2
+    // local sum of my rows: item = (row r of my slice, logical 4-column group m)
+    const int r_lo = rank * slice;
+    for (int p = (int)threadIdx.x; p < slice * (BM / 4); p += nthreads_) {
+        const int r = p / (BM / 4), m = p % (BM / 4);
+        const int prow = r_lo + r;
+        const int j = prow / BN, L = prow % BN;
+        const int kl = NAT ? L : iperm16(L);
+        // logical columns 4m..4m+3 -> physical columns (K-major path: block
+        // b = 4m/16, t = 4m%16 -> physical 16b + t/2 + {0, 8, 1, 9})
+        const int b16 = (4 * m) >> 4, t = (4 * m) & 15;
+        const int p0 = NAT ? 4 * m : 16 * b16 + (t >> 1);
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int src = 0; src < cs; ++src) {
+            const float* row = Rcv + (size_t)(src * slice + r) * LD;
+            float4 e;
+            if (NAT) {
+                e = *reinterpret_cast<const float4*>(row + p0);
+            } else {
+                const float2 a = *reinterpret_cast<const float2*>(row + p0);
+                const float2 c = *reinterpret_cast<const float2*>(row + p0 + 8);
+                e = make_float4(a.x, c.x, a.y, c.y);
+            }
+            acc.x += e.x; acc.y += e.y; acc.z += e.z; acc.w += e.w;
+        }
+        const int kg = cc.kb * BN + kl, cgl = cc.cb * BM + 4 * m;
+        if (kg < g.K && cgl < g.C)
+            *reinterpret_cast<float4*>(bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0 + j) * g.C + cgl) = acc;
+    }
+}
+
 template <int A0, int N0, int R0, int A1, int N1, int R1, int BM, bool BF>
 __global__ void __launch_bounds__(nthreads<BM>(), 1)
 bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX0,
@@ -729,6 +831,9 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         if (has_residual(g, cc.col))
             for (int j = 0; j < N0 / N1; ++j) jobs[njobs++] = Job{1, g.k1, g.res_col0, fw0 + j * N1, true};
     }
+    // single-job tile with a cluster split: fused epilogue + push reduction
+    const bool fused = kCluster && WINRS_F16_PUSH && WINRS_F16_DYN && njobs == 1 && g.csplit > 1 &&
+                       TX_WARPS >= push_warps<BM>();
     // this cluster rank's chunk range of a job
     auto chunk_range = [&](const Job& J, int* lo, int* hi) {
         const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
@@ -887,7 +992,8 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         const int kv = g.K - cc.kb * BN, cv = g.C - cc.cb * BM;
         int jlo[1 + 9], jhi[1 + 9];
         for (int jb = 0; jb < njobs; ++jb) chunk_range(jobs[jb], &jlo[jb], &jhi[jb]);
-        int jb = 0, unit_base = 0, gch_base = 0, epi = 0;
+        int jb = 0, unit_base = 0, gch_base = 0, epi = 0, rr_iter = 0;
+        (void)rr_iter;
         auto run_epilogue = [&](int e) {
             const Job& J = jobs[e];
             mbar_wait(&bars->acc_full, (uint32_t)(e & 1));
@@ -903,16 +1009,21 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         };
         for (;;) {
             int gi = 0;
-            if (lane == 0) gi = atomicAdd(&bars->unit_ctr, 1);
-            gi = __shfl_sync(0xffffffffu, gi, 0);
+            if constexpr (WINRS_F16_RR == 1 || (WINRS_F16_RR == 2 && A0 == 4)) {
+                // round-robin: warp w takes units w, w + T, w + 2T, ... (no atomics)
+                gi = (warp - 2) + TX_WARPS * rr_iter++;
+            } else {
+                if (lane == 0) gi = atomicAdd(&bars->unit_ctr, 1);
+                gi = __shfl_sync(0xffffffffu, gi, 0);
+            }
             while (jb < njobs && gi >= unit_base + (jhi[jb] - jlo[jb]) * NU) {
                 unit_base += (jhi[jb] - jlo[jb]) * NU;
                 gch_base += jhi[jb] - jlo[jb];
                 ++jb;
             }
             // epilogues of the jobs whose units are all handed out (warps 2..5:
-            // one TMEM lane quarter each)
-            if (warp < 6)
+            // one TMEM lane quarter each); the fused push path does its own
+            if (warp < 6 && !fused)
                 while (epi < jb) run_epilogue(epi++);
             if (jb >= njobs) break;
             const int rel = gi - unit_base;
@@ -954,10 +1065,17 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             if (lane == 0) mbar_arrive(&bars->op_full[so]);
         }
         if (threadIdx.x == 64) PTRACE(3);
-        asm volatile("bar.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
-        if (warp < 6) {
-            final_out<N0, BM, NAT>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
-            if (threadIdx.x == 64) PTRACE(4);
+        if (fused) {
+            if (warp == 2) {   // the accumulators are final before the CTA-wide sync below
+                mbar_wait(&bars->acc_full, 0u);
+                tc_fence_after();
+            }
+        } else {
+            asm volatile("bar.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
+            if (warp < 6) {
+                final_out<N0, BM, NAT>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
+                if (threadIdx.x == 64) PTRACE(4);
+            }
         }
     } else {
         // ===================== transformers (+ epilogue) =====================
@@ -1029,8 +1147,17 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     __syncthreads();
     if (threadIdx.x == 0) PTRACE(5);
     if constexpr (kCluster) {
-        if (g.csplit > 1)
+        if (fused) {
+            tc_fence_after();
+            int lo, hi;
+            chunk_range(jobs[0], &lo, &hi);
+            cluster_push_reduce<A0, N0, R0, N0, BM, NAT>(g, bucket, cc, fw0, rank, tmem_base, hi <= lo,
+                                                        reinterpret_cast<float*>(smem), nthreads<BM>());
+            tc_fence_before();
+            __syncthreads();
+        } else if (g.csplit > 1) {
             cluster_reduce<N0, BM>(g, bucket, cc, fw0, rank, reinterpret_cast<const float*>(smem), nthreads<BM>());
+        }
     }
     if (threadIdx.x == 0) PTRACE(6);
     if (warp == 1) {
