@@ -50,6 +50,9 @@ constexpr int KC = 16;           // depth entries per chunk = UMMA K
 #ifndef WINRS_F16_PUSH
 #define WINRS_F16_PUSH 0         // 1: fused epilogue + one-way DSMEM push reduction for cluster-split single-job tiles (measured: no gain, DSMEM-bandwidth bound either way)
 #endif
+#ifndef WINRS_F16_DIRECT
+#define WINRS_F16_DIRECT 1       // single-job tiles: OT straight to the staging tile / bucket (no TMEM stash, no final pass)
+#endif
 #ifndef WINRS_F16_RR
 #define WINRS_F16_RR 2           // 1: static round-robin unit assignment instead of the shared counter; 2: for alpha = 4 only
                                  // (measured on B200: round-robin 6-12% faster for alpha = 4, 15% slower for alpha = 8)
@@ -615,6 +618,71 @@ __device__ __forceinline__ void epilogue(int j_off, bool first, bool empty, uint
     }
 }
 
+template <int BM> __host__ __device__ constexpr int out_ld();
+// ---- direct epilogue (single-job tiles): accumulators -> OT (FP32) -> the
+// cluster staging tile (csplit > 1) or the bucket, with no TMEM output stash
+// and no separate final pass.  Warps 2..5 (one TMEM lane quarter each) take
+// 16 physical columns at a time: two 8-column halves are read and
+// transformed, then de-interleaved into 16 logical columns (K-major path:
+// physical 16b + i holds c = 16b + 2i, 16b + 8 + i holds c = 16b + 2i + 1)
+// and written as float4s.  After acc_full no ring access is outstanding
+// (every unit stored before its op_full arrival), so the staging tile may
+// overlay the rings.
+template <int A, int NN, int RR, int BM, bool NAT>
+__device__ __forceinline__ void epilogue_direct(const Geometry& g, float* bucket, const CtaCoord& cc, int fw0,
+                                                uint32_t tmem_base, int warp, bool empty, float* Out) {
+    using WT = Wino<A, NN, RR>;
+    const int quarter = warp & 3, lane = threadIdx.x & 31;
+    const int L = quarter * 32 + lane;
+    const int kl = NAT ? L : iperm16(L);
+    const int kg = cc.kb * BN + kl;
+    const uint32_t lane_base = tmem_base + ((uint32_t)(quarter * 32) << 16);
+#pragma unroll 1
+    for (int c0 = 0; c0 < BM; c0 += 16) {
+        float y[NN][16];
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            float v[A][8];
+            if (!empty) {
+#pragma unroll
+                for (int x = 0; x < A; ++x) tmem_ld8(lane_base + (uint32_t)(x * BM + c0 + 8 * h), v[x]);
+                tmem_wait_ld();
+            } else {
+#pragma unroll
+                for (int x = 0; x < A; ++x)
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) v[x][i] = 0.f;
+            }
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                float vv[A], yy[NN];
+#pragma unroll
+                for (int x = 0; x < A; ++x) vv[x] = v[x][i];
+                WT::ot(vv, yy);
+#pragma unroll
+                for (int j = 0; j < NN; ++j) y[j][NAT ? 8 * h + i : 2 * i + h] = yy[j];
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < NN; ++j) {
+            if (g.csplit > 1) {
+                float4* o = reinterpret_cast<float4*>(Out + ((long long)j * BN + kl) * out_ld<BM>() + c0);
+#pragma unroll
+                for (int q = 0; q < 4; ++q) o[q] = make_float4(y[j][4 * q], y[j][4 * q + 1], y[j][4 * q + 2], y[j][4 * q + 3]);
+            } else {
+                const int cg = cc.cb * BM + c0;
+                if (kg < g.K && cg < g.C) {   // C % 8 == 0: 8-column groups are all in or all out
+                    float4* d4 = reinterpret_cast<float4*>(bucket + (((long long)kg * g.R + cc.fh) * g.S + fw0 + j) * g.C + cg);
+                    const int nq = cg + 16 <= g.C ? 4 : 2;
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        if (q < nq) d4[q] = make_float4(y[j][4 * q], y[j][4 * q + 1], y[j][4 * q + 2], y[j][4 * q + 3]);
+                }
+            }
+        }
+    }
+}
+
 // Output staging tile in shared memory for the cluster reduction: [n0][BN][BM+4].
 // It overlays the rings (and, when larger, the mbarriers): it is only written
 // after the last job, when all of them are idle.
@@ -858,7 +926,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                      :: "r"(smem_u32(&bars->tmem_base)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
-    {   // clear the operand ring once (rows past K / C are never transformed)
+    if (g.K - cc.kb * BN < BN || g.C - cc.cb * BM < BM) {   // clear the operand ring once (rows past K / C are never transformed)
         uint4* op = reinterpret_cast<uint4*>(smem + SM::op_off);
         for (int i = threadIdx.x; i < SM::S_OP * SM::OP / 16; i += nthreads<BM>()) op[i] = make_uint4(0, 0, 0, 0);
         fence_proxy_async();   // generic-proxy zeros visible to the tensor core's async proxy
@@ -994,12 +1062,18 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         for (int jb = 0; jb < njobs; ++jb) chunk_range(jobs[jb], &jlo[jb], &jhi[jb]);
         int jb = 0, unit_base = 0, gch_base = 0, epi = 0, rr_iter = 0;
         (void)rr_iter;
+        // (the staging tile must not reach the mbarriers / unit counter, which
+        // other warps may still touch while the epilogue runs)
+        constexpr bool kOutBelowBars = (size_t)N0 * BN * out_ld<BM>() * 4 <= (size_t)SM::bar_off;
+        const bool direct = WINRS_F16_DIRECT && njobs == 1 && !fused && (g.csplit <= 1 || kOutBelowBars);
         auto run_epilogue = [&](int e) {
             const Job& J = jobs[e];
             mbar_wait(&bars->acc_full, (uint32_t)(e & 1));
             tc_fence_after();
             const bool empty = jhi[e] <= jlo[e];
-            if (J.phase == 0)
+            if (direct)
+                epilogue_direct<A0, N0, R0, BM, NAT>(g, bucket, cc, fw0, tmem_base, warp, empty, reinterpret_cast<float*>(smem));
+            else if (J.phase == 0)
                 epilogue<A0, N0, R0, N0, BM>(0, true, empty, tmem_base, warp);
             else if constexpr (A1 != 0)
                 epilogue<A1, N1, R1, N0, BM>(J.fw0 - fw0, false, empty, tmem_base, warp);
@@ -1070,7 +1144,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 mbar_wait(&bars->acc_full, 0u);
                 tc_fence_after();
             }
-        } else {
+        } else if (!direct) {
             asm volatile("bar.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
             if (warp < 6) {
                 final_out<N0, BM, NAT>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
