@@ -78,16 +78,17 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
         mY1 = mY0;
     }
     if (g.csplit <= 1) {
-        k<<<(unsigned)grid, nthreads<BM>(), sm, stream>>>(a, mX0, mY0, mX1, mY1);
+        k<<<(unsigned)grid, kthreads<A0, N0, R0, A1, BM>(), sm, stream>>>(a, mX0, mY0, mX1, mY1);
         return cudaGetLastError();
     }
-    return launch_cluster(k, (unsigned)grid, (unsigned)nthreads<BM>(), sm, stream, g.csplit, a, mX0, mY0, mX1, mY1);
+    return launch_cluster(k, (unsigned)grid, (unsigned)kthreads<A0, N0, R0, A1, BM>(), sm, stream, g.csplit, a, mX0, mY0,
+                          mX1, mY1);
 }
 
 }  // namespace f16k
 
 #define WINRS_TC_ENTRY(DT, BF, PFX, A0, N0, R0, A1, N1, R1, BM)                                     \
-    {DT, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::nthreads<BM>(), 1,              \
+    {DT, A0, N0, R0, A1, N1, R1, ::winrs::f16k::BN, BM, ::winrs::f16k::kthreads<A0, N0, R0, A1, BM>(), 1, \
      ::winrs::f16k::csplit_fits<N0, BM>() ? 1 : 0, ::winrs::f16k::smem_total<A0, N0, R0, BM>(),       \
      &::winrs::f16k::launch<A0, N0, R0, A1, N1, R1, BM, BF>,                                          \
      PFX "_O" #A0 "(" #N0 "," #R0 ")+O" #A1 "(" #N1 "," #R1 ")_128x" #BM}

@@ -50,6 +50,9 @@ constexpr int KC = 16;           // depth entries per chunk = UMMA K
 #ifndef WINRS_F16_PUSH
 #define WINRS_F16_PUSH 0         // 1: fused epilogue + one-way DSMEM push reduction for cluster-split single-job tiles (measured: no gain, DSMEM-bandwidth bound either way)
 #endif
+#ifndef WINRS_F16_UPAIR
+#define WINRS_F16_UPAIR 2        // dynamic schedule: a unit covers both depth octets of its row block (2: alpha = 4 kernels only)
+#endif
 #ifndef WINRS_F16_DIRECT
 #define WINRS_F16_DIRECT 1       // single-job tiles: OT straight to the staging tile / bucket (no TMEM stash, no final pass)
 #endif
@@ -101,14 +104,37 @@ __host__ __device__ constexpr bool native_path() {
 constexpr int NAT_IPT = WINRS_NAT_IPT;   // (channel octet, depth) items per thread per unit
 template <int BM> __host__ __device__ constexpr int nat_ft_units() { return (BN / 8) * KC / (32 * NAT_IPT); }
 template <int BM> __host__ __device__ constexpr int nat_it_units() { return (BM / 8) * KC / (32 * NAT_IPT); }
-template <int BM, bool NAT> __host__ __device__ constexpr int units_per_chunk() {
-    return NAT ? nat_ft_units<BM>() + nat_it_units<BM>() : n_units<BM>();
+// Paired units (dynamic schedule): one grab covers both depth octets of a
+// row block (FT always; IT when a block spans a whole warp of c pairs), so a
+// chunk has half as many units and half the barrier hand-offs.
+// Measured on B200: 2-9 % faster for the alpha = 4 kernels, much slower for
+// alpha = 8 (too few units per chunk to keep the transformer warps busy).
+template <int A0, int R0> __host__ __device__ constexpr bool pair_units() {
+    return WINRS_F16_DYN && (WINRS_F16_UPAIR == 1 || (WINRS_F16_UPAIR == 2 && A0 == 4 && R0 == 2));
+}
+template <int BM, bool P> __host__ __device__ constexpr bool it_paired() { return P && BM / 2 >= 32; }
+template <int BM, bool P> __host__ __device__ constexpr int ft_units_p() { return P ? ft_warps<BM>() / 2 : ft_warps<BM>(); }
+template <int BM, bool P> __host__ __device__ constexpr int it_units_p() { return it_paired<BM, P>() ? it_warps<BM>() / 2 : it_warps<BM>(); }
+template <int BM, bool NAT, bool P = false> __host__ __device__ constexpr int units_per_chunk() {
+    return NAT ? nat_ft_units<BM>() + nat_it_units<BM>() : ft_units_p<BM, P>() + it_units_p<BM, P>();
 }
 
-template <int BM> __host__ __device__ constexpr int tx_warps() {
-    return !WINRS_F16_DYN ? n_units<BM>() : WINRS_F16_TXW > 0 ? WINRS_F16_TXW : BM >= 128 ? 14 : 10;
+// Transformer warps.  The ring waits are parity waits, so a unit of chunk c
+// must not start before the raw data of chunk c - S_RAW has landed: with
+// units handed out in order, at most TX - 1 other units are in flight, which
+// the kernel bounds statically (TX <= (S_RAW - 1) * units_per_chunk + 1).
+// With paired / native units (4 per chunk at B_M = 128) that caps TX at 12.
+template <int BM, bool FEW = false> __host__ __device__ constexpr int tx_warps() {
+    return !WINRS_F16_DYN ? n_units<BM>() : WINRS_F16_TXW > 0 ? WINRS_F16_TXW : BM >= 128 ? (FEW ? 12 : 14) : 10;
 }
-template <int BM> __host__ __device__ constexpr int nthreads() { return 64 + 32 * tx_warps<BM>(); }
+template <int BM, bool FEW = false> __host__ __device__ constexpr int nthreads() { return 64 + 32 * tx_warps<BM, FEW>(); }
+// FEW: 4 units per chunk at B_M = 128 (paired or native units)
+template <int A0, int N0, int R0, int A1, int BM> __host__ __device__ constexpr bool few_units() {
+    return pair_units<A0, R0>() || native_path<A0, N0, R0, A1, BM>();
+}
+template <int A0, int N0, int R0, int A1, int BM> __host__ __device__ constexpr int kthreads() {
+    return nthreads<BM, few_units<A0, N0, R0, A1, BM>()>();
+}
 
 struct Args {
     Geometry g;
@@ -424,6 +450,34 @@ __device__ __forceinline__ void transform_role(const uint8_t* raw, uint8_t* op, 
         unit_transform<1, A, NN, RR, A, DQ_IT, BF>(rawX, BM, A * BM, op + A * OPA, OPB, q, quad, mid);
     }
 }
+// Dynamic schedule with paired units: unit u -> one or two roles (IT first).
+// mid_op (wait for the operand stage) runs before the first stores, mid_raw
+// (release the raw stage) after the last raw loads of the unit.
+template <int A, int NN, int RR, int BM, bool BF, bool P, class MidOp, class MidRaw>
+__device__ __forceinline__ void transform_unit_paired(const uint8_t* raw, uint8_t* op, int u, int lane, int kv, int cv,
+                                                      const MidOp& mid_op, const MidRaw& mid_raw) {
+    const auto both = [&]() { mid_raw(); mid_op(); };
+    if (u < it_units_p<BM, P>()) {
+        if (it_paired<BM, P>()) {   // block u, octets 0 and 1 (roles octet * nblk + block)
+            constexpr int NB = (BM / 2) / 32;
+            transform_role<A, NN, RR, BM, BF>(raw, op, u, lane, kv, cv, mid_op);
+            transform_role<A, NN, RR, BM, BF>(raw, op, NB + u, lane, kv, cv, mid_raw);
+        } else {
+            transform_role<A, NN, RR, BM, BF>(raw, op, u, lane, kv, cv, both);
+        }
+    } else {
+        const int f2 = u - it_units_p<BM, P>();
+        if (P) {   // block f2 % nb, octets 2*(f2 / nb) + {0, 1} (roles octet * nb + block)
+            constexpr int NB = BN / 64;
+            const int blk = f2 % NB, oct = 2 * (f2 / NB);
+            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - (oct * NB + blk), lane, kv, cv, mid_op);
+            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - ((oct + 1) * NB + blk), lane, kv, cv, mid_raw);
+        } else {
+            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - f2, lane, kv, cv, both);
+        }
+    }
+}
+
 // Static schedule: transformer warp tw always runs the same unit.
 template <int A, int NN, int RR, int BM, bool BF>
 __device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tw, int lane, int kv, int cv) {
@@ -856,14 +910,18 @@ __device__ __forceinline__ void cluster_push_reduce(const Geometry& g, float* bu
 }
 
 template <int A0, int N0, int R0, int A1, int N1, int R1, int BM, bool BF>
-__global__ void __launch_bounds__(nthreads<BM>(), 1)
+__global__ void __launch_bounds__((kthreads<A0, N0, R0, A1, BM>()), 1)
 bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX0,
                const __grid_constant__ CUtensorMap tmY0, const __grid_constant__ CUtensorMap tmX1,
                const __grid_constant__ CUtensorMap tmY1) {
     using SM = Smem<A0, R0, BM>;
     constexpr int S_RAW = SM::S_RAW;
-    constexpr int TX_WARPS = tx_warps<BM>();
+    constexpr int TX_WARPS = tx_warps<BM, few_units<A0, N0, R0, A1, BM>()>();
+    constexpr int NTHR = kthreads<A0, N0, R0, A1, BM>();
     static_assert(A1 * BM <= stash_col<N0, BM>(), "residual accumulators overlap the TMEM output stash");
+    static_assert(!WINRS_F16_DYN ||
+                  TX_WARPS <= (S_RAW - 1) * units_per_chunk<BM, native_path<A0, N0, R0, A1, BM>(), pair_units<A0, R0>()>() + 1,
+                  "in-order unit hand-out could run a full raw ring ahead of the TMA (parity-wait aliasing)");
     constexpr bool kCluster = csplit_fits<N0, BM>();
     constexpr bool NAT = native_path<A0, N0, R0, A1, BM>();
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -909,7 +967,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     };
 
     if (threadIdx.x == 0) {
-        constexpr int NU = units_per_chunk<BM, NAT>();
+        constexpr int NU = units_per_chunk<BM, NAT, pair_units<A0, R0>()>();
         for (int s = 0; s < S_RAW; ++s) { mbar_init(&bars->raw_full[s], 1); mbar_init(&bars->raw_empty[s], NU); }
         for (int s = 0; s < SM::S_OP; ++s) { mbar_init(&bars->op_full[s], NU); mbar_init(&bars->op_empty[s], 1); }
         bars->unit_ctr = 0;
@@ -928,7 +986,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     }
     if (g.K - cc.kb * BN < BN || g.C - cc.cb * BM < BM) {   // clear the operand ring once (rows past K / C are never transformed)
         uint4* op = reinterpret_cast<uint4*>(smem + SM::op_off);
-        for (int i = threadIdx.x; i < SM::S_OP * SM::OP / 16; i += nthreads<BM>()) op[i] = make_uint4(0, 0, 0, 0);
+        for (int i = threadIdx.x; i < SM::S_OP * SM::OP / 16; i += NTHR) op[i] = make_uint4(0, 0, 0, 0);
         fence_proxy_async();   // generic-proxy zeros visible to the tensor core's async proxy
     }
     tc_fence_before();
@@ -1056,7 +1114,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         // sub-partition takes more: the chunk rate follows the average unit
         // cost instead of the slowest fixed role.  Ring stage / parity follow
         // from the global chunk index, as in the producer and MMA loops.
-        constexpr int NU = units_per_chunk<BM, NAT>();
+        constexpr int NU = units_per_chunk<BM, NAT, pair_units<A0, R0>()>();
         const int kv = g.K - cc.kb * BN, cv = g.C - cc.cb * BM;
         int jlo[1 + 9], jhi[1 + 9];
         for (int jb = 0; jb < njobs; ++jb) chunk_range(jobs[jb], &jlo[jb], &jhi[jb]);
@@ -1114,21 +1172,24 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             // wait for the MMAs of the chunk that last used this operand stage.
             // A skipped unit also waits, so its op_full arrival cannot land in
             // the previous phase of the stage.
-            const auto mid = [&]() {
+            const auto mid_raw = [&]() {
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&bars->raw_empty[sr]);
+            };
+            const auto mid_op = [&]() {
                 mbar_wait(&bars->op_empty[so], (uint32_t)(((gch / SM::S_OP) & 1) ^ 1));
 #ifdef WINRS_TRACE
                 if (lane == 0 && blockIdx.x == 0 && gch < 256) g_trace_w[gch][warp][1] = gtime();
 #endif
             };
+            const auto mid = [&]() { mid_raw(); mid_op(); };
 #ifdef WINRS_NO_TX     // debug: transformer units keep only the barrier protocol
             if (true) mid();
             else
 #endif
             if constexpr (NAT) native_unit<BM, BF>(raw, op, u, lane, kv, cv, mid);
-            else if (jobs[jb].phase == 0) transform_unit<A0, N0, R0, BM, BF>(raw, op, u, lane, kv, cv, mid);
-            else if constexpr (A1 != 0) transform_unit<A1, N1, R1, BM, BF>(raw, op, u, lane, kv, cv, mid);
+            else if (jobs[jb].phase == 0) transform_unit_paired<A0, N0, R0, BM, BF, pair_units<A0, R0>()>(raw, op, u, lane, kv, cv, mid_op, mid_raw);
+            else if constexpr (A1 != 0) transform_unit_paired<A1, N1, R1, BM, BF, pair_units<A0, R0>()>(raw, op, u, lane, kv, cv, mid_op, mid_raw);
 #ifndef WINRS_NO_FENCE
             fence_proxy_async();
 #endif
@@ -1226,11 +1287,11 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             int lo, hi;
             chunk_range(jobs[0], &lo, &hi);
             cluster_push_reduce<A0, N0, R0, N0, BM, NAT>(g, bucket, cc, fw0, rank, tmem_base, hi <= lo,
-                                                        reinterpret_cast<float*>(smem), nthreads<BM>());
+                                                        reinterpret_cast<float*>(smem), NTHR);
             tc_fence_before();
             __syncthreads();
         } else if (g.csplit > 1) {
-            cluster_reduce<N0, BM>(g, bucket, cc, fw0, rank, reinterpret_cast<const float*>(smem), nthreads<BM>());
+            cluster_reduce<N0, BM>(g, bucket, cc, fw0, rank, reinterpret_cast<const float*>(smem), NTHR);
         }
     }
     if (threadIdx.x == 0) PTRACE(6);
