@@ -22,39 +22,73 @@ __device__ __forceinline__ void kahan_add(float& s, float& c, float x) {
     s = t;
 }
 
+// The bucket loads of a group of 8 are issued together (they are independent)
+// and then added in z order, so a thread waits for one memory latency per 8
+// buckets instead of one per bucket; small dW uses one float per thread so
+// the grid still covers the SMs.  The summation order is unchanged.
+constexpr int ZB = 8;
+
+template <class V>
+__device__ __forceinline__ void kahan_v(V& s, V& c, const V& x);
+template <>
+__device__ __forceinline__ void kahan_v<float4>(float4& s, float4& c, const float4& x) {
+    kahan_add(s.x, c.x, x.x);
+    kahan_add(s.y, c.y, x.y);
+    kahan_add(s.z, c.z, x.z);
+    kahan_add(s.w, c.w, x.w);
+}
+template <>
+__device__ __forceinline__ void kahan_v<float>(float& s, float& c, const float& x) {
+    kahan_add(s, c, x);
+}
+template <class V> __device__ __forceinline__ V vzero();
+template <> __device__ __forceinline__ float4 vzero<float4>() { return make_float4(0.f, 0.f, 0.f, 0.f); }
+template <> __device__ __forceinline__ float vzero<float>() { return 0.f; }
+
+// V = float4: i indexes float4 groups of the first n/4*4 elements; V = float: all n elements.
+template <class V>
 __global__ void __launch_bounds__(256)
 bucket_reduce_kernel(float* __restrict__ dW, const float* __restrict__ ws, long long n, int Z) {
-    const long long n4 = n >> 2;
+    constexpr int W = sizeof(V) / 4;
+    const long long nv = n / W;
     const long long stride = (long long)gridDim.x * blockDim.x;
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride) {
-        float4 s = reinterpret_cast<const float4*>(dW)[i];
-        float4 c = make_float4(0.f, 0.f, 0.f, 0.f);
-        for (int z = 1; z < Z; ++z) {
-            const float4 x = __ldcs(reinterpret_cast<const float4*>(ws + (long long)(z - 1) * n) + i);
-            kahan_add(s.x, c.x, x.x);
-            kahan_add(s.y, c.y, x.y);
-            kahan_add(s.z, c.z, x.z);
-            kahan_add(s.w, c.w, x.w);
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += stride) {
+        V s = reinterpret_cast<const V*>(dW)[i];
+        V c = vzero<V>();
+        for (int z0 = 1; z0 < Z; z0 += ZB) {
+            V x[ZB];
+#pragma unroll
+            for (int j = 0; j < ZB; ++j)
+                if (z0 + j < Z) x[j] = __ldcs(reinterpret_cast<const V*>(ws + (long long)(z0 + j - 1) * n) + i);
+#pragma unroll
+            for (int j = 0; j < ZB; ++j)
+                if (z0 + j < Z) kahan_v<V>(s, c, x[j]);
         }
-        reinterpret_cast<float4*>(dW)[i] = s;
+        reinterpret_cast<V*>(dW)[i] = s;
     }
-    // scalar tail (n % 4 elements)
-    for (long long i = (n4 << 2) + (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-        float s = dW[i], c = 0.f;
-        for (int z = 1; z < Z; ++z) kahan_add(s, c, ws[(long long)(z - 1) * n + i]);
-        dW[i] = s;
+    if (W > 1) {   // scalar tail (n % 4 elements)
+        for (long long i = nv * W + (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+            float s = dW[i], c = 0.f;
+            for (int z = 1; z < Z; ++z) kahan_add(s, c, ws[(long long)(z - 1) * n + i]);
+            dW[i] = s;
+        }
     }
 }
 
 cudaError_t launch_bucket_reduce(float* dW, const float* ws, long long n, int Z, int num_sms,
                                  cudaStream_t stream) {
     if (Z <= 1) return cudaSuccess;
-    const long long n4 = (n + 3) / 4;
-    long long blocks = (n4 + 255) / 256;
     const long long cap = (long long)num_sms * 8;
+    // one float per thread while a float4 per thread would leave SMs idle
+    const bool scalar = (n / 4 + 255) / 256 < num_sms;
+    const long long items = scalar ? n : n / 4 + (n % 4 ? 1 : 0);
+    long long blocks = (items + 255) / 256;
     if (blocks > cap) blocks = cap - cap % num_sms;
     if (blocks < 1) blocks = 1;
-    bucket_reduce_kernel<<<(unsigned)blocks, 256, 0, stream>>>(dW, ws, n, Z);
+    if (scalar)
+        bucket_reduce_kernel<float><<<(unsigned)blocks, 256, 0, stream>>>(dW, ws, n, Z);
+    else
+        bucket_reduce_kernel<float4><<<(unsigned)blocks, 256, 0, stream>>>(dW, ws, n, Z);
     return cudaGetLastError();
 }
 
