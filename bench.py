@@ -224,6 +224,33 @@ def run_winrs(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         step_ms = float(t.item())
 
+    # Secondary numbers: warm-L2 per-layer time (no flush between
+    # calls) and, for N > 1, the compute-only time without the all_reduce.
+    def time_layers(flush_l2, with_allreduce, reps=5):
+        out = []
+        for it2 in items:
+            ts = []
+            for _ in range(reps):
+                if flush_l2:
+                    flush.fill_(3)
+                else:   # keep the GPU busy while the host launches (no memory traffic)
+                    torch.cuda._sleep(100000)
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                if with_allreduce:
+                    run_bfc(it2, stream)
+                elif kshard:
+                    run_bfc(it2, stream)
+                else:
+                    W.bfc(it2["plan"], it2["X"], it2["dY"], it2["dW"], it2["ws"], stream)
+                b.record(stream)
+                torch.cuda.synchronize()
+                ts.append(a.elapsed_time(b))
+            out.append(statistics.median(ts))
+        return out
+    warm_ms = time_layers(False, world > 1)
+    compute_only_ms = time_layers(True, False) if world > 1 else None
+
     # Dominant kernel's live duration: time the fused kernel alone (no
     # all_reduce) for the layer with the largest share, CUDA events on the stream.
     dom = max(range(len(items)), key=lambda j: per_layer_ms[j])
@@ -321,7 +348,9 @@ def run_winrs(args):
                        "parallelism": (f"kshard{world}" if kshard else f"dp{world}") if world > 1 else "single",
                        "l2": "flushed (256 MiB write) before every layer call; flush outside timed events",
                        "workspace_cap": float(os.environ.get("WINRS_WS_CAP", "0.04")),
-                       "layers": [{"name": x["layer"].name, "ms": per_layer_ms[j],
+                       "warm_l2_ms_per_step": sum(warm_ms),
+                       "compute_only_ms_per_step": sum(compute_only_ms) if compute_only_ms else None,
+                       "layers": [{"name": x["layer"].name, "ms": per_layer_ms[j], "warm_ms": warm_ms[j],
                                    "tflops": x["layer"].direct_flops / (per_layer_ms[j] * 1e-3) / 1e12,
                                    "workspace_bytes": x["plan"].workspace_bytes, "plan": repr(x["plan"]),
                                    "kernel": x["plan"].kernel_name} for j, x in enumerate(items)]},
