@@ -3,6 +3,9 @@
 #include <cuda_runtime.h>
 #include <cstdlib>
 #include <mutex>
+#ifndef WINRS_F16_YB64
+#define WINRS_F16_YB64 1   // 64-row dY boxes when K <= 64
+#endif
 #include "bfc_f16.cuh"
 #include "launch_util.cuh"
 #include "registry.h"
@@ -65,13 +68,14 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
     a.dW = dW;
     a.ws = ws;
     a.nb = images_per_box(g.N);
+    a.ybn = (g.K <= 64 && !native_path<A0, N0, R0, A1, BM>() && WINRS_F16_YB64) ? 64 : BN;
     CUtensorMap mX0, mY0, mX1, mY1;
     if (!make_map(&mX0, X, g.N, g.H, g.W, g.C, BM, A0, a.nb, 0, BF) ||
-        !make_map(&mY0, dY, g.N, g.Ho, g.Wo, g.K, BN, R0, a.nb, g.ldy, BF))
+        !make_map(&mY0, dY, g.N, g.Ho, g.Wo, g.K, a.ybn, R0, a.nb, g.ldy, BF))
         return cudaErrorInvalidValue;
     if (A1 != 0) {
         if (!make_map(&mX1, X, g.N, g.H, g.W, g.C, BM, A1 ? A1 : A0, a.nb, 0, BF) ||
-            !make_map(&mY1, dY, g.N, g.Ho, g.Wo, g.K, BN, R1 ? R1 : R0, a.nb, g.ldy, BF))
+            !make_map(&mY1, dY, g.N, g.Ho, g.Wo, g.K, a.ybn, R1 ? R1 : R0, a.nb, g.ldy, BF))
             return cudaErrorInvalidValue;
     } else {
         mX1 = mX0;

@@ -141,6 +141,7 @@ struct Args {
     float* dW;
     float* ws;
     int nb;          // images per TMA box (divides N and KC)
+    int ybn;         // k rows per dY box: B_N, or 64 when K <= 64 (no zero-filled rows to land in SMEM)
 };
 
 // ----------------------------------------------------------------------------- PTX helpers
@@ -432,7 +433,7 @@ __device__ __forceinline__ int tx_role(int tw) {
 // role >= 0: IT unit `role`; role < 0: FT unit -1 - role.
 template <int A, int NN, int RR, int BM, bool BF, class Mid = NoMid>
 __device__ __forceinline__ void transform_role(const uint8_t* raw, uint8_t* op, int role, int lane, int kv, int cv,
-                                               const Mid& mid = Mid()) {
+                                               const Mid& mid = Mid(), int yb = BN) {
     constexpr int RAW_Y = KC * RR * BN * 2;
     const uint16_t* rawY = reinterpret_cast<const uint16_t*>(raw);            // [KC][RR][BN]
     const uint16_t* rawX = reinterpret_cast<const uint16_t*>(raw + RAW_Y);    // [KC][A][BM]
@@ -440,7 +441,7 @@ __device__ __forceinline__ void transform_role(const uint8_t* raw, uint8_t* op, 
     if (role < 0) {
         const int f = -1 - role;   // FT warp: 32 k pairs x one octet
         if ((f % (BN / 64)) * 64 >= kv) { mid(); return; }
-        unit_transform<0, A, NN, RR, RR, DQ_FT, BF>(rawY, BN, RR * BN, op, OPA, (f % (BN / 64)) * 32 + lane,
+        unit_transform<0, A, NN, RR, RR, DQ_FT, BF>(rawY, yb, RR * yb, op, OPA, (f % (BN / 64)) * 32 + lane,
                                                 f / (BN / 64), mid);
     } else {                       // IT warp: 32 c pairs (or BM/2 pairs x 32/(BM/2) quads) x quads
         constexpr int PW = BM / 2 < 32 ? BM / 2 : 32;
@@ -455,33 +456,33 @@ __device__ __forceinline__ void transform_role(const uint8_t* raw, uint8_t* op, 
 // (release the raw stage) after the last raw loads of the unit.
 template <int A, int NN, int RR, int BM, bool BF, bool P, class MidOp, class MidRaw>
 __device__ __forceinline__ void transform_unit_paired(const uint8_t* raw, uint8_t* op, int u, int lane, int kv, int cv,
-                                                      const MidOp& mid_op, const MidRaw& mid_raw) {
+                                                      const MidOp& mid_op, const MidRaw& mid_raw, int yb) {
     const auto both = [&]() { mid_raw(); mid_op(); };
     if (u < it_units_p<BM, P>()) {
         if (it_paired<BM, P>()) {   // block u, octets 0 and 1 (roles octet * nblk + block)
             constexpr int NB = (BM / 2) / 32;
-            transform_role<A, NN, RR, BM, BF>(raw, op, u, lane, kv, cv, mid_op);
-            transform_role<A, NN, RR, BM, BF>(raw, op, NB + u, lane, kv, cv, mid_raw);
+            transform_role<A, NN, RR, BM, BF>(raw, op, u, lane, kv, cv, mid_op, yb);
+            transform_role<A, NN, RR, BM, BF>(raw, op, NB + u, lane, kv, cv, mid_raw, yb);
         } else {
-            transform_role<A, NN, RR, BM, BF>(raw, op, u, lane, kv, cv, both);
+            transform_role<A, NN, RR, BM, BF>(raw, op, u, lane, kv, cv, both, yb);
         }
     } else {
         const int f2 = u - it_units_p<BM, P>();
         if (P) {   // block f2 % nb, octets 2*(f2 / nb) + {0, 1} (roles octet * nb + block)
             constexpr int NB = BN / 64;
             const int blk = f2 % NB, oct = 2 * (f2 / NB);
-            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - (oct * NB + blk), lane, kv, cv, mid_op);
-            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - ((oct + 1) * NB + blk), lane, kv, cv, mid_raw);
+            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - (oct * NB + blk), lane, kv, cv, mid_op, yb);
+            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - ((oct + 1) * NB + blk), lane, kv, cv, mid_raw, yb);
         } else {
-            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - f2, lane, kv, cv, both);
+            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - f2, lane, kv, cv, both, yb);
         }
     }
 }
 
 // Static schedule: transformer warp tw always runs the same unit.
 template <int A, int NN, int RR, int BM, bool BF>
-__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tw, int lane, int kv, int cv) {
-    transform_role<A, NN, RR, BM, BF>(raw, op, tx_role<BM>(tw), lane, kv, cv);
+__device__ __forceinline__ void transform_chunk(const uint8_t* raw, uint8_t* op, int tw, int lane, int kv, int cv, int yb) {
+    transform_role<A, NN, RR, BM, BF>(raw, op, tx_role<BM>(tw), lane, kv, cv, NoMid(), yb);
 }
 // Dynamic schedule: unit u of a chunk, the (costlier) IT units first.
 template <int A, int NN, int RR, int BM, bool BF, class Mid>
@@ -1019,7 +1020,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             const long long depth = (long long)(rows > 0 ? rows : 0) * J.units * g.N;
             int c_lo, c_hi;
             chunk_range(J, &c_lo, &c_hi);
-            const uint32_t bytes = (uint32_t)(KC * (RRj * BN + Aj * BM) * 2);
+            const uint32_t bytes = (uint32_t)(KC * (RRj * args.ybn + Aj * BM) * 2);
             // This lane's box start d = ch*KC + b and its (n, h, u), advanced
             // incrementally (one division per job, not per chunk: the
             // producer shares its SM sub-partition with transformer warps).
@@ -1044,7 +1045,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     const int nn = in ? n : g.N, hh = in ? h : hs;
                     const int w0 = J.w_first + (in ? u : 0) * RRj;
                     if ((lane & 1) == 0)
-                        tma_load_4d(raw + b * RRj * BN * 2, mY, &bars->raw_full[s], cc.kb * BN, w0, hh, nn);
+                        tma_load_4d(raw + b * RRj * args.ybn * 2, mY, &bars->raw_full[s], cc.kb * BN, w0, hh, nn);
                     else
                         tma_load_4d(raw + KC * RRj * BN * 2 + b * Aj * BM * 2, mX, &bars->raw_full[s], cc.cb * BM,
                                     w0 + J.fw0 - g.pad, hh + cc.fh - g.pad, nn);
@@ -1188,8 +1189,8 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             else
 #endif
             if constexpr (NAT) native_unit<BM, BF>(raw, op, u, lane, kv, cv, mid);
-            else if (jobs[jb].phase == 0) transform_unit_paired<A0, N0, R0, BM, BF, pair_units<A0, R0>()>(raw, op, u, lane, kv, cv, mid_op, mid_raw);
-            else if constexpr (A1 != 0) transform_unit_paired<A1, N1, R1, BM, BF, pair_units<A0, R0>()>(raw, op, u, lane, kv, cv, mid_op, mid_raw);
+            else if (jobs[jb].phase == 0) transform_unit_paired<A0, N0, R0, BM, BF, pair_units<A0, R0>()>(raw, op, u, lane, kv, cv, mid_op, mid_raw, args.ybn);
+            else if constexpr (A1 != 0) transform_unit_paired<A1, N1, R1, BM, BF, pair_units<A0, R0>()>(raw, op, u, lane, kv, cv, mid_op, mid_raw, args.ybn);
 #ifndef WINRS_NO_FENCE
             fence_proxy_async();
 #endif
@@ -1236,8 +1237,8 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
 #endif
                 const uint8_t* raw = smem + SM::raw_off + sr * SM::RAW;
                 uint8_t* op = smem + SM::op_off + so * SM::OP;
-                if (J.phase == 0) transform_chunk<A0, N0, R0, BM, BF>(raw, op, tw, lane, kv, cv);
-                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM, BF>(raw, op, tw, lane, kv, cv);
+                if (J.phase == 0) transform_chunk<A0, N0, R0, BM, BF>(raw, op, tw, lane, kv, cv, args.ybn);
+                else if constexpr (A1 != 0) transform_chunk<A1, N1, R1, BM, BF>(raw, op, tw, lane, kv, cv, args.ybn);
                 if (threadIdx.x == 64) TRACE(3, ch - c_lo + jb * 64, 0);
                 if (threadIdx.x == 64 + 32 * 2) TRACE(3, ch - c_lo + jb * 64, 1);   // an IT warp
                 fence_proxy_async();
