@@ -230,10 +230,12 @@ __device__ __forceinline__ void producer_phase(const Geometry& g, const float* _
     }
     for (int ch = 0; ch < nchunks; ++ch) {
         // the slot of chunk ch+S_RAW-1 was read by every thread's transform of ch-1
+        __syncwarp();   // bar.sync is .aligned: the warp must be converged
         asm volatile("bar.sync 1, %0;" :: "n"(NP) : "memory");
         if (ch + S_RAW - 1 < nchunks) issue((ch + S_RAW - 1) % S_RAW);
         cp_async_commit();
         cp_async_wait<S_RAW - 1>();                                   // this thread's copies of chunk ch
+        __syncwarp();   // bar.sync is .aligned: the warp must be converged
         asm volatile("bar.sync 1, %0;" :: "n"(NP) : "memory");       // everyone's copies of chunk ch
         const int ts = tcount % S_T;
         mbar_wait(&ring.t_empty[ts], ((tcount / S_T) & 1) ^ 1);
@@ -329,6 +331,7 @@ __device__ __forceinline__ void gemm_phase(const Geometry& g, float* __restrict_
     }
     // All of this job's ring writes are done (the producer only fills chunks of
     // this job, each consumed above), so the ring memory can hold the OT staging.
+    __syncwarp();   // bar.sync is .aligned: the warp must be converged
     asm volatile("bar.sync 2, %0;" :: "n"(NT) : "memory");
 
     // ---- OT in rounds (one 4-wide k-group of every thread per round)
@@ -345,6 +348,7 @@ __device__ __forceinline__ void gemm_phase(const Geometry& g, float* __restrict_
                 t.x = lo.x; t.y = lo.y; t.z = hi.x; t.w = hi.y;
                 *reinterpret_cast<float4*>(As + (xi * KR + tk * 4 + e) * BM + (gn * L::TPC + tc) * 4) = t;
             }
+        __syncwarp();   // bar.sync is .aligned: the warp must be converged
         asm volatile("bar.sync 2, %0;" :: "n"(NT) : "memory");
         for (int p = gtid; p < KR * BM; p += NT) {
             const int kl = p / BM, c = p % BM;
@@ -359,6 +363,7 @@ __device__ __forceinline__ void gemm_phase(const Geometry& g, float* __restrict_
                 *dst = P.accumulate ? *dst + y[j] : y[j];
             }
         }
+        __syncwarp();   // bar.sync is .aligned: the warp must be converged
         asm volatile("bar.sync 2, %0;" :: "n"(NT) : "memory");
     }
 }
@@ -477,6 +482,7 @@ bfc_f32_kernel(const Geometry g, const float* __restrict__ X, const float* __res
         // the transformer warpgroup hands registers to the GEMM warpgroups
         asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" :: "n"(REG_P));
         producer_phase<A0, N0, R0, BN, BM, C::SR, C::BD>(g, X, dY, cc, P0, smem, ring, tcount);
+        __syncwarp();   // bar.sync is .aligned: the warp must be converged
         asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");   // job boundary (ring reused by the OT)
         if constexpr (A1 != 0) {
             if (resid) {
@@ -485,6 +491,7 @@ bfc_f32_kernel(const Geometry g, const float* __restrict__ X, const float* __res
                     const PhaseCtx P1{hs, he, g.res_col0, g.k1, fw0 + j * N1, j * N1, rank, true};
                     producer_phase<(A1 ? A1 : A0), (N1 ? N1 : N0), (R1 ? R1 : R0), BN, BM, C::SR, C::BD>(g, X, dY, cc, P1, smem, ring,
                                                                                          tcount);
+                    __syncwarp();   // bar.sync is .aligned: the warp must be converged
                     asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");
                 }
             }
@@ -492,6 +499,7 @@ bfc_f32_kernel(const Geometry g, const float* __restrict__ X, const float* __res
     } else {
         asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" :: "n"(REG_G));
         gemm_phase<A0, N0, R0, BN, BM, C::SR, C::BD>(g, Out, cc, P0, smem, ring, tcount);
+        __syncwarp();   // bar.sync is .aligned: the warp must be converged
         asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");
         if constexpr (A1 != 0) {
             if (resid) {
@@ -500,6 +508,7 @@ bfc_f32_kernel(const Geometry g, const float* __restrict__ X, const float* __res
                     const PhaseCtx P1{hs, he, g.res_col0, g.k1, fw0 + j * N1, j * N1, rank, true};
                     gemm_phase<(A1 ? A1 : A0), (N1 ? N1 : N0), (R1 ? R1 : R0), BN, BM, C::SR, C::BD>(g, Out, cc, P1, smem, ring,
                                                                                      tcount);
+                    __syncwarp();   // bar.sync is .aligned: the warp must be converged
                     asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");
                 }
             }
