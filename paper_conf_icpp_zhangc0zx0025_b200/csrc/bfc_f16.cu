@@ -54,13 +54,25 @@ static int images_per_box(int N) {
     return 1;
 }
 
-template <int A0, int N0, int R0, int A1, int N1, int R1, int BM, bool BF>
-cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BM, bool BF, int YB>
+static cudaError_t launch_yb(const Geometry& g, const Args& a, const CUtensorMap& mX0, const CUtensorMap& mY0,
+                             const CUtensorMap& mX1, const CUtensorMap& mY1, cudaStream_t stream) {
     static std::atomic<unsigned long long> done{0};
-    auto k = bfc_f16_kernel<A0, N0, R0, A1, N1, R1, BM, BF>;
-    constexpr size_t sm = smem_total<A0, N0, R0, BM>();
+    auto k = bfc_f16_kernel<A0, N0, R0, A1, N1, R1, BM, BF, YB>;
+    constexpr size_t sm = smem_total<A0, N0, R0, BM, YB>();
     cudaError_t e = ensure_smem_attr(k, sm, done);
     if (e != cudaSuccess) return e;
+    const long long grid = num_ctas(g);
+    if (g.csplit <= 1) {
+        k<<<(unsigned)grid, kthreads<A0, N0, R0, A1, BM>(), sm, stream>>>(a, mX0, mY0, mX1, mY1);
+        return cudaGetLastError();
+    }
+    return launch_cluster(k, (unsigned)grid, (unsigned)kthreads<A0, N0, R0, A1, BM>(), sm, stream, g.csplit, a, mX0, mY0,
+                          mX1, mY1);
+}
+
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BM, bool BF>
+cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
     const long long grid = num_ctas(g);
     if (grid <= 0) return cudaSuccess;
     Args a;
@@ -81,12 +93,10 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
         mX1 = mX0;
         mY1 = mY0;
     }
-    if (g.csplit <= 1) {
-        k<<<(unsigned)grid, kthreads<A0, N0, R0, A1, BM>(), sm, stream>>>(a, mX0, mY0, mX1, mY1);
-        return cudaGetLastError();
+    if constexpr (yb64_variant<A0, R0, A1, BM>()) {
+        if (a.ybn == 64) return launch_yb<A0, N0, R0, A1, N1, R1, BM, BF, 64>(g, a, mX0, mY0, mX1, mY1, stream);
     }
-    return launch_cluster(k, (unsigned)grid, (unsigned)kthreads<A0, N0, R0, A1, BM>(), sm, stream, g.csplit, a, mX0, mY0,
-                          mX1, mY1);
+    return launch_yb<A0, N0, R0, A1, N1, R1, BM, BF, BN>(g, a, mX0, mY0, mX1, mY1, stream);
 }
 
 }  // namespace f16k

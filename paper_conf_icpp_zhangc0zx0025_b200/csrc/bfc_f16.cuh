@@ -79,9 +79,9 @@ constexpr int DQ_IT = WINRS_F16_DQ;      // depth entries per IT unit
 // A chunk's transform work is split into warp-sized units: FT units (32 k
 // pairs x one depth group) and IT units (32 c pairs, or BM/2 pairs x several
 // groups, x depth groups).
-template <int BM> __host__ __device__ constexpr int ft_warps() { return (BN / 2) * (KC / DQ_FT) / 32; }
+template <int BM, int YB = BN> __host__ __device__ constexpr int ft_warps() { return (YB / 2) * (KC / DQ_FT) / 32; }
 template <int BM> __host__ __device__ constexpr int it_warps() { return (BM / 2) * (KC / DQ_IT) / 32; }
-template <int BM> __host__ __device__ constexpr int n_units() { return ft_warps<BM>() + it_warps<BM>(); }
+template <int BM, int YB = BN> __host__ __device__ constexpr int n_units() { return ft_warps<BM, YB>() + it_warps<BM>(); }
 // More warps than units per chunk let several chunks be in flight, which
 // hides the shared-memory latency of the transforms; measured best on B200
 // (A/B of 8..16 warps over the ResNet-50 / VGG-16 layers): 10 warps for the
@@ -113,10 +113,12 @@ template <int A0, int R0> __host__ __device__ constexpr bool pair_units() {
     return WINRS_F16_DYN && (WINRS_F16_UPAIR == 1 || (WINRS_F16_UPAIR == 2 && A0 == 4 && R0 == 2));
 }
 template <int BM, bool P> __host__ __device__ constexpr bool it_paired() { return P && BM / 2 >= 32; }
-template <int BM, bool P> __host__ __device__ constexpr int ft_units_p() { return P ? ft_warps<BM>() / 2 : ft_warps<BM>(); }
+template <int BM, bool P, int YB = BN> __host__ __device__ constexpr int ft_units_p() {
+    return P ? ft_warps<BM, YB>() / 2 : ft_warps<BM, YB>();
+}
 template <int BM, bool P> __host__ __device__ constexpr int it_units_p() { return it_paired<BM, P>() ? it_warps<BM>() / 2 : it_warps<BM>(); }
-template <int BM, bool NAT, bool P = false> __host__ __device__ constexpr int units_per_chunk() {
-    return NAT ? nat_ft_units<BM>() + nat_it_units<BM>() : ft_units_p<BM, P>() + it_units_p<BM, P>();
+template <int BM, bool NAT, bool P = false, int YB = BN> __host__ __device__ constexpr int units_per_chunk() {
+    return NAT ? nat_ft_units<BM>() + nat_it_units<BM>() : ft_units_p<BM, P, YB>() + it_units_p<BM, P>();
 }
 
 // Transformer warps.  The ring waits are parity waits, so a unit of chunk c
@@ -271,9 +273,9 @@ __device__ __forceinline__ F2 ld_h2(const __half* p) {
 }
 
 // ----------------------------------------------------------------------------- shared memory plan
-template <int A0, int R0, int BM>
+template <int A0, int R0, int BM, int YB = BN>
 struct Smem {
-    static constexpr int RAW_Y = KC * R0 * BN * 2;       // bytes per raw stage (dY)
+    static constexpr int RAW_Y = KC * R0 * YB * 2;       // bytes per raw stage (dY; YB k rows per box)
     static constexpr int RAW_X = KC * A0 * BM * 2;       // bytes per raw stage (X)
     static constexpr int RAW = RAW_Y + RAW_X;
     static constexpr int OPA = BN * KC * 2;              // one A_xi slab (4 KB)
@@ -431,18 +433,18 @@ __device__ __forceinline__ int tx_role(int tw) {
 // transforms: those operand rows stay zero (the op ring is cleared once at
 // kernel start) and their accumulator rows are never written out.
 // role >= 0: IT unit `role`; role < 0: FT unit -1 - role.
-template <int A, int NN, int RR, int BM, bool BF, class Mid = NoMid>
+template <int A, int NN, int RR, int BM, bool BF, class Mid = NoMid, int YB = BN>
 __device__ __forceinline__ void transform_role(const uint8_t* raw, uint8_t* op, int role, int lane, int kv, int cv,
                                                const Mid& mid = Mid(), int yb = BN) {
-    constexpr int RAW_Y = KC * RR * BN * 2;
+    constexpr int RAW_Y = KC * RR * YB * 2;
     const uint16_t* rawY = reinterpret_cast<const uint16_t*>(raw);            // [KC][RR][BN]
     const uint16_t* rawX = reinterpret_cast<const uint16_t*>(raw + RAW_Y);    // [KC][A][BM]
     constexpr int OPA = BN * KC * 2, OPB = BM * KC * 2;
     if (role < 0) {
         const int f = -1 - role;   // FT warp: 32 k pairs x one octet
-        if ((f % (BN / 64)) * 64 >= kv) { mid(); return; }
-        unit_transform<0, A, NN, RR, RR, DQ_FT, BF>(rawY, yb, RR * yb, op, OPA, (f % (BN / 64)) * 32 + lane,
-                                                f / (BN / 64), mid);
+        if ((f % (YB / 64)) * 64 >= kv) { mid(); return; }
+        unit_transform<0, A, NN, RR, RR, DQ_FT, BF>(rawY, yb, RR * yb, op, OPA, (f % (YB / 64)) * 32 + lane,
+                                                f / (YB / 64), mid);
     } else {                       // IT warp: 32 c pairs (or BM/2 pairs x 32/(BM/2) quads) x quads
         constexpr int PW = BM / 2 < 32 ? BM / 2 : 32;
         const int q = (role % ((BM / 2) / PW)) * PW + (lane % PW);
@@ -454,27 +456,27 @@ __device__ __forceinline__ void transform_role(const uint8_t* raw, uint8_t* op, 
 // Dynamic schedule with paired units: unit u -> one or two roles (IT first).
 // mid_op (wait for the operand stage) runs before the first stores, mid_raw
 // (release the raw stage) after the last raw loads of the unit.
-template <int A, int NN, int RR, int BM, bool BF, bool P, class MidOp, class MidRaw>
+template <int A, int NN, int RR, int BM, bool BF, bool P, int YB, class MidOp, class MidRaw>
 __device__ __forceinline__ void transform_unit_paired(const uint8_t* raw, uint8_t* op, int u, int lane, int kv, int cv,
                                                       const MidOp& mid_op, const MidRaw& mid_raw, int yb) {
     const auto both = [&]() { mid_raw(); mid_op(); };
     if (u < it_units_p<BM, P>()) {
         if (it_paired<BM, P>()) {   // block u, octets 0 and 1 (roles octet * nblk + block)
             constexpr int NB = (BM / 2) / 32;
-            transform_role<A, NN, RR, BM, BF>(raw, op, u, lane, kv, cv, mid_op, yb);
-            transform_role<A, NN, RR, BM, BF>(raw, op, NB + u, lane, kv, cv, mid_raw, yb);
+            transform_role<A, NN, RR, BM, BF, decltype(mid_op), YB>(raw, op, u, lane, kv, cv, mid_op, yb);
+            transform_role<A, NN, RR, BM, BF, decltype(mid_raw), YB>(raw, op, NB + u, lane, kv, cv, mid_raw, yb);
         } else {
-            transform_role<A, NN, RR, BM, BF>(raw, op, u, lane, kv, cv, both, yb);
+            transform_role<A, NN, RR, BM, BF, decltype(both), YB>(raw, op, u, lane, kv, cv, both, yb);
         }
     } else {
         const int f2 = u - it_units_p<BM, P>();
         if (P) {   // block f2 % nb, octets 2*(f2 / nb) + {0, 1} (roles octet * nb + block)
-            constexpr int NB = BN / 64;
+            constexpr int NB = YB / 64;
             const int blk = f2 % NB, oct = 2 * (f2 / NB);
-            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - (oct * NB + blk), lane, kv, cv, mid_op, yb);
-            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - ((oct + 1) * NB + blk), lane, kv, cv, mid_raw, yb);
+            transform_role<A, NN, RR, BM, BF, decltype(mid_op), YB>(raw, op, -1 - (oct * NB + blk), lane, kv, cv, mid_op, yb);
+            transform_role<A, NN, RR, BM, BF, decltype(mid_raw), YB>(raw, op, -1 - ((oct + 1) * NB + blk), lane, kv, cv, mid_raw, yb);
         } else {
-            transform_role<A, NN, RR, BM, BF>(raw, op, -1 - f2, lane, kv, cv, both, yb);
+            transform_role<A, NN, RR, BM, BF, decltype(both), YB>(raw, op, -1 - f2, lane, kv, cv, both, yb);
         }
     }
 }
@@ -746,9 +748,16 @@ template <int BM> __host__ __device__ constexpr int out_ld() { return BM + 4; }
 template <int N0, int BM> __host__ __device__ constexpr bool csplit_fits() {
     return (size_t)N0 * BN * out_ld<BM>() * 4 <= 227u * 1024u;
 }
-template <int A0, int N0, int R0, int BM> __host__ __device__ constexpr size_t smem_total() {
+template <int A0, int N0, int R0, int BM, int YB = BN> __host__ __device__ constexpr size_t smem_total() {
     const size_t out = csplit_fits<N0, BM>() ? (size_t)N0 * BN * out_ld<BM>() * 4 : 0;
-    return Smem<A0, R0, BM>::bytes > out ? Smem<A0, R0, BM>::bytes : out;
+    return Smem<A0, R0, BM, YB>::bytes > out ? Smem<A0, R0, BM, YB>::bytes : out;
+}
+// The YB = 64 variant (K <= 64: 64-row dY raw stages, only the FT units of
+// the first 64-row block, a deeper raw ring) for the alpha = 8 single-kernel
+// pairs; the others run the B_N-row layout.
+template <int A0, int R0, int A1, int BM> __host__ __device__ constexpr bool yb64_variant() {
+    return WINRS_F16_DYN && A0 == 8 && A1 == 0 && BM >= 64 &&
+           tx_warps<BM>() <= (Smem<A0, R0, BM, 64>::S_RAW - 1) * units_per_chunk<BM, false, false, 64>() + 1;
 }
 
 // ---- final pass (warps 2..5): staged tile -> bucket (no cluster split) or ->
@@ -910,18 +919,19 @@ __device__ __forceinline__ void cluster_push_reduce(const Geometry& g, float* bu
     }
 }
 
-template <int A0, int N0, int R0, int A1, int N1, int R1, int BM, bool BF>
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BM, bool BF, int YB = BN>
 __global__ void __launch_bounds__((kthreads<A0, N0, R0, A1, BM>()), 1)
 bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX0,
                const __grid_constant__ CUtensorMap tmY0, const __grid_constant__ CUtensorMap tmX1,
                const __grid_constant__ CUtensorMap tmY1) {
-    using SM = Smem<A0, R0, BM>;
+    using SM = Smem<A0, R0, BM, YB>;
+    static_assert(YB == BN || (YB == 64 && yb64_variant<A0, R0, A1, BM>()), "64-row dY stages: alpha = 8 single-kernel pairs");
     constexpr int S_RAW = SM::S_RAW;
     constexpr int TX_WARPS = tx_warps<BM, few_units<A0, N0, R0, A1, BM>()>();
     constexpr int NTHR = kthreads<A0, N0, R0, A1, BM>();
     static_assert(A1 * BM <= stash_col<N0, BM>(), "residual accumulators overlap the TMEM output stash");
     static_assert(!WINRS_F16_DYN ||
-                  TX_WARPS <= (S_RAW - 1) * units_per_chunk<BM, native_path<A0, N0, R0, A1, BM>(), pair_units<A0, R0>()>() + 1,
+                  TX_WARPS <= (S_RAW - 1) * units_per_chunk<BM, native_path<A0, N0, R0, A1, BM>(), pair_units<A0, R0>(), YB>() + 1,
                   "in-order unit hand-out could run a full raw ring ahead of the TMA (parity-wait aliasing)");
     constexpr bool kCluster = csplit_fits<N0, BM>();
     constexpr bool NAT = native_path<A0, N0, R0, A1, BM>();
@@ -968,7 +978,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     };
 
     if (threadIdx.x == 0) {
-        constexpr int NU = units_per_chunk<BM, NAT, pair_units<A0, R0>()>();
+        constexpr int NU = units_per_chunk<BM, NAT, pair_units<A0, R0>(), YB>();
         for (int s = 0; s < S_RAW; ++s) { mbar_init(&bars->raw_full[s], 1); mbar_init(&bars->raw_empty[s], NU); }
         for (int s = 0; s < SM::S_OP; ++s) { mbar_init(&bars->op_full[s], NU); mbar_init(&bars->op_empty[s], 1); }
         bars->unit_ctr = 0;
@@ -1047,7 +1057,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     if ((lane & 1) == 0)
                         tma_load_4d(raw + b * RRj * args.ybn * 2, mY, &bars->raw_full[s], cc.kb * BN, w0, hh, nn);
                     else
-                        tma_load_4d(raw + KC * RRj * BN * 2 + b * Aj * BM * 2, mX, &bars->raw_full[s], cc.cb * BM,
+                        tma_load_4d(raw + KC * RRj * YB * 2 + b * Aj * BM * 2, mX, &bars->raw_full[s], cc.cb * BM,
                                     w0 + J.fw0 - g.pad, hh + cc.fh - g.pad, nn);
                     if (lane == 0) TRACE(0, ch - c_lo + jb * 64, 2);
                     if (lane == 1) TRACE(0, ch - c_lo + jb * 64, 3);
@@ -1115,7 +1125,7 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         // sub-partition takes more: the chunk rate follows the average unit
         // cost instead of the slowest fixed role.  Ring stage / parity follow
         // from the global chunk index, as in the producer and MMA loops.
-        constexpr int NU = units_per_chunk<BM, NAT, pair_units<A0, R0>()>();
+        constexpr int NU = units_per_chunk<BM, NAT, pair_units<A0, R0>(), YB>();
         const int kv = g.K - cc.kb * BN, cv = g.C - cc.cb * BM;
         int jlo[1 + 9], jhi[1 + 9];
         for (int jb = 0; jb < njobs; ++jb) chunk_range(jobs[jb], &jlo[jb], &jhi[jb]);
@@ -1189,8 +1199,8 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             else
 #endif
             if constexpr (NAT) native_unit<BM, BF>(raw, op, u, lane, kv, cv, mid);
-            else if (jobs[jb].phase == 0) transform_unit_paired<A0, N0, R0, BM, BF, pair_units<A0, R0>()>(raw, op, u, lane, kv, cv, mid_op, mid_raw, args.ybn);
-            else if constexpr (A1 != 0) transform_unit_paired<A1, N1, R1, BM, BF, pair_units<A0, R0>()>(raw, op, u, lane, kv, cv, mid_op, mid_raw, args.ybn);
+            else if (jobs[jb].phase == 0) transform_unit_paired<A0, N0, R0, BM, BF, pair_units<A0, R0>(), YB>(raw, op, u, lane, kv, cv, mid_op, mid_raw, args.ybn);
+            else if constexpr (A1 != 0) transform_unit_paired<A1, N1, R1, BM, BF, pair_units<A0, R0>(), YB>(raw, op, u, lane, kv, cv, mid_op, mid_raw, args.ybn);
 #ifndef WINRS_NO_FENCE
             fence_proxy_async();
 #endif

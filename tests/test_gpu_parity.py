@@ -161,6 +161,24 @@ FORCED_F16 = [
 ]
 
 
+# K <= 64: 64-row dY raw stages (the alpha = 8 YB = 64 kernel variant) with
+# ragged K and C, the B_N = 128 kernels with 64-row boxes (128x32 tile,
+# Omega_4(3,2)), cluster split and buckets.
+K64_F16 = [
+    ({"K": 64, "C": 64}, {"WINRS_FORCE_PAIR": "8,3,6,0,0,0", "WINRS_FORCE_TILE": "128x64"}),
+    ({"K": 40, "C": 72}, {"WINRS_FORCE_PAIR": "8,3,6,0,0,0", "WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "4"}),
+    ({"K": 8, "C": 136}, {"WINRS_FORCE_PAIR": "8,3,6,0,0,0", "WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_Z": "3"}),
+    ({"K": 56, "C": 64}, {"WINRS_FORCE_PAIR": "8,3,6,0,0,0", "WINRS_FORCE_TILE": "128x32"}),
+    ({"K": 64, "C": 128}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "2"}),
+]
+
+
+@pytest.mark.parametrize("shape,env", K64_F16, ids=lambda v: ",".join(f"{k}={x}" for k, x in v.items()) if isinstance(v, dict) else str(v))
+def test_k_le_64_f16(shape, env, monkeypatch):
+    layer = wl.LAYERS["r50_c64_56_f16"].with_(N=2, H=22, W=23, name="k64_" + str(shape["K"]), **shape)
+    _full_check(layer, env=env, monkeypatch=monkeypatch)
+
+
 @pytest.mark.parametrize("env", FORCED_F16, ids=lambda e: ",".join(f"{k[12:]}={v}" for k, v in e.items()))
 def test_forced_plans_f16(env, monkeypatch):
     layer = wl.LAYERS["r50_c64_56_f16"].with_(N=2, H=30, W=29, C=72, K=136, name="forced16")
