@@ -12,7 +12,7 @@ __device__ __forceinline__ uint64_t desc(uint32_t a, uint32_t lbo, uint32_t sbo,
            (1ull << 46) | ((uint64_t)layout << 61);
 }
 
-template <int N, bool TS = false>
+template <int N, bool TS = false, int M = 128>
 __global__ void __launch_bounds__(128, 1) k(unsigned long long* out, int iters, int per, uint32_t lbo, uint32_t sbo, int layout) {
     extern __shared__ __align__(1024) uint8_t sm[];
     __shared__ uint64_t bar;
@@ -31,7 +31,7 @@ __global__ void __launch_bounds__(128, 1) k(unsigned long long* out, int iters, 
     asm volatile("tcgen05.fence::before_thread_sync;");
     __syncthreads();
     asm volatile("tcgen05.fence::after_thread_sync;");
-    const uint32_t idesc = (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+    const uint32_t idesc = (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
     if (threadIdx.x == 0) {
         const uint32_t a0 = smem_u32(sm), b0 = smem_u32(sm + 32 * 1024);
         uint32_t ph = 0;
@@ -63,13 +63,13 @@ __global__ void __launch_bounds__(128, 1) k(unsigned long long* out, int iters, 
     if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tbase));
 }
 
-template <int N, bool TS = false>
+template <int N, bool TS = false, int M = 128>
 void run(int per, uint32_t lbo, uint32_t sbo, int layout, const char* name) {
     unsigned long long* d;
     cudaMalloc(&d, 8 * 148);
-    cudaFuncSetAttribute(k<N, TS>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024 + 1024);
+    cudaFuncSetAttribute(k<N, TS, M>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024 + 1024);
     const int iters = 200;
-    k<N, TS><<<148, 128, 64 * 1024 + 1024>>>(d, iters, per, lbo, sbo, layout);
+    k<N, TS, M><<<148, 128, 64 * 1024 + 1024>>>(d, iters, per, lbo, sbo, layout);
     cudaError_t e = cudaDeviceSynchronize();
     unsigned long long h[148];
     cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
@@ -78,18 +78,16 @@ void run(int per, uint32_t lbo, uint32_t sbo, int layout, const char* name) {
     avg /= 148;
     const double cyc = avg / iters / per;
     printf("%-28s N=%3d per=%2d: %7.1f cycles/MMA  -> %6.0f MAC/clk/SM (%s)\n", name, N, per, cyc,
-           128.0 * N * 16 / cyc, cudaGetErrorString(e));
+           (double)M * N * 16 / cyc, cudaGetErrorString(e));
     cudaFree(d);
 }
 
 int main() {
     for (int per : {8, 32}) {
-        run<64>(per, 128, 256, 0, "SS noswz");
-        run<64>(per, 16, 256, 6, "SS swz32 sbo256");
-        run<128>(per, 16, 256, 6, "SS swz32 sbo256");
-        run<64, true>(per, 128, 256, 0, "TS(A in TMEM) B noswz");
-        run<128, true>(per, 128, 256, 0, "TS(A in TMEM) B noswz");
-        run<64, true>(per, 16, 256, 6, "TS(A in TMEM) B swz32");
+        run<64>(per, 128, 256, 0, "SS noswz M128");
+        run<64, false, 64>(per, 128, 256, 0, "SS noswz M64");
+        run<128>(per, 128, 256, 0, "SS noswz M128");
+        run<128, false, 64>(per, 128, 256, 0, "SS noswz M64");
     }
     return 0;
 }
