@@ -60,6 +60,9 @@ constexpr int KC = 16;           // depth entries per chunk = UMMA K
 #define WINRS_F16_RR 2           // 1: static round-robin unit assignment instead of the shared counter; 2: for alpha = 4 only
                                  // (measured on B200: round-robin 6-12% faster for alpha = 4, 15% slower for alpha = 8)
 #endif
+#ifndef WINRS_F16_DEEPRAW
+#define WINRS_F16_DEEPRAW 1      // paired Omega_4(3,2) at B_M = 128: 3 operand + 5 raw stages, 14 transformer warps
+#endif
 #ifndef WINRS_F16_RAWMAX
 #define WINRS_F16_RAWMAX 4       // cap on raw (TMA) ring stages
 #endif
@@ -130,9 +133,15 @@ template <int BM, bool FEW = false> __host__ __device__ constexpr int tx_warps()
     return !WINRS_F16_DYN ? n_units<BM>() : WINRS_F16_TXW > 0 ? WINRS_F16_TXW : BM >= 128 ? (FEW ? 12 : 14) : 10;
 }
 template <int BM, bool FEW = false> __host__ __device__ constexpr int nthreads() { return 64 + 32 * tx_warps<BM, FEW>(); }
-// FEW: 4 units per chunk at B_M = 128 (paired or native units)
+// Deep raw ring for the paired Omega_4(3,2) kernels at B_M = 128: 5 raw
+// stages keep the parity bound with 14 transformer warps (17 >= 14).
+template <int A0, int R0, int BM> __host__ __device__ constexpr bool deep_raw() {
+    return WINRS_F16_DEEPRAW && pair_units<A0, R0>() && BM >= 128;
+}
+// FEW: 4 units per chunk at B_M = 128 (paired or native units) with the
+// 4-stage raw ring -> 12 transformer warps.
 template <int A0, int N0, int R0, int A1, int BM> __host__ __device__ constexpr bool few_units() {
-    return pair_units<A0, R0>() || native_path<A0, N0, R0, A1, BM>();
+    return (pair_units<A0, R0>() && !deep_raw<A0, R0, BM>()) || native_path<A0, N0, R0, A1, BM>();
 }
 template <int A0, int N0, int R0, int A1, int BM> __host__ __device__ constexpr int kthreads() {
     return nthreads<BM, few_units<A0, N0, R0, A1, BM>()>();
@@ -273,7 +282,8 @@ __device__ __forceinline__ F2 ld_h2(const __half* p) {
 }
 
 // ----------------------------------------------------------------------------- shared memory plan
-template <int A0, int R0, int BM, int YB = BN>
+// DR (deep raw ring): 3 operand stages and up to 5 raw stages instead of 4 + 4.
+template <int A0, int R0, int BM, int YB = BN, bool DR = false>
 struct Smem {
     static constexpr int RAW_Y = KC * R0 * YB * 2;       // bytes per raw stage (dY; YB k rows per box)
     static constexpr int RAW_X = KC * A0 * BM * 2;       // bytes per raw stage (X)
@@ -285,9 +295,10 @@ struct Smem {
     // operand stages: the deeper the ring, the less the transformers wait for
     // the MMAs of the chunk S_OP back; keep >= 3 raw stages for TMA latency.
     static constexpr int S_OP = WINRS_F16_SOP > 0 ? WINRS_F16_SOP
-                              : (LIMIT - 4 * OP) / RAW >= 3 ? 4 : (LIMIT - 3 * OP) / RAW >= 3 ? 3 : 2;
+                              : DR ? 3 : (LIMIT - 4 * OP) / RAW >= 3 ? 4 : (LIMIT - 3 * OP) / RAW >= 3 ? 3 : 2;
     // as many raw (TMA) stages as fit: the raw ring is the latency-hiding depth
-    static constexpr int S_RAW = (LIMIT - S_OP * OP) / RAW > WINRS_F16_RAWMAX ? WINRS_F16_RAWMAX : (LIMIT - S_OP * OP) / RAW;
+    static constexpr int RAWMAX = DR ? 5 : WINRS_F16_RAWMAX;
+    static constexpr int S_RAW = (LIMIT - S_OP * OP) / RAW > RAWMAX ? RAWMAX : (LIMIT - S_OP * OP) / RAW;
     static_assert(S_RAW >= 2 && S_RAW <= 8, "raw ring: 2..8 stages");
     static constexpr int raw_off = 0;
     static constexpr int op_off = S_RAW * RAW;
@@ -750,7 +761,8 @@ template <int N0, int BM> __host__ __device__ constexpr bool csplit_fits() {
 }
 template <int A0, int N0, int R0, int BM, int YB = BN> __host__ __device__ constexpr size_t smem_total() {
     const size_t out = csplit_fits<N0, BM>() ? (size_t)N0 * BN * out_ld<BM>() * 4 : 0;
-    return Smem<A0, R0, BM, YB>::bytes > out ? Smem<A0, R0, BM, YB>::bytes : out;
+    using SMx = Smem<A0, R0, BM, YB, deep_raw<A0, R0, BM>()>;
+    return SMx::bytes > out ? SMx::bytes : out;
 }
 // The YB = 64 variant (K <= 64: 64-row dY raw stages, only the FT units of
 // the first 64-row block, a deeper raw ring) for the alpha = 8 single-kernel
@@ -924,7 +936,7 @@ __global__ void __launch_bounds__((kthreads<A0, N0, R0, A1, BM>()), 1)
 bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX0,
                const __grid_constant__ CUtensorMap tmY0, const __grid_constant__ CUtensorMap tmX1,
                const __grid_constant__ CUtensorMap tmY1) {
-    using SM = Smem<A0, R0, BM, YB>;
+    using SM = Smem<A0, R0, BM, YB, deep_raw<A0, R0, BM>()>;
     static_assert(YB == BN || (YB == 64 && yb64_variant<A0, R0, A1, BM>()), "64-row dY stages: alpha = 8 single-kernel pairs");
     constexpr int S_RAW = SM::S_RAW;
     constexpr int TX_WARPS = tx_warps<BM, few_units<A0, N0, R0, A1, BM>()>();
