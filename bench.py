@@ -24,7 +24,6 @@ import argparse
 import json
 import os
 import statistics
-import subprocess
 import sys
 import threading
 import time
@@ -77,52 +76,80 @@ def _workload(name: str, dtype: str):
 
 
 class ClockSampler:
-    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+    """SM clocks and clock-event (throttle) reasons sampled during the timed region.
 
-    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
-              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-              "clocks_event_reasons.sw_power_cap")
+    In-process NVML (pynvml): a background thread polls every ~1 ms, and the
+    timed loop calls ``sample()`` itself while it waits for the queued steps
+    to drain, so even a timed region of a few milliseconds gets samples taken
+    while the GPU is busy.  nvidia-smi (~100 ms minimum period, ~0.5 s start
+    up) never landed a sample inside the short ResNet-50 step.
+    """
 
-    def __init__(self, index: int):
-        self.index = index
+    REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
+               ("sw_power_cap", 0x4), ("hw_power_brake_slowdown", 0x80))
+
+    def __init__(self, cuda_index: int):
         self.rows = []
-        self.proc = None
+        self.h = None
+        self.nvml = None
+        self.stop_flag = False
         self.t = None
+        self.lock = threading.Lock()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nvml = pynvml
+            self.h = self._handle(cuda_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.h = None
+
+    def _handle(self, cuda_index):
+        pynvml = self.nvml
+        try:
+            import torch
+            p = torch.cuda.get_device_properties(cuda_index)
+            bus = f"{p.pci_domain_id:08X}:{p.pci_bus_id:02X}:{p.pci_device_id:02X}.0"
+            return pynvml.nvmlDeviceGetHandleByPciBusId(bus)
+        except Exception:
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES", "")
+            ids = [v.strip() for v in vis.split(",") if v.strip()]
+            idx = int(ids[cuda_index]) if cuda_index < len(ids) and ids[cuda_index].isdigit() else cuda_index
+            return pynvml.nvmlDeviceGetHandleByIndex(idx)
+
+    def sample(self):
+        if self.h is None:
+            return
+        try:
+            sm = self.nvml.nvmlDeviceGetClockInfo(self.h, self.nvml.NVML_CLOCK_SM)
+            rs = self.nvml.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+        except Exception:
+            return
+        with self.lock:
+            self.rows.append((sm, rs))
+
+    def _loop(self):
+        while not self.stop_flag:
+            self.sample()
+            time.sleep(0.001)
 
     def start(self):
-        try:
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
-                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
-            self.t.start()
-        except Exception:
-            self.proc = None
-
-    def _read(self):
-        for line in self.proc.stdout:
-            self.rows.append([x.strip() for x in line.split(",")])
+        if self.h is None:
+            return
+        self.t = threading.Thread(target=self._loop, daemon=True)
+        self.t.start()
 
     def stop(self):
-        if self.proc is None:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        time.sleep(0.15)
-        self.proc.terminate()
-        try:
-            self.proc.wait(timeout=2)
-        except Exception:
-            self.proc.kill()
-        sm = [float(r[0]) for r in self.rows if len(r) >= 7 and r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if len(r) >= 7 and r[1].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = set()
-        for r in self.rows:
-            if len(r) >= 7:
-                for nme, v in zip(names, r[3:7]):
-                    if v.lower() == "active":
-                        reasons.add(nme)
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+        if self.h is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"], "samples": 0}
+        self.stop_flag = True
+        if self.t is not None:
+            self.t.join(timeout=2)
+        sm = [r[0] for r in self.rows]
+        reasons = sorted({n for _, rs in self.rows for n, bit in self.REASONS if rs & bit})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": self.max_mhz,
+                "sm_min_mhz": min(sm) if sm else None, "reasons": reasons, "samples": len(sm),
+                "source": "nvml"}
 
 
 def run_winrs(args):
@@ -211,6 +238,9 @@ def run_winrs(args):
     torch.cuda.synchronize()
     for s in range(args.steps):
         one_step(ev[s])
+    if rank == 0:
+        while not ev[-1][-1][1].query():                           # GPU still draining the steps
+            clocks.sample()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
