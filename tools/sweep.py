@@ -56,7 +56,9 @@ for l in layers:
                     ts.append(a.elapsed_time(b))
             ms = statistics.median(ts)
             print(json.dumps({"layer": l.name, "pair": p.kernel_name, "tile": t, "csplit": p.info["csplit"], "Z": p.info["Z"],
-                              "ctas": p.info["ctas_main"], "ewm": p.info["ewm_flops"], "us": round(ms * 1e3, 1),
+                              "ctas": p.info["ctas_main"], "ws": p.workspace_bytes,
+                              "data": l.N * (l.H * l.W * l.C + p.info["Ho"] * p.info["Wo"] * l.K) * (4 if l.dtype == "f32" else 2),
+                              "ewm": p.info["ewm_flops"], "us": round(ms * 1e3, 1),
                               "tflops": round(l.direct_flops / ms / 1e9, 1)}), flush=True)
 os.environ.pop("WINRS_FORCE_TILE", None)
 os.environ.pop("WINRS_FORCE_CSPLIT", None)
