@@ -61,7 +61,9 @@ constexpr int KC = 16;           // depth entries per chunk = UMMA K
                                  // (measured on B200: round-robin 6-12% faster for alpha = 4, 15% slower for alpha = 8)
 #endif
 #ifndef WINRS_F16_DEEPRAW
-#define WINRS_F16_DEEPRAW 1      // paired Omega_4(3,2) at B_M = 128: 3 operand + 5 raw stages, 14 transformer warps
+#define WINRS_F16_DEEPRAW 0      // paired Omega_4(3,2) at B_M = 128: 3 operand + 5 raw stages, 14 transformer warps.
+                                 // Off: 14 > 3 * 4 breaks the operand-ring parity bound (intermittent hang
+                                 // under cold L2 on B200, tools/hang_repro.py); the static_assert now rejects it.
 #endif
 #ifndef WINRS_F16_RAWMAX
 #define WINRS_F16_RAWMAX 4       // cap on raw (TMA) ring stages
@@ -945,6 +947,22 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     static_assert(!WINRS_F16_DYN ||
                   TX_WARPS <= (S_RAW - 1) * units_per_chunk<BM, native_path<A0, N0, R0, A1, BM>(), pair_units<A0, R0>(), YB>() + 1,
                   "in-order unit hand-out could run a full raw ring ahead of the TMA (parity-wait aliasing)");
+    // Operand ring: a unit of chunk c waits (by parity) for the MMAs of chunk
+    // c - S_OP.  While one unit of chunk s is held up, the MMAs stop at s, so
+    // units of chunks s+S_OP .. s+2*S_OP-1 block in that wait; a unit of chunk
+    // s + 2*S_OP would see the completed phase of chunk s - S_OP and overwrite
+    // an operand stage the tensor core has not read.  Reaching it needs more
+    // than S_OP * units_per_chunk + 1 warps (in-order hand-out) or a
+    // round-robin stride above S_OP * units_per_chunk.  Otherwise the raw ring
+    // must gate it: with S_RAW == 2 * S_OP the TMA of chunk s + 2*S_OP waits
+    // for chunk s's own raw release, so the held unit would have to stall a
+    // whole TMA round trip between its raw release and its operand arrival
+    // ("operand-ring parity"; the YB = 64 and alpha = 8,
+    // B_M = 64 kernels rely on this gate).
+    constexpr int NU_ = units_per_chunk<BM, native_path<A0, N0, R0, A1, BM>(), pair_units<A0, R0>(), YB>();
+    constexpr bool RR_ = WINRS_F16_RR == 1 || (WINRS_F16_RR == 2 && A0 == 4);
+    static_assert(!WINRS_F16_DYN || TX_WARPS <= SM::S_OP * NU_ + (RR_ ? 0 : 1) || S_RAW == 2 * SM::S_OP,
+                  "transformer units could run two operand-ring phases ahead of the MMAs (parity-wait aliasing)");
     constexpr bool kCluster = csplit_fits<N0, BM>();
     constexpr bool NAT = native_path<A0, N0, R0, A1, BM>();
     extern __shared__ __align__(1024) uint8_t smem[];

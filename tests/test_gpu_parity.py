@@ -5,6 +5,8 @@ Gate (BASELINE.json north_star): max|err| <= 1e-4 * max|ref| for FP32 inputs,
 <= 2e-2 * max|ref| for FP16 inputs (FP32 accumulation).  Inputs follow the
 paper's accuracy protocol (P@50685): U[0,1], dY x 1e-2 for FP16.
 """
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -259,3 +261,18 @@ def test_bf16_full_size_sampled():
     idx = wl.sample_indices(layer, 256)
     ref = O.bfc_c_sampled(X, dY, layer.R, layer.S, layer.pad, idx)
     assert O.rel_max_err(got.ravel()[idx], ref) <= TOL["bf16"]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("z,tile,cs", [(4, "128x128", 8), (7, "128x128", 8), (4, "128x128", 4)])
+def test_no_hang_partial_tile_alpha4_cold_l2(z, tile, cs):
+    """Regression: the deep-raw-ring Omega_4(3,2) kernel (14 transformer warps,
+    3 operand stages) broke the operand-ring parity bound and hung within a few
+    hundred cold-L2 calls on these forced ResNet-50 L1 plans.  Run 1500 calls
+    in a child process under a hard timeout so a hang fails instead of blocking."""
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, os.path.join(root, "tools", "hang_repro.py"), "r50_c64_56_f16",
+                        str(z), tile, str(cs), "1500"], capture_output=True, text=True, timeout=240, cwd=root)
+    assert r.returncode == 0 and "done 1500" in r.stdout, r.stdout + r.stderr
