@@ -238,6 +238,8 @@ def run_winrs(args):
     torch.cuda.synchronize()
     for s in range(args.steps):
         one_step(ev[s])
+        if rank == 0:
+            clocks.sample()                                        # GPU busy with the queued layers
     if rank == 0:
         while not ev[-1][-1][1].query():                           # GPU still draining the steps
             clocks.sample()
