@@ -1,0 +1,106 @@
+// Instantiations, TMA tensor maps and launch of the second-generation
+// FP16 / BF16 tensor-core kernel (bfc_tc2.cuh).
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <mutex>
+#include "bfc_tc2.cuh"
+#include "launch_util.cuh"
+#include "registry.h"
+
+namespace winrs {
+namespace tc2 {
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static EncodeTiledFn encode_fn() {
+    static EncodeTiledFn fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<EncodeTiledFn>(p);
+    });
+    return fn;
+}
+
+// 4-D NHWC 16-bit tensor [N][H][W][Ch] (pixel stride ld >= Ch elements) as
+// TMA dims {Ch, N, H, W} (so a box lands as [cols][rows][images][channels]),
+// box {64, bn, 1, bw}, 128-byte swizzle: every (col, image) is one 128-byte
+// row of a UMMA MN-major SW128 atom.  Out-of-bounds elements read as zero.
+static bool make_map(CUtensorMap* m, const void* base, int N, int H, int W, int Ch, int ld, int bw, int bn, bool bf) {
+    EncodeTiledFn fn = encode_fn();
+    if (!fn) return false;
+    const cuuint64_t dims[4] = {(cuuint64_t)Ch, (cuuint64_t)N, (cuuint64_t)H, (cuuint64_t)W};
+    const cuuint64_t strides[3] = {(cuuint64_t)H * W * ld * 2, (cuuint64_t)W * ld * 2, (cuuint64_t)ld * 2};
+    const cuuint32_t box[4] = {64u, (cuuint32_t)bn, 1u, (cuuint32_t)bw};
+    const cuuint32_t es[4] = {1u, 1u, 1u, 1u};
+    return fn(m, bf ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void*>(base),
+              dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// Images per TMA box: one box per stage and atom, so the box's [cols][images]
+// rows are exactly a column-major run of 16-row operand atoms (N % 16 == 0).
+static int images_per_box(int N) { return N % KC == 0 ? KC : 0; }
+
+template <int F, int NK, bool BF>
+cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
+    using L = Lay<F, NK>;
+    const long long grid = num_ctas(g);
+    if (grid <= 0) return cudaSuccess;
+    Args a;
+    a.g = g;
+    a.dW = dW;
+    a.ws = ws;
+    a.nb = images_per_box(g.N);
+    if (a.nb == 0 || g.a0 != 4 || g.n0 != 3 || g.r0 != 2 || g.a1 != 0) return cudaErrorInvalidValue;
+    CUtensorMap mX, mY;
+    if (!make_map(&mX, X, g.N, g.H, g.W, g.C, g.C, 4, a.nb, BF) ||
+        !make_map(&mY, dY, g.N, g.Ho, g.Wo, g.K, g.ldy, 2, a.nb, BF))
+        return cudaErrorInvalidValue;
+    static std::atomic<unsigned long long> done{0};
+    auto k = bfc_tc2_kernel<F, NK, BF>;
+    cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
+    if (e != cudaSuccess) return e;
+    if (g.csplit <= 1) {
+        k<<<(unsigned)grid, NTHREADS, L::BYTES, stream>>>(a, mX, mY);
+        return cudaGetLastError();
+    }
+    return launch_cluster(k, (unsigned)grid, (unsigned)NTHREADS, (size_t)L::BYTES, stream, g.csplit, a, mX, mY);
+}
+
+}  // namespace tc2
+
+#define WINRS_TC2_ENTRY(DT, BF, PFX, F, NK)                                                              \
+    {DT, 4, 3, 2, 0, 0, 0, NK, ::winrs::tc2::MROWS / F, ::winrs::tc2::NTHREADS, 1, 1,                    \
+     (size_t)::winrs::tc2::Lay<F, NK>::BYTES, &::winrs::tc2::launch<F, NK, BF>,                           \
+     PFX "_O4(3,2)_v2_" #NK "x" #F "fh", F}
+
+#ifdef WINRS_TC2_TRACE
+extern "C" __attribute__((visibility("default"))) int winrs_tc2_trace(int cta, long long* out) {
+    if (cta >= 0) return (int)cudaMemcpyToSymbol(tc2::g_tc2_trace_cta, &cta, sizeof(int));
+    return (int)cudaMemcpyFromSymbol(out, tc2::g_tc2_trace, sizeof(tc2::g_tc2_trace));
+}
+#endif
+
+const KernelEntry* tc2_entries(int* n) {
+    // tile = NK k columns x (128 / F) c rows x F filter rows
+    static const KernelEntry e[] = {
+        WINRS_TC2_ENTRY(1, false, "f16tc", 1, 128),
+        WINRS_TC2_ENTRY(1, false, "f16tc", 1, 64),
+        WINRS_TC2_ENTRY(1, false, "f16tc", 2, 128),
+        WINRS_TC2_ENTRY(1, false, "f16tc", 2, 64),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 1, 128),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 1, 64),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 128),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 64),
+    };
+    *n = sizeof(e) / sizeof(e[0]);
+    return e;
+}
+
+}  // namespace winrs

@@ -1,0 +1,490 @@
+// Second-generation FP16 / BF16 tensor-core WinRS BFC kernel for sm_100a
+// (tcgen05 + TMEM + TMA + mbarrier), kernel Omega_4(3,2) (Figure 6,
+// P@28451; the F_W = 3 member of the ported FP16 set, P@28616).
+//
+// What it computes (§3 eq. (6), P@31000-32161): for a CTA tile
+// (segment z, filter-row group, c-block, k-block) and every unit u of r0 = 2
+// dY columns of every clipped dY row h of the segment and every image n,
+//     v[xi][m][k] += Xhat[xi](n, h + fh(m) - pad, u)[c(m)] * What[xi](n, h, u)[k]
+// with What = G w (FT of the dY unit, P@30202 Alg. 3) and Xhat = D^T x (IT of
+// the alpha = 4 X window, P@30341), then dW_z[k][fh][s][c] = (A^T v)[s] (OT,
+// P@31000).  The transforms (R20):
+//     FT  What = (w0 + w1, w0 - w1, w0, w1)
+//     IT  Xhat = (x1 + x2, x2 - x1, x0 - x2, x3 - x1)
+//     OT  y0 = (v0 + v1)/2 + v2,  y1 = (v0 - v1)/2,  y2 = (v0 + v1)/2 + v3
+// (interpolation points 1, -1, 0, inf: the Cook-Toom F(3,2) of
+// tools/gen_winograd.py with the eq. (7) row scaling moved from G and D^T into
+// A, so every FT / IT output is ONE add or subtract of two inputs).
+//
+// B200 design (each choice measured on B200):
+//   * The EWM is a 4-batched GEMM with M = 128 TMEM lanes = X rows (fh slot,
+//     c) and N = NK = 64 / 128 k columns (all 512 TMEM columns at NK = 128).
+//   * The IT runs INSIDE the tensor core: by linearity
+//         v0 = x1 W0 + x2 W0,  v1 = x2 W1 - x1 W1,
+//         v2 = x0 W2 - x2 W2,  v3 = x3 W3 - x1 W3,
+//     8 MMAs per 16-deep stage whose A operands are the raw X columns x_t,
+//     landed by TMA directly in the UMMA operand layout (MN-major, 128-byte
+//     swizzle), the minus signs being the instruction descriptor's negate-A
+//     bit.  Measured (WINRS_TC2_NO_MMA / _NO_STS ablations): the tensor core's
+//     shared-memory reads do not compete with TMA / LDS / STS traffic, while
+//     thread-side operand stores cost a third of every stage, so trading the
+//     IT's 16 KB of loads + 16 KB of stores per stage for 4 extra MMAs is a
+//     net win.  The products are exact and accumulate in FP32: the IT adds no
+//     rounding at all.
+//   * The FT stays on threads (What[0,1] = w0 +- w1 in packed 16-bit adds:
+//     one correctly rounded add, the FP16 value P@38729's "computed in FP32,
+//     then converted" produces); What[2,3] are the raw dY columns (TMA).
+//   * For C <= 64 two filter rows share the M = 128 tile (F = 2: rows
+//     [0,64) are fh0's X windows, [64,128) fh0+1's) so K = C = 64 layers do
+//     not waste half of every MMA.
+//   * One ring of S stages (KC = 16 depth entries each); a stage holds the TMA
+//     data and the FT operands of the same 16 depth entries, so it has exactly
+//     one owner at a time: TMA -> FT threads -> MMA -> (commit) TMA.  Every
+//     FT warp processes every stage in order and only the MMA commit frees a
+//     stage, so a warp can never be a full ring ahead of the MMAs and no
+//     phase-parity wait can alias (safe by construction; round 1's
+//     dynamically handed-out units needed a timing argument).
+//
+// Warp roles (320 threads, one CTA per SM):
+//   warp 0     TMA producer (one lane per box)
+//   warp 1     TMEM allocator + MMA issuer
+//   warps 2-9  FT (256 threads: at most one (k octet, depth) item per stage),
+//              then the epilogue (tcgen05.ld -> OT -> bucket, or -> shared
+//              staging tile -> DSMEM cluster reduction).
+#pragma once
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include "dsmem.cuh"
+#include "winrs_internal.h"
+
+namespace winrs {
+namespace tc2 {
+
+constexpr int KC = 16;                 // depth entries per stage = UMMA K
+constexpr int MROWS = 128;             // UMMA M = TMEM lanes
+constexpr int NTX = 8;                 // transformer warps
+constexpr int NTHREADS = 64 + 32 * NTX;
+constexpr int NSOUT = 3;               // n0: outputs per unit (S = 3)
+
+template <int F, int NK>
+struct Lay {
+    static constexpr int BC = MROWS / F;                 // channels c per fh slot
+    // One stage = 16 depth entries (images n of one (h, u)), three regions of
+    // 64-channel swizzle atoms [atom][col][n (16 rows of 128 B)]:
+    //   X   [2 atoms][4 cols x_t]   16 KB   A operand of column t: +t*2 KB, atoms 8 KB apart
+    //                                        (atom = c half for F = 1, fh slot for F = 2)
+    //   Y   [NK/64 atoms][w0, w1]   8/4 KB  What[2], What[3]: +0 / +2 KB, atoms 4 KB apart
+    //   FT  [NK/64 atoms][W0, W1]   8/4 KB  What[0], What[1] (stored by the FT threads)
+    static constexpr int ATOM = KC * 128;                // 2 KB: 64 channels x 16 depth rows
+    static constexpr int X_LBO = 4 * ATOM;               // 8 KB
+    static constexpr int Y_LBO = 2 * ATOM;               // 4 KB
+    static constexpr int OFF_Y = 2 * X_LBO;              // 16 KB
+    static constexpr int OFF_F = OFF_Y + (NK / 64) * Y_LBO;
+    static constexpr int STAGE = OFF_F + (NK / 64) * Y_LBO;   // 32 / 24 KB
+    static constexpr int LIMIT = 227 * 1024 - 1024 - 256;
+    static constexpr int S = LIMIT / STAGE > 8 ? 8 : LIMIT / STAGE;
+    static constexpr int RING = S * STAGE;
+    static constexpr int OUT = NSOUT * NK * MROWS * 4;   // staging tile [s][k][m] fp32 (cluster split)
+    static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
+    static constexpr int BYTES = BAR_OFF + 256 + 1024;   // + alignment slack
+    static constexpr int TX_BYTES = OFF_F;               // TMA bytes per stage
+    static constexpr int TMEM_COLS = 4 * NK;
+    static_assert(STAGE % 1024 == 0, "stages must keep the 1 KB swizzle-atom alignment");
+    static_assert(S >= 4, "ring too shallow");
+    static_assert(MROWS == F * BC && BC % 64 == 0, "fh slots of whole 64-channel atoms");
+};
+
+struct Args {
+    Geometry g;
+    float* dW;
+    float* ws;
+    int nb;            // images per TMA box (divides N and KC, >= 8)
+};
+
+struct Bars {
+    uint64_t full[8];       // TMA data landed
+    uint64_t opfull[8];     // FT operands stored (8 warp arrivals)
+    uint64_t empty[8];      // MMAs of the stage done (commit)
+    uint64_t accfull;
+    uint32_t tmem_base;
+};
+
+// ----------------------------------------------------------------------------- PTX helpers
+__device__ __forceinline__ uint32_t su(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t n) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(su(b)), "r"(n));
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(su(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(su(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+    asm volatile(
+        "{\n.reg .pred P;\nW_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1, %2;\n"
+        "@!P bra W_%=;\n}\n" :: "r"(su(b)), "r"(parity), "r"(1000000) : "memory");
+}
+__device__ __forceinline__ void tma4(uint32_t dst, const CUtensorMap* m, uint64_t* bar, int c0, int c1, int c2, int c3) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];"
+        :: "r"(dst), "l"(reinterpret_cast<uint64_t>(m)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(su(bar)) : "memory");
+}
+// One lane of a converged warp (elect.sync).  Issuing tcgen05.mma / TMA from
+// an elected lane of a converged warp lets the compiler keep the operands in
+// uniform registers; inside `if (lane == 0)` every operand goes through an
+// R2UR waterfall loop (~50-70 cycles per instruction, measured: the MMA issue
+// and the TMA issue each took ~500 cycles per stage that way).
+__device__ __forceinline__ bool elect_one() {
+    uint32_t pred;
+    asm volatile("{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\nselp.u32 %0, 1, 0, p;\n}\n" : "=r"(pred));
+    return pred != 0;
+}
+__device__ __forceinline__ void fence_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tc_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// UMMA shared-memory descriptor, MN-major, 128-byte swizzle: atoms of 64 MN
+// elements x 8 K rows (1 KB); LBO = MN-atom stride, SBO = K-atom stride
+// (probed on B200, tools/microbench/umma_mn.cu), version bit 46, layout 2.
+__device__ __forceinline__ uint64_t desc_sw128(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+    return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+           ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46) | (2ull << 61);
+}
+// kind::f16 instruction descriptor: D f32, A/B f16 (0) or bf16 (1), both
+// MN-major (bits 15, 16), N >> 3 at bit 17, M >> 4 at bit 24.
+// Bit 13: negate A (the IT's minus signs).
+template <int NK, bool BF, bool NEG = false>
+__host__ __device__ constexpr uint32_t idesc() {
+    return (1u << 4) | ((BF ? 1u : 0u) << 7) | ((BF ? 1u : 0u) << 10) | ((NEG ? 1u : 0u) << 13) | (1u << 15) |
+           (1u << 16) | ((uint32_t)(NK >> 3) << 17) | ((uint32_t)(MROWS >> 4) << 24);
+}
+template <int NK, bool BF, bool NEG = false>
+__device__ __forceinline__ void umma(uint32_t d, uint64_t a, uint64_t b, uint32_t acc) {
+    asm volatile(
+        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
+        :: "r"(d), "l"(a), "l"(b), "r"(idesc<NK, BF, NEG>()), "r"(acc));
+}
+__device__ __forceinline__ void umma_commit(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" :: "r"(su(bar)) : "memory");
+}
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, float* v) {
+    uint32_t r[8];
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+                 : "r"(taddr));
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
+// Byte offset of the 16-byte chunk (8 channels, octet o) at depth d of an
+// MN-major SW128 operand whose 64-channel atoms are `lbo` bytes apart (KC =
+// 16: two 1 KB K-atoms per atom; the chunk index is XORed with the row).
+__device__ __forceinline__ uint32_t opoff(int o, int d, int lbo) {
+    return (uint32_t)((o >> 3) * lbo + (d >> 3) * 1024 + (d & 7) * 128 + (((o & 7) ^ (d & 7)) << 4));
+}
+
+// Packed 16-bit add / subtract of four pairs (one rounding per element).
+template <bool BF> struct P16;
+template <> struct P16<false> {
+    __device__ static __forceinline__ uint32_t add(uint32_t a, uint32_t b) {
+        uint32_t r; asm("add.rn.f16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b)); return r;
+    }
+    __device__ static __forceinline__ uint32_t sub(uint32_t a, uint32_t b) {
+        uint32_t r; asm("sub.rn.f16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b)); return r;
+    }
+};
+template <> struct P16<true> {
+    __device__ static __forceinline__ uint32_t add(uint32_t a, uint32_t b) {
+        uint32_t r; asm("add.rn.bf16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b)); return r;
+    }
+    __device__ static __forceinline__ uint32_t sub(uint32_t a, uint32_t b) {
+        uint32_t r; asm("sub.rn.bf16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b)); return r;
+    }
+};
+template <bool BF>
+__device__ __forceinline__ uint4 vadd(const uint4& a, const uint4& b) {
+    return make_uint4(P16<BF>::add(a.x, b.x), P16<BF>::add(a.y, b.y), P16<BF>::add(a.z, b.z), P16<BF>::add(a.w, b.w));
+}
+template <bool BF>
+__device__ __forceinline__ uint4 vsub(const uint4& a, const uint4& b) {
+    return make_uint4(P16<BF>::sub(a.x, b.x), P16<BF>::sub(a.y, b.y), P16<BF>::sub(a.z, b.z), P16<BF>::sub(a.w, b.w));
+}
+__device__ __forceinline__ uint4 lds16(uint32_t a) {
+    uint4 v;
+    asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void sts16(uint32_t a, const uint4& v) {
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" :: "r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+
+#ifdef WINRS_TC2_TRACE
+// Debug-build timeline (clock64) of CTA `g_tc2_trace_cta`, per stage:
+// [0] producer past `empty`, [1] TMAs issued, [2] transformer warp 2 past `full`,
+// [3] its `opfull` arrival, [4] MMA warp past `opfull`, [5] MMAs + commit issued.
+__device__ long long g_tc2_trace[512][8];
+__device__ int g_tc2_trace_cta;
+#define TC2_TRACE(ch, ev) do { if (blockIdx.x == (unsigned)g_tc2_trace_cta && (ch) < 512) g_tc2_trace[ch][ev] = clock64(); } while (0)
+#else
+#define TC2_TRACE(ch, ev) do { } while (0)
+#endif
+
+// Depth entry d of a CTA -> (n, h, u): n fastest (d = ((h - hs) * units + u) * N + n).
+__device__ __forceinline__ void depth_nhu(int d, int N, int units, int hs, int* n, int* h, int* u) {
+    *n = d % N;
+    const int t = d / N;
+    *u = t % units;
+    *h = hs + t / units;
+}
+
+template <int F, int NK, bool BF>
+__global__ void __launch_bounds__(NTHREADS, 1)
+bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX,
+               const __grid_constant__ CUtensorMap tmY) {
+    using L = Lay<F, NK>;
+    extern __shared__ uint8_t smem_raw[];
+    // 1 KB-aligned base (SW128 atoms, TMA swizzle pattern)
+    const uint32_t raw_s = su(smem_raw);
+    uint8_t* smem = smem_raw + (((raw_s + 1023u) & ~1023u) - raw_s);
+    const uint32_t sbase = su(smem);
+    Bars* bars = reinterpret_cast<Bars*>(smem + L::BAR_OFF);
+    const Geometry& g = args.g;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 64) TC2_TRACE(511, 0);
+
+    const int rank = (int)(blockIdx.x % g.csplit);
+    const CtaCoord cc = decode_cta(g, blockIdx.x / g.csplit);
+    const int seg = cc.band * g.seg_cols + cc.col;
+    float* bucket = seg == 0 ? args.dW : args.ws + (long long)(seg - 1) * g.dw_elems;
+    int hs, he, w_first, units;
+    group_rows(g, cc.band, cc.fh, &hs, &he);
+    seg_units(g, cc.col, &w_first, &units);
+    const long long depth = (long long)(he > hs ? he - hs : 0) * units * g.N;
+    int c_lo, c_hi;
+    split_chunks((int)((depth + KC - 1) / KC), rank, g.csplit, &c_lo, &c_hi);
+    const bool empty_range = c_hi <= c_lo;
+    const int fw0 = cc.ft * NSOUT;       // first output column of this fw-tile (S = 3 * ftiles)
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < L::S; ++s) {
+            mbar_init(&bars->full[s], 1);
+            mbar_init(&bars->opfull[s], NTX);
+            mbar_init(&bars->empty[s], 1);
+        }
+        mbar_init(&bars->accfull, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 0 && lane == 0) {
+        asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+        asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+                     :: "r"(su(&bars->tmem_base)), "r"(L::TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_before();
+    __syncthreads();
+    tc_after();
+    const uint32_t tmem = bars->tmem_base;
+    if (threadIdx.x == 64) TC2_TRACE(511, 1);
+
+    if (warp == 0) {
+        // ============================ TMA producer ============================
+        // Converged warp, one elected lane issues the stage's boxes: X atoms
+        // 0 and 1 (c halves, or fh slots for F = 2) and the dY k atoms, each
+        // [64 ch][16 images][1 row][cols], i.e. one 128-byte swizzled row per
+        // (col, image) = the UMMA operand layout.  (n, u, h) advance
+        // incrementally (per-stage integer divisions cost ~700 cycles on an
+        // SM sub-partition shared with other warps: WINRS_TC2_TRACE timeline.)
+        long long d = (long long)c_lo * KC;
+        int n = 0, h = hs, u = 0;
+        if (d < depth) depth_nhu((int)d, g.N, units, hs, &n, &h, &u);
+        int s = 0;
+        uint32_t ph = 0;
+        for (int ch = c_lo; ch < c_hi; ++ch) {
+            mbar_wait(&bars->empty[s], ph ^ 1);
+            TC2_TRACE(ch - c_lo, 0);
+            uint64_t* fb = &bars->full[s];
+            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            const bool in = d < depth;               // past the end: image N (zero fill)
+            const int nn = in ? n : g.N, hh = in ? h : hs;
+            const int w0 = w_first + (in ? u : 0) * 2;
+            if (elect_one()) {
+#ifdef WINRS_TC2_NO_TMA   // debug ablation: stages carry no data (barrier protocol kept)
+                mbar_arrive(fb);
+#else
+                mbar_expect_tx(fb, (uint32_t)L::TX_BYTES);
+#pragma unroll
+                for (int a = 0; a < 2; ++a) {
+                    // X window columns x0..x3 of atom a; an fh slot past the last
+                    // filter row reads rows far outside (zero fill)
+                    const int fh = F == 2 ? cc.fh + a : cc.fh;
+                    const int c0 = F == 2 ? cc.cb * 64 : cc.cb * 128 + a * 64;
+                    const int xrow = fh < g.R ? hh + fh - g.pad : -(1 << 20);
+                    tma4(st + a * L::X_LBO, &tmX, fb, c0, nn, xrow, w0 + fw0 - g.pad);
+                }
+#pragma unroll
+                for (int ka = 0; ka < NK / 64; ++ka)   // dY unit columns w0, w0 + 1 of k atom ka
+                    tma4(st + L::OFF_Y + ka * L::Y_LBO, &tmY, fb, cc.kb * NK + ka * 64, nn, hh, w0);
+#endif
+            }
+            __syncwarp();
+            TC2_TRACE(ch - c_lo, 1);
+            d += KC;
+            n += KC;
+            while (n >= g.N) {
+                n -= g.N;
+                if (++u == units) { u = 0; ++h; }
+            }
+            if (++s == L::S) { s = 0; ph ^= 1; }
+        }
+    } else if (warp == 1) {
+        // ============================ MMA issuer ==============================
+        // Converged warp; descriptors are computed uniformly, one elected lane
+        // issues the MMAs and the commit.
+        int s = 0;
+        uint32_t ph = 0;
+        for (int ch = c_lo; ch < c_hi; ++ch) {
+            mbar_wait(&bars->opfull[s], ph);
+            TC2_TRACE(ch - c_lo, 4);
+            tc_after();
+            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            const uint32_t acc = ch > c_lo ? 1u : 0u;
+            // A: raw X column x_t (M = 128: two atoms X_LBO apart); B: What[xi]
+            const uint64_t x0 = desc_sw128(st, L::X_LBO, 1024);
+            const uint64_t x1 = x0 + (L::ATOM >> 4), x2 = x0 + (2 * L::ATOM >> 4), x3 = x0 + (3 * L::ATOM >> 4);
+            const uint64_t w0d = desc_sw128(st + L::OFF_F, L::Y_LBO, 1024), w1d = w0d + (L::ATOM >> 4);
+            const uint64_t w2d = desc_sw128(st + L::OFF_Y, L::Y_LBO, 1024), w3d = w2d + (L::ATOM >> 4);
+            if (elect_one()) {
+#ifndef WINRS_TC2_NO_MMA   // debug ablation: no tensor-core work (barrier protocol kept)
+                umma<NK, BF>(tmem + 0 * NK, x1, w0d, acc);          // v0 = (x1 + x2) W0
+                umma<NK, BF>(tmem + 0 * NK, x2, w0d, 1u);
+                umma<NK, BF>(tmem + 1 * NK, x2, w1d, acc);          // v1 = (x2 - x1) W1
+                umma<NK, BF, true>(tmem + 1 * NK, x1, w1d, 1u);
+                umma<NK, BF>(tmem + 2 * NK, x0, w2d, acc);          // v2 = (x0 - x2) W2
+                umma<NK, BF, true>(tmem + 2 * NK, x2, w2d, 1u);
+                umma<NK, BF>(tmem + 3 * NK, x3, w3d, acc);          // v3 = (x3 - x1) W3
+                umma<NK, BF, true>(tmem + 3 * NK, x1, w3d, 1u);
+#else
+                (void)x0; (void)x1; (void)x2; (void)x3; (void)w0d; (void)w1d; (void)w2d; (void)w3d; (void)acc;
+#endif
+                umma_commit(&bars->empty[s]);
+            }
+            __syncwarp();
+            TC2_TRACE(ch - c_lo, 5);
+            if (++s == L::S) { s = 0; ph ^= 1; }
+        }
+        if (elect_one()) umma_commit(&bars->accfull);   // arrives once all issued MMAs completed
+        __syncwarp();
+    } else {
+        // ================================= FT =================================
+        // item: depth df, k octet fo (t < 2 NK); What[0] = w0 + w1, What[1] = w0 - w1
+        const int t = threadIdx.x - 64;             // 0..255
+        constexpr int KO = NK / 8;
+        const bool has_ft = t < KO * KC;
+        const int df = t / KO, fo = t % KO;
+        const uint32_t ft_off = opoff(fo, df, L::Y_LBO);
+        int s = 0;
+        uint32_t ph = 0;
+        for (int ch = c_lo; ch < c_hi; ++ch) {
+            mbar_wait(&bars->full[s], ph);
+            if (threadIdx.x == 64) TC2_TRACE(ch - c_lo, 2);
+            if (has_ft) {
+                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+                const uint4 w0 = lds16(st + L::OFF_Y + ft_off), w1 = lds16(st + L::OFF_Y + L::ATOM + ft_off);
+#ifndef WINRS_TC2_NO_STS   // debug ablation: no operand stores
+                sts16(st + L::OFF_F + ft_off, vadd<BF>(w0, w1));
+                sts16(st + L::OFF_F + L::ATOM + ft_off, vsub<BF>(w0, w1));
+#endif
+                fence_async();     // generic-proxy stores -> visible to the tensor core (async proxy)
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&bars->opfull[s]);
+            if (threadIdx.x == 64) TC2_TRACE(ch - c_lo, 3);
+            if (++s == L::S) { s = 0; ph ^= 1; }
+        }
+        // ============================ epilogue ================================
+        mbar_wait(&bars->accfull, 0);
+        tc_after();
+        if (threadIdx.x == 64) TC2_TRACE(511, 2);
+        const int q = warp & 3;                      // TMEM lane quarter of this warp
+        const int half = (warp - 2) >> 2;            // k half
+        const int m = q * 32 + lane;
+        const int fh = cc.fh + m / L::BC;
+        const int c = cc.cb * L::BC + m % L::BC;
+        const bool row_ok = fh < g.R && c < g.C;
+        float* Out = reinterpret_cast<float*>(smem);  // staging [s][k][m] (overlays the idle ring)
+        const uint32_t lane_base = tmem + ((uint32_t)(q * 32) << 16);
+#pragma unroll 1
+        for (int k0 = half * (NK / 2); k0 < (half + 1) * (NK / 2); k0 += 8) {
+            float v[4][8];
+            if (!empty_range) {
+#pragma unroll
+                for (int x = 0; x < 4; ++x) tmem_ld8(lane_base + (uint32_t)(x * NK + k0), v[x]);
+                tmem_wait_ld();
+            } else {
+#pragma unroll
+                for (int x = 0; x < 4; ++x)
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) v[x][i] = 0.f;
+            }
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const float sp = 0.5f * (v[0][i] + v[1][i]);
+                const float y0 = sp + v[2][i], y1 = 0.5f * (v[0][i] - v[1][i]), y2 = sp + v[3][i];
+                if (g.csplit > 1) {
+                    Out[(0 * NK + k0 + i) * MROWS + m] = y0;
+                    Out[(1 * NK + k0 + i) * MROWS + m] = y1;
+                    Out[(2 * NK + k0 + i) * MROWS + m] = y2;
+                } else {
+                    const int k = cc.kb * NK + k0 + i;
+                    if (row_ok && k < g.K) {
+                        float* o = bucket + (((long long)k * g.R + fh) * g.S + fw0) * g.C + c;
+                        o[0] = y0;
+                        o[g.C] = y1;
+                        o[2 * g.C] = y2;
+                    }
+                }
+            }
+        }
+    }
+    tc_before();
+    __syncthreads();
+    if (threadIdx.x == 64) TC2_TRACE(511, 3);
+    if (g.csplit > 1) {
+        // ---- deterministic cluster reduction: rank r sums rows (s, k) of its
+        // slice over ranks 0..cs-1 in order (dsmem_sum4) and writes them.
+        constexpr int ROWS = NSOUT * NK, M4 = MROWS / 4;
+        cluster_sync_all();
+        if (threadIdx.x == 64) TC2_TRACE(511, 4);
+        const int r_lo = ROWS * rank / g.csplit, r_hi = ROWS * (rank + 1) / g.csplit;
+        const uint32_t out_s = sbase;
+        for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHREADS) {
+            const int row = p / M4, m4 = p % M4;
+            const int sidx = row / NK, kl = row % NK;
+            const float4 acc = dsmem_sum4(out_s + (uint32_t)((row * MROWS + m4 * 4) * 4), g.csplit);
+            const int m = m4 * 4;
+            const int fh = cc.fh + m / L::BC, c = cc.cb * L::BC + m % L::BC, k = cc.kb * NK + kl;
+            if (fh < g.R && c < g.C && k < g.K)
+                *reinterpret_cast<float4*>(bucket + (((long long)k * g.R + fh) * g.S + fw0 + sidx) * g.C + c) = acc;
+        }
+        if (threadIdx.x == 64) TC2_TRACE(511, 5);
+        cluster_sync_all();
+    }
+    if (threadIdx.x == 64) TC2_TRACE(511, 6);
+    if (warp == 1) {
+        tc_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem), "r"(L::TMEM_COLS));
+    }
+}
+
+}  // namespace tc2
+}  // namespace winrs

@@ -189,6 +189,8 @@ static void fill_geometry(const Problem& p, const KernelEntry& e, const PairChoi
     g->kblocks = (int)cdiv(p.K, e.bn);
     g->cblocks = (int)cdiv(p.C, e.bm);
     g->ftiles = p.S / e.n0;
+    g->fhs = e.fhs > 0 ? e.fhs : 1;
+    g->fhg = (int)cdiv(p.R, g->fhs);
     g->Z = g->bands * g->seg_cols;
     g->csplit = 1;
     g->chunk = p.dtype == 0 ? 8 : 16;
@@ -200,9 +202,9 @@ static void fill_geometry(const Problem& p, const KernelEntry& e, const PairChoi
 static long long min_tile_chunks(const Geometry& g) {
     long long best = -1;
     for (int band = 0; band < g.bands; ++band)
-        for (int fh = 0; fh < g.R; ++fh) {
+        for (int fh = 0; fh < g.R; fh += g.fhs) {
             int hs, he;
-            band_rows(g, band, fh, &hs, &he);
+            group_rows(g, band, fh, &hs, &he);
             for (int col = 0; col < g.seg_cols; ++col) {
                 int wf, units;
                 seg_units(g, col, &wf, &units);
@@ -235,7 +237,12 @@ struct SharedModel {
     double slots4, slots8;   // resident 4- / 8-CTA clusters on 148 SMs
 };
 
-static TimeModel time_model(int dtype, int bn, int bm) {
+static TimeModel time_model(const KernelEntry& e) {
+    const int dtype = e.dtype, bn = e.bn, bm = e.bm;
+    if (e.fhs > 0) {   // bfc_tc2.cuh: rate over the whole 128-row UMMA tile (fhs filter rows)
+        if (bn >= 128) return {3.0e-6, 10.0e12};
+        return {2.5e-6, 7.0e12};
+    }
     if (dtype != 0) {
         if (bm >= 128) return {11.02e-6, 3.095e12};
         if (bm >= 64) return {6.19e-6, 1.545e12};
@@ -262,9 +269,12 @@ static long long cluster_slots(int cs, int occ, int num_sms, const SharedModel& 
 }
 
 static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
-    const TimeModel m = time_model(e.dtype, e.bn, e.bm);
-    const SharedModel sh = shared_model(e.dtype);
-    const double per_chunk = (double)g.chunk * e.bn * e.bm * 2.0 / m.rate_sm;
+    const TimeModel m = time_model(e);
+    SharedModel sh = shared_model(e.dtype);
+    const int fhs = e.fhs > 0 ? e.fhs : 1;
+    const double per_chunk = (double)g.chunk * e.bn * e.bm * fhs * 2.0 / m.rate_sm;
+    if (e.fhs > 0)   // DSMEM reduction of the n0 x B_N x 128 FP32 output tile at ~20 B/clk/SM
+        sh.cluster_s = 1.0e-6 + (double)g.n0 * e.bn * 128 * 4 / 40e9;
     const double t0 = g.a0 * per_chunk, t1 = (g.a1 ? g.a1 : 1) * per_chunk;
     const long long mult = (long long)g.kblocks * g.cblocks * g.ftiles;
     const int jobs_res = g.a1 ? g.n0 / g.n1 : 0;
@@ -287,9 +297,9 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
     };
     for (int band = 0; band < g.bands; ++band)
         for (int col = 0; col < g.seg_cols; ++col)
-            for (int fh = 0; fh < g.R; ++fh) {
+            for (int fh = 0; fh < g.R; fh += g.fhs) {
                 int hs, he, wf, units;
-                band_rows(g, band, fh, &hs, &he);
+                group_rows(g, band, fh, &hs, &he);
                 seg_units(g, col, &wf, &units);
                 const long long rows = he - hs;
                 const long long cm = (rows * units * g.N + g.chunk - 1) / g.chunk;
@@ -370,7 +380,8 @@ static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairC
         last_bands = g.bands; last_cols = g.seg_cols; last_sh = seg_h; last_sw = seg_w;
         const long long mc = min_tile_chunks(g);
         for (int cs = 1; cs <= 8; cs *= 2) {
-            if (fcs ? cs != fcs : (cs > 1 && (!e.csplit_ok || mc < cs))) continue;
+            if (cs > 1 && !e.csplit_ok) continue;   // never launch a cluster the kernel cannot reduce (even if forced)
+            if (fcs ? cs != fcs : (cs > 1 && mc < cs)) continue;
             g.csplit = cs;
             const double t = model_time(g, e, num_sms);
             if (!have || t < best_t * (1.0 - 1e-9)) {
@@ -384,7 +395,7 @@ static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairC
         int z_used = 1, seg_h = p.Ho, seg_w = pc.k0 * e.r0;
         alg2(p, e.r0, pc.k0, z_lo, &z_used, &seg_h, &seg_w);
         fill_geometry(p, e, pc, seg_h, seg_w, &out->geom);
-        out->geom.csplit = fcs ? fcs : 1;
+        out->geom.csplit = fcs && e.csplit_ok ? fcs : 1;
         best_t = model_time(out->geom, e, num_sms);
     }
     out->entry = &e;
@@ -427,6 +438,10 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
         });
         for (const KernelEntry* e : tiles) {
             if (force_tile && (e->bn != fbn || e->bm != fbm)) continue;
+            if (e->fhs > 0 && p.N % 16 != 0) continue;   // tc2: one 16-image TMA box per stage and atom
+            if (const char* v = getenv("WINRS_TC_GEN")) {   // debug: restrict to one tensor-core generation
+                if (e->dtype != 0 && ((atoi(v) == 2) != (e->fhs > 0))) continue;
+            }
             PlanResult r;
             const double t = plan_with_tile(p, *e, cand, num_sms, &r);
             if (!have || t < best_t * (1.0 - 1e-9)) { best = r; best_t = t; have = true; }

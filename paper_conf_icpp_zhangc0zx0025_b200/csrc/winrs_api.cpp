@@ -270,17 +270,21 @@ winrs_status_t winrs_debug_emulate(winrs_plan_t plan, const double* X, const dou
         const int seg = cc.band * g.seg_cols + cc.col;
         double* bucket = buckets.data() + (size_t)seg * g.dw_elems;
         int hs, he, wf, units;
-        band_rows(g, cc.band, cc.fh, &hs, &he);
+        group_rows(g, cc.band, cc.fh, &hs, &he);   // fh group: the union of its rows' ranges
         seg_units(g, cc.col, &wf, &units);
         const int fw0 = cc.ft * g.n0;
         // cluster ranks each compute a partial tile; the tile is their sum
-        for (int rank = 0; rank < g.csplit; ++rank) {
-            std::fill(part.begin(), part.end(), 0.0);
-            f0(g, X, dY, part.data(), cc, hs, he, wf, units, fw0, false, rank);
-            if (f1 && has_residual(g, cc.col))
-                for (int j = 0; j < g.n0 / g.n1; ++j)
-                    f1(g, X, dY, part.data(), cc, hs, he, g.res_col0, g.k1, fw0 + j * g.n1, true, rank);
-            for (long long i = 0; i < g.dw_elems; ++i) bucket[i] += part[i];
+        for (int f = 0; f < g.fhs && cc.fh + f < g.R; ++f) {
+            CtaCoord cf = cc;
+            cf.fh = cc.fh + f;
+            for (int rank = 0; rank < g.csplit; ++rank) {
+                std::fill(part.begin(), part.end(), 0.0);
+                f0(g, X, dY, part.data(), cf, hs, he, wf, units, fw0, false, rank);
+                if (f1 && has_residual(g, cc.col))
+                    for (int j = 0; j < g.n0 / g.n1; ++j)
+                        f1(g, X, dY, part.data(), cf, hs, he, g.res_col0, g.k1, fw0 + j * g.n1, true, rank);
+                for (long long i = 0; i < g.dw_elems; ++i) bucket[i] += part[i];
+            }
         }
     }
     for (long long i = 0; i < g.dw_elems; ++i) {

@@ -11,8 +11,12 @@
 //     column segment as a second phase that adds into the same bucket, so no
 //     extra workspace and no second launch is needed.  Columns >= Wo inside
 //     the last unit are zero-masked (R6).
-//   * CTA = (segment, fh, fw-tile, c-block, k-block); it computes the
-//     B_N x B_M x n0 tile dW_z[kb*B_N.., fh, ft*n0 .. ft*n0+n0, cb*B_M..].
+//   * CTA = (segment, fh group, fw-tile, c-block, k-block); it computes the
+//     B_N x B_M x n0 tile dW_z[kb*B_N.., fh, ft*n0 .. ft*n0+n0, cb*B_M..] for
+//     each filter row fh of its group.  A group is `fhs` consecutive filter
+//     rows (1 for every kernel except the stacked tcgen05 kernel of
+//     bfc_tc2.cuh, which puts 2 rows' X windows into one 128-row UMMA tile
+//     when C <= 64).
 //   * Height clipping (P@32013-33698, Figure 7): a CTA only visits dY rows h
 //     whose X row h+fh-pad lies inside [0, H).
 //   * Cluster split (B200 addition): the depth of one tile can
@@ -49,6 +53,7 @@ struct Geometry {
     // CTA tiling
     int tile_k, tile_c;         // B_N (k), B_M (c)
     int kblocks, cblocks, ftiles;   // ceil(K/B_N), ceil(C/B_M), S/n0
+    int fhs, fhg;               // filter rows per CTA (fh group size) and groups ceil(R / fhs)
     int Z;                      // buckets
     int csplit;                 // CTAs per tile (thread-block cluster size), >= 1
     int chunk;                  // depth entries per main-loop chunk (8 FP32, 16 FP16)
@@ -65,14 +70,14 @@ WINRS_HD CtaCoord decode_cta(const Geometry& g, long long bid) {
     c.kb = (int)(bid % g.kblocks); bid /= g.kblocks;
     c.cb = (int)(bid % g.cblocks); bid /= g.cblocks;
     c.ft = (int)(bid % g.ftiles);  bid /= g.ftiles;
-    c.fh = (int)(bid % g.R);       bid /= g.R;
+    c.fh = (int)(bid % g.fhg) * g.fhs; bid /= g.fhg;   // first filter row of the group
     c.col = (int)(bid % g.seg_cols);
     c.band = (int)(bid / g.seg_cols);
     return c;
 }
 
 WINRS_HD long long num_tiles(const Geometry& g) {
-    return (long long)g.kblocks * g.cblocks * g.ftiles * g.R * g.seg_cols * g.bands;
+    return (long long)g.kblocks * g.cblocks * g.ftiles * g.fhg * g.seg_cols * g.bands;
 }
 WINRS_HD long long num_ctas(const Geometry& g) { return num_tiles(g) * g.csplit; }
 
@@ -90,6 +95,25 @@ WINRS_HD void band_rows(const Geometry& g, int band, int fh, int* hs, int* he) {
     int b = g.H + g.pad - fh; if (b > h1) b = h1;
     *hs = a;
     *he = b > a ? b : a;
+}
+
+// dY rows a CTA of an fh group walks: the union of its rows' clipped ranges
+// (for a row outside a member's range that member's X row lies in the zero
+// padding, so it contributes nothing; the kernel reads it as TMA zero fill).
+WINRS_HD void group_rows(const Geometry& g, int band, int fh0, int* hs, int* he) {
+    int a = 0, b = 0;
+    bool any = false;
+    for (int f = 0; f < g.fhs && fh0 + f < g.R; ++f) {
+        int x, y;
+        band_rows(g, band, fh0 + f, &x, &y);
+        if (y <= x) continue;
+        if (!any || x < a) a = x;
+        if (!any || y > b) b = y;
+        any = true;
+    }
+    if (!any) band_rows(g, band, fh0, &a, &b);
+    *hs = a;
+    *he = b;
 }
 
 // Omega_a0 units of a column segment: first dY column and unit count.
