@@ -769,9 +769,16 @@ template <int A0, int N0, int R0, int BM, int YB = BN> __host__ __device__ const
 // The YB = 64 variant (K <= 64: 64-row dY raw stages, only the FT units of
 // the first 64-row block, a deeper raw ring) for the alpha = 8 single-kernel
 // pairs; the others run the B_N-row layout.
+// Both ring-parity bounds must hold (raw ring: in-order hand-out; operand
+// ring: TX <= S_OP * units + 1).  Round 1 shipped YB = 64 under a timing
+// argument (S_RAW == 2 S_OP) instead of the operand-ring bound; the variant
+// is now compiled out unless the proven bound holds (with 10 transformer
+// warps and 4 units per chunk it does not, so K <= 64 layers run the B_N
+// layout; the default plans for them use the bfc_tc2.cuh kernel anyway).
 template <int A0, int R0, int A1, int BM> __host__ __device__ constexpr bool yb64_variant() {
     return WINRS_F16_DYN && A0 == 8 && A1 == 0 && BM >= 64 &&
-           tx_warps<BM>() <= (Smem<A0, R0, BM, 64>::S_RAW - 1) * units_per_chunk<BM, false, false, 64>() + 1;
+           tx_warps<BM>() <= (Smem<A0, R0, BM, 64>::S_RAW - 1) * units_per_chunk<BM, false, false, 64>() + 1 &&
+           tx_warps<BM>() <= Smem<A0, R0, BM, 64>::S_OP * units_per_chunk<BM, false, false, 64>() + 1;
 }
 
 // ---- final pass (warps 2..5): staged tile -> bucket (no cluster split) or ->
@@ -957,11 +964,12 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     // must gate it: with S_RAW == 2 * S_OP the TMA of chunk s + 2*S_OP waits
     // for chunk s's own raw release, so the held unit would have to stall a
     // whole TMA round trip between its raw release and its operand arrival
-    // ("operand-ring parity"; the YB = 64 and alpha = 8,
-    // B_M = 64 kernels rely on this gate).
+    // ("operand-ring parity").  No instantiation relies on
+    // that timing gate any more: the bound below is a proof obligation for
+    // every compiled kernel.
     constexpr int NU_ = units_per_chunk<BM, native_path<A0, N0, R0, A1, BM>(), pair_units<A0, R0>(), YB>();
     constexpr bool RR_ = WINRS_F16_RR == 1 || (WINRS_F16_RR == 2 && A0 == 4);
-    static_assert(!WINRS_F16_DYN || TX_WARPS <= SM::S_OP * NU_ + (RR_ ? 0 : 1) || S_RAW == 2 * SM::S_OP,
+    static_assert(!WINRS_F16_DYN || TX_WARPS <= SM::S_OP * NU_ + (RR_ ? 0 : 1),
                   "transformer units could run two operand-ring phases ahead of the MMAs (parity-wait aliasing)");
     constexpr bool kCluster = csplit_fits<N0, BM>();
     constexpr bool NAT = native_path<A0, N0, R0, A1, BM>();

@@ -106,7 +106,7 @@ struct Args {
 
 struct Bars {
     uint64_t full[8];       // TMA data landed
-    uint64_t opfull[8];     // FT operands stored (8 warp arrivals)
+    uint64_t opfull[8];     // FT operands stored (one warp per stage)
     uint64_t empty[8];      // MMAs of the stage done (commit)
     uint64_t accfull;
     uint32_t tmem_base;
@@ -275,7 +275,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     if (threadIdx.x == 0) {
         for (int s = 0; s < L::S; ++s) {
             mbar_init(&bars->full[s], 1);
-            mbar_init(&bars->opfull[s], NTX);
+            mbar_init(&bars->opfull[s], 1);
             mbar_init(&bars->empty[s], 1);
         }
         mbar_init(&bars->accfull, 1);
@@ -386,30 +386,46 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         __syncwarp();
     } else {
         // ================================= FT =================================
-        // item: depth df, k octet fo (t < 2 NK); What[0] = w0 + w1, What[1] = w0 - w1
-        const int t = threadIdx.x - 64;             // 0..255
-        constexpr int KO = NK / 8;
-        const bool has_ft = t < KO * KC;
-        const int df = t / KO, fo = t % KO;
-        const uint32_t ft_off = opoff(fo, df, L::Y_LBO);
-        int s = 0;
+        // What[0] = w0 + w1, What[1] = w0 - w1 for the stage's NK k x 16 depth
+        // entries.  FT warp w owns ring slot w (w < S): it takes the whole
+        // stages ch = c_lo + w, c_lo + w + S, ... (all FT items of a stage: IPT
+        // per lane), so S stages are in flight on the FT side at once: warps
+        // splitting every stage in lockstep put the whole LDS -> STS -> proxy
+        // fence round trip (~400-700 cycles, WINRS_TC2_TRACE) on each stage's
+        // critical path.  One warp per slot keeps the ring safe by construction:
+        // slot w is refilled only after the MMAs of this warp's previous stage
+        // in it, so its parity wait can never see a phase two rounds ahead.
+        constexpr int KO = NK / 8;                  // k octets
+        constexpr int IPT = KO * KC / 32;           // items per lane: 8 (NK 128) / 4 (NK 64)
+        static_assert(L::S <= NTX, "one FT warp per ring slot");
+        const int tw = warp - 2;
         uint32_t ph = 0;
-        for (int ch = c_lo; ch < c_hi; ++ch) {
+        for (int ch = c_lo + tw; tw < L::S && ch < c_hi; ch += L::S) {
+            const int s = tw;
             mbar_wait(&bars->full[s], ph);
-            if (threadIdx.x == 64) TC2_TRACE(ch - c_lo, 2);
-            if (has_ft) {
-                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
-                const uint4 w0 = lds16(st + L::OFF_Y + ft_off), w1 = lds16(st + L::OFF_Y + L::ATOM + ft_off);
-#ifndef WINRS_TC2_NO_STS   // debug ablation: no operand stores
-                sts16(st + L::OFF_F + ft_off, vadd<BF>(w0, w1));
-                sts16(st + L::OFF_F + L::ATOM + ft_off, vsub<BF>(w0, w1));
-#endif
-                fence_async();     // generic-proxy stores -> visible to the tensor core (async proxy)
+            ph ^= 1;
+            if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
+            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            uint4 w0[IPT], w1[IPT];
+            uint32_t off[IPT];
+#pragma unroll
+            for (int i = 0; i < IPT; ++i) {
+                const int t = i * 32 + lane;        // item: depth t / KO, k octet t % KO
+                off[i] = opoff(t % KO, t / KO, L::Y_LBO);
+                w0[i] = lds16(st + L::OFF_Y + off[i]);
+                w1[i] = lds16(st + L::OFF_Y + L::ATOM + off[i]);
             }
+#pragma unroll
+            for (int i = 0; i < IPT; ++i) {
+#ifndef WINRS_TC2_NO_STS   // debug ablation: no operand stores
+                sts16(st + L::OFF_F + off[i], vadd<BF>(w0[i], w1[i]));
+                sts16(st + L::OFF_F + L::ATOM + off[i], vsub<BF>(w0[i], w1[i]));
+#endif
+            }
+            fence_async();     // generic-proxy stores -> visible to the tensor core (async proxy)
             __syncwarp();
             if (lane == 0) mbar_arrive(&bars->opfull[s]);
-            if (threadIdx.x == 64) TC2_TRACE(ch - c_lo, 3);
-            if (++s == L::S) { s = 0; ph ^= 1; }
+            if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 3);
         }
         // ============================ epilogue ================================
         mbar_wait(&bars->accfull, 0);

@@ -239,9 +239,14 @@ struct SharedModel {
 
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
-    if (e.fhs > 0) {   // bfc_tc2.cuh: rate over the whole 128-row UMMA tile (fhs filter rows)
-        if (bn >= 128) return {3.0e-6, 10.0e12};
-        return {2.5e-6, 7.0e12};
+    if (e.fhs > 0) {
+        // bfc_tc2.cuh, rate over the whole 128-row UMMA tile (fhs filter rows).
+        // Measured on B200 (tools/trace_tc2.py, WINRS_TC2_TRACE): a 16-deep stage
+        // takes ~820 cycles at NK = 128 and ~600 at NK = 64 -- the shared-memory
+        // port (~128 B/clk: 8 MMAs' operand reads + TMA fill + FT traffic,
+        // DESIGN.md §6.4); fixed = setup + pipeline fill + epilogue.
+        if (bn >= 128) return {4.5e-6, 5.0e12};
+        return {4.0e-6, 3.4e12};
     }
     if (dtype != 0) {
         if (bm >= 128) return {11.02e-6, 3.095e12};
@@ -264,7 +269,8 @@ static long long cluster_slots(int cs, int occ, int num_sms, const SharedModel& 
     if (cs == 1) s = (long long)occ * num_sms;
     else if (cs == 2) s = (long long)occ * num_sms / 2;
     else if (cs == 4) s = (long long)(occ * sm.slots4 * f);
-    else s = (long long)(occ * sm.slots8 * f);
+    else if (cs == 8) s = (long long)(occ * sm.slots8 * f);
+    else s = (long long)(occ * 0.9 * num_sms / cs);   // 3, 6: clusters within a GPC, some SMs stranded
     return std::max(1LL, s);
 }
 
@@ -273,8 +279,8 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
     SharedModel sh = shared_model(e.dtype);
     const int fhs = e.fhs > 0 ? e.fhs : 1;
     const double per_chunk = (double)g.chunk * e.bn * e.bm * fhs * 2.0 / m.rate_sm;
-    if (e.fhs > 0)   // DSMEM reduction of the n0 x B_N x 128 FP32 output tile at ~20 B/clk/SM
-        sh.cluster_s = 1.0e-6 + (double)g.n0 * e.bn * 128 * 4 / 40e9;
+    if (e.fhs > 0)   // rank skew + DSMEM reduction of the n0 x B_N x 128 FP32 output tile (~20 B/clk/SM)
+        sh.cluster_s = 1.5e-6 + (double)g.n0 * e.bn * 128 * 4 / 30e9;
     const double t0 = g.a0 * per_chunk, t1 = (g.a1 ? g.a1 : 1) * per_chunk;
     const long long mult = (long long)g.kblocks * g.cblocks * g.ftiles;
     const int jobs_res = g.a1 ? g.n0 / g.n1 : 0;
@@ -324,7 +330,7 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
 static int forced_csplit() {
     if (const char* f = getenv("WINRS_FORCE_CSPLIT")) {
         const int v = atoi(f);
-        if (v == 1 || v == 2 || v == 4 || v == 8) return v;
+        if (v >= 1 && v <= 8 && v != 5 && v != 7) return v;
     }
     return 0;
 }
@@ -379,7 +385,7 @@ static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairC
         if (g.bands == last_bands && g.seg_cols == last_cols && seg_h == last_sh && seg_w == last_sw) continue;
         last_bands = g.bands; last_cols = g.seg_cols; last_sh = seg_h; last_sw = seg_w;
         const long long mc = min_tile_chunks(g);
-        for (int cs = 1; cs <= 8; cs *= 2) {
+        for (int cs : {1, 2, 3, 4, 6, 8}) {
             if (cs > 1 && !e.csplit_ok) continue;   // never launch a cluster the kernel cannot reduce (even if forced)
             if (fcs ? cs != fcs : (cs > 1 && mc < cs)) continue;
             g.csplit = cs;

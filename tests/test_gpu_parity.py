@@ -14,6 +14,7 @@ import torch
 import paper_conf_icpp_zhangc0zx0025_b200 as W
 from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
 from oracle import oracle as O
+from conftest import record_err
 
 pytestmark = pytest.mark.gpu
 
@@ -42,6 +43,7 @@ def _full_check(layer, dist="u01", env=None, monkeypatch=None, tol=None):
     p, got = _run(layer, X, dY, env, monkeypatch)
     ref = O.bfc_c(X, dY, layer.R, layer.S, layer.pad)
     err = O.rel_max_err(got, ref)
+    record_err(f"{layer.name}[{layer.dtype},{dist}]" + (f" {env}" if env else ""), err, p.kernel_name)
     assert err <= (tol or TOL[layer.dtype]), (layer, p, err)
     return p, err
 
@@ -115,6 +117,7 @@ def test_full_size_sampled(layer):
     idx = wl.sample_indices(layer, 384)
     ref = O.bfc_c_sampled(X, dY, layer.R, layer.S, layer.pad, idx)
     err = O.rel_max_err(got.ravel()[idx], ref)
+    record_err(f"{layer.name} full size, {len(idx)} sampled outputs", err, p.kernel_name)
     assert err <= TOL[layer.dtype], (layer.name, p, err)
     assert np.isfinite(got).all()
 
@@ -205,6 +208,7 @@ def test_full_size_sampled_f16(layer):
     idx = wl.sample_indices(layer, 256)
     ref = O.bfc_c_sampled(X, dY, layer.R, layer.S, layer.pad, idx)
     err = O.rel_max_err(got.ravel()[idx], ref)
+    record_err(f"{layer.name} full size, {len(idx)} sampled outputs", err, p.kernel_name)
     assert err <= TOL[layer.dtype], (layer.name, p, err)
     assert np.isfinite(got).all()
 
@@ -227,7 +231,9 @@ def test_k_sharded_slices_concatenate_to_oracle(layer, world):
     assert [k0 for k0, _ in parts] == sorted(k0 for k0, _ in parts)
     got = torch.cat([d for _, d in parts], dim=0).cpu().numpy()
     ref = O.bfc_c(X, dY, layer.R, layer.S, layer.pad)
-    assert O.rel_max_err(got, ref) <= TOL[layer.dtype]
+    err = O.rel_max_err(got, ref)
+    record_err(f"{layer.name} K-sharded x{world}", err)
+    assert err <= TOL[layer.dtype]
 
 
 # ============================================================== FP16 widths 2..9
@@ -260,7 +266,9 @@ def test_bf16_full_size_sampled():
     p, got = _run(layer, X, dY)
     idx = wl.sample_indices(layer, 256)
     ref = O.bfc_c_sampled(X, dY, layer.R, layer.S, layer.pad, idx)
-    assert O.rel_max_err(got.ravel()[idx], ref) <= TOL["bf16"]
+    err = O.rel_max_err(got.ravel()[idx], ref)
+    record_err(f"{layer.name} full size, {len(idx)} sampled outputs", err, p.kernel_name)
+    assert err <= TOL["bf16"]
 
 
 @pytest.mark.gpu

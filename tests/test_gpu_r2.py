@@ -1,0 +1,224 @@
+"""GPU parity, round 2: the second-generation tensor-core kernel
+(bfc_tc2.cuh), pad = 0 layers, every reachable FP32 kernel for F_W = 6 / 8,
+exactness on structured inputs, and bitwise reproducibility under repeated
+cold-L2 calls.  Every check compares the CUDA path (C ABI via the ctypes
+binding) with the FP64 oracle on the same inputs, element by element.
+
+Gate (BASELINE.json north_star): max|err| <= 1e-4 max|ref| (FP32 inputs),
+<= 2e-2 max|ref| (FP16 / BF16 inputs, FP32 accumulation).
+"""
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_icpp_zhangc0zx0025_b200 as W
+from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+from oracle import oracle as O
+from conftest import record_err
+
+pytestmark = pytest.mark.gpu
+
+TOL = {"f32": 1e-4, "f16": 2e-2, "bf16": 2e-2}
+ENV_KEYS = ("WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_TC_GEN")
+
+
+def _dev(a, dtype):
+    t = torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    return t.to(torch.bfloat16) if dtype == "bf16" else t
+
+
+def _plan(layer, env, monkeypatch):
+    for k in ENV_KEYS:
+        monkeypatch.delenv(k, raising=False)
+    for k, v in (env or {}).items():
+        monkeypatch.setenv(k, v)
+    return W.plan(layer.N, layer.C, layer.H, layer.W, layer.K, layer.R, layer.S, layer.pad, layer.dtype)
+
+
+def _check(layer, monkeypatch, env=None, dist="u01", X=None, dY=None, exact=False, expect_kernel=None):
+    if X is None:
+        X, dY = wl.make_inputs(layer, dist)
+    p = _plan(layer, env, monkeypatch)
+    if expect_kernel:
+        assert expect_kernel in p.kernel_name, (p.kernel_name, expect_kernel)
+    dW = W.bfc(p, _dev(X, layer.dtype), _dev(dY, layer.dtype))
+    torch.cuda.synchronize()
+    got = dW.cpu().numpy().astype(np.float64)
+    ref = O.bfc_c(X, dY, layer.R, layer.S, layer.pad)
+    err = O.rel_max_err(got, ref)
+    record_err(f"{layer.name}[{layer.dtype}] {env or ''}", err, f"{p.kernel_name} Z={p.info['Z']} cs={p.info['csplit']}")
+    if exact:
+        assert np.array_equal(got, ref), (layer.name, p.kernel_name, err, np.max(np.abs(got - ref)))
+    assert err <= TOL[layer.dtype], (layer.name, p.kernel_name, err)
+    assert np.isfinite(got).all()
+    return p, err
+
+
+# ====================================================== bfc_tc2.cuh (second-generation tensor-core kernel)
+BASE = wl.LAYERS["r50_c64_56_f16"]
+TC2 = [
+    ("l1", dict(N=16), {}),
+    ("l1_f2", dict(N=16), {"WINRS_FORCE_TILE": "64x64"}),
+    ("l1_f1_cs2", dict(N=16), {"WINRS_FORCE_TILE": "64x128", "WINRS_FORCE_CSPLIT": "2"}),
+    ("l2_nk128_cs1", dict(N=16, C=128, K=128, H=28, W=28), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "1"}),
+    ("l2_nk128_cs3", dict(N=16, C=128, K=128, H=28, W=28), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "3"}),
+    ("l2_nk128_cs4", dict(N=16, C=128, K=128, H=28, W=28), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "4"}),
+    ("l3", dict(N=16, C=256, K=256, H=14, W=14), {}),
+    ("l3_cs6", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "6"}),
+    ("l4_odd_wo", dict(N=16, C=512, K=512, H=7, W=7), {}),
+    ("ragged_ck", dict(N=16, C=72, K=200, H=20, W=17), {}),
+    ("ragged_f2", dict(N=16, C=40, K=136, H=20, W=17), {"WINRS_FORCE_TILE": "128x64"}),
+    ("pad0", dict(N=16, C=64, K=64, H=20, W=20, pad=0), {}),
+    ("pad0_f1", dict(N=16, C=128, K=64, H=19, W=21, pad=0), {"WINRS_FORCE_TILE": "64x128"}),
+    ("s6_ftiles2", dict(N=16, C=64, K=64, H=16, W=16, R=3, S=6, pad=2), {"WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
+    ("r5_f2", dict(N=16, C=64, K=128, H=16, W=16, R=5, S=3, pad=2), {"WINRS_FORCE_TILE": "128x64"}),
+    ("r1", dict(N=16, C=64, K=64, H=12, W=12, R=1, S=3, pad=0), {}),
+    ("n32_z5", dict(N=32, C=64, K=64, H=30, W=30), {"WINRS_FORCE_Z": "5"}),
+    ("n48_cs8", dict(N=48, C=128, K=64, H=12, W=12), {"WINRS_FORCE_CSPLIT": "8"}),
+]
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+@pytest.mark.parametrize("name,ov,env", TC2, ids=[c[0] for c in TC2])
+def test_tc2(name, ov, env, dtype, monkeypatch):
+    layer = BASE.with_(name="tc2_" + name, dtype=dtype, **ov)
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2"), expect_kernel="_v2_")
+
+
+@pytest.mark.parametrize("name,ov,env", TC2[:8], ids=[c[0] for c in TC2[:8]])
+def test_tc2_signed(name, ov, env, monkeypatch):
+    layer = BASE.with_(name="tc2s_" + name, **ov)
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2"), dist="signed", expect_kernel="_v2_")
+
+
+def test_tc2_default_plans_use_tc2(monkeypatch):
+    """The planner's picks for the ResNet-50 / VGG-16 FP16 layers are the
+    second-generation kernel (the bench's headline path)."""
+    for l in wl.RESNET50_F16 + wl.VGG16_F16:
+        p = _plan(l, {}, monkeypatch)
+        assert "_v2_" in p.kernel_name, (l.name, p.kernel_name)
+
+
+# ====================================================== pad = 0 (pad=0 variants of the wide config)
+PAD0 = [(l.with_(N=2, C=40, K=36, H=17, W=19, pad=0, name=l.name + "_pad0")) for l in wl.WIDE_F32] + [
+    wl.LAYERS["r50_c64_56_f32"].with_(N=2, H=20, W=23, pad=0, name="r50_l1_pad0"),
+    wl.LAYERS["r50_c256_14_f32"].with_(N=2, C=72, K=64, pad=0, name="r50_l3_pad0"),
+]
+
+
+@pytest.mark.parametrize("layer", PAD0, ids=lambda l: l.name)
+@pytest.mark.parametrize("dtype", ["f32", "f16"])
+def test_pad0(layer, dtype, monkeypatch):
+    _check(layer.with_(dtype=dtype), monkeypatch)
+
+
+def test_pad0_f16_n16_tc2(monkeypatch):
+    layer = wl.LAYERS["r50_c64_56_f16"].with_(N=16, H=21, W=22, pad=0, name="r50_l1_pad0_n16")
+    _check(layer, monkeypatch)
+
+
+# ====================================================== FP32 kernels for F_W = 6, 8
+FW68 = [
+    (6, "8,6,3,0,0,0"),       # Omega_8(6,3)
+    (6, "16,6,11,0,0,0"),     # Omega_16(6,11)
+    (8, "16,8,9,0,0,0"),      # Omega_16(8,9)
+    (8, "8,4,5,4,2,3"),       # Omega_8(4,5) + Omega_4(2,3)
+    (8, "8,4,5,0,0,0"),       # Omega_8(4,5)
+    (6, "8,6,3,4,3,2"),       # Omega_8(6,3) + Omega_4(3,2)
+    (8, "16,8,9,8,4,5"),      # Omega_16(8,9) + Omega_8(4,5)
+    (6, None),                # the planner's own choice
+    (8, None),
+]
+
+
+@pytest.mark.parametrize("S,pair", FW68, ids=lambda v: str(v))
+def test_fp32_fw6_fw8(S, pair, monkeypatch):
+    layer = wl.LAYERS["wide_r5_f32"].with_(N=2, C=40, K=36, H=21, W=26, R=S, S=S, pad=S // 2, name=f"f32_w{S}")
+    env = {"WINRS_FORCE_PAIR": pair} if pair else {}
+    p, _ = _check(layer, monkeypatch, env)
+    if pair:
+        a = [int(x) for x in pair.split(",")]
+        assert (p.info["alpha0"], p.info["n0"], p.info["r0"]) == tuple(a[:3])
+
+
+# ====================================================== exactness on structured inputs
+def _int_inputs(layer, lo=0, hi=8, seed=11):
+    g = np.random.Generator(np.random.PCG64(seed))
+    X = g.integers(lo, hi, size=(layer.N, layer.H, layer.W, layer.C)).astype(np.float32)
+    dY = np.zeros((layer.N, layer.Ho, layer.Wo, layer.K), dtype=np.float32)
+    return X, dY
+
+
+EXACT = [
+    ("f32", {"WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
+    ("f16", {"WINRS_TC_GEN": "2"}),
+    ("bf16", {"WINRS_TC_GEN": "2"}),
+    ("f16", {"WINRS_TC_GEN": "1", "WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
+]
+
+
+@pytest.mark.parametrize("dtype,env", EXACT, ids=lambda v: str(v))
+def test_all_ones_exact(dtype, env, monkeypatch):
+    """X = dY = 1: dW[k,r,s,c] = N cnt_H(r) cnt_W(s), integers < 2^24.  With
+    the Omega_4(3,2) transforms (coefficients +-1, 1/2, 2) every intermediate
+    is exact, so the GPU result equals the closed form bit for bit."""
+    layer = wl.LAYERS["r50_c64_56_f16"].with_(N=16, C=64, K=64, H=18, W=17, dtype=dtype, name="ones")
+    X = np.ones((layer.N, layer.H, layer.W, layer.C), np.float32)
+    dY = np.ones((layer.N, layer.Ho, layer.Wo, layer.K), np.float32)
+    _check(layer, monkeypatch, env, X=X.astype(wl.np_dtype(dtype)), dY=dY.astype(wl.np_dtype(dtype)), exact=True)
+
+
+@pytest.mark.parametrize("dtype,env", EXACT, ids=lambda v: str(v))
+def test_impulse_exact(dtype, env, monkeypatch):
+    """dY = a few unit impulses, X = small integers: dW[k0] = the padded X
+    window at each impulse (layout, correlation, padding), exactly."""
+    layer = wl.LAYERS["r50_c64_56_f16"].with_(N=16, C=64, K=64, H=15, W=16, dtype=dtype, name="impulse")
+    X, dY = _int_inputs(layer)
+    for (n, h, w, k) in [(0, 0, 0, 0), (3, layer.Ho - 1, layer.Wo - 1, 63), (7, 5, 6, 17), (15, 0, layer.Wo - 1, 40)]:
+        dY[n, h, w, k] = 1.0
+    _check(layer, monkeypatch, env, X=X.astype(wl.np_dtype(dtype)), dY=dY.astype(wl.np_dtype(dtype)), exact=True)
+
+
+def test_impulse_fp32_alpha8_tolerance(monkeypatch):
+    """Omega_8 transforms have non-dyadic coefficients: impulse results are
+    within the FP32 gate rather than bit-exact."""
+    layer = wl.LAYERS["r50_c64_56_f32"].with_(N=2, H=15, W=16, name="impulse_a8")
+    X, dY = _int_inputs(layer)
+    dY[1, 3, 4, 5] = 1.0
+    _check(layer, monkeypatch, {"WINRS_FORCE_PAIR": "8,3,6,4,3,2"}, X=X, dY=dY)
+
+
+# ====================================================== reproducibility under repeated cold-L2 calls
+@pytest.mark.parametrize("layer_name,env", [
+    ("r50_c64_56_f16", {}),                                   # tc2, Z > 1, cluster split
+    ("r50_c256_14_f16", {}),                                  # tc2, NK = 128, cs = 8
+    ("r50_c64_56_f16", {"WINRS_TC_GEN": "1"}),                # round-1 kernel default plan
+    ("r50_c128_28_f16", {"WINRS_TC_GEN": "1"}),
+])
+def test_repeated_calls_bitwise(layer_name, env, monkeypatch):
+    """400 cold-L2 calls of the default plan: every dW equals the first one bit
+    for bit (determinism for a fixed plan, R16; a ring-protocol race
+    would show up as a changed or non-finite dW, or as a hang)."""
+    layer = wl.LAYERS[layer_name]
+    X, dY = wl.make_inputs(layer)
+    p = _plan(layer, env, monkeypatch)
+    Xg, Gg = _dev(X, layer.dtype), _dev(dY, layer.dtype)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    ws = torch.empty(max(16, p.workspace_bytes), dtype=torch.uint8, device="cuda")
+    first = W.bfc(p, Xg, Gg, workspace=ws).clone()
+    out = torch.empty_like(first)
+    bad = 0
+    for i in range(400):
+        flush.fill_(i & 255)
+        W.bfc(p, Xg, Gg, out, ws)
+        if i % 50 == 49 or i == 399:
+            torch.cuda.synchronize()
+        bad += int(not torch.equal(out, first))
+    assert bad == 0, (p.kernel_name, bad)
+    idx = wl.sample_indices(layer, 128)
+    ref = O.bfc_c_sampled(X, dY, layer.R, layer.S, layer.pad, idx)
+    err = O.rel_max_err(first.cpu().numpy().astype(np.float64).ravel()[idx], ref)
+    record_err(f"{layer_name} 400 cold-L2 calls bitwise equal {env}", err, p.kernel_name)
+    assert err <= TOL[layer.dtype]

@@ -48,7 +48,7 @@ def main():
         cfgs = [("auto", None, None, None), ("gen1", None, None, None), ("gen2", None, None, None)]
         if not quick:
             zs = [1, 2, 3, 4, 6, 8, 12, 16, 24, 32]
-            cfgs += [("f", t, cs, z) for t in TILES for cs in (1, 2, 4, 8) for z in zs]
+            cfgs += [("f", t, cs, z) for t in TILES for cs in (1, 2, 3, 4, 6, 8) for z in zs]
         seen = set()
         for kind, t, cs, z in cfgs:
             for k in ("WINRS_FORCE_Z", "WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_TC_GEN"):
