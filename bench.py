@@ -3,20 +3,32 @@
 effective TFLOPS = direct-conv FLOPs 2*N*C*K*Ho*Wo*R*S / device time, plus
 workspace bytes).
 
-A "step" is one pass of the whole hot path (plan is prebuilt; fused kernels +
-bucket reduction) over every layer of the workload, inputs resident in HBM.
-Default workload: configs[1] of BASELINE.json — the four ResNet-50 3x3 layers
-at N=64 (C=K=64/128/256/512, H=W=56/28/14/7, pad 1).  L2 is flushed (a
-256 MiB write) before every layer call and each call is timed with CUDA events
-on the launch stream (the flush is outside the timed events).
+A "step" is one pass of the whole hot path (plan prebuilt; fused kernel +
+bucket reduction [+ one NCCL all_reduce of dW when N > 1]) over every layer of
+the workload, inputs resident in HBM.  L2 is flushed (a 256 MiB write) before
+every layer call and each call is timed with CUDA events on the launch stream
+(the flush is outside the timed events).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--dtype f16|f32] [--impl winrs|reference]
+Default workload: the largest single-GPU BASELINE config, VGG-16's 3x3 layers
+2-13 at N=128 in FP16 (configs[2]; BASELINE's metric names no config).  The
+ResNet-50 layers (configs[1], FP16 and FP32) and the wide-dW config
+(configs[3], FP32) are measured alongside in the same run and reported under
+config.alongside (--no-alongside skips them).
 
-N > 1 (torchrun): each rank runs the same per-rank workload on its own batch
-shard (weak scaling: global batch = N * 64) followed by one NCCL all_reduce of
-each layer's dW — the batch-sharded data-parallel BFC; time = max over ranks.
---impl reference runs the FP64 CPU oracle (the only reference this paper-only
-tier has) on a bounded sample of the same workload, rank 0 only.
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload vgg|r50|wide|r50l3]
+                    [--dtype f16|bf16|f32] [--impl winrs|reference] [--parallel dp|kshard]
+
+--gpus N > 1 without a torchrun environment re-launches itself under
+torch.distributed.run (one rank per GPU, NCCL, 127.0.0.1).  dp (default):
+every rank runs the per-rank workload on its own batch shard and all-reduces
+each layer's dW (weak scaling: global batch = N x per-rank batch), except
+--workload r50l3, BASELINE configs[4]: the FIXED global batch N=512 of
+ResNet-50 layer 3 split over the ranks (strong scaling), reported with and
+without the all_reduce.  kshard: every rank holds the full batch and computes
+its slice of the output channels (strong, no communication).  Time = max over
+ranks.  --impl reference runs the FP64 CPU oracle (the only reference this
+paper-only tier has) on a bounded sample of the same workload, rank 0 only.
+--dry-run exercises only the launch / rank plumbing (gloo, no GPU work).
 """
 from __future__ import annotations
 
@@ -27,6 +39,8 @@ import statistics
 import sys
 import threading
 import time
+
+import numpy as np
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
@@ -152,68 +166,123 @@ class ClockSampler:
                 "source": "nvml"}
 
 
-def run_winrs(args):
+# L2 -> SM fill rate used for the t_L2 diagnostic: TMA boxes of the tc2 kernel,
+# 148 CTAs, tools/microbench/tma_rate3.cu mode 0 on B200 (81 B/clk/SM x 148 x 1.965 GHz).
+L2_SM_GBS = 23650.0
+
+
+def _rows_valid(l, fh):
+    return sum(1 for h in range(l.Ho) if 0 <= h + fh - l.pad < l.H)
+
+
+def _rows_union(l, fhs):
+    return sum(1 for h in range(l.Ho) if any(0 <= h + f - l.pad < l.H for f in fhs))
+
+
+def layer_roofline(l, p, ms, peaks):
+    """The BASELINE roofline of one layer call:
+    T_roof = max(algorithmic bytes / HBM, Winograd EWM FLOPs / pipe peak), and
+    the diagnostic bounds t_ALU (transform lane-ops / FP32 lanes) and t_L2
+    (L2 -> SM bytes / measured fill rate), all against the measured time."""
+    info = p.info
+    esz = 4 if l.dtype == "f32" else 2
+    Z = info["Z"]
+    dw = 4 * l.K * l.R * l.S * l.C
+    alg_bytes = esz * (l.N * l.H * l.W * l.C + l.N * l.Ho * l.Wo * l.K) + dw * (1 if Z == 1 else 2 * Z + 1)
+    ewm = info["ewm_flops"]
+    clk_ghz = float(peaks.get("sm_max_mhz", 1965.0)) / 1e3
+    fp32_peak = 148 * 128 * 2 * clk_ghz * 1e9            # FLOP/s (lanes x FMA)
+    lanes = 148 * 128 * clk_ghz * 1e9                    # lane-ops/s
+    t_hbm = alg_bytes / (peaks["hbm_gbs"] * 1e9)
+    if l.dtype == "f32":
+        t_pipe, bound, pk = ewm / fp32_peak, "alu", fp32_peak / 1e12
+    else:
+        t_pipe, bound, pk = ewm / (peaks["bf16_tflops"] * 1e12), "tensor", peaks["bf16_tflops"]
+    if t_hbm > t_pipe:
+        bound = "hbm"
+    t_roof = max(t_hbm, t_pipe)
+    # depth entries x tiles the kernel walks, for the diagnostics
+    name = p.kernel_name
+    a, n0, r0 = info["alpha0"], info["n0"], info["r0"]
+    units = info["k0"] + info["k1"]
+    bn, bm = info["tile_k0"], info["tile_c0"]
+    kb, cb = -(-l.K // bn), -(-l.C // bm)
+    ft = l.S // n0
+    if "_v2_" in name:
+        fhs = int(name.split("x")[-1].rstrip("fh"))
+        rows = sum(_rows_union(l, range(g, min(l.R, g + fhs))) for g in range(0, l.R, fhs))
+        depth = rows * units * l.N * kb * cb * ft
+        l2_bytes = depth / 16 * (16384 + bn * 64)         # per 16-deep stage: X 16 KB + dY NK*64 B
+        alu_ops = depth * bn                              # FT: W0, W1 = w0 +- w1, packed half2
+    else:
+        rows = sum(_rows_valid(l, fh) for fh in range(l.R))
+        depth = rows * units * l.N * kb * cb * ft
+        ft_ops = {2: 1, 4: 2, 8: 22, 16: 90}.get(a, a * r0)    # FT adds/FMAs per channel (generated code)
+        it_ops = {2: 2, 4: 4, 8: 28, 16: 110}.get(a, a * a)
+        cvt = 0 if l.dtype == "f32" else (r0 + a / 2 + a / 2 + a / 2)   # unpack + pack (FP16 path)
+        alu_ops = depth * (bn * (ft_ops + cvt) + bm * (it_ops + cvt))
+        l2_bytes = depth * (r0 * bn + a * bm) * esz
+    t_alu = alu_ops / lanes
+    t_l2 = l2_bytes / (L2_SM_GBS * 1e9)
+    sec = ms * 1e-3
+    return {"layer": l.name, "kernel": name, "bound": bound, "frac": t_roof / sec,
+            "t_roof_us": t_roof * 1e6, "t_hbm_us": t_hbm * 1e6, "t_pipe_us": t_pipe * 1e6,
+            "t_alu_us": t_alu * 1e6, "t_l2_us": t_l2 * 1e6, "measured_us": ms * 1e3,
+            "alg_bytes": alg_bytes, "ewm_flops": ewm, "pipe_peak_tflops": pk}
+
+
+def measure(layers, args, ctx, primary=True):
+    """Time one workload: per-layer cold-L2 CUDA-event times over the steps,
+    warm-L2 times, CUDA-graph replays, (N > 1) compute-only times, the dominant
+    kernel alone, and the end-to-end host-buffer path.  Returns a dict."""
     import torch
     import torch.distributed as dist
     import paper_conf_icpp_zhangc0zx0025_b200 as W
     from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
-
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    ndev = torch.cuda.device_count()
-    torch.cuda.set_device(local % ndev)
-    dev = torch.device("cuda", local % ndev)
-    if world > 1:
-        # NCCL over NVLink/NVSwitch; WINRS_DIST_BACKEND=gloo only to exercise the
-        # multi-rank path on a single-GPU box (ranks sharing one device).
-        backend = os.environ.get("WINRS_DIST_BACKEND", "nccl")
-        if backend == "nccl":
-            dist.init_process_group("nccl", device_id=dev)
-        else:
-            dist.init_process_group(backend)
-    layers = _workload(args.workload, args.dtype)
-    tdt = torch.float32 if args.dtype == "f32" else torch.float16
-
-    # Inputs resident in HBM, plans prebuilt.  dp: each rank has its own
-    # seeded batch shard (weak scaling); kshard: every rank holds the full
-    # batch and computes its slice of the output channels (strong scaling, no
-    # communication: BASELINE's K-sharding alternative).
-    kshard = args.parallel == "kshard" and world > 1
+    world, rank, dev, kshard, strong = ctx["world"], ctx["rank"], ctx["dev"], ctx["kshard"], ctx["strong"]
+    steps = args.steps if primary else max(3, min(args.steps, 5))
+    warmup = args.warmup if primary else 3
     items = []
     for l in layers:
-        X, dY = wl.make_inputs(l, seed_offset=0 if kshard else 1000 * rank)
         align = 4 if l.dtype == "f32" else 8
+        k0, k1, n0, n1 = 0, l.K, 0, l.N
+        if strong:     # fixed global batch: this rank's contiguous image slice (NHWC: contiguous)
+            n0, n1 = W.shard_range(l.N, world, rank)
+            X, dY = wl.make_inputs(l)
+            X, dY = np.ascontiguousarray(X[n0:n1]), np.ascontiguousarray(dY[n0:n1])
+        else:
+            X, dY = wl.make_inputs(l, seed_offset=0 if kshard else 1000 * rank)
         if kshard:
             a, b = W.shard_range(l.K // align, world, rank)
             k0, k1 = a * align, b * align
-        else:
-            k0, k1 = 0, l.K
-        p = W.plan(l.N, l.C, l.H, l.W, k1 - k0, l.R, l.S, l.pad, l.dtype)
+        ll = l.with_(N=n1 - n0)
+        p = W.plan(ll.N, l.C, l.H, l.W, k1 - k0, l.R, l.S, l.pad, l.dtype)
         Xt, Gt = torch.from_numpy(X), torch.from_numpy(dY)
         if l.dtype == "bf16":   # workloads carries bf16 values in float32
             Xt, Gt = Xt.to(torch.bfloat16), Gt.to(torch.bfloat16)
-        Xg = Xt.to(dev)
-        Gg = Gt.to(dev)
         dW = torch.empty((k1 - k0, l.R, l.S, l.C), dtype=torch.float32, device=dev)
         ws = torch.empty(max(p.workspace_bytes, 16), dtype=torch.uint8, device=dev)
-        items.append(dict(layer=l, plan=p, X=Xg, dY=Gg, dW=dW, ws=ws, Xh=Xt.pin_memory(),
-                          Gh=Gt.pin_memory(), dWh=torch.empty(dW.shape).pin_memory(),
-                          k0=k0, k1=k1, flops=l.direct_flops * (k1 - k0) / l.K))
+        items.append(dict(layer=l, local=ll, plan=p, X=Xt.to(dev), dY=Gt.to(dev), dW=dW, ws=ws,
+                          Xh=Xt.pin_memory(), Gh=Gt.pin_memory(), dWh=torch.empty(dW.shape).pin_memory(),
+                          k0=k0, k1=k1))
+    stream = torch.cuda.current_stream(dev)
 
-    def run_bfc(it, stream):
+    def bfc_only(it, s):
         if kshard:   # channel slice of dY read in place (ldy = K), no communication
             from paper_conf_icpp_zhangc0zx0025_b200 import _lib
             _lib.check(_lib.lib().winrs_bfc_strided(it["plan"].handle, it["X"].data_ptr(),
                                                     it["dY"].data_ptr() + it["k0"] * it["dY"].element_size(),
                                                     it["layer"].K, it["dW"].data_ptr(), it["ws"].data_ptr(),
-                                                    stream.cuda_stream), "winrs_bfc_strided")
+                                                    s.cuda_stream), "winrs_bfc_strided")
         else:
-            W.bfc(it["plan"], it["X"], it["dY"], it["dW"], it["ws"], stream)
-            if world > 1:
-                dist.all_reduce(it["dW"])
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-    stream = torch.cuda.current_stream(dev)
+            W.bfc(it["plan"], it["X"], it["dY"], it["dW"], it["ws"], s)
+
+    def run_bfc(it, s):
+        bfc_only(it, s)
+        if world > 1 and not kshard:
+            dist.all_reduce(it["dW"])      # the data-parallel step's one exchange (NCCL over NVLink)
+
+    flush = ctx["flush"]
 
     def one_step(timed_events=None):
         for j, it in enumerate(items):
@@ -224,41 +293,32 @@ def run_winrs(args):
             if timed_events is not None:
                 timed_events[j][1].record(stream)
 
-    for _ in range(args.warmup):
+    for _ in range(warmup):
         one_step()
     torch.cuda.synchronize()
-
-    clocks = ClockSampler(local)
-    if rank == 0:
+    clocks = ClockSampler(ctx["local"]) if primary and rank == 0 else None
+    if clocks:
         clocks.start()
     ev = [[[torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)] for _ in items]
-          for _ in range(args.steps)]
+          for _ in range(steps)]
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    for s in range(args.steps):
+    for s in range(steps):
         one_step(ev[s])
-        if rank == 0:
+        if clocks:
             clocks.sample()                                        # GPU busy with the queued layers
-    if rank == 0:
+    if clocks:
         while not ev[-1][-1][1].query():                           # GPU still draining the steps
             clocks.sample()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    clk = clocks.stop() if rank == 0 else None
-
-    per_layer_ms = [sum(ev[s][j][0].elapsed_time(ev[s][j][1]) for s in range(args.steps)) / args.steps
+    clk = clocks.stop() if clocks else None
+    per_layer_ms = [sum(ev[s][j][0].elapsed_time(ev[s][j][1]) for s in range(steps)) / steps
                     for j in range(len(items))]
-    step_ms = sum(per_layer_ms)
-    if world > 1:
-        t = torch.tensor([step_ms], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        step_ms = float(t.item())
 
-    # Secondary numbers: warm-L2 per-layer time (no flush between
-    # calls) and, for N > 1, the compute-only time without the all_reduce.
-    def time_layers(flush_l2, with_allreduce, reps=5):
+    def time_layers(flush_l2, fn, reps=5):
         out = []
         for it2 in items:
             ts = []
@@ -269,35 +329,50 @@ def run_winrs(args):
                     torch.cuda._sleep(100000)
                 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 a.record(stream)
-                if with_allreduce:
-                    run_bfc(it2, stream)
-                elif kshard:
-                    run_bfc(it2, stream)
-                else:
-                    W.bfc(it2["plan"], it2["X"], it2["dY"], it2["dW"], it2["ws"], stream)
+                fn(it2, stream)
                 b.record(stream)
                 torch.cuda.synchronize()
                 ts.append(a.elapsed_time(b))
             out.append(statistics.median(ts))
         return out
-    warm_ms = time_layers(False, world > 1)
-    compute_only_ms = time_layers(True, False) if world > 1 else None
+    warm_ms = time_layers(False, run_bfc)
+    compute_only_ms = time_layers(True, bfc_only) if world > 1 and not kshard else None
 
-    # Dominant kernel's live duration: time the fused kernel alone (no
-    # all_reduce) for the layer with the largest share, CUDA events on the stream.
+    # CUDA-graph replays: each layer's winrs_bfc launches captured
+    # once, replayed cold-L2; device time per replay from CUDA events.
+    graph = None
+    if primary and not args.no_graphs:
+        graph = []
+        reps = args.graph_reps or (1000 if sum(per_layer_ms) < 1.0 else 100)
+        cap = torch.cuda.Stream(dev)
+        for it2 in items:
+            g = torch.cuda.CUDAGraph()
+            cap.wait_stream(stream)
+            with torch.cuda.graph(g, stream=cap):
+                bfc_only(it2, cap)
+            stream.wait_stream(cap)
+            for _ in range(20):
+                g.replay()
+            torch.cuda.synchronize()
+            evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+            for a, b in evs:
+                flush.fill_(5)
+                a.record(stream)
+                g.replay()
+                b.record(stream)
+            torch.cuda.synchronize()
+            ts = [a.elapsed_time(b) for a, b in evs]
+            graph.append({"mean_ms": statistics.fmean(ts), "median_ms": statistics.median(ts), "replays": reps})
+            del g
+
+    # The dominant layer's kernel(s) alone (no all_reduce), CUDA events on the stream.
     dom = max(range(len(items)), key=lambda j: per_layer_ms[j])
-    it = items[dom]
-    p = it["plan"]
-    info = p.info
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     kt = []
-    for _ in range(max(3, args.steps)):
+    for _ in range(max(3, steps)):
         flush.fill_(1)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        if kshard:
-            run_bfc(it, stream)
-        else:
-            W.bfc(p, it["X"], it["dY"], it["dW"], it["ws"], stream)
+        bfc_only(items[dom], stream)
         e1.record(stream)
         torch.cuda.synchronize()
         kt.append(e0.elapsed_time(e1))
@@ -305,7 +380,7 @@ def run_winrs(args):
 
     # End to end through the C ABI with host buffers (pinned), copies inside.
     e2e_ms = []
-    for _ in range(max(2, min(args.steps, 5))):
+    for _ in range(max(2, min(steps, 5))):
         tot = 0.0
         for it2 in items:
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -315,10 +390,8 @@ def run_winrs(args):
             if kshard or world > 1:   # H2D, the BFC (+ all_reduce for dp), D2H of (this rank's) dW
                 dX.copy_(it2["Xh"], non_blocking=True)
                 dG.copy_(it2["Gh"], non_blocking=True)
-                it3 = dict(it2, X=dX, dY=dG)
-                run_bfc(it3, stream)
+                run_bfc(dict(it2, X=dX, dY=dG), stream)
                 it2["dWh"].copy_(it2["dW"], non_blocking=True)
-                stream.synchronize()
             else:
                 W.bfc_host(it2["plan"], it2["Xh"], it2["Gh"], it2["dWh"], dX, dG, it2["dW"], it2["ws"], stream)
             b.record(stream)
@@ -326,77 +399,168 @@ def run_winrs(args):
             tot += a.elapsed_time(b)
         e2e_ms.append(tot)
     e2e = statistics.median(e2e_ms)
-    if world > 1:
-        t = torch.tensor([e2e], device=dev)
+
+    def max_over_ranks(v):
+        if world == 1 or v is None:
+            return v
+        t = torch.tensor([float(v)], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e = float(t.item())
+        return float(t.item())
+    step_ms = max_over_ranks(sum(per_layer_ms))
+    e2e = max_over_ranks(e2e)
+    co = max_over_ranks(sum(compute_only_ms)) if compute_only_ms else None
+    h2d = sum(it2["X"].numel() * it2["X"].element_size() + it2["dY"].numel() * it2["dY"].element_size()
+              for it2 in items)
+    d2h = sum(it2["dW"].numel() * 4 for it2 in items)   # this rank's dW (slice under kshard)
+    # whole-job FLOPs: every rank's local work
+    if strong or kshard:   # fixed global problem split over the ranks
+        job_flops = sum(it2["layer"].direct_flops for it2 in items)
+    else:                  # weak: every rank runs the full per-rank workload
+        job_flops = sum(it2["layer"].direct_flops for it2 in items) * world
+    return dict(items=items, per_layer_ms=per_layer_ms, warm_ms=warm_ms, compute_only_ms=compute_only_ms,
+                graph=graph, dom=dom, dom_ms=dom_ms, e2e_ms=e2e, step_ms=step_ms, compute_only_step_ms=co,
+                clocks=clk, h2d=h2d, d2h=d2h, job_flops=job_flops, steps=steps)
+
+
+def summarize(m, peaks, args):
+    items = m["items"]
+    layers = []
+    for j, x in enumerate(items):
+        rf = layer_roofline(x["local"], x["plan"], m["per_layer_ms"][j], peaks)
+        d = {"name": x["layer"].name, "ms": m["per_layer_ms"][j], "warm_ms": m["warm_ms"][j],
+             "tflops": x["local"].direct_flops * (x["k1"] - x["k0"]) / x["layer"].K / (m["per_layer_ms"][j] * 1e-3) / 1e12,
+             "workspace_bytes": x["plan"].workspace_bytes, "plan": repr(x["plan"]), "kernel": x["plan"].kernel_name,
+             "roofline_frac": rf["frac"], "bound": rf["bound"], "t_roof_us": rf["t_roof_us"],
+             "t_alu_us": rf["t_alu_us"], "t_l2_us": rf["t_l2_us"]}
+        if m["graph"]:
+            d["graph_replay_ms"] = m["graph"][j]["mean_ms"]
+            d["graph_replay_median_ms"] = m["graph"][j]["median_ms"]
+            d["graph_replays"] = m["graph"][j]["replays"]
+        if m["compute_only_ms"]:
+            d["compute_only_ms"] = m["compute_only_ms"][j]
+        layers.append(d)
+    return layers
+
+
+def run_winrs(args):
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    ndev = torch.cuda.device_count()
+    torch.cuda.set_device(local % ndev)
+    dev = torch.device("cuda", local % ndev)
+    backend = None
+    if world > 1:
+        # NCCL over NVLink/NVSwitch; gloo only when ranks must share a device
+        # (fewer GPUs than ranks: a multi-rank check on a 1-GPU box).
+        backend = os.environ.get("WINRS_DIST_BACKEND", "nccl" if ndev >= world else "gloo")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
+    kshard = args.parallel == "kshard" and world > 1
+    strong = args.workload == "r50l3" and world > 1 and not kshard
+    ctx = dict(world=world, rank=rank, local=local, dev=dev, kshard=kshard, strong=strong,
+               flush=torch.empty(256 << 20, dtype=torch.uint8, device=dev))
+    layers = _workload(args.workload, args.dtype)
+    m = measure(layers, args, ctx, primary=True)
+    alongside = []
+    if world == 1 and not args.no_alongside and args.workload == "vgg":
+        for wk, dt in (("r50", "f16"), ("r50", "f32"), ("wide", "f32")):
+            a = measure(_workload(wk, dt), args, ctx, primary=False)
+            alongside.append((wk, dt, a))
 
     if rank == 0:
-        flops = sum(it["layer"].direct_flops for it in items) * (1 if kshard else world)
-        value = flops / (step_ms * 1e-3) / 1e12
         peaks, src = _peaks()
-        esz = 4 if args.dtype == "f32" else 2   # f16 / bf16
-        l = it["layer"]
-        alg_bytes = esz * (l.N * l.H * l.W * l.C + l.N * l.Ho * l.Wo * l.K) + 4 * l.K * l.R * l.S * l.C * (
-            1 if info["Z"] == 1 else 2 * info["Z"] + 1)
-        if args.dtype == "f32":
-            peak = 148 * 128 * 2 * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6 / 1e12
-            roof = {"bound": "alu", "achieved": info["ewm_flops"] / (dom_ms * 1e-3) / 1e12, "peak": peak,
-                    "unit": "TFLOP/s", "peak_source": "148 SMs x 128 FP32 lanes x 2 x sm_max_mhz (DESIGN.md)",
-                    "kernel": p.kernel_name, "layer": l.name}
+        value = m["job_flops"] / (m["step_ms"] * 1e-3) / 1e12
+        per_layer = summarize(m, peaks, args)
+        it = m["items"][m["dom"]]
+        rf = layer_roofline(it["local"], it["plan"], m["dom_ms"], peaks)
+        if rf["bound"] == "hbm":
+            roof = {"bound": "hbm", "achieved": rf["alg_bytes"] / (m["dom_ms"] * 1e-3) / 1e9, "peak": peaks["hbm_gbs"],
+                    "unit": "GB/s", "peak_source": src + " hbm_gbs (copy)"}
+        elif rf["bound"] == "alu":
+            roof = {"bound": "alu", "achieved": rf["ewm_flops"] / (m["dom_ms"] * 1e-3) / 1e12, "peak": rf["pipe_peak_tflops"],
+                    "unit": "TFLOP/s", "peak_source": "148 SMs x 128 FP32 lanes x 2 x sm_max_mhz (DESIGN.md §6)"}
         else:
-            t_hbm = alg_bytes / (peaks["hbm_gbs"] * 1e9)
-            t_tc = info["ewm_flops"] / (peaks["bf16_tflops"] * 1e12)
-            if t_hbm >= t_tc:
-                roof = {"bound": "hbm", "achieved": alg_bytes / (dom_ms * 1e-3) / 1e9, "peak": peaks["hbm_gbs"],
-                        "unit": "GB/s", "peak_source": src}
-            else:
-                roof = {"bound": "tensor", "achieved": info["ewm_flops"] / (dom_ms * 1e-3) / 1e12,
-                        "peak": peaks["bf16_tflops"], "unit": "TFLOP/s", "peak_source": src + " (fp16 = bf16 rate)"}
-            roof.update(kernel=p.kernel_name, layer=l.name)
+            roof = {"bound": "tensor", "achieved": rf["ewm_flops"] / (m["dom_ms"] * 1e-3) / 1e12,
+                    "peak": peaks["bf16_tflops"], "unit": "TFLOP/s", "peak_source": src + " bf16_tflops (fp16 = bf16 rate)"}
         roof["frac"] = roof["achieved"] / roof["peak"]
-        roof["traffic"], roof["traffic_source"] = _ncu_traffic(args.dtype, l.name)
-        roof["alg_bytes"] = alg_bytes
-        roof["ewm_flops"] = info["ewm_flops"]
-        roof["kernel_ms"] = dom_ms
-        h2d = sum(it2["X"].numel() * it2["X"].element_size() + it2["dY"].numel() * it2["dY"].element_size()
-                  for it2 in items)
-        d2h = sum(it2["dW"].numel() * 4 for it2 in items)   # this rank's dW (slice under kshard)
+        roof["traffic"], roof["traffic_source"] = _ncu_traffic(args.dtype, it["layer"].name)
+        roof.update(kernel=it["plan"].kernel_name, layer=it["layer"].name, alg_bytes=rf["alg_bytes"],
+                    ewm_flops=rf["ewm_flops"], kernel_ms=m["dom_ms"], t_alu_us=rf["t_alu_us"], t_l2_us=rf["t_l2_us"],
+                    per_layer_frac={d["name"]: round(d["roofline_frac"], 4) for d in per_layer},
+                    worst_layer=min(per_layer, key=lambda d: d["roofline_frac"])["name"])
+        cfg = {"workload": f"{args.workload}_{args.dtype}: " + ", ".join(x["layer"].name for x in m["items"]),
+               "global_batch": (m["items"][0]["layer"].N if (strong or kshard) else m["items"][0]["layer"].N * world),
+               "parallelism": (f"kshard{world}" if kshard else f"dp{world}") if world > 1 else "single",
+               "backend": backend,
+               "l2": "flushed (256 MiB write) before every layer call; flush outside timed events",
+               "workspace_cap": float(os.environ.get("WINRS_WS_CAP", "0.04")),
+               "warm_l2_ms_per_step": sum(m["warm_ms"]),
+               "layers": per_layer}
+        if m["graph"]:
+            cfg["graph_replay_ms_per_step"] = sum(g["mean_ms"] for g in m["graph"])
+            cfg["graph_replay_tflops"] = m["job_flops"] / world / (cfg["graph_replay_ms_per_step"] * 1e-3) / 1e12 \
+                if world == 1 else None
+        if m["compute_only_step_ms"]:
+            cfg["compute_only_ms_per_step"] = m["compute_only_step_ms"]
+            cfg["compute_only_tflops"] = m["job_flops"] / (m["compute_only_step_ms"] * 1e-3) / 1e12
+            cfg["allreduce_share"] = 1.0 - m["compute_only_step_ms"] / m["step_ms"]
+        for wk, dt, a in alongside:
+            cfg.setdefault("alongside", []).append({
+                "workload": f"{wk}_{dt}", "value": a["job_flops"] / (a["step_ms"] * 1e-3) / 1e12, "unit": "TFLOPS",
+                "ms_per_step": a["step_ms"], "steps": a["steps"],
+                "e2e_tflops": a["job_flops"] / (a["e2e_ms"] * 1e-3) / 1e12,
+                "layers": summarize(a, peaks, args)})
         out = {
             "metric": METRIC,
             "value": value,
             "unit": "TFLOPS",
             "n_gpus": world,
-            "steps": args.steps,
+            "steps": m["steps"],
             "warmup": args.warmup,
-            "ms_per_step": step_ms,
+            "ms_per_step": m["step_ms"],
             "higher_is_better": True,
-            "scaling": "strong" if kshard else "weak",
+            "scaling": "strong" if (kshard or strong) else "weak",
             "vs_baseline": None,
             "dtype": args.dtype,
             "data": "synthetic (seeded U[0,1), dY x 1e-2 for f16; PAPER.md P@50685)",
-            "config": {"workload": f"{args.workload}_{args.dtype}: " + ", ".join(x["layer"].name for x in items),
-                       "global_batch": layers[0].N * (1 if kshard else world),
-                       "parallelism": (f"kshard{world}" if kshard else f"dp{world}") if world > 1 else "single",
-                       "l2": "flushed (256 MiB write) before every layer call; flush outside timed events",
-                       "workspace_cap": float(os.environ.get("WINRS_WS_CAP", "0.04")),
-                       "warm_l2_ms_per_step": sum(warm_ms),
-                       "compute_only_ms_per_step": sum(compute_only_ms) if compute_only_ms else None,
-                       "layers": [{"name": x["layer"].name, "ms": per_layer_ms[j], "warm_ms": warm_ms[j],
-                                   "tflops": x["layer"].direct_flops / (per_layer_ms[j] * 1e-3) / 1e12,
-                                   "workspace_bytes": x["plan"].workspace_bytes, "plan": repr(x["plan"]),
-                                   "kernel": x["plan"].kernel_name} for j, x in enumerate(items)]},
+            "config": cfg,
             "roofline": roof,
-            "e2e": {"value": flops / (e2e * 1e-3) / 1e12, "unit": "TFLOPS", "h2d_bytes_per_step": h2d,
-                    "d2h_bytes_per_step": d2h, "ms_per_step": e2e},
-            "gpu_launches": sum(x["plan"].launch_count for x in items) * args.steps,
-            "clocks": clk,
+            "e2e": {"value": m["job_flops"] / (m["e2e_ms"] * 1e-3) / 1e12, "unit": "TFLOPS",
+                    "h2d_bytes_per_step": m["h2d"], "d2h_bytes_per_step": m["d2h"], "ms_per_step": m["e2e_ms"]},
+            "gpu_launches": sum(x["plan"].launch_count for x in m["items"]) * m["steps"],
+            "clocks": m["clocks"],
         }
         if not args.no_cpu_baseline:
             out["cpu_baseline"] = cpu_baseline(layers, budget_s=args.cpu_seconds)
         print(json.dumps(out))
     if world > 1:
         dist.destroy_process_group()
+
+
+def run_dry(args):
+    """--dry-run: the launch / rank plumbing only (gloo, CPU tensors)."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        dist.init_process_group("gloo")
+        t = torch.tensor([float(rank + 1)])
+        dist.all_reduce(t)
+        total = float(t.item())
+        dist.barrier()
+        dist.destroy_process_group()
+    else:
+        total = 1.0
+    if rank == 0:
+        print(json.dumps({"metric": METRIC, "dry_run": True, "n_gpus": world, "ranks_sum": total,
+                          "workload": args.workload, "parallel": args.parallel}))
 
 
 def cpu_baseline(layers, budget_s: float = 8.0):
@@ -459,22 +623,39 @@ def run_reference(args):
     }))
 
 
+def _free_port():
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="winrs", choices=["winrs", "reference"])
-    ap.add_argument("--workload", default="r50", choices=["r50", "vgg", "wide", "r50l3"])
+    ap.add_argument("--workload", default="vgg", choices=["vgg", "r50", "wide", "r50l3"])
     ap.add_argument("--dtype", default=os.environ.get("WINRS_BENCH_DTYPE", "f16"), choices=["f32", "f16", "bf16"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-alongside", action="store_true", help="skip the ResNet-50 / wide workloads measured alongside")
+    ap.add_argument("--no-graphs", action="store_true", help="skip the CUDA-graph replay timing")
+    ap.add_argument("--graph-reps", type=int, default=0)
     ap.add_argument("--cpu-seconds", type=float, default=8.0)
     ap.add_argument("--parallel", default="dp", choices=["dp", "kshard"],
-                    help="N>1: dp = batch shards + one all_reduce of dW (weak); kshard = output-channel "
+                    help="N>1: dp = batch shards + one all_reduce of dW; kshard = output-channel "
                          "shards of the full batch, no communication (strong)")
     ap.add_argument("--ws-cap", type=float, default=None,
                     help="planner workspace cap as a fraction of X+dY bytes (default: the paper's 4%%)")
+    ap.add_argument("--dry-run", action="store_true", help="launch plumbing only (gloo, no GPU work)")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # one rank per GPU: re-launch under torch.distributed.run on this node
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+        import subprocess
+        sys.exit(subprocess.call(cmd))
     if args.ws_cap is not None:
         os.environ["WINRS_WS_CAP"] = str(args.ws_cap)
     if args.warmup < 3:
@@ -483,7 +664,9 @@ def main():
         args.dtype = "f32"
     if args.workload in ("vgg", "r50l3"):
         args.dtype = "f16"
-    if args.impl == "reference":
+    if args.dry_run:
+        run_dry(args)
+    elif args.impl == "reference":
         run_reference(args)
     else:
         run_winrs(args)

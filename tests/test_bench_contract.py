@@ -35,3 +35,17 @@ def test_reference_arm_json_line():
 def test_reference_arm_nonzero_rank_is_silent():
     out = _run(["--impl", "reference", "--steps", "1", "--warmup", "0"], env={"RANK": "1", "WORLD_SIZE": "2"})
     assert out.strip() == ""
+
+
+def test_gpus_flag_self_launches_ranks():
+    """--gpus 2 without a torchrun environment re-launches itself under
+    torch.distributed.run with 2 ranks; rank 0 prints one line with n_gpus 2."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK", "MASTER_ADDR",
+                                                            "MASTER_PORT")}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--dry-run",
+                        "--workload", "r50l3"], capture_output=True, text=True, cwd=ROOT, env=env, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.strip().startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["dry_run"] is True and d["ranks_sum"] == 3.0

@@ -102,7 +102,7 @@ def test_tc2_default_plans_use_tc2(monkeypatch):
 
 
 # ====================================================== pad = 0 (pad=0 variants of the wide config)
-PAD0 = [(l.with_(N=2, C=40, K=36, H=17, W=19, pad=0, name=l.name + "_pad0")) for l in wl.WIDE_F32] + [
+PAD0 = [(l.with_(N=2, C=40, K=48, H=17, W=19, pad=0, name=l.name + "_pad0")) for l in wl.WIDE_F32] + [
     wl.LAYERS["r50_c64_56_f32"].with_(N=2, H=20, W=23, pad=0, name="r50_l1_pad0"),
     wl.LAYERS["r50_c256_14_f32"].with_(N=2, C=72, K=64, pad=0, name="r50_l3_pad0"),
 ]
