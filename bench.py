@@ -208,12 +208,13 @@ def layer_roofline(l, p, ms, peaks):
     bn, bm = info["tile_k0"], info["tile_c0"]
     kb, cb = -(-l.K // bn), -(-l.C // bm)
     ft = l.S // n0
-    if "_v2_" in name:
-        fhs = int(name.split("x")[-1].rstrip("fh"))
+    if "_v2" in name:
+        cg = int(name.split("_v2")[1][0])                 # CTAs per UMMA (2: cta_group::2 pair)
+        fhs = int(name.split("x")[-1].rstrip("fh")) * cg if bm == 64 else 1
         rows = sum(_rows_union(l, range(g, min(l.R, g + fhs))) for g in range(0, l.R, fhs))
-        depth = rows * units * l.N * kb * cb * ft
-        l2_bytes = depth / 16 * (16384 + bn * 64)         # per 16-deep stage: X 16 KB + dY NK*64 B
-        alu_ops = depth * bn                              # FT: W0, W1 = w0 +- w1, packed half2
+        depth = rows * units * l.N * kb * cb * ft        # depth entries x (pair) tiles
+        l2_bytes = depth / 16 * (cg * 16384 + bn * 64)    # per 16-deep stage: X 16 KB per CTA + dY NK*64 B
+        alu_ops = depth * (bn + 128 * cg * 2)             # FT: W0, W1 = w0 +- w1; IT: 4 outputs per row (half2)
     else:
         rows = sum(_rows_valid(l, fh) for fh in range(l.R))
         depth = rows * units * l.N * kb * cb * ft

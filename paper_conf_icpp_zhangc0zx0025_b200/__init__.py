@@ -19,7 +19,7 @@ from dataclasses import dataclass
 from . import _lib
 from ._lib import WinrsError, DTYPES
 
-__all__ = ["Plan", "plan", "plan_for_device", "bfc", "bfc_host", "as_kcrs", "bfc_data_parallel", "shard_range",
+__all__ = ["Plan", "plan", "plan_for_device", "bfc", "bfc_host", "as_kcrs", "as_krsc", "bfc_data_parallel", "shard_range",
            "bfc_k_sharded",
            "WinrsError", "version", "emulate", "transform", "kernel_names"]
 
@@ -104,8 +104,28 @@ def _as_nhwc(t, n, h, w, c, name):
                      f"[{n},{c},{h},{w}], got shape {tuple(t.shape)} strides {t.stride()}")
 
 
+def _as_krsc(t, k, c, r, s_, name):
+    """Return a tensor whose memory is KRSC [k,r,s,c] (no copy): a contiguous
+    KRSC tensor, or a logical [K,C,R,S] channels_last tensor."""
+    if tuple(t.shape) == (k, r, s_, c) and t.is_contiguous():
+        return t
+    if tuple(t.shape) == (k, c, r, s_):
+        import torch
+        if t.is_contiguous(memory_format=torch.channels_last):
+            return t.permute(0, 2, 3, 1)
+    raise ValueError(f"{name}: expected KRSC [{k},{r},{s_},{c}] contiguous or channels_last "
+                     f"[{k},{c},{r},{s_}], got shape {tuple(t.shape)} strides {t.stride()}")
+
+
 def bfc(p: Plan, X, dY, dW=None, workspace=None, stream=None):
-    """winrs_bfc on torch CUDA tensors; returns dW [K,R,S,C] float32."""
+    """winrs_bfc on torch CUDA tensors.
+
+    X, dY: logical NCHW with channels_last strides, or NHWC-contiguous.
+    Returns dW with logical [K,C,R,S] shape and channels_last strides, FP32
+    (physical order KRSC, the C ABI's layout; `as_krsc` gives that view).  A
+    caller-supplied dW (KRSC-contiguous or channels_last KCRS) is written in
+    place and returned as given.  Everything runs on `stream` (default: the
+    current stream); tensors allocated here are recorded on it."""
     import torch
     i = p.info
     tdt = {"f32": torch.float32, "f16": torch.float16, "bf16": torch.bfloat16}[p.dtype]
@@ -113,20 +133,51 @@ def bfc(p: Plan, X, dY, dW=None, workspace=None, stream=None):
     Gn = _as_nhwc(dY, i["N"], i["Ho"], i["Wo"], i["K"], "dY")
     if Xn.dtype != tdt or Gn.dtype != tdt:
         raise TypeError(f"X and dY must be {tdt} for this plan")
-    if not (Xn.is_cuda and Gn.is_cuda):
-        raise ValueError("X and dY must be CUDA tensors (use bfc_host for host buffers)")
-    if dW is None:
-        dW = torch.empty((i["K"], i["R"], i["S"], i["C"]), dtype=torch.float32, device=Xn.device)
-    elif not (dW.dtype == torch.float32 and dW.is_contiguous() and dW.numel() == i["K"] * i["R"] * i["S"] * i["C"]):
-        raise ValueError("dW must be a contiguous float32 KRSC tensor")
-    wsb = p.workspace_bytes
-    if wsb and workspace is None:
-        workspace = torch.empty(wsb, dtype=torch.uint8, device=Xn.device)
+    if not (Xn.is_cuda and Gn.is_cuda) or Gn.device != Xn.device:
+        raise ValueError("X and dY must be CUDA tensors on one device (use bfc_host for host buffers)")
     if stream is None:
         stream = torch.cuda.current_stream(Xn.device)
     sp = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
-    _lib.check(_lib.lib().winrs_bfc(p.handle, Xn.data_ptr(), Gn.data_ptr(), dW.data_ptr(),
+    ts = stream if isinstance(stream, torch.cuda.Stream) else None
+    ret = dW
+    if dW is None:
+        with torch.cuda.stream(ts) if ts is not None else _nullctx():
+            dk = torch.empty((i["K"], i["R"], i["S"], i["C"]), dtype=torch.float32, device=Xn.device)
+        ret = dk.permute(0, 3, 1, 2)          # logical KCRS, channels_last
+    else:
+        if dW.dtype != torch.float32 or not dW.is_cuda or dW.device != Xn.device:
+            raise ValueError("dW must be a float32 CUDA tensor on X's device")
+        dk = _as_krsc(dW, i["K"], i["C"], i["R"], i["S"], "dW")
+    wsb = p.workspace_bytes
+    if wsb:
+        if workspace is None:
+            with torch.cuda.stream(ts) if ts is not None else _nullctx():
+                workspace = torch.empty(wsb, dtype=torch.uint8, device=Xn.device)
+        elif not workspace.is_cuda or workspace.device != Xn.device or \
+                workspace.numel() * workspace.element_size() < wsb:
+            raise ValueError(f"workspace must be >= {wsb} bytes on X's device")
+    _lib.check(_lib.lib().winrs_bfc(p.handle, Xn.data_ptr(), Gn.data_ptr(), dk.data_ptr(),
                                     workspace.data_ptr() if wsb else None, sp), "winrs_bfc")
+    if ts is not None:   # the caching allocator must not recycle these before `stream` is done with them
+        dk.record_stream(ts)
+        if wsb:
+            workspace.record_stream(ts)
+    return ret
+
+
+class _nullctx:
+    def __enter__(self):
+        return None
+
+    def __exit__(self, *a):
+        return False
+
+
+def as_krsc(dW):
+    """bfc()'s logical [K,C,R,S] channels_last result -> its KRSC [K,R,S,C]
+    storage view (the C ABI / oracle layout), no copy.  KRSC input passes."""
+    if dW.dim() == 4 and dW.stride(1) == 1 and not dW.is_contiguous():
+        return dW.permute(0, 2, 3, 1)
     return dW
 
 
@@ -199,7 +250,7 @@ def bfc_data_parallel(X_shard, dY_shard, R: int, S: int, pad: int, dtype: str = 
         p = plan(N, C, H, W, K, R, S, pad, dtype)
     dW = bfc(p, X_shard, dY_shard)
     if dist.is_initialized() and dist.get_world_size(group) > 1:
-        dist.all_reduce(dW, op=dist.ReduceOp.SUM, group=group)
+        dist.all_reduce(as_krsc(dW), op=dist.ReduceOp.SUM, group=group)   # the contiguous KRSC storage
     return dW
 
 

@@ -47,9 +47,9 @@ static bool make_map(CUtensorMap* m, const void* base, int N, int H, int W, int 
 // rows are exactly a column-major run of 16-row operand atoms (N % 16 == 0).
 static int images_per_box(int N) { return N % KC == 0 ? KC : 0; }
 
-template <int F, int NK, bool BF>
+template <int F, int NK, bool BF, int CG>
 cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
-    using L = Lay<F, NK>;
+    using L = Lay<F, NK, CG>;
     const long long grid = num_ctas(g);
     if (grid <= 0) return cudaSuccess;
     Args a;
@@ -63,22 +63,36 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
         !make_map(&mY, dY, g.N, g.Ho, g.Wo, g.K, g.ldy, 2, a.nb, BF))
         return cudaErrorInvalidValue;
     static std::atomic<unsigned long long> done{0};
-    auto k = bfc_tc2_kernel<F, NK, BF>;
+    auto k = bfc_tc2_kernel<F, NK, BF, CG>;
     cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
     if (e != cudaSuccess) return e;
-    if (g.csplit <= 1) {
+    const int cluster = CG * g.csplit;
+    if (cluster <= 1) {
         k<<<(unsigned)grid, NTHREADS, L::BYTES, stream>>>(a, mX, mY);
         return cudaGetLastError();
     }
-    return launch_cluster(k, (unsigned)grid, (unsigned)NTHREADS, (size_t)L::BYTES, stream, g.csplit, a, mX, mY);
+    if (cluster > 8) {   // 16-CTA clusters (a pair per rank of an 8-way depth split): non-portable size
+        static std::atomic<unsigned long long> np{0};
+        int dev = 0;
+        cudaGetDevice(&dev);
+        if (!(np.load() & (1ull << (dev & 63)))) {
+            e = cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+            if (e != cudaSuccess) return e;
+            np.fetch_or(1ull << (dev & 63));
+        }
+    }
+    return launch_cluster(k, (unsigned)grid, (unsigned)NTHREADS, (size_t)L::BYTES, stream, cluster, a, mX, mY);
 }
 
 }  // namespace tc2
 
-#define WINRS_TC2_ENTRY(DT, BF, PFX, F, NK)                                                              \
-    {DT, 4, 3, 2, 0, 0, 0, NK, ::winrs::tc2::MROWS / F, ::winrs::tc2::NTHREADS, 1, 1,                    \
-     (size_t)::winrs::tc2::Lay<F, NK>::BYTES, &::winrs::tc2::launch<F, NK, BF>,                           \
-     PFX "_O4(3,2)_v2_" #NK "x" #F "fh", F}
+// tile = NK k columns x (128 / F) c rows x F filter rows (one CTA), or for a
+// cta_group::2 pair (CG = 2) 256 c rows (F = 1) or 4 filter rows (F = 2).
+#define WINRS_TC2_ENTRY(DT, BF, PFX, F, NK, CG)                                                          \
+    {DT, 4, 3, 2, 0, 0, 0, NK, (F == 1 ? ::winrs::tc2::MROWS * CG : ::winrs::tc2::MROWS / F),            \
+     ::winrs::tc2::NTHREADS, 1, 1, (size_t)::winrs::tc2::Lay<F, NK, CG>::BYTES,                          \
+     &::winrs::tc2::launch<F, NK, BF, CG>,                                                                \
+     PFX "_O4(3,2)_v2" #CG "_" #NK "x" #F "fh", (F == 1 ? 1 : F * CG), CG}
 
 #ifdef WINRS_TC2_TRACE
 extern "C" __attribute__((visibility("default"))) int winrs_tc2_trace(int cta, long long* out) {
@@ -90,14 +104,18 @@ extern "C" __attribute__((visibility("default"))) int winrs_tc2_trace(int cta, l
 const KernelEntry* tc2_entries(int* n) {
     // tile = NK k columns x (128 / F) c rows x F filter rows
     static const KernelEntry e[] = {
-        WINRS_TC2_ENTRY(1, false, "f16tc", 1, 128),
-        WINRS_TC2_ENTRY(1, false, "f16tc", 1, 64),
-        WINRS_TC2_ENTRY(1, false, "f16tc", 2, 128),
-        WINRS_TC2_ENTRY(1, false, "f16tc", 2, 64),
-        WINRS_TC2_ENTRY(2, true, "bf16tc", 1, 128),
-        WINRS_TC2_ENTRY(2, true, "bf16tc", 1, 64),
-        WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 128),
-        WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 64),
+        WINRS_TC2_ENTRY(1, false, "f16tc", 1, 128, 1),
+        WINRS_TC2_ENTRY(1, false, "f16tc", 1, 64, 1),
+        WINRS_TC2_ENTRY(1, false, "f16tc", 2, 128, 1),
+        WINRS_TC2_ENTRY(1, false, "f16tc", 2, 64, 1),
+        WINRS_TC2_ENTRY(1, false, "f16tc", 1, 128, 2),
+        WINRS_TC2_ENTRY(1, false, "f16tc", 2, 128, 2),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 1, 128, 1),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 1, 64, 1),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 128, 1),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 64, 1),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 1, 128, 2),
+        WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 128, 2),
     };
     *n = sizeof(e) / sizeof(e[0]);
     return e;

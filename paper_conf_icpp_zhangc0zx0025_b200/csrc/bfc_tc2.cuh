@@ -68,10 +68,16 @@ constexpr int MROWS = 128;             // UMMA M = TMEM lanes
 constexpr int NTX = 8;                 // transformer warps
 constexpr int NTHREADS = 64 + 32 * NTX;
 constexpr int NSOUT = 3;               // n0: outputs per unit (S = 3)
+#ifndef WINRS_TC2_ITM
+#define WINRS_TC2_ITM 0    // 1: IT inside the tensor core (8 MMAs per stage on the raw X columns, by linearity);
+                           // 0: IT on the FT warps, in place over the raw X slabs (4 MMAs per stage: the
+                           //    alpha = 4 Winograd EWM).  A/B on B200 in DESIGN.md §6.4.
+#endif
 
-template <int F, int NK>
+template <int F, int NK, int CG = 1>
 struct Lay {
     static constexpr int BC = MROWS / F;                 // channels c per fh slot
+    static constexpr int NKL = NK / CG;                  // k rows of the What operand held by this CTA
     // One stage = 16 depth entries (images n of one (h, u)), three regions of
     // 64-channel swizzle atoms [atom][col][n (16 rows of 128 B)]:
     //   X   [2 atoms][4 cols x_t]   16 KB   A operand of column t: +t*2 KB, atoms 8 KB apart
@@ -82,8 +88,8 @@ struct Lay {
     static constexpr int X_LBO = 4 * ATOM;               // 8 KB
     static constexpr int Y_LBO = 2 * ATOM;               // 4 KB
     static constexpr int OFF_Y = 2 * X_LBO;              // 16 KB
-    static constexpr int OFF_F = OFF_Y + (NK / 64) * Y_LBO;
-    static constexpr int STAGE = OFF_F + (NK / 64) * Y_LBO;   // 32 / 24 KB
+    static constexpr int OFF_F = OFF_Y + (NKL / 64) * Y_LBO;
+    static constexpr int STAGE = OFF_F + (NKL / 64) * Y_LBO;   // 32 / 24 KB (cta pair: 24 KB)
     static constexpr int LIMIT = 227 * 1024 - 1024 - 256;
     static constexpr int S = LIMIT / STAGE > 8 ? 8 : LIMIT / STAGE;
     static constexpr int RING = S * STAGE;
@@ -95,6 +101,7 @@ struct Lay {
     static_assert(STAGE % 1024 == 0, "stages must keep the 1 KB swizzle-atom alignment");
     static_assert(S >= 4, "ring too shallow");
     static_assert(MROWS == F * BC && BC % 64 == 0, "fh slots of whole 64-channel atoms");
+    static_assert(NKL % 64 == 0, "whole 64-channel k atoms per CTA");
 };
 
 struct Args {
@@ -158,20 +165,46 @@ __device__ __forceinline__ uint64_t desc_sw128(uint32_t addr, uint32_t lbo, uint
 // kind::f16 instruction descriptor: D f32, A/B f16 (0) or bf16 (1), both
 // MN-major (bits 15, 16), N >> 3 at bit 17, M >> 4 at bit 24.
 // Bit 13: negate A (the IT's minus signs).
-template <int NK, bool BF, bool NEG = false>
+// cta_group::2: M = 256 over a CTA pair (each CTA's 128 A rows and NK / 2 B
+// rows; each CTA's TMEM holds its 128 rows x NK accumulator columns).
+template <int NK, bool BF, bool NEG = false, int CG = 1>
 __host__ __device__ constexpr uint32_t idesc() {
     return (1u << 4) | ((BF ? 1u : 0u) << 7) | ((BF ? 1u : 0u) << 10) | ((NEG ? 1u : 0u) << 13) | (1u << 15) |
-           (1u << 16) | ((uint32_t)(NK >> 3) << 17) | ((uint32_t)(MROWS >> 4) << 24);
+           (1u << 16) | ((uint32_t)(NK >> 3) << 17) | ((uint32_t)((MROWS * CG) >> 4) << 24);
 }
-template <int NK, bool BF, bool NEG = false>
+template <int NK, bool BF, bool NEG = false, int CG = 1>
 __device__ __forceinline__ void umma(uint32_t d, uint64_t a, uint64_t b, uint32_t acc) {
-    asm volatile(
-        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
-        :: "r"(d), "l"(a), "l"(b), "r"(idesc<NK, BF, NEG>()), "r"(acc));
+    if constexpr (CG == 1)
+        asm volatile(
+            "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+            "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
+            :: "r"(d), "l"(a), "l"(b), "r"(idesc<NK, BF, NEG, CG>()), "r"(acc));
+    else
+        asm volatile(
+            "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+            "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n"
+            :: "r"(d), "l"(a), "l"(b), "r"(idesc<NK, BF, NEG, CG>()), "r"(acc));
 }
-__device__ __forceinline__ void umma_commit(uint64_t* bar) {
-    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" :: "r"(su(bar)) : "memory");
+// Commit: arrives on `bar` once every MMA issued so far completed; for a CTA
+// pair on the barrier at the same offset in both CTAs (mask = the pair).
+template <int CG = 1>
+__device__ __forceinline__ void umma_commit(uint64_t* bar, uint16_t mask = 3) {
+    if constexpr (CG == 1)
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" :: "r"(su(bar)) : "memory");
+    else
+        asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
+                     :: "r"(su(bar)), "h"(mask) : "memory");
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+// Arrive on the mbarrier at local shared offset `bar` of cluster CTA `rank`.
+__device__ __forceinline__ void mbar_arrive_cluster(uint64_t* bar, uint32_t rank) {
+    uint32_t remote;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(su(bar)), "r"(rank));
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" :: "r"(remote) : "memory");
 }
 __device__ __forceinline__ void tmem_ld8(uint32_t taddr, float* v) {
     uint32_t r[8];
@@ -244,11 +277,11 @@ __device__ __forceinline__ void depth_nhu(int d, int N, int units, int hs, int* 
     *h = hs + t / units;
 }
 
-template <int F, int NK, bool BF>
+template <int F, int NK, bool BF, int CG = 1>
 __global__ void __launch_bounds__(NTHREADS, 1)
 bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX,
                const __grid_constant__ CUtensorMap tmY) {
-    using L = Lay<F, NK>;
+    using L = Lay<F, NK, CG>;
     extern __shared__ uint8_t smem_raw[];
     // 1 KB-aligned base (SW128 atoms, TMA swizzle pattern)
     const uint32_t raw_s = su(smem_raw);
@@ -259,8 +292,20 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 64) TC2_TRACE(511, 0);
 
-    const int rank = (int)(blockIdx.x % g.csplit);
-    const CtaCoord cc = decode_cta(g, blockIdx.x / g.csplit);
+    // Cluster = CG x csplit CTAs: a CTA pair (cta_group::2, CG = 2: ranks 2j,
+    // 2j + 1; the even one issues the MMAs) per depth-split rank j.
+    const int crank = CG * g.csplit > 1 ? (int)cluster_rank() : 0;
+    const int e = CG == 2 ? (crank & 1) : 0;                 // half of the pair
+    const int rank = CG == 2 ? (crank >> 1) : (int)(blockIdx.x % g.csplit);   // depth-split rank
+    const uint32_t leader = (uint32_t)(crank & ~(CG - 1));
+    const uint16_t pair_mask = (uint16_t)(3u << leader);
+    const CtaCoord cc = decode_cta(g, blockIdx.x / (CG * g.csplit));
+    // this CTA's 128 A rows: F = 1: channels c_base.. of filter row fh_base;
+    // F = 2: fh slots fh_base, fh_base + 1 of channels c_base..c_base + 63.
+    // A pair covers 256 channels (F = 1) or 4 filter rows (F = 2).
+    const int fh_base = cc.fh + (F == 2 ? 2 * e : 0);
+    const int c_base = F == 2 ? cc.cb * 64 : cc.cb * (128 * CG) + e * 128;
+    const int k_base = cc.kb * NK + e * L::NKL;              // this CTA's What rows
     const int seg = cc.band * g.seg_cols + cc.col;
     float* bucket = seg == 0 ? args.dW : args.ws + (long long)(seg - 1) * g.dw_elems;
     int hs, he, w_first, units;
@@ -281,17 +326,26 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         mbar_init(&bars->accfull, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
+    if (CG == 2 && threadIdx.x == 0 && e == 0)   // the leader's opfull gathers both CTAs' FT warps
+        for (int s = 0; s < L::S; ++s) mbar_init(&bars->opfull[s], 2);
     if (warp == 0 && lane == 0) {
         asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
         asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
     }
     if (warp == 1) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
-                     :: "r"(su(&bars->tmem_base)), "r"(L::TMEM_COLS));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        if constexpr (CG == 2) {
+            asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;"
+                         :: "r"(su(&bars->tmem_base)), "r"(L::TMEM_COLS));
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+        } else {
+            asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+                         :: "r"(su(&bars->tmem_base)), "r"(L::TMEM_COLS));
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        }
     }
     tc_before();
     __syncthreads();
+    if (CG == 2) cluster_sync_all();   // peer barriers initialised before any remote arrive / multicast commit
     tc_after();
     const uint32_t tmem = bars->tmem_base;
     if (threadIdx.x == 64) TC2_TRACE(511, 1);
@@ -326,14 +380,14 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 for (int a = 0; a < 2; ++a) {
                     // X window columns x0..x3 of atom a; an fh slot past the last
                     // filter row reads rows far outside (zero fill)
-                    const int fh = F == 2 ? cc.fh + a : cc.fh;
-                    const int c0 = F == 2 ? cc.cb * 64 : cc.cb * 128 + a * 64;
+                    const int fh = F == 2 ? fh_base + a : fh_base;
+                    const int c0 = F == 2 ? c_base : c_base + a * 64;
                     const int xrow = fh < g.R ? hh + fh - g.pad : -(1 << 20);
                     tma4(st + a * L::X_LBO, &tmX, fb, c0, nn, xrow, w0 + fw0 - g.pad);
                 }
 #pragma unroll
-                for (int ka = 0; ka < NK / 64; ++ka)   // dY unit columns w0, w0 + 1 of k atom ka
-                    tma4(st + L::OFF_Y + ka * L::Y_LBO, &tmY, fb, cc.kb * NK + ka * 64, nn, hh, w0);
+                for (int ka = 0; ka < L::NKL / 64; ++ka)   // dY unit columns w0, w0 + 1 of k atom ka
+                    tma4(st + L::OFF_Y + ka * L::Y_LBO, &tmY, fb, k_base + ka * 64, nn, hh, w0);
 #endif
             }
             __syncwarp();
@@ -349,7 +403,9 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     } else if (warp == 1) {
         // ============================ MMA issuer ==============================
         // Converged warp; descriptors are computed uniformly, one elected lane
-        // issues the MMAs and the commit.
+        // issues the MMAs and the commit (a pair: the leader only, for both).
+        if (CG == 2 && e != 0) goto mma_done;
+        {
         int s = 0;
         uint32_t ph = 0;
         for (int ch = c_lo; ch < c_hi; ++ch) {
@@ -365,25 +421,34 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             const uint64_t w2d = desc_sw128(st + L::OFF_Y, L::Y_LBO, 1024), w3d = w2d + (L::ATOM >> 4);
             if (elect_one()) {
 #ifndef WINRS_TC2_NO_MMA   // debug ablation: no tensor-core work (barrier protocol kept)
-                umma<NK, BF>(tmem + 0 * NK, x1, w0d, acc);          // v0 = (x1 + x2) W0
-                umma<NK, BF>(tmem + 0 * NK, x2, w0d, 1u);
-                umma<NK, BF>(tmem + 1 * NK, x2, w1d, acc);          // v1 = (x2 - x1) W1
-                umma<NK, BF, true>(tmem + 1 * NK, x1, w1d, 1u);
-                umma<NK, BF>(tmem + 2 * NK, x0, w2d, acc);          // v2 = (x0 - x2) W2
-                umma<NK, BF, true>(tmem + 2 * NK, x2, w2d, 1u);
-                umma<NK, BF>(tmem + 3 * NK, x3, w3d, acc);          // v3 = (x3 - x1) W3
-                umma<NK, BF, true>(tmem + 3 * NK, x1, w3d, 1u);
+              if (!WINRS_TC2_ITM) {   // Xhat[xi] (IT done in place by the FT warps) x What[xi]
+                umma<NK, BF, false, CG>(tmem + 0 * NK, x0, w0d, acc);
+                umma<NK, BF, false, CG>(tmem + 1 * NK, x1, w1d, acc);
+                umma<NK, BF, false, CG>(tmem + 2 * NK, x2, w2d, acc);
+                umma<NK, BF, false, CG>(tmem + 3 * NK, x3, w3d, acc);
+              } else {
+                umma<NK, BF, false, CG>(tmem + 0 * NK, x1, w0d, acc);          // v0 = (x1 + x2) W0
+                umma<NK, BF, false, CG>(tmem + 0 * NK, x2, w0d, 1u);
+                umma<NK, BF, false, CG>(tmem + 1 * NK, x2, w1d, acc);          // v1 = (x2 - x1) W1
+                umma<NK, BF, true, CG>(tmem + 1 * NK, x1, w1d, 1u);
+                umma<NK, BF, false, CG>(tmem + 2 * NK, x0, w2d, acc);          // v2 = (x0 - x2) W2
+                umma<NK, BF, true, CG>(tmem + 2 * NK, x2, w2d, 1u);
+                umma<NK, BF, false, CG>(tmem + 3 * NK, x3, w3d, acc);          // v3 = (x3 - x1) W3
+                umma<NK, BF, true, CG>(tmem + 3 * NK, x1, w3d, 1u);
+              }
 #else
                 (void)x0; (void)x1; (void)x2; (void)x3; (void)w0d; (void)w1d; (void)w2d; (void)w3d; (void)acc;
 #endif
-                umma_commit(&bars->empty[s]);
+                umma_commit<CG>(&bars->empty[s], pair_mask);
             }
             __syncwarp();
             TC2_TRACE(ch - c_lo, 5);
             if (++s == L::S) { s = 0; ph ^= 1; }
         }
-        if (elect_one()) umma_commit(&bars->accfull);   // arrives once all issued MMAs completed
+        if (elect_one()) umma_commit<CG>(&bars->accfull, pair_mask);   // arrives once all issued MMAs completed
         __syncwarp();
+        }
+    mma_done:;
     } else {
         // ================================= FT =================================
         // What[0] = w0 + w1, What[1] = w0 - w1 for the stage's NK k x 16 depth
@@ -395,8 +460,8 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         // critical path.  One warp per slot keeps the ring safe by construction:
         // slot w is refilled only after the MMAs of this warp's previous stage
         // in it, so its parity wait can never see a phase two rounds ahead.
-        constexpr int KO = NK / 8;                  // k octets
-        constexpr int IPT = KO * KC / 32;           // items per lane: 8 (NK 128) / 4 (NK 64)
+        constexpr int KO = L::NKL / 8;              // k octets of this CTA's What rows
+        constexpr int IPT = KO * KC / 32;           // items per lane: 8 (NK 128) / 4 (NK 64 or a pair)
         static_assert(L::S <= NTX, "one FT warp per ring slot");
         const int tw = warp - 2;
         uint32_t ph = 0;
@@ -406,6 +471,32 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             ph ^= 1;
             if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
             const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            if (!WINRS_TC2_ITM) {
+                // IT in place: item (row octet o, depth d) reads x0..x3 of its 8 rows
+                // and overwrites them with Xhat = (x1 + x2, x2 - x1, x0 - x2, x3 - x1)
+                // (no other item touches those bytes); 256 items, 8 per lane, in
+                // two batches of 4 to bound the live registers.
+#pragma unroll
+                for (int bt = 0; bt < 2; ++bt) {
+                    uint4 xv[4][4];
+                    uint32_t xo[4];
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const int t = (bt * 4 + i) * 32 + lane;     // depth t / 16, row octet t % 16
+                        const int o = t & 15;
+                        xo[i] = st + (uint32_t)((o >> 3) * L::X_LBO) + opoff(o & 7, t >> 4, 0);
+#pragma unroll
+                        for (int c = 0; c < 4; ++c) xv[i][c] = lds16(xo[i] + c * L::ATOM);
+                    }
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        sts16(xo[i], vadd<BF>(xv[i][1], xv[i][2]));
+                        sts16(xo[i] + L::ATOM, vsub<BF>(xv[i][2], xv[i][1]));
+                        sts16(xo[i] + 2 * L::ATOM, vsub<BF>(xv[i][0], xv[i][2]));
+                        sts16(xo[i] + 3 * L::ATOM, vsub<BF>(xv[i][3], xv[i][1]));
+                    }
+                }
+            }
             uint4 w0[IPT], w1[IPT];
             uint32_t off[IPT];
 #pragma unroll
@@ -424,7 +515,10 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             }
             fence_async();     // generic-proxy stores -> visible to the tensor core (async proxy)
             __syncwarp();
-            if (lane == 0) mbar_arrive(&bars->opfull[s]);
+            if (lane == 0) {
+                if (CG == 2) mbar_arrive_cluster(&bars->opfull[s], leader);
+                else mbar_arrive(&bars->opfull[s]);
+            }
             if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 3);
         }
         // ============================ epilogue ================================
@@ -434,8 +528,8 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         const int q = warp & 3;                      // TMEM lane quarter of this warp
         const int half = (warp - 2) >> 2;            // k half
         const int m = q * 32 + lane;
-        const int fh = cc.fh + m / L::BC;
-        const int c = cc.cb * L::BC + m % L::BC;
+        const int fh = fh_base + m / L::BC;
+        const int c = c_base + m % L::BC;
         const bool row_ok = fh < g.R && c < g.C;
         float* Out = reinterpret_cast<float*>(smem);  // staging [s][k][m] (overlays the idle ring)
         const uint32_t lane_base = tmem + ((uint32_t)(q * 32) << 16);
@@ -486,9 +580,9 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHREADS) {
             const int row = p / M4, m4 = p % M4;
             const int sidx = row / NK, kl = row % NK;
-            const float4 acc = dsmem_sum4(out_s + (uint32_t)((row * MROWS + m4 * 4) * 4), g.csplit);
+            const float4 acc = dsmem_sum4(out_s + (uint32_t)((row * MROWS + m4 * 4) * 4), g.csplit, CG, e);
             const int m = m4 * 4;
-            const int fh = cc.fh + m / L::BC, c = cc.cb * L::BC + m % L::BC, k = cc.kb * NK + kl;
+            const int fh = fh_base + m / L::BC, c = c_base + m % L::BC, k = cc.kb * NK + kl;
             if (fh < g.R && c < g.C && k < g.K)
                 *reinterpret_cast<float4*>(bucket + (((long long)k * g.R + fh) * g.S + fw0 + sidx) * g.C + c) = acc;
         }
@@ -496,9 +590,13 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         cluster_sync_all();
     }
     if (threadIdx.x == 64) TC2_TRACE(511, 6);
+    if (CG == 2 && g.csplit <= 1) cluster_sync_all();   // the pair's MMAs wrote both TMEMs
     if (warp == 1) {
         tc_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem), "r"(L::TMEM_COLS));
+        if constexpr (CG == 2)
+            asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" :: "r"(tmem), "r"(L::TMEM_COLS));
+        else
+            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem), "r"(L::TMEM_COLS));
     }
 }
 

@@ -11,13 +11,14 @@ namespace winrs {
 // `saddr` of each rank.  All remote loads are issued before the first add, so
 // the cs DSMEM round trips overlap instead of serialising on the adds; the
 // adds then run in rank order (bitwise reproducible).
-__device__ __forceinline__ float4 dsmem_sum4(uint32_t saddr, int cs) {
+// Ranks stride * q + offset (a CTA pair's halves reduce separately).
+__device__ __forceinline__ float4 dsmem_sum4(uint32_t saddr, int cs, int stride = 1, int offset = 0) {
     float4 v[8];
 #pragma unroll
     for (int q = 0; q < 8; ++q) {
         if (q < cs) {
             uint32_t remote;
-            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(saddr), "r"(q));
+            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(saddr), "r"(stride * q + offset));
             asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
                          : "=f"(v[q].x), "=f"(v[q].y), "=f"(v[q].z), "=f"(v[q].w) : "r"(remote) : "memory");
         }

@@ -12,7 +12,7 @@
 //      eq. (5); readings R9, R10).
 //
 // Debug overrides (tests only): WINRS_FORCE_Z=<z>, WINRS_FORCE_TILE=<bn>x<bm>, WINRS_FORCE_CSPLIT=<1|2|4|8>,
-// WINRS_FORCE_PAIR=a0,n0,r0,a1,n1,r1.  Policy: WINRS_WS_CAP=<fraction> replaces the
+// WINRS_FORCE_PAIR=a0,n0,r0,a1,n1,r1, WINRS_TC_GEN=1|2 (tensor-core kernel generation), WINRS_FORCE_CG=1|2.  Policy: WINRS_WS_CAP=<fraction> replaces the
 // 4% workspace cap (R11).
 #include <algorithm>
 #include <cmath>
@@ -190,6 +190,7 @@ static void fill_geometry(const Problem& p, const KernelEntry& e, const PairChoi
     g->cblocks = (int)cdiv(p.C, e.bm);
     g->ftiles = p.S / e.n0;
     g->fhs = e.fhs > 0 ? e.fhs : 1;
+    g->cg = e.cg > 0 ? e.cg : 1;
     g->fhg = (int)cdiv(p.R, g->fhs);
     g->Z = g->bands * g->seg_cols;
     g->csplit = 1;
@@ -239,13 +240,15 @@ struct SharedModel {
 
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
+    if (e.fhs > 0 && e.cg == 2)   // bfc_tc2.cuh CTA pair: rate of the pair over its 256-row tile
+        return {4.5e-6, 11.0e12};
     if (e.fhs > 0) {
         // bfc_tc2.cuh, rate over the whole 128-row UMMA tile (fhs filter rows).
         // Measured on B200 (tools/trace_tc2.py, WINRS_TC2_TRACE): a 16-deep stage
         // takes ~820 cycles at NK = 128 and ~600 at NK = 64 -- the shared-memory
         // port (~128 B/clk: 8 MMAs' operand reads + TMA fill + FT traffic,
         // DESIGN.md §6.4); fixed = setup + pipeline fill + epilogue.
-        if (bn >= 128) return {4.5e-6, 5.0e12};
+        if (bn >= 128) return {4.5e-6, 5.5e12};
         return {4.0e-6, 3.4e12};
     }
     if (dtype != 0) {
@@ -266,6 +269,7 @@ static SharedModel shared_model(int dtype) {
 static long long cluster_slots(int cs, int occ, int num_sms, const SharedModel& sm) {
     const double f = (double)num_sms / 148.0;
     long long s;
+    if (cs > 8) return std::max(1LL, (long long)(occ * 8 * f));   // 16-CTA clusters: one per GPC
     if (cs == 1) s = (long long)occ * num_sms;
     else if (cs == 2) s = (long long)occ * num_sms / 2;
     else if (cs == 4) s = (long long)(occ * sm.slots4 * f);
@@ -284,7 +288,7 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
     const double t0 = g.a0 * per_chunk, t1 = (g.a1 ? g.a1 : 1) * per_chunk;
     const long long mult = (long long)g.kblocks * g.cblocks * g.ftiles;
     const int jobs_res = g.a1 ? g.n0 / g.n1 : 0;
-    const long long slots = cluster_slots(g.csplit, e.occ, num_sms, sh);
+    const long long slots = cluster_slots(g.csplit * g.cg, e.occ, num_sms, sh) ;
     // min-heap of slot free times (list scheduling in launch order: band, col, fh outer; kb fastest)
     std::vector<double> heap((size_t)slots, 0.0);
     auto push_root = [&](double v) {   // replace the minimum (root) by v and sift down
@@ -387,6 +391,7 @@ static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairC
         const long long mc = min_tile_chunks(g);
         for (int cs : {1, 2, 3, 4, 6, 8}) {
             if (cs > 1 && !e.csplit_ok) continue;   // never launch a cluster the kernel cannot reduce (even if forced)
+            if (e.cg == 2 && cs > 4) continue;   // 16-CTA clusters (pairs x 8): ~half the clusters co-resident (measured 2x slower)
             if (fcs ? cs != fcs : (cs > 1 && mc < cs)) continue;
             g.csplit = cs;
             const double t = model_time(g, e, num_sms);
@@ -447,6 +452,9 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
             if (e->fhs > 0 && p.N % 16 != 0) continue;   // tc2: one 16-image TMA box per stage and atom
             if (const char* v = getenv("WINRS_TC_GEN")) {   // debug: restrict to one tensor-core generation
                 if (e->dtype != 0 && ((atoi(v) == 2) != (e->fhs > 0))) continue;
+            }
+            if (const char* v = getenv("WINRS_FORCE_CG")) {  // debug: tc2 CTA pair (2) or single CTA (1)
+                if (e->fhs > 0 && atoi(v) != (e->cg > 0 ? e->cg : 1)) continue;
             }
             PlanResult r;
             const double t = plan_with_tile(p, *e, cand, num_sms, &r);

@@ -22,8 +22,9 @@ struct KernelEntry {
     size_t smem;               // dynamic shared memory bytes
     LaunchFn launch;
     const char* name;
-    int fhs;                   // filter rows per CTA (fh group; 0 = 1: one row); > 0 marks the
+    int fhs;                   // filter rows per tile (fh group; 0 = 1: one row); > 0 marks the
                                // second-generation tcgen05 kernels (bfc_tc2.cuh), which need N % 16 == 0
+    int cg;                    // CTAs per UMMA: 2 = cta_group::2 pair (0 = 1)
 };
 
 // All entries (FP32 and FP16), terminated by count.

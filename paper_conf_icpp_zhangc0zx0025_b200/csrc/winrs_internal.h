@@ -55,7 +55,8 @@ struct Geometry {
     int kblocks, cblocks, ftiles;   // ceil(K/B_N), ceil(C/B_M), S/n0
     int fhs, fhg;               // filter rows per CTA (fh group size) and groups ceil(R / fhs)
     int Z;                      // buckets
-    int csplit;                 // CTAs per tile (thread-block cluster size), >= 1
+    int csplit;                 // depth-split ranks per tile (thread-block cluster), >= 1
+    int cg;                     // CTAs per UMMA (2: a cta_group::2 pair per depth rank), >= 1
     int chunk;                  // depth entries per main-loop chunk (8 FP32, 16 FP16)
     long long dw_elems;         // K*R*S*C
 };
@@ -79,7 +80,7 @@ WINRS_HD CtaCoord decode_cta(const Geometry& g, long long bid) {
 WINRS_HD long long num_tiles(const Geometry& g) {
     return (long long)g.kblocks * g.cblocks * g.ftiles * g.fhg * g.seg_cols * g.bands;
 }
-WINRS_HD long long num_ctas(const Geometry& g) { return num_tiles(g) * g.csplit; }
+WINRS_HD long long num_ctas(const Geometry& g) { return num_tiles(g) * g.csplit * (g.cg > 1 ? g.cg : 1); }
 
 // Chunk range [lo, hi) of cluster rank `rank` out of `nchunks` chunks.
 WINRS_HD void split_chunks(int nchunks, int rank, int csplit, int* lo, int* hi) {

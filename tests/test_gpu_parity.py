@@ -33,7 +33,7 @@ def _run(layer, X, dY, env=None, monkeypatch=None):
     p = W.plan(layer.N, layer.C, layer.H, layer.W, layer.K, layer.R, layer.S, layer.pad, layer.dtype)
     Xg = _dev(X, layer.dtype)
     Gg = _dev(dY, layer.dtype)
-    dW = W.bfc(p, Xg, Gg)
+    dW = W.as_krsc(W.bfc(p, Xg, Gg))
     torch.cuda.synchronize()
     return p, dW.cpu().numpy().astype(np.float64)
 

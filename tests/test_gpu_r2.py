@@ -21,7 +21,7 @@ from conftest import record_err
 pytestmark = pytest.mark.gpu
 
 TOL = {"f32": 1e-4, "f16": 2e-2, "bf16": 2e-2}
-ENV_KEYS = ("WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_TC_GEN")
+ENV_KEYS = ("WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_TC_GEN", "WINRS_FORCE_CG")
 
 
 def _dev(a, dtype):
@@ -43,7 +43,7 @@ def _check(layer, monkeypatch, env=None, dist="u01", X=None, dY=None, exact=Fals
     p = _plan(layer, env, monkeypatch)
     if expect_kernel:
         assert expect_kernel in p.kernel_name, (p.kernel_name, expect_kernel)
-    dW = W.bfc(p, _dev(X, layer.dtype), _dev(dY, layer.dtype))
+    dW = W.as_krsc(W.bfc(p, _dev(X, layer.dtype), _dev(dY, layer.dtype)))
     torch.cuda.synchronize()
     got = dW.cpu().numpy().astype(np.float64)
     ref = O.bfc_c(X, dY, layer.R, layer.S, layer.pad)
@@ -84,13 +84,13 @@ TC2 = [
 @pytest.mark.parametrize("name,ov,env", TC2, ids=[c[0] for c in TC2])
 def test_tc2(name, ov, env, dtype, monkeypatch):
     layer = BASE.with_(name="tc2_" + name, dtype=dtype, **ov)
-    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2"), expect_kernel="_v2_")
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2"), expect_kernel="_v2")
 
 
 @pytest.mark.parametrize("name,ov,env", TC2[:8], ids=[c[0] for c in TC2[:8]])
 def test_tc2_signed(name, ov, env, monkeypatch):
     layer = BASE.with_(name="tc2s_" + name, **ov)
-    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2"), dist="signed", expect_kernel="_v2_")
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2"), dist="signed", expect_kernel="_v2")
 
 
 def test_tc2_default_plans_use_tc2(monkeypatch):
@@ -98,7 +98,7 @@ def test_tc2_default_plans_use_tc2(monkeypatch):
     second-generation kernel (the bench's headline path)."""
     for l in wl.RESNET50_F16 + wl.VGG16_F16:
         p = _plan(l, {}, monkeypatch)
-        assert "_v2_" in p.kernel_name, (l.name, p.kernel_name)
+        assert "_v2" in p.kernel_name, (l.name, p.kernel_name)
 
 
 # ====================================================== pad = 0 (SURVEY §8(d): pad=0 variants of the wide config)
@@ -219,6 +219,6 @@ def test_repeated_calls_bitwise(layer_name, env, monkeypatch):
     assert bad == 0, (p.kernel_name, bad)
     idx = wl.sample_indices(layer, 128)
     ref = O.bfc_c_sampled(X, dY, layer.R, layer.S, layer.pad, idx)
-    err = O.rel_max_err(first.cpu().numpy().astype(np.float64).ravel()[idx], ref)
+    err = O.rel_max_err(W.as_krsc(first).cpu().numpy().astype(np.float64).ravel()[idx], ref)
     record_err(f"{layer_name} 400 cold-L2 calls bitwise equal {env}", err, p.kernel_name)
     assert err <= TOL[layer.dtype]

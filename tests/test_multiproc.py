@@ -93,7 +93,7 @@ def _worker_gpu(rank, world, port, q):
                              l.R, l.S, l.pad, l.dtype)
     torch.cuda.synchronize()
     if rank == 0:
-        q.put(dW.cpu().numpy())
+        q.put(W.as_krsc(dW).cpu().numpy())
     dist.barrier()
     dist.destroy_process_group()
 

@@ -22,6 +22,12 @@ METRICS = [
     ("lts__t_bytes.sum", "L2 bytes"),
     ("l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum", "smem bank confl."),
     ("smsp__inst_executed.sum", "warp inst"),
+    ("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed", "smem LSU wavefronts %"),
+    ("l1tex__data_pipe_tc_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed", "smem tensor-core wavefronts %"),
+    ("l1tex__m_xbar2l1tex_read_bytes.sum.pct_of_peak_sustained_elapsed", "xbar->L1 (TMA fill) %"),
+    ("lts__t_sectors.avg.pct_of_peak_sustained_elapsed", "L2 sectors %"),
+    ("sm__cycles_active.avg", "SM active cycles"),
+    ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue active %"),
     ("smsp__average_warps_issue_stalled_wait_per_issue_active.ratio", "stall wait"),
     ("smsp__average_warps_issue_stalled_short_scoreboard_per_issue_active.ratio", "stall short_sb"),
     ("smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio", "stall long_sb"),

@@ -29,7 +29,7 @@ for l in cases:
         except Exception as e:   # a forced pair that does not apply to this shape
             print(l.name, env, "skipped:", e, flush=True)
             continue
-        dW = W.bfc(p, torch.from_numpy(X).cuda(), torch.from_numpy(dY).cuda())
+        dW = W.as_krsc(W.bfc(p, torch.from_numpy(X).cuda(), torch.from_numpy(dY).cuda()))
         torch.cuda.synchronize()
         err = O.rel_max_err(dW.cpu().numpy(), O.bfc_c(X, dY, l.R, l.S, l.pad))
         print(l.name, env, p, "err %.2e" % err, flush=True)

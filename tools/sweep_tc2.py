@@ -16,7 +16,8 @@ sys.path.insert(0, ROOT)
 import paper_conf_icpp_zhangc0zx0025_b200 as W  # noqa: E402
 from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl  # noqa: E402
 
-TILES = ["128x128", "64x128", "128x64", "64x64"]   # NK x (128 / fhs)
+# (tile NK x bm, CTAs per UMMA): single CTA NK x (128 / F), or a cta_group::2 pair
+TILES = [("128x128", 1), ("64x128", 1), ("128x64", 1), ("64x64", 1), ("128x256", 2), ("128x64", 2)]
 
 
 def time_plan(p, Xg, Gg, flush, reps=10):
@@ -47,18 +48,19 @@ def main():
         data = l.N * (l.H * l.W * l.C + (l.H + 2 * l.pad - l.R + 1) * (l.W + 2 * l.pad - l.S + 1) * l.K) * 2
         cfgs = [("auto", None, None, None), ("gen1", None, None, None), ("gen2", None, None, None)]
         if not quick:
-            zs = [1, 2, 3, 4, 6, 8, 12, 16, 24, 32]
+            zs = [1, 2, 4, 7, 8, 14, 16, 28, 56]
             cfgs += [("f", t, cs, z) for t in TILES for cs in (1, 2, 3, 4, 6, 8) for z in zs]
         seen = set()
         for kind, t, cs, z in cfgs:
-            for k in ("WINRS_FORCE_Z", "WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_TC_GEN"):
+            for k in ("WINRS_FORCE_Z", "WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_TC_GEN", "WINRS_FORCE_CG"):
                 os.environ.pop(k, None)
             if kind == "gen1":
                 os.environ["WINRS_TC_GEN"] = "1"
             elif kind != "auto":
                 os.environ["WINRS_TC_GEN"] = "2"
             if kind == "f":
-                os.environ.update({"WINRS_FORCE_TILE": t, "WINRS_FORCE_CSPLIT": str(cs), "WINRS_FORCE_Z": str(z)})
+                os.environ.update({"WINRS_FORCE_TILE": t[0], "WINRS_FORCE_CG": str(t[1]), "WINRS_FORCE_CSPLIT": str(cs),
+                                   "WINRS_FORCE_Z": str(z)})
             try:
                 p = W.plan(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype)
             except Exception:
@@ -69,7 +71,7 @@ def main():
             seen.add(key)
             us = time_plan(p, Xg, Gg, flush)
             flops = p.info["direct_flops"]
-            print(json.dumps({"layer": name, "kind": kind, "tile": t, "cs": p.info["csplit"], "Z": p.info["Z"],
+            print(json.dumps({"layer": name, "kind": kind, "tile": t and list(t), "cs": p.info["csplit"], "Z": p.info["Z"],
                               "kernel": p.kernel_name, "ctas": p.info["ctas_main"], "model_us": round(p.model_us, 1),
                               "us": round(us, 2), "tflops": round(flops / us / 1e6, 1)}), flush=True)
 

@@ -33,6 +33,12 @@ CASES = [
     ("r5_f2", dict(N=16, C=64, K=128, H=16, W=16, R=5, S=3, pad=2), {"WINRS_FORCE_TILE": "128x64"}),
     ("n32_z5", dict(N=32, C=64, K=64, H=30, W=30), {"WINRS_FORCE_Z": "5"}),
     ("n48_cs8", dict(N=48, C=128, K=64, H=12, W=12), {"WINRS_FORCE_CSPLIT": "8"}),
+    ("pair_l3", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_CSPLIT": "1"}),
+    ("pair_l3_cs4", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_CSPLIT": "4"}),
+    ("pair_f1_ragged", dict(N=16, C=200, K=136, H=12, W=13), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_TILE": "128x256"}),
+    ("pair_f2", dict(N=16, C=64, K=128, H=20, W=20), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_TILE": "128x64"}),
+    ("pair_f2_cs2_r5", dict(N=32, C=128, K=128, H=12, W=12, R=5, S=3, pad=2), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "2"}),
+    ("pair_cs8", dict(N=16, C=256, K=128, H=12, W=12), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_CSPLIT": "8"}),
 ]
 
 
@@ -45,7 +51,7 @@ def main():
         if sel and name not in sel:
             continue
         for dt in ("f16", "bf16"):
-            for k in ("WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR"):
+            for k in ("WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_FORCE_CG"):
                 os.environ.pop(k, None)
             os.environ.update(env)
             layer = BASE.with_(name=name, dtype=dt, **ov)
@@ -53,7 +59,7 @@ def main():
             p = W.plan(layer.N, layer.C, layer.H, layer.W, layer.K, layer.R, layer.S, layer.pad, dt)
             to = (lambda a: torch.from_numpy(a).cuda().to(torch.bfloat16)) if dt == "bf16" else (lambda a: torch.from_numpy(a).cuda())
             t0 = time.time()
-            dW = W.bfc(p, to(X), to(dY))
+            dW = W.as_krsc(W.bfc(p, to(X), to(dY)))
             torch.cuda.synchronize()
             got = dW.cpu().numpy().astype(np.float64)
             ref = O.bfc_c(X, dY, layer.R, layer.S, layer.pad)
