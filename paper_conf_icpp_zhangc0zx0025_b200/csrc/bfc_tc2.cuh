@@ -269,6 +269,20 @@ __device__ int g_tc2_trace_cta;
 #define TC2_TRACE(ch, ev) do { } while (0)
 #endif
 
+#ifdef WINRS_TC2_JITTER
+// Debug build: pseudo-random sleeps in every role, every stage, so the ring
+// protocol is exercised under arbitrary relative warp timing (stress test:
+// results must stay bitwise identical to an undisturbed run).
+__device__ __forceinline__ void jitter(int ch, int who) {
+    uint32_t x = (uint32_t)ch * 2654435761u ^ (uint32_t)who * 40503u ^ (uint32_t)blockIdx.x * 97u;
+    x ^= x >> 13; x *= 0x5bd1e995u; x ^= x >> 15;
+    if ((x & 3) == 0) __nanosleep(64 + (x >> 20) % 2048);
+}
+#define TC2_JITTER(ch, who) jitter((ch), (who))
+#else
+#define TC2_JITTER(ch, who) do { } while (0)
+#endif
+
 // Depth entry d of a CTA -> (n, h, u): n fastest (d = ((h - hs) * units + u) * N + n).
 __device__ __forceinline__ void depth_nhu(int d, int N, int units, int hs, int* n, int* h, int* u) {
     *n = d % N;
@@ -365,6 +379,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         uint32_t ph = 0;
         for (int ch = c_lo; ch < c_hi; ++ch) {
             mbar_wait(&bars->empty[s], ph ^ 1);
+            TC2_JITTER(ch, 0);
             TC2_TRACE(ch - c_lo, 0);
             uint64_t* fb = &bars->full[s];
             const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
@@ -410,6 +425,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         uint32_t ph = 0;
         for (int ch = c_lo; ch < c_hi; ++ch) {
             mbar_wait(&bars->opfull[s], ph);
+            TC2_JITTER(ch, 1);
             TC2_TRACE(ch - c_lo, 4);
             tc_after();
             const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
@@ -469,6 +485,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             const int s = tw;
             mbar_wait(&bars->full[s], ph);
             ph ^= 1;
+            TC2_JITTER(ch, warp);
             if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
             const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
             if (!WINRS_TC2_ITM) {

@@ -14,13 +14,20 @@ cases = [
     wl.LAYERS["r50_c64_56_f16"].with_(N=3, H=9, W=20, C=8, K=8),
     # Omega_4(3,2) paired / round-robin units, 128x128 tile, ragged K and C
     wl.LAYERS["r50_c256_14_f16"].with_(N=2, H=14, W=14, C=136, K=200),
+    # bfc_tc2.cuh (N % 16 == 0): stacked fh (F = 2), NK 64 / 128, a cta_group::2 pair
+    wl.LAYERS["r50_c64_56_f16"].with_(N=16, H=10, W=11),
+    wl.LAYERS["r50_c256_14_f16"].with_(N=16, H=7, W=7, C=256, K=128),
+    wl.LAYERS["r50_c256_14_f16"].with_(N=16, H=6, W=9, C=200, K=136, dtype="bf16"),
 ]
-envs = [{}, {"WINRS_FORCE_CSPLIT": "2"}, {"WINRS_FORCE_Z": "3"}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_CSPLIT": "4"}]
+envs = [{}, {"WINRS_FORCE_CSPLIT": "2"}, {"WINRS_FORCE_Z": "3"}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_CSPLIT": "4"},
+        {"WINRS_FORCE_CG": "2", "WINRS_FORCE_CSPLIT": "2"}]
 for l in cases:
     for env in envs:
-        for k in ("WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR"):
+        for k in ("WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_FORCE_CG"):
             os.environ.pop(k, None)
         if "WINRS_FORCE_PAIR" in env and l.dtype != "f16":
+            continue
+        if "WINRS_FORCE_CG" in env and l.N % 16:
             continue
         os.environ.update(env)
         X, dY = wl.make_inputs(l)
@@ -29,7 +36,8 @@ for l in cases:
         except Exception as e:   # a forced pair that does not apply to this shape
             print(l.name, env, "skipped:", e, flush=True)
             continue
-        dW = W.as_krsc(W.bfc(p, torch.from_numpy(X).cuda(), torch.from_numpy(dY).cuda()))
+        to = (lambda a: torch.from_numpy(a).cuda().to(torch.bfloat16)) if l.dtype == "bf16" else (lambda a: torch.from_numpy(a).cuda())
+        dW = W.as_krsc(W.bfc(p, to(X), to(dY)))
         torch.cuda.synchronize()
         err = O.rel_max_err(dW.cpu().numpy(), O.bfc_c(X, dY, l.R, l.S, l.pad))
         print(l.name, env, p, "err %.2e" % err, flush=True)
