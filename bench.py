@@ -208,7 +208,12 @@ def layer_roofline(l, p, ms, peaks):
     bn, bm = info["tile_k0"], info["tile_c0"]
     kb, cb = -(-l.K // bn), -(-l.C // bm)
     ft = l.S // n0
-    if "_v2" in name:
+    if "_v2s_" in name:                                   # swapped CTA pair: 256 k x 128 c, 1 filter row
+        rows = sum(_rows_valid(l, fh) for fh in range(l.R))
+        depth = rows * units * l.N * kb * cb * ft
+        l2_bytes = depth / 16 * 2 * (8192 + 8192)         # per pair stage: each CTA X 8 KB + dY 8 KB
+        alu_ops = depth * (256 + 128 * 2)                 # FT over 256 k, IT over 128 c (half2)
+    elif "_v2" in name:
         cg = int(name.split("_v2")[1][0])                 # CTAs per UMMA (2: cta_group::2 pair)
         fhs = int(name.split("x")[-1].rstrip("fh")) * cg if bm == 64 else 1
         rows = sum(_rows_union(l, range(g, min(l.R, g + fhs))) for g in range(0, l.R, fhs))

@@ -84,6 +84,41 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
     return launch_cluster(k, (unsigned)grid, (unsigned)NTHREADS, (size_t)L::BYTES, stream, cluster, a, mX, mY);
 }
 
+// The swapped CTA pair (bfc_tc2s_kernel): tile = 256 k x 128 c x 1 filter row.
+template <bool BF>
+cudaError_t launch_sw(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
+    using L = LaySw;
+    const long long grid = num_ctas(g);
+    if (grid <= 0) return cudaSuccess;
+    Args a;
+    a.g = g;
+    a.dW = dW;
+    a.ws = ws;
+    a.nb = images_per_box(g.N);
+    if (a.nb == 0 || g.a0 != 4 || g.n0 != 3 || g.r0 != 2 || g.a1 != 0 || g.cg != 2 || g.fhs != 1)
+        return cudaErrorInvalidValue;
+    CUtensorMap mX, mY;
+    if (!make_map(&mX, X, g.N, g.H, g.W, g.C, g.C, 4, a.nb, BF) ||
+        !make_map(&mY, dY, g.N, g.Ho, g.Wo, g.K, g.ldy, 2, a.nb, BF))
+        return cudaErrorInvalidValue;
+    static std::atomic<unsigned long long> done{0};
+    auto k = bfc_tc2s_kernel<BF>;
+    cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
+    if (e != cudaSuccess) return e;
+    const int cluster = 2 * g.csplit;
+    if (cluster > 8) {
+        static std::atomic<unsigned long long> np{0};
+        int dev = 0;
+        cudaGetDevice(&dev);
+        if (!(np.load() & (1ull << (dev & 63)))) {
+            e = cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+            if (e != cudaSuccess) return e;
+            np.fetch_or(1ull << (dev & 63));
+        }
+    }
+    return launch_cluster(k, (unsigned)grid, (unsigned)NTHREADS, (size_t)L::BYTES, stream, cluster, a, mX, mY);
+}
+
 }  // namespace tc2
 
 // tile = NK k columns x (128 / F) c rows x F filter rows (one CTA), or for a
@@ -116,6 +151,11 @@ const KernelEntry* tc2_entries(int* n) {
         WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 64, 1),
         WINRS_TC2_ENTRY(2, true, "bf16tc", 1, 128, 2),
         WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 128, 2),
+        // swapped CTA pair: 256 k x 128 c (What rows split, the Xhat side shared)
+        {1, 4, 3, 2, 0, 0, 0, 256, 128, ::winrs::tc2::NTHREADS, 1, 1, (size_t)::winrs::tc2::LaySw::BYTES,
+         &::winrs::tc2::launch_sw<false>, "f16tc_O4(3,2)_v2s_256x128", 1, 2},
+        {2, 4, 3, 2, 0, 0, 0, 256, 128, ::winrs::tc2::NTHREADS, 1, 1, (size_t)::winrs::tc2::LaySw::BYTES,
+         &::winrs::tc2::launch_sw<true>, "bf16tc_O4(3,2)_v2s_256x128", 1, 2},
     };
     *n = sizeof(e) / sizeof(e[0]);
     return e;

@@ -617,5 +617,287 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     }
 }
 
+
+// ============================================================================
+// Swapped CTA pair ("v2s"): the same computation with the operand roles
+// exchanged.  M = 256 What rows (k: 128 per CTA), N = 128 Xhat columns
+// (c: 64 per CTA), cta_group::2.  In a pair the B operand is shared, so each
+// SM now fetches and transforms only HALF of the X side -- the expensive side
+// (4 window columns and the 4-output IT per channel against 2 columns and 2
+// computed outputs for What): per SM and 16-deep stage 16 KB of TMA fill, 16 KB
+// of IT and 16 KB of FT traffic instead of 24 + 32 + 16 KB for one CTA
+// (§6.4: the shared-memory port bounds the stage).  For K >= 256 tiles
+// (ResNet-50 L3 / L4, VGG-16 conv3-5).
+struct LaySw {
+    static constexpr int ATOM = KC * 128;                // 2 KB: 64 channels x 16 depth rows
+    static constexpr int OFF_X = 0;                      // X columns x0..x3 of this CTA's 64 c: [col][n]
+    static constexpr int OFF_Y = 4 * ATOM;               // raw dY columns: [k atom 0/1][w0, w1][n]
+    static constexpr int Y_LBO = 2 * ATOM;               // 4 KB between the two k atoms
+    static constexpr int OFF_F = OFF_Y + 2 * Y_LBO;      // What[0], What[1]: same shape
+    static constexpr int STAGE = OFF_F + 2 * Y_LBO;      // 24 KB
+    static constexpr int S = 8;
+    static constexpr int RING = S * STAGE;               // 192 KB
+    static constexpr int OUT_LD = 128 + 4;               // staging row stride (floats): float4 stores of 8
+                                                         // lanes on consecutive k rows hit distinct banks
+    static constexpr int OUT = NSOUT * 128 * OUT_LD * 4;  // staging [s][k 128][c 128 (+4)] fp32, 198 KB
+    static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
+    static constexpr int BYTES = BAR_OFF + 256 + 1024;
+    static constexpr int TX_BYTES = OFF_F;               // 16 KB per stage
+    static constexpr int TMEM_COLS = 512;                // 4 xi x N = 128
+    static_assert(BYTES <= 227 * 1024, "smem");
+};
+
+template <bool BF>
+__global__ void __launch_bounds__(NTHREADS, 1)
+bfc_tc2s_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX,
+                const __grid_constant__ CUtensorMap tmY) {
+    using L = LaySw;
+    constexpr int NN = 128;                              // UMMA N (c per pair)
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t raw_s = su(smem_raw);
+    uint8_t* smem = smem_raw + (((raw_s + 1023u) & ~1023u) - raw_s);
+    const uint32_t sbase = su(smem);
+    Bars* bars = reinterpret_cast<Bars*>(smem + L::BAR_OFF);
+    const Geometry& g = args.g;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 64) TC2_TRACE(511, 0);
+
+    const int crank = (int)cluster_rank();
+    const int e = crank & 1;
+    const int rank = crank >> 1;                         // depth-split rank
+    const uint32_t leader = (uint32_t)(crank & ~1);
+    const uint16_t pair_mask = (uint16_t)(3u << leader);
+    const CtaCoord cc = decode_cta(g, blockIdx.x / (2 * g.csplit));
+    const int k_base = cc.kb * 256 + e * 128;            // this CTA's What rows (TMEM lanes)
+    const int c_base = cc.cb * 128 + e * 64;             // this CTA's half of the Xhat columns
+    const int fh = cc.fh;
+    const int seg = cc.band * g.seg_cols + cc.col;
+    float* bucket = seg == 0 ? args.dW : args.ws + (long long)(seg - 1) * g.dw_elems;
+    int hs, he, w_first, units;
+    group_rows(g, cc.band, cc.fh, &hs, &he);
+    seg_units(g, cc.col, &w_first, &units);
+    const long long depth = (long long)(he > hs ? he - hs : 0) * units * g.N;
+    int c_lo, c_hi;
+    split_chunks((int)((depth + KC - 1) / KC), rank, g.csplit, &c_lo, &c_hi);
+    const bool empty_range = c_hi <= c_lo;
+    const int fw0 = cc.ft * NSOUT;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < L::S; ++s) {
+            mbar_init(&bars->full[s], 1);
+            mbar_init(&bars->opfull[s], e == 0 ? 2 : 1);   // the leader gathers both CTAs' FT warps
+            mbar_init(&bars->empty[s], 1);
+        }
+        mbar_init(&bars->accfull, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 0 && lane == 0) {
+        asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
+        asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
+    }
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;"
+                     :: "r"(su(&bars->tmem_base)), "r"(L::TMEM_COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+    }
+    tc_before();
+    __syncthreads();
+    cluster_sync_all();
+    tc_after();
+    const uint32_t tmem = bars->tmem_base;
+    if (threadIdx.x == 64) TC2_TRACE(511, 1);
+
+    if (warp == 0) {
+        // ---- TMA: X columns x0..x3 of this CTA's 64 channels; dY w0, w1 of its 128 k
+        long long d = (long long)c_lo * KC;
+        int n = 0, h = hs, u = 0;
+        if (d < depth) depth_nhu((int)d, g.N, units, hs, &n, &h, &u);
+        int s = 0;
+        uint32_t ph = 0;
+        for (int ch = c_lo; ch < c_hi; ++ch) {
+            mbar_wait(&bars->empty[s], ph ^ 1);
+            TC2_JITTER(ch, 0);
+            TC2_TRACE(ch - c_lo, 0);
+            uint64_t* fb = &bars->full[s];
+            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            const bool in = d < depth;
+            const int nn = in ? n : g.N, hh = in ? h : hs;
+            const int w0 = w_first + (in ? u : 0) * 2;
+            if (elect_one()) {
+                mbar_expect_tx(fb, (uint32_t)L::TX_BYTES);
+                tma4(st + L::OFF_X, &tmX, fb, c_base, nn, hh + fh - g.pad, w0 + fw0 - g.pad);
+                tma4(st + L::OFF_Y, &tmY, fb, k_base, nn, hh, w0);
+                tma4(st + L::OFF_Y + L::Y_LBO, &tmY, fb, k_base + 64, nn, hh, w0);
+            }
+            __syncwarp();
+            TC2_TRACE(ch - c_lo, 1);
+            d += KC;
+            n += KC;
+            while (n >= g.N) {
+                n -= g.N;
+                if (++u == units) { u = 0; ++h; }
+            }
+            if (++s == L::S) { s = 0; ph ^= 1; }
+        }
+    } else if (warp == 1) {
+        // ---- MMA (the pair's leader): D[xi] (256 k x 128 c) += What[xi] . Xhat[xi]
+        if (e == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            for (int ch = c_lo; ch < c_hi; ++ch) {
+                mbar_wait(&bars->opfull[s], ph);
+                TC2_JITTER(ch, 1);
+                TC2_TRACE(ch - c_lo, 4);
+                tc_after();
+                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+                const uint32_t acc = ch > c_lo ? 1u : 0u;
+                const uint64_t a0 = desc_sw128(st + L::OFF_F, L::Y_LBO, 1024), a1 = a0 + (L::ATOM >> 4);
+                const uint64_t a2 = desc_sw128(st + L::OFF_Y, L::Y_LBO, 1024), a3 = a2 + (L::ATOM >> 4);
+                const uint64_t b0 = desc_sw128(st + L::OFF_X, 8 * 1024, 1024);
+                if (elect_one()) {
+#ifndef WINRS_TC2_NO_MMA
+                    umma<NN, BF, false, 2>(tmem + 0 * NN, a0, b0, acc);
+                    umma<NN, BF, false, 2>(tmem + 1 * NN, a1, b0 + (L::ATOM >> 4), acc);
+                    umma<NN, BF, false, 2>(tmem + 2 * NN, a2, b0 + (2 * L::ATOM >> 4), acc);
+                    umma<NN, BF, false, 2>(tmem + 3 * NN, a3, b0 + (3 * L::ATOM >> 4), acc);
+#else
+                    (void)a0; (void)a1; (void)a2; (void)a3; (void)b0; (void)acc;
+#endif
+                    umma_commit<2>(&bars->empty[s], pair_mask);
+                }
+                __syncwarp();
+                TC2_TRACE(ch - c_lo, 5);
+                if (++s == L::S) { s = 0; ph ^= 1; }
+            }
+            if (elect_one()) umma_commit<2>(&bars->accfull, pair_mask);
+            __syncwarp();
+        }
+    } else {
+        // ---- FT warp w owns ring slot w: IT in place over its 64 c (4 items/lane),
+        // FT What[0,1] = w0 +- w1 over its 128 k (8 items/lane)
+        const int tw = warp - 2;
+        uint32_t ph = 0;
+        for (int ch = c_lo + tw; ch < c_hi; ch += L::S) {
+            const int s = tw;
+            mbar_wait(&bars->full[s], ph);
+            ph ^= 1;
+            TC2_JITTER(ch, warp);
+            if (lane == 0) TC2_TRACE(ch - c_lo, 2);
+            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            {
+                uint4 xv[4][4];
+                uint32_t xo[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const int t = i * 32 + lane;                // depth t / 8, c octet t % 8
+                    xo[i] = st + L::OFF_X + opoff(t & 7, t >> 3, 0);
+#pragma unroll
+                    for (int c = 0; c < 4; ++c) xv[i][c] = lds16(xo[i] + c * L::ATOM);
+                }
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    sts16(xo[i], vadd<BF>(xv[i][1], xv[i][2]));
+                    sts16(xo[i] + L::ATOM, vsub<BF>(xv[i][2], xv[i][1]));
+                    sts16(xo[i] + 2 * L::ATOM, vsub<BF>(xv[i][0], xv[i][2]));
+                    sts16(xo[i] + 3 * L::ATOM, vsub<BF>(xv[i][3], xv[i][1]));
+                }
+            }
+            {
+                uint4 w0[8], w1[8];
+                uint32_t off[8];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const int t = i * 32 + lane;                // depth t / 16, k octet t % 16
+                    off[i] = opoff(t & 15, t >> 4, L::Y_LBO);
+                    w0[i] = lds16(st + L::OFF_Y + off[i]);
+                    w1[i] = lds16(st + L::OFF_Y + L::ATOM + off[i]);
+                }
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    sts16(st + L::OFF_F + off[i], vadd<BF>(w0[i], w1[i]));
+                    sts16(st + L::OFF_F + L::ATOM + off[i], vsub<BF>(w0[i], w1[i]));
+                }
+            }
+            fence_async();
+            __syncwarp();
+            if (lane == 0) mbar_arrive_cluster(&bars->opfull[s], leader);
+            if (lane == 0) TC2_TRACE(ch - c_lo, 3);
+        }
+        // ---- epilogue: TMEM lane = k, columns = xi * 128 + c (c of the whole pair)
+        mbar_wait(&bars->accfull, 0);
+        tc_after();
+        if (threadIdx.x == 64) TC2_TRACE(511, 2);
+        const int q = warp & 3;
+        const int half = (warp - 2) >> 2;                // c half of the 128 columns
+        const int kl = q * 32 + lane;                    // local k row
+        const int k = k_base + kl;
+        float* Out = reinterpret_cast<float*>(smem);      // staging [s][kl][c 128 (+4)]
+        const uint32_t lane_base = tmem + ((uint32_t)(q * 32) << 16);
+#pragma unroll 1
+        for (int cl0 = half * 64; cl0 < half * 64 + 64; cl0 += 8) {
+            float v[4][8];
+            if (!empty_range) {
+#pragma unroll
+                for (int x = 0; x < 4; ++x) tmem_ld8(lane_base + (uint32_t)(x * NN + cl0), v[x]);
+                tmem_wait_ld();
+            } else {
+#pragma unroll
+                for (int x = 0; x < 4; ++x)
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) v[x][i] = 0.f;
+            }
+            float y[3][8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const float sp = 0.5f * (v[0][i] + v[1][i]);
+                y[0][i] = sp + v[2][i];
+                y[1][i] = 0.5f * (v[0][i] - v[1][i]);
+                y[2][i] = sp + v[3][i];
+            }
+            // pair column cl -> channel: CTA e' holds c_pair [e' * 64, e' * 64 + 64)
+            const int cg = cc.cb * 128 + cl0;
+#pragma unroll
+            for (int j = 0; j < 3; ++j) {
+                if (g.csplit > 1) {
+                    float4* o = reinterpret_cast<float4*>(Out + (j * 128 + kl) * L::OUT_LD + cl0);
+                    o[0] = make_float4(y[j][0], y[j][1], y[j][2], y[j][3]);
+                    o[1] = make_float4(y[j][4], y[j][5], y[j][6], y[j][7]);
+                } else if (k < g.K && cg < g.C && fh < g.R) {   // C % 8 == 0: octets all in or all out
+                    float4* o = reinterpret_cast<float4*>(bucket + (((long long)k * g.R + fh) * g.S + fw0 + j) * g.C + cg);
+                    o[0] = make_float4(y[j][0], y[j][1], y[j][2], y[j][3]);
+                    o[1] = make_float4(y[j][4], y[j][5], y[j][6], y[j][7]);
+                }
+            }
+        }
+    }
+    tc_before();
+    __syncthreads();
+    if (threadIdx.x == 64) TC2_TRACE(511, 3);
+    if (g.csplit > 1) {
+        // ---- depth-split reduction over the ranks with the same pair half e
+        constexpr int ROWS = NSOUT * 128, C4 = 128 / 4;
+        cluster_sync_all();
+        if (threadIdx.x == 64) TC2_TRACE(511, 4);
+        const int r_lo = ROWS * rank / g.csplit, r_hi = ROWS * (rank + 1) / g.csplit;
+        for (int p = r_lo * C4 + (int)threadIdx.x; p < r_hi * C4; p += NTHREADS) {
+            const int row = p / C4, c4 = p % C4;
+            const int j = row / 128, kl = row % 128;
+            const float4 acc = dsmem_sum4(sbase + (uint32_t)((row * L::OUT_LD + c4 * 4) * 4), g.csplit, 2, e);
+            const int k = k_base + kl, c = cc.cb * 128 + c4 * 4;
+            if (k < g.K && c < g.C && fh < g.R)
+                *reinterpret_cast<float4*>(bucket + (((long long)k * g.R + fh) * g.S + fw0 + j) * g.C + c) = acc;
+        }
+        if (threadIdx.x == 64) TC2_TRACE(511, 5);
+        cluster_sync_all();
+    } else {
+        cluster_sync_all();
+    }
+    if (threadIdx.x == 64) TC2_TRACE(511, 6);
+    if (warp == 1) {
+        tc_after();
+        asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" :: "r"(tmem), "r"(L::TMEM_COLS));
+    }
+}
+
 }  // namespace tc2
 }  // namespace winrs

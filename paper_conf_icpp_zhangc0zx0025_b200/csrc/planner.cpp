@@ -240,6 +240,8 @@ struct SharedModel {
 
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
+    if (e.fhs > 0 && e.cg == 2 && bn == 256)   // swapped CTA pair (256 k x 128 c): X side shared
+        return {4.5e-6, 16.0e12};
     if (e.fhs > 0 && e.cg == 2)   // bfc_tc2.cuh CTA pair: rate of the pair over its 256-row tile
         return {4.5e-6, 11.0e12};
     if (e.fhs > 0) {
@@ -283,8 +285,8 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
     SharedModel sh = shared_model(e.dtype);
     const int fhs = e.fhs > 0 ? e.fhs : 1;
     const double per_chunk = (double)g.chunk * e.bn * e.bm * fhs * 2.0 / m.rate_sm;
-    if (e.fhs > 0)   // rank skew + DSMEM reduction of the n0 x B_N x 128 FP32 output tile (~20 B/clk/SM)
-        sh.cluster_s = 1.5e-6 + (double)g.n0 * e.bn * 128 * 4 / 30e9;
+    if (e.fhs > 0)   // rank skew + DSMEM reduction of the n0 x 128 x 128 (per SM) FP32 output tile (~20 B/clk/SM)
+        sh.cluster_s = 1.5e-6 + (double)g.n0 * (e.bn > 128 ? 128 : e.bn) * 128 * 4 / 30e9;
     const double t0 = g.a0 * per_chunk, t1 = (g.a1 ? g.a1 : 1) * per_chunk;
     const long long mult = (long long)g.kblocks * g.cblocks * g.ftiles;
     const int jobs_res = g.a1 ? g.n0 / g.n1 : 0;

@@ -77,6 +77,15 @@ TC2 = [
     ("r1", dict(N=16, C=64, K=64, H=12, W=12, R=1, S=3, pad=0), {}),
     ("n32_z5", dict(N=32, C=64, K=64, H=30, W=30), {"WINRS_FORCE_Z": "5"}),
     ("n48_cs8", dict(N=48, C=128, K=64, H=12, W=12), {"WINRS_FORCE_CSPLIT": "8"}),
+    # cta_group::2 pairs: What rows split (256 c / 4 filter rows) and the swapped pair (256 k x 128 c)
+    ("pair_l3", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_TILE": "128x256", "WINRS_FORCE_CSPLIT": "1"}),
+    ("pair_f2_cs2_r5", dict(N=32, C=128, K=128, H=12, W=12, R=5, S=3, pad=2),
+     {"WINRS_FORCE_CG": "2", "WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "2"}),
+    ("pair_cs4_ragged", dict(N=16, C=200, K=136, H=12, W=13), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_TILE": "128x256", "WINRS_FORCE_CSPLIT": "4"}),
+    ("swap_l3", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_CSPLIT": "1"}),
+    ("swap_cs4", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_CSPLIT": "4"}),
+    ("swap_ragged", dict(N=16, C=200, K=328, H=12, W=13), {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_CSPLIT": "2"}),
+    ("swap_pad0_s6", dict(N=16, C=128, K=256, H=12, W=14, S=6, pad=0), {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
 ]
 
 
@@ -194,6 +203,7 @@ def test_impulse_fp32_alpha8_tolerance(monkeypatch):
 @pytest.mark.parametrize("layer_name,env", [
     ("r50_c64_56_f16", {}),                                   # tc2, Z > 1, cluster split
     ("r50_c256_14_f16", {}),                                  # tc2, NK = 128, cs = 8
+    ("r50_c512_7_f16", {}),                                   # tc2 swapped cta_group::2 pair, cs = 2
     ("r50_c64_56_f16", {"WINRS_TC_GEN": "1"}),                # round-1 kernel default plan
     ("r50_c128_28_f16", {"WINRS_TC_GEN": "1"}),
 ])

@@ -39,6 +39,11 @@ CASES = [
     ("pair_f2", dict(N=16, C=64, K=128, H=20, W=20), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_TILE": "128x64"}),
     ("pair_f2_cs2_r5", dict(N=32, C=128, K=128, H=12, W=12, R=5, S=3, pad=2), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "2"}),
     ("pair_cs8", dict(N=16, C=256, K=128, H=12, W=12), {"WINRS_FORCE_CG": "2", "WINRS_FORCE_CSPLIT": "8"}),
+    ("swap_l3", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_CSPLIT": "1"}),
+    ("swap_l3_cs4", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_CSPLIT": "4"}),
+    ("swap_ragged", dict(N=16, C=200, K=328, H=12, W=13), {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_CSPLIT": "2"}),
+    ("swap_l4_z", dict(N=32, C=128, K=256, H=7, W=7), {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_CSPLIT": "3"}),
+    ("swap_pad0_s6", dict(N=16, C=128, K=256, H=12, W=14, S=6, pad=0), {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
 ]
 
 
