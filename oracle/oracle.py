@@ -22,9 +22,18 @@ Three independent formulations, all FP64:
                           definition with a library contraction as the step.
 * ``bfc_bruteforce``   — pure-Python loops, tiny shapes only.
 
-Plus ``bfc_c_sampled`` (selected dW elements, for full-size parity).
+Plus ``bfc_c_sampled`` (selected dW elements, for full-size parity), and the
+N-D (3-D) definition of PAPER.md §3's Level-2 dimension reduction (P@17805:
+an N-D BFC reduces to 2-D BFCs over the extra spatial axis)::
 
-Pins (tests/test_oracle.py): brute force == C == numpy; impulse; all-ones
+    Do = D + 2 pad - T + 1
+    dW[k, t, r, s, c] = sum_{n, d, h, w} Xp[n, d+t-pad, h+r-pad, w+s-pad, c] * dY[n, d, h, w, k]
+
+``bfc3d_numpy`` (one tensordot per filter tap) and ``bfc3d_bruteforce``; layouts
+NDHWC / NDHWC / KTRSC (Table 1 extended by the depth axis, R23).
+
+Pins (tests/test_oracle.py): brute force == C == numpy (2-D and 3-D); torch
+conv3d_weight in FP64; the D = 1 reduction of the 3-D definition; impulse; all-ones
 closed form; adjoint identity against an independent forward convolution;
 linearity; dY = 0; the Ho = Wo = 1 GEMM special case; torch.nn.grad
 conv2d_weight in FP64.  No function here is "parity unpinned".
@@ -158,6 +167,61 @@ def bfc_bruteforce(X, dY, R: int, S: int, pad: int) -> np.ndarray:
                                 acc += Xl[n][i][j][c] * Gl[n][h][w][k]
                     out[k][r][s][c] = acc
     return np.array(out, dtype=np.float64)
+
+
+def out_dims3(D, H, W, T, R, S, pad):
+    return D + 2 * pad - T + 1, H + 2 * pad - R + 1, W + 2 * pad - S + 1
+
+
+def bfc3d_numpy(X: np.ndarray, dY: np.ndarray, T: int, R: int, S: int, pad: int) -> np.ndarray:
+    """3-D BFC, the plain definition: zero-pad X on the three spatial axes, then
+    for every filter tap (t, r, s) contract the shifted window with dY over
+    (n, d, h, w).  X: [N,D,H,W,C], dY: [N,Do,Ho,Wo,K] -> dW [K,T,R,S,C] (FP64)."""
+    X = X.astype(np.float64)
+    dY = dY.astype(np.float64)
+    N, D, H, W, C = X.shape
+    _, Do, Ho, Wo, K = dY.shape
+    assert (Do, Ho, Wo) == out_dims3(D, H, W, T, R, S, pad)
+    Xp = np.zeros((N, D + 2 * pad, H + 2 * pad, W + 2 * pad, C), dtype=np.float64)
+    Xp[:, pad:pad + D, pad:pad + H, pad:pad + W, :] = X
+    dW = np.empty((K, T, R, S, C), dtype=np.float64)
+    for t in range(T):
+        for r in range(R):
+            for s in range(S):
+                win = Xp[:, t:t + Do, r:r + Ho, s:s + Wo, :]
+                dW[:, t, r, s, :] = np.tensordot(dY, win, axes=([0, 1, 2, 3], [0, 1, 2, 3]))
+    return dW
+
+
+def bfc3d_bruteforce(X, dY, T: int, R: int, S: int, pad: int) -> np.ndarray:
+    """Pure-Python loops over every index of the 3-D definition (tiny shapes)."""
+    N, D, H, W, C = X.shape
+    _, Do, Ho, Wo, K = dY.shape
+    assert (Do, Ho, Wo) == out_dims3(D, H, W, T, R, S, pad)
+    Xl = np.asarray(X, dtype=np.float64).tolist()
+    Gl = np.asarray(dY, dtype=np.float64).tolist()
+    out = np.zeros((K, T, R, S, C), dtype=np.float64)
+    for k in range(K):
+        for t in range(T):
+            for r in range(R):
+                for s in range(S):
+                    for c in range(C):
+                        acc = 0.0
+                        for n in range(N):
+                            for d in range(Do):
+                                a = d + t - pad
+                                if not 0 <= a < D:
+                                    continue
+                                for h in range(Ho):
+                                    i = h + r - pad
+                                    if not 0 <= i < H:
+                                        continue
+                                    for w in range(Wo):
+                                        j = w + s - pad
+                                        if 0 <= j < W:
+                                            acc += Xl[n][a][i][j][c] * Gl[n][d][h][w][k]
+                        out[k, t, r, s, c] = acc
+    return out
 
 
 def rel_max_err(got: np.ndarray, ref: np.ndarray) -> float:

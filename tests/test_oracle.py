@@ -162,3 +162,58 @@ def test_error_metrics():
 def test_rejects_bad_shapes():
     with pytest.raises(AssertionError):
         O.bfc_c(np.zeros((1, 4, 4, 1)), np.zeros((1, 3, 3, 1)), 3, 3, 1)   # dY should be 4x4
+
+
+# ============================================================== N-D (3-D) definition
+SHAPES3 = [
+    # N, C, D, H, W, K, T, R, S, pad
+    (1, 2, 3, 4, 5, 2, 3, 3, 3, 1),
+    (2, 3, 4, 3, 4, 2, 2, 1, 3, 0),
+    (1, 2, 2, 5, 4, 3, 3, 2, 2, 2),
+]
+
+
+@pytest.mark.parametrize("shape", SHAPES3)
+def test_3d_numpy_bruteforce_torch_agree(shape):
+    """3-D definition: brute force == numpy == torch.nn.grad.conv3d_weight (FP64,
+    a library routine; NCDHW / KCTRS permuted to NDHWC / KTRSC)."""
+    N, C, D, H, W, K, T, R, S, pad = shape
+    Do, Ho, Wo = O.out_dims3(D, H, W, T, R, S, pad)
+    X = _rand((N, D, H, W, C), 11)
+    dY = _rand((N, Do, Ho, Wo, K), 12)
+    bf = O.bfc3d_bruteforce(X, dY, T, R, S, pad)
+    nb = O.bfc3d_numpy(X, dY, T, R, S, pad)
+    ref = torch.nn.grad.conv3d_weight(torch.from_numpy(X).permute(0, 4, 1, 2, 3), (K, C, T, R, S),
+                                      torch.from_numpy(dY).permute(0, 4, 1, 2, 3), padding=pad)
+    ref = ref.permute(0, 2, 3, 4, 1).numpy()
+    assert np.allclose(nb, bf, rtol=1e-13, atol=1e-13)
+    assert np.allclose(nb, ref, rtol=1e-12, atol=1e-12)
+
+
+def test_3d_reduces_to_2d_when_depth_is_one():
+    """Level-2 dimension reduction, special case D = 1, T = 3, pad = 1: Do = 1,
+    the depth taps t = 0, 2 only see padding (zero), and the middle tap is the
+    2-D BFC of the single slice."""
+    N, C, H, W, K, R, S, pad = 2, 3, 6, 5, 4, 3, 3, 1
+    X = _rand((N, 1, H, W, C), 13)
+    Do, Ho, Wo = O.out_dims3(1, H, W, 3, R, S, pad)
+    assert Do == 1
+    dY = _rand((N, 1, Ho, Wo, K), 14)
+    got = O.bfc3d_numpy(X, dY, 3, R, S, pad)
+    assert np.all(got[:, 0] == 0) and np.all(got[:, 2] == 0)
+    assert np.allclose(got[:, 1], O.bfc_c(X[:, 0], dY[:, 0], R, S, pad), rtol=1e-13, atol=1e-13)
+
+
+def test_3d_impulse():
+    """dY = e_{n0,d0,h0,w0,k0} => dW[k0,t,r,s,c] = Xpad[n0, d0+t-pad, h0+r-pad, w0+s-pad, c]."""
+    N, C, D, H, W, K, T, R, S, pad = 2, 3, 4, 5, 5, 2, 3, 3, 3, 1
+    Do, Ho, Wo = O.out_dims3(D, H, W, T, R, S, pad)
+    X = _rand((N, D, H, W, C), 15)
+    dY = np.zeros((N, Do, Ho, Wo, K))
+    n0, d0, h0, w0, k0 = 1, 0, 2, 4, 1
+    dY[n0, d0, h0, w0, k0] = 1.0
+    got = O.bfc3d_numpy(X, dY, T, R, S, pad)
+    Xp = np.zeros((N, D + 2 * pad, H + 2 * pad, W + 2 * pad, C))
+    Xp[:, pad:pad + D, pad:pad + H, pad:pad + W] = X
+    assert np.array_equal(got[k0], Xp[n0, d0:d0 + T, h0:h0 + R, w0:w0 + S, :])
+    assert np.all(got[1 - k0] == 0)
