@@ -97,8 +97,10 @@ typedef struct {
     long long ctas_main, ctas_resid, ctas_reduce;
     int csplit;                    /* CTAs per tile: thread-block cluster depth split   */
     size_t workspace_bytes;        /* (Z-1) * 4 * K*R*S*C, 0 when Z == 1                  */
-    double direct_flops;           /* 2*N*C*K*Ho*Wo*R*S (P@43462)                         */
+    double direct_flops;           /* 2*N*C*K*Ho*Wo*R*S (P@43462) (x D_o*T for N-D)       */
     double ewm_flops;              /* Winograd-domain EWM flops actually issued           */
+    int D, T, Do;                  /* N-D plans (winrs_plan3d): depth of X, of the filter  */
+                                   /* and of dY; 1, 1, 1 for the 2-D plans                */
 } winrs_plan_info_t;
 
 /* Create a plan for the current CUDA device.
@@ -115,6 +117,22 @@ WINRS_API winrs_status_t winrs_plan(int N, int C, int H, int W, int K, int R, in
 WINRS_API winrs_status_t winrs_plan_for_device(int N, int C, int H, int W, int K, int R, int S, int pad,
                                      winrs_dtype_t dtype, const winrs_device_t* dev,
                                      winrs_plan_t* out);
+
+/* N-D (3-D) BFC by Level-2 dimension reduction (§3 P@17805-18294: an
+ * N-D problem reduces to the 2-D machinery over the extra spatial axis):
+ *   X  [N][D][H][W][C] (NDHWC), dY [N][Do][Ho][Wo][K] (NDHWC),
+ *   dW [K][T][R][S][C] FP32 (KTRSC), Do = D + 2 pad - T + 1 (one symmetric pad),
+ *   dW[k][t][r][s][c] = sum_{n,d,h,w} Xp[n][d+t-pad][h+r-pad][w+s-pad][c] dY[n][d][h][w][k].
+ * The T x R filter planes become T*R "filter rows" of the 2-D decomposition and
+ * the N x Do dY slices its images; a row's depth offset t reads X slice d+t-pad
+ * (zero outside [0, D)).  Run with winrs_bfc.  UNSUPPORTED beyond the 2-D rules
+ * for FP32 and when Do % 16 != 0 (FP16 / BF16: the second-generation tensor-core
+ * kernel loads 16 depth slices of one image per TMA box). */
+WINRS_API winrs_status_t winrs_plan3d(int N, int C, int D, int H, int W, int K, int T, int R, int S, int pad,
+                            winrs_dtype_t dtype, winrs_plan_t* out);
+WINRS_API winrs_status_t winrs_plan3d_for_device(int N, int C, int D, int H, int W, int K, int T, int R, int S,
+                                       int pad, winrs_dtype_t dtype, const winrs_device_t* dev,
+                                       winrs_plan_t* out);
 
 /* Copy the plan description into *info (host memory). */
 WINRS_API winrs_status_t winrs_plan_info(winrs_plan_t plan, winrs_plan_info_t* info);

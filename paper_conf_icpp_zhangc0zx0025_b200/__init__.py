@@ -19,7 +19,7 @@ from dataclasses import dataclass
 from . import _lib
 from ._lib import WinrsError, DTYPES
 
-__all__ = ["Plan", "plan", "plan_for_device", "bfc", "bfc_host", "as_kcrs", "as_krsc", "bfc_data_parallel", "shard_range",
+__all__ = ["Plan", "plan", "plan_for_device", "plan3d", "plan3d_for_device", "bfc", "bfc_host", "as_kcrs", "as_krsc", "bfc_data_parallel", "shard_range",
            "bfc_k_sharded",
            "WinrsError", "version", "emulate", "transform", "kernel_names"]
 
@@ -92,6 +92,39 @@ def plan_for_device(N, C, H, W, K, R, S, pad, dtype: str = "f32", num_sms: int =
     return Plan(h)
 
 
+def plan3d(N, C, D, H, W, K, T, R, S, pad, dtype: str = "f16") -> Plan:
+    """winrs_plan3d: N-D (3-D) BFC by Level-2 dimension reduction (PAPER.md
+    P@17805).  X [N,D,H,W,C], dY [N,Do,Ho,Wo,K], dW [K,T,R,S,C]."""
+    h = ctypes.c_void_p()
+    _lib.check(_lib.lib().winrs_plan3d(N, C, D, H, W, K, T, R, S, pad, DTYPES[dtype], ctypes.byref(h)),
+               "winrs_plan3d")
+    return Plan(h)
+
+
+def plan3d_for_device(N, C, D, H, W, K, T, R, S, pad, dtype: str = "f16", num_sms: int = 148, cc=(10, 0)) -> Plan:
+    dev = _lib.DeviceT(num_sms, cc[0], cc[1])
+    h = ctypes.c_void_p()
+    _lib.check(_lib.lib().winrs_plan3d_for_device(N, C, D, H, W, K, T, R, S, pad, DTYPES[dtype], ctypes.byref(dev),
+                                                  ctypes.byref(h)), "winrs_plan3d_for_device")
+    return Plan(h)
+
+
+def _as_cl(t, dims_last, name):
+    """A tensor whose memory is channels-last `dims_last` = (b, *spatial, ch):
+    that contiguous shape, or the logical (b, ch, *spatial) with channels_last
+    (2-D) / channels_last_3d (3-D) strides.  No copy."""
+    if tuple(t.shape) == tuple(dims_last) and t.is_contiguous():
+        return t
+    logical = (dims_last[0], dims_last[-1]) + tuple(dims_last[1:-1])
+    if tuple(t.shape) == logical:
+        perm = (0,) + tuple(range(2, len(logical))) + (1,)
+        v = t.permute(*perm)
+        if v.is_contiguous():
+            return v
+    raise ValueError(f"{name}: expected channels-last {tuple(dims_last)} (contiguous, or logical {logical} "
+                     f"with channels_last strides), got shape {tuple(t.shape)} strides {t.stride()}")
+
+
 def _as_nhwc(t, n, h, w, c, name):
     """Return a tensor whose memory is NHWC [n,h,w,c] (no copy)."""
     if tuple(t.shape) == (n, h, w, c) and t.is_contiguous():
@@ -129,8 +162,15 @@ def bfc(p: Plan, X, dY, dW=None, workspace=None, stream=None):
     import torch
     i = p.info
     tdt = {"f32": torch.float32, "f16": torch.float16, "bf16": torch.bfloat16}[p.dtype]
-    Xn = _as_nhwc(X, i["N"], i["H"], i["W"], i["C"], "X")
-    Gn = _as_nhwc(dY, i["N"], i["Ho"], i["Wo"], i["K"], "dY")
+    nd = i["T"] > 1 or i["D"] > 1
+    if nd:   # N-D plan: NDHWC / NDHWC / KTRSC
+        Xn = _as_cl(X, (i["N"], i["D"], i["H"], i["W"], i["C"]), "X")
+        Gn = _as_cl(dY, (i["N"], i["Do"], i["Ho"], i["Wo"], i["K"]), "dY")
+        wshape = (i["K"], i["T"], i["R"], i["S"], i["C"])
+    else:
+        Xn = _as_nhwc(X, i["N"], i["H"], i["W"], i["C"], "X")
+        Gn = _as_nhwc(dY, i["N"], i["Ho"], i["Wo"], i["K"], "dY")
+        wshape = (i["K"], i["R"], i["S"], i["C"])
     if Xn.dtype != tdt or Gn.dtype != tdt:
         raise TypeError(f"X and dY must be {tdt} for this plan")
     if not (Xn.is_cuda and Gn.is_cuda) or Gn.device != Xn.device:
@@ -142,12 +182,12 @@ def bfc(p: Plan, X, dY, dW=None, workspace=None, stream=None):
     ret = dW
     if dW is None:
         with torch.cuda.stream(ts) if ts is not None else _nullctx():
-            dk = torch.empty((i["K"], i["R"], i["S"], i["C"]), dtype=torch.float32, device=Xn.device)
-        ret = dk.permute(0, 3, 1, 2)          # logical KCRS, channels_last
+            dk = torch.empty(wshape, dtype=torch.float32, device=Xn.device)
+        ret = dk.permute(0, len(wshape) - 1, *range(1, len(wshape) - 1))   # logical K, C, spatial: channels last
     else:
         if dW.dtype != torch.float32 or not dW.is_cuda or dW.device != Xn.device:
             raise ValueError("dW must be a float32 CUDA tensor on X's device")
-        dk = _as_krsc(dW, i["K"], i["C"], i["R"], i["S"], "dW")
+        dk = _as_cl(dW, wshape, "dW")
     wsb = p.workspace_bytes
     if wsb:
         if workspace is None:
@@ -174,10 +214,11 @@ class _nullctx:
 
 
 def as_krsc(dW):
-    """bfc()'s logical [K,C,R,S] channels_last result -> its KRSC [K,R,S,C]
-    storage view (the C ABI / oracle layout), no copy.  KRSC input passes."""
-    if dW.dim() == 4 and dW.stride(1) == 1 and not dW.is_contiguous():
-        return dW.permute(0, 2, 3, 1)
+    """bfc()'s logical [K,C,R,S] (or [K,C,T,R,S]) channels-last result -> its
+    KRSC [K,R,S,C] (KTRSC) storage view (the C ABI / oracle layout), no copy.
+    Channels-last-contiguous input passes."""
+    if dW.dim() >= 4 and dW.stride(1) == 1 and not dW.is_contiguous():
+        return dW.permute(0, *range(2, dW.dim()), 1)
     return dW
 
 
@@ -270,8 +311,13 @@ def emulate(p: Plan, X, dY):
     i = p.info
     Xd = np.ascontiguousarray(X, dtype=np.float64)
     Gd = np.ascontiguousarray(dY, dtype=np.float64)
-    assert Xd.shape == (i["N"], i["H"], i["W"], i["C"]) and Gd.shape == (i["N"], i["Ho"], i["Wo"], i["K"])
-    out = np.empty((i["K"], i["R"], i["S"], i["C"]), dtype=np.float64)
+    if i["T"] > 1 or i["D"] > 1:   # N-D plan: NDHWC in, KTRSC out
+        assert Xd.shape == (i["N"], i["D"], i["H"], i["W"], i["C"])
+        assert Gd.shape == (i["N"], i["Do"], i["Ho"], i["Wo"], i["K"])
+        out = np.empty((i["K"], i["T"], i["R"], i["S"], i["C"]), dtype=np.float64)
+    else:
+        assert Xd.shape == (i["N"], i["H"], i["W"], i["C"]) and Gd.shape == (i["N"], i["Ho"], i["Wo"], i["K"])
+        out = np.empty((i["K"], i["R"], i["S"], i["C"]), dtype=np.float64)
     _lib.check(_lib.lib().winrs_debug_emulate(p.handle, Xd.ctypes.data, Gd.ctypes.data, out.ctypes.data),
                "winrs_debug_emulate")
     return out

@@ -38,7 +38,8 @@ class PlanInfoT(ctypes.Structure):
                  "tile_k0", "tile_c0", "tile_k1", "tile_c1")] + [
         ("ctas_main", ctypes.c_longlong), ("ctas_resid", ctypes.c_longlong),
         ("ctas_reduce", ctypes.c_longlong), ("csplit", ctypes.c_int), ("workspace_bytes", ctypes.c_size_t),
-        ("direct_flops", ctypes.c_double), ("ewm_flops", ctypes.c_double)]
+        ("direct_flops", ctypes.c_double), ("ewm_flops", ctypes.c_double),
+        ("D", ctypes.c_int), ("T", ctypes.c_int), ("Do", ctypes.c_int)]
 
 
 # (name, restype, argtypes) of every exported symbol, in header order.
@@ -46,6 +47,8 @@ _i, _p, _s = ctypes.c_int, ctypes.c_void_p, ctypes.c_size_t
 SYMBOLS = [
     ("winrs_plan", _i, [_i] * 8 + [_i, ctypes.POINTER(_p)]),
     ("winrs_plan_for_device", _i, [_i] * 8 + [_i, ctypes.POINTER(DeviceT), ctypes.POINTER(_p)]),
+    ("winrs_plan3d", _i, [_i] * 10 + [_i, ctypes.POINTER(_p)]),
+    ("winrs_plan3d_for_device", _i, [_i] * 10 + [_i, ctypes.POINTER(DeviceT), ctypes.POINTER(_p)]),
     ("winrs_plan_info", _i, [_p, ctypes.POINTER(PlanInfoT)]),
     ("winrs_workspace_bytes", _s, [_p]),
     ("winrs_bfc", _i, [_p, _p, _p, _p, _p, _p]),

@@ -27,25 +27,38 @@ static EncodeTiledFn encode_fn() {
     return fn;
 }
 
-// 4-D NHWC 16-bit tensor [N][H][W][Ch] (pixel stride ld >= Ch elements) as
-// TMA dims {Ch, N, H, W} (so a box lands as [cols][rows][images][channels]),
-// box {64, bn, 1, bw}, 128-byte swizzle: every (col, image) is one 128-byte
-// row of a UMMA MN-major SW128 atom.  Out-of-bounds elements read as zero.
-static bool make_map(CUtensorMap* m, const void* base, int N, int H, int W, int Ch, int ld, int bw, int bn, bool bf) {
+// 16-bit channels-last tensor as the 5-D TMA map {Ch, A, B, H, W} (A inner
+// image axis, B outer: 2-D [N][H][W][Ch] -> A = N, B = 1; N-D [Nb][D][H][W][Ch]
+// -> A = D, B = Nb), pixel stride ld >= Ch elements; box {64, bn, 1, 1, bw}
+// with the 128-byte swizzle: every (col, image) is one 128-byte row of a UMMA
+// MN-major SW128 atom.  Out-of-bounds elements (padding, depth taps outside
+// [0, D), masked columns, channel tails, past-the-end images) read as zero.
+static bool make_map(CUtensorMap* m, const void* base, int A, int B, int H, int W, int Ch, int ld, int bw, int bn, bool bf) {
     EncodeTiledFn fn = encode_fn();
     if (!fn) return false;
-    const cuuint64_t dims[4] = {(cuuint64_t)Ch, (cuuint64_t)N, (cuuint64_t)H, (cuuint64_t)W};
-    const cuuint64_t strides[3] = {(cuuint64_t)H * W * ld * 2, (cuuint64_t)W * ld * 2, (cuuint64_t)ld * 2};
-    const cuuint32_t box[4] = {64u, (cuuint32_t)bn, 1u, (cuuint32_t)bw};
-    const cuuint32_t es[4] = {1u, 1u, 1u, 1u};
-    return fn(m, bf ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4, const_cast<void*>(base),
+    const cuuint64_t dims[5] = {(cuuint64_t)Ch, (cuuint64_t)A, (cuuint64_t)B, (cuuint64_t)H, (cuuint64_t)W};
+    const cuuint64_t img = (cuuint64_t)H * W * ld * 2;
+    const cuuint64_t strides[4] = {img, img * A, (cuuint64_t)W * ld * 2, (cuuint64_t)ld * 2};
+    const cuuint32_t box[5] = {64u, (cuuint32_t)bn, 1u, 1u, (cuuint32_t)bw};
+    const cuuint32_t es[5] = {1u, 1u, 1u, 1u, 1u};
+    return fn(m, bf ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 5, const_cast<void*>(base),
               dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
+// The X and dY maps of a plan (2-D or N-D).
+static bool make_maps(const Geometry& g, const void* X, const void* dY, bool bf, CUtensorMap* mX, CUtensorMap* mY) {
+    const bool nd = g.T > 1 || g.D > 1;
+    return make_map(mX, X, nd ? g.D : g.N, nd ? g.Nb : 1, g.H, g.W, g.C, g.C, 4, KC, bf) &&
+           make_map(mY, dY, nd ? g.Do : g.N, nd ? g.Nb : 1, g.Ho, g.Wo, g.K, g.ldy, 2, KC, bf);
+}
 
 // Images per TMA box: one box per stage and atom, so the box's [cols][images]
-// rows are exactly a column-major run of 16-row operand atoms (N % 16 == 0).
-static int images_per_box(int N) { return N % KC == 0 ? KC : 0; }
+// rows are exactly a column-major run of 16-row operand atoms (N % 16 == 0;
+// N-D: Do % 16 == 0, 16 depth slices of one batch image).
+static int images_per_box(const Geometry& g) {
+    const bool nd = g.T > 1 || g.D > 1;
+    return (nd ? g.Do : g.N) % KC == 0 ? KC : 0;
+}
 
 template <int F, int NK, bool BF, int CG>
 cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
@@ -56,12 +69,10 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
     a.g = g;
     a.dW = dW;
     a.ws = ws;
-    a.nb = images_per_box(g.N);
+    a.nb = images_per_box(g);
     if (a.nb == 0 || g.a0 != 4 || g.n0 != 3 || g.r0 != 2 || g.a1 != 0) return cudaErrorInvalidValue;
     CUtensorMap mX, mY;
-    if (!make_map(&mX, X, g.N, g.H, g.W, g.C, g.C, 4, a.nb, BF) ||
-        !make_map(&mY, dY, g.N, g.Ho, g.Wo, g.K, g.ldy, 2, a.nb, BF))
-        return cudaErrorInvalidValue;
+    if (!make_maps(g, X, dY, BF, &mX, &mY)) return cudaErrorInvalidValue;
     static std::atomic<unsigned long long> done{0};
     auto k = bfc_tc2_kernel<F, NK, BF, CG>;
     cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
@@ -94,13 +105,11 @@ cudaError_t launch_sw(const Geometry& g, const void* X, const void* dY, float* d
     a.g = g;
     a.dW = dW;
     a.ws = ws;
-    a.nb = images_per_box(g.N);
+    a.nb = images_per_box(g);
     if (a.nb == 0 || g.a0 != 4 || g.n0 != 3 || g.r0 != 2 || g.a1 != 0 || g.cg != 2 || g.fhs != 1)
         return cudaErrorInvalidValue;
     CUtensorMap mX, mY;
-    if (!make_map(&mX, X, g.N, g.H, g.W, g.C, g.C, 4, a.nb, BF) ||
-        !make_map(&mY, dY, g.N, g.Ho, g.Wo, g.K, g.ldy, 2, a.nb, BF))
-        return cudaErrorInvalidValue;
+    if (!make_maps(g, X, dY, BF, &mX, &mY)) return cudaErrorInvalidValue;
     static std::atomic<unsigned long long> done{0};
     auto k = bfc_tc2s_kernel<BF>;
     cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);

@@ -151,6 +151,36 @@ __device__ __forceinline__ bool elect_one() {
     asm volatile("{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\nselp.u32 %0, 1, 0, p;\n}\n" : "=r"(pred));
     return pred != 0;
 }
+__device__ __forceinline__ void tma5(uint32_t dst, const CUtensorMap* m, uint64_t* bar, int c0, int c1, int c2, int c3,
+                                     int c4) {
+    asm volatile(
+        "cp.async.bulk.tensor.5d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5, %6}], [%7];"
+        :: "r"(dst), "l"(reinterpret_cast<uint64_t>(m)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(su(bar))
+        : "memory");
+}
+// Image index img of the 2-D decomposition -> (inner, outer) TMA coordinates:
+// 2-D plans: (img, 0) of maps {ch, N, 1, H, W}; N-D plans (PAPER.md P@17805,
+// Level-2 dimension reduction): (depth slice img % Do, batch img / Do) of maps
+// {ch, D or Do, Nb, H, W}.  Past the end: outer = Nb (zero fill).
+struct ImgCoord {
+    int a, b;
+};
+__device__ __forceinline__ ImgCoord img_coord(const Geometry& g, int img, bool in) {
+    const bool nd = g.T > 1 || g.D > 1;
+    const int inner = nd ? g.Do : g.N;
+    ImgCoord c;
+    c.a = in ? img % inner : 0;
+    c.b = in ? img / inner : (nd ? g.Nb : 1);
+    return c;
+}
+// X's inner coordinate for filter row fh: the depth slice shifted by the row's
+// depth tap fh / Rh (N-D), and the X row h + (fh % Rh) - pad.
+__device__ __forceinline__ int x_inner(const Geometry& g, int a, int fh) {
+    return (g.T > 1 || g.D > 1) ? a + fh / g.Rh - g.pad : a;
+}
+__device__ __forceinline__ int x_row(const Geometry& g, int h, int fh) {
+    return fh < g.R ? h + fh % g.Rh - g.pad : -(1 << 20);   // a slot past the last filter row: zero fill
+}
 __device__ __forceinline__ void fence_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void tc_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
@@ -383,8 +413,9 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             TC2_TRACE(ch - c_lo, 0);
             uint64_t* fb = &bars->full[s];
             const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
-            const bool in = d < depth;               // past the end: image N (zero fill)
-            const int nn = in ? n : g.N, hh = in ? h : hs;
+            const bool in = d < depth;               // past the end: outer image coordinate out of range (zero fill)
+            const ImgCoord ic = img_coord(g, n, in);
+            const int hh = in ? h : hs;
             const int w0 = w_first + (in ? u : 0) * 2;
             if (elect_one()) {
 #ifdef WINRS_TC2_NO_TMA   // debug ablation: stages carry no data (barrier protocol kept)
@@ -397,12 +428,12 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     // filter row reads rows far outside (zero fill)
                     const int fh = F == 2 ? fh_base + a : fh_base;
                     const int c0 = F == 2 ? c_base : c_base + a * 64;
-                    const int xrow = fh < g.R ? hh + fh - g.pad : -(1 << 20);
-                    tma4(st + a * L::X_LBO, &tmX, fb, c0, nn, xrow, w0 + fw0 - g.pad);
+                    tma5(st + a * L::X_LBO, &tmX, fb, c0, x_inner(g, ic.a, fh), ic.b, x_row(g, hh, fh),
+                         w0 + fw0 - g.pad);
                 }
 #pragma unroll
                 for (int ka = 0; ka < L::NKL / 64; ++ka)   // dY unit columns w0, w0 + 1 of k atom ka
-                    tma4(st + L::OFF_Y + ka * L::Y_LBO, &tmY, fb, k_base + ka * 64, nn, hh, w0);
+                    tma5(st + L::OFF_Y + ka * L::Y_LBO, &tmY, fb, k_base + ka * 64, ic.a, ic.b, hh, w0);
 #endif
             }
             __syncwarp();
@@ -721,13 +752,14 @@ bfc_tc2s_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
             uint64_t* fb = &bars->full[s];
             const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
             const bool in = d < depth;
-            const int nn = in ? n : g.N, hh = in ? h : hs;
+            const ImgCoord ic = img_coord(g, n, in);
+            const int hh = in ? h : hs;
             const int w0 = w_first + (in ? u : 0) * 2;
             if (elect_one()) {
                 mbar_expect_tx(fb, (uint32_t)L::TX_BYTES);
-                tma4(st + L::OFF_X, &tmX, fb, c_base, nn, hh + fh - g.pad, w0 + fw0 - g.pad);
-                tma4(st + L::OFF_Y, &tmY, fb, k_base, nn, hh, w0);
-                tma4(st + L::OFF_Y + L::Y_LBO, &tmY, fb, k_base + 64, nn, hh, w0);
+                tma5(st + L::OFF_X, &tmX, fb, c_base, x_inner(g, ic.a, fh), ic.b, x_row(g, hh, fh), w0 + fw0 - g.pad);
+                tma5(st + L::OFF_Y, &tmY, fb, k_base, ic.a, ic.b, hh, w0);
+                tma5(st + L::OFF_Y + L::Y_LBO, &tmY, fb, k_base + 64, ic.a, ic.b, hh, w0);
             }
             __syncwarp();
             TC2_TRACE(ch - c_lo, 1);

@@ -196,6 +196,11 @@ static void fill_geometry(const Problem& p, const KernelEntry& e, const PairChoi
     g->csplit = 1;
     g->chunk = p.dtype == 0 ? 8 : 16;
     g->dw_elems = (long long)p.K * p.R * p.S * p.C;
+    g->Rh = p.Rh > 0 ? p.Rh : p.R;
+    g->T = p.T;
+    g->D = p.D;
+    g->Do = p.Do;
+    g->Nb = p.Nb > 0 ? p.Nb : p.N;
 }
 
 // Fewest chunks any tile of the Omega_a0 phase walks (its segment's clipped
@@ -452,6 +457,8 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
         for (const KernelEntry* e : tiles) {
             if (force_tile && (e->bn != fbn || e->bm != fbm)) continue;
             if (e->fhs > 0 && p.N % 16 != 0) continue;   // tc2: one 16-image TMA box per stage and atom
+            const bool nd = p.T > 1 || p.D > 1;
+            if (nd && (e->fhs <= 0 || p.Do % 16 != 0)) continue;   // N-D: tc2 kernels, 16 slices of one image per box
             if (const char* v = getenv("WINRS_TC_GEN")) {   // debug: restrict to one tensor-core generation
                 if (e->dtype != 0 && ((atoi(v) == 2) != (e->fhs > 0))) continue;
             }

@@ -6,9 +6,12 @@
 
 namespace winrs {
 
+// For an N-D problem N = Nb * Do images and R = T * Rh filter rows (the 2-D
+// decomposition the kernels run); Nb, Rh, T, D, Do describe the original axes.
 struct Problem {
     int N, C, H, W, K, R, S, pad, Ho, Wo;
     int dtype;
+    int Nb = 0, Rh = 0, T = 1, D = 1, Do = 1;
 };
 
 struct PlanResult {

@@ -21,12 +21,16 @@ struct winrs_plan_s {
 
 using namespace winrs;
 
+// D, T: the N-D depth axes (1, 1 for a 2-D plan); see winrs_plan3d.
 static winrs_status_t build_plan(int N, int C, int H, int W, int K, int R, int S, int pad,
-                                 winrs_dtype_t dtype, const winrs_device_t* dev, winrs_plan_t* out) {
+                                 winrs_dtype_t dtype, const winrs_device_t* dev, winrs_plan_t* out,
+                                 int D = 1, int T = 1) {
     if (!out) return WINRS_ERR_INVALID_ARG;
     *out = nullptr;
-    if (N <= 0 || C <= 0 || H <= 0 || W <= 0 || K <= 0 || R <= 0 || S <= 0 || pad < 0)
+    if (N <= 0 || C <= 0 || H <= 0 || W <= 0 || K <= 0 || R <= 0 || S <= 0 || pad < 0 || D <= 0 || T <= 0)
         return WINRS_ERR_INVALID_ARG;
+    const int Do = D + 2 * (T > 1 || D > 1 ? pad : 0) - T + 1;
+    if (Do < 1) return WINRS_ERR_INVALID_ARG;
     if (dtype != WINRS_F32 && dtype != WINRS_F16 && dtype != WINRS_BF16) return WINRS_ERR_INVALID_ARG;
     const int Ho = H + 2 * pad - R + 1, Wo = W + 2 * pad - S + 1;
     if (Ho < 1 || Wo < 1) return WINRS_ERR_INVALID_ARG;
@@ -34,8 +38,13 @@ static winrs_status_t build_plan(int N, int C, int H, int W, int K, int R, int S
     if (dev->cc_major != 10 || dev->cc_minor != 0) return WINRS_ERR_UNSUPPORTED;   // sm_100a build
     const int align = dtype == WINRS_F32 ? 4 : 8;                                  // 16-byte vectors
     if (C % align || K % align) return WINRS_ERR_UNSUPPORTED;
-    if ((long long)N * Ho * Wo >= (1LL << 31)) return WINRS_ERR_UNSUPPORTED;   // 32-bit depth index
-    Problem p{N, C, H, W, K, R, S, pad, Ho, Wo, (int)dtype};
+    const bool nd = T > 1 || D > 1;
+    if (nd && dtype == WINRS_F32) return WINRS_ERR_UNSUPPORTED;   // N-D: the tensor-core kernels
+    if ((long long)N * Do * Ho * Wo >= (1LL << 31) || (long long)R * T > (1 << 20))
+        return WINRS_ERR_UNSUPPORTED;   // 32-bit depth index
+    // N-D -> the 2-D decomposition: N*Do images, T*R filter rows
+    Problem p{N * Do, C, H, W, K, R * T, S, pad, Ho, Wo, (int)dtype};
+    p.Nb = N; p.Rh = R; p.T = T; p.D = D; p.Do = Do;
     PlanResult pr;
     const winrs_status_t st = make_plan(p, dev->num_sms, &pr);
     if (st != WINRS_OK) return st;
@@ -47,6 +56,7 @@ static winrs_status_t build_plan(int N, int C, int H, int W, int K, int R, int S
     winrs_plan_info_t& in = pl->info;
     memset(&in, 0, sizeof(in));
     in.N = N; in.C = C; in.H = H; in.W = W; in.K = K; in.R = R; in.S = S; in.pad = pad;
+    in.D = D; in.T = T; in.Do = Do;
     in.dtype = dtype; in.Ho = Ho; in.Wo = Wo;
     in.alpha0 = g.a0; in.n0 = g.n0; in.r0 = g.r0; in.k0 = g.k0;
     in.alpha1 = g.a1; in.n1 = g.n1; in.r1 = g.r1; in.k1 = g.k1;
@@ -61,7 +71,7 @@ static winrs_status_t build_plan(int N, int C, int H, int W, int K, int R, int S
     in.ctas_resid = 0;   // the residual phase runs inside the main launch's last-column CTAs
     in.ctas_reduce = g.Z > 1 ? 1 : 0;
     in.workspace_bytes = g.Z > 1 ? (size_t)(g.Z - 1) * 4u * (size_t)g.dw_elems : 0;
-    in.direct_flops = 2.0 * N * (double)C * K * Ho * Wo * R * S;
+    in.direct_flops = 2.0 * N * (double)Do * C * K * Ho * Wo * R * T * S;
     in.ewm_flops = pr.ewm_flops;
     *out = pl;
     return WINRS_OK;
@@ -87,6 +97,26 @@ winrs_status_t winrs_plan(int N, int C, int H, int W, int K, int R, int S, int p
         return WINRS_ERR_CUDA;
     }
     return build_plan(N, C, H, W, K, R, S, pad, dtype, &dev, out);
+}
+
+winrs_status_t winrs_plan3d_for_device(int N, int C, int D, int H, int W, int K, int T, int R, int S, int pad,
+                                       winrs_dtype_t dtype, const winrs_device_t* dev, winrs_plan_t* out) {
+    return build_plan(N, C, H, W, K, R, S, pad, dtype, dev, out, D, T);
+}
+
+winrs_status_t winrs_plan3d(int N, int C, int D, int H, int W, int K, int T, int R, int S, int pad,
+                            winrs_dtype_t dtype, winrs_plan_t* out) {
+    if (!out) return WINRS_ERR_INVALID_ARG;
+    int d = 0;
+    if (cudaGetDevice(&d) != cudaSuccess) { cudaGetLastError(); return WINRS_ERR_CUDA; }
+    winrs_device_t dev{};
+    if (cudaDeviceGetAttribute(&dev.num_sms, cudaDevAttrMultiProcessorCount, d) != cudaSuccess ||
+        cudaDeviceGetAttribute(&dev.cc_major, cudaDevAttrComputeCapabilityMajor, d) != cudaSuccess ||
+        cudaDeviceGetAttribute(&dev.cc_minor, cudaDevAttrComputeCapabilityMinor, d) != cudaSuccess) {
+        cudaGetLastError();
+        return WINRS_ERR_CUDA;
+    }
+    return build_plan(N, C, H, W, K, R, S, pad, dtype, &dev, out, D, T);
 }
 
 winrs_status_t winrs_plan_info(winrs_plan_t plan, winrs_plan_info_t* info) {
@@ -137,9 +167,9 @@ winrs_status_t winrs_bfc_host(winrs_plan_t plan, const void* host_X, const void*
     if (!plan || !host_X || !host_dY || !host_dW || !dev_X || !dev_dY || !dev_dW) return WINRS_ERR_INVALID_ARG;
     const winrs_plan_info_t& in = plan->info;
     const size_t esz = in.dtype == WINRS_F32 ? 4 : 2;
-    const size_t bx = esz * (size_t)in.N * in.H * in.W * in.C;
-    const size_t by = esz * (size_t)in.N * in.Ho * in.Wo * in.K;
-    const size_t bw = 4 * (size_t)in.K * in.R * in.S * in.C;
+    const size_t bx = esz * (size_t)in.N * in.D * in.H * in.W * in.C;
+    const size_t by = esz * (size_t)in.N * in.Do * in.Ho * in.Wo * in.K;
+    const size_t bw = 4 * (size_t)in.K * in.T * in.R * in.S * in.C;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     if (cudaMemcpyAsync(dev_X, host_X, bx, cudaMemcpyHostToDevice, s) != cudaSuccess ||
         cudaMemcpyAsync(dev_dY, host_dY, by, cudaMemcpyHostToDevice, s) != cudaSuccess) {
@@ -209,13 +239,21 @@ void emu_phase(const Geometry& g, const double* X, const double* dY, double* buc
                     WT::ft(w, o);
                     for (int x = 0; x < A; ++x) gt[(size_t)x * BN + k] = o[x];
                 }
-                const int xrow = h + cc.fh - g.pad;
+                // N-D: filter row fh = (depth tap fh / Rh, height tap fh % Rh); image n =
+                // (batch n / Do, dY depth slice n % Do) reads X slice (n % Do) + t - pad
+                const int rh = g.Rh > 0 ? g.Rh : g.R;
+                const int xrow = h + cc.fh % rh - g.pad;
+                const bool nd = g.T > 1 || g.D > 1;
+                const int Do = g.Do > 0 ? g.Do : 1;
+                const int xd = (n % Do) + (nd ? cc.fh / rh - g.pad : 0);
+                const bool dok = xd >= 0 && xd < (g.D > 0 ? g.D : 1);
+                const long long ximg = (long long)(n / Do) * (g.D > 0 ? g.D : 1) + xd;
                 for (int c = 0; c < BM; ++c) {
                     double xv[A], o[A];
                     for (int t = 0; t < A; ++t) {
                         const int col = w0 + fw0 - g.pad + t, ccn = c0 + c;
-                        xv[t] = (col >= 0 && col < g.W && ccn < g.C && xrow >= 0 && xrow < g.H)
-                                    ? X[(((size_t)n * g.H + xrow) * g.W + col) * g.C + ccn] : 0.0;
+                        xv[t] = (dok && col >= 0 && col < g.W && ccn < g.C && xrow >= 0 && xrow < g.H)
+                                    ? X[(((size_t)ximg * g.H + xrow) * g.W + col) * g.C + ccn] : 0.0;
                     }
                     WT::it(xv, o);
                     for (int x = 0; x < A; ++x) xt[(size_t)x * BM + c] = o[x];

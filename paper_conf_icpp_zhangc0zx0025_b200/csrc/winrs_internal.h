@@ -59,6 +59,10 @@ struct Geometry {
     int cg;                     // CTAs per UMMA (2: a cta_group::2 pair per depth rank), >= 1
     int chunk;                  // depth entries per main-loop chunk (8 FP32, 16 FP16)
     long long dw_elems;         // K*R*S*C
+    // N-D (Level-2 dimension reduction, PAPER.md P@17805): R = T * Rh filter rows
+    // (depth tap fh / Rh, height tap fh % Rh); N = Nb * Do images (depth slice
+    // img % Do of batch image img / Do).  2-D: T = D = Do = 1, Rh = R, Nb = N.
+    int Rh, T, D, Do, Nb;
 };
 
 struct CtaCoord {
@@ -88,12 +92,14 @@ WINRS_HD void split_chunks(int nchunks, int rank, int csplit, int* lo, int* hi) 
     *hi = (int)((long long)nchunks * (rank + 1) / csplit);
 }
 
-// Valid (clipped) dY rows [hs, he) of a band for filter row fh.
+// Valid (clipped) dY rows [hs, he) of a band for filter row fh (height tap
+// fh % Rh; an N-D plan's depth tap fh / Rh is clipped by the zero fill).
 WINRS_HD void band_rows(const Geometry& g, int band, int fh, int* hs, int* he) {
     const int h0 = band * g.seg_h;
     const int h1 = (band == g.bands - 1) ? g.Ho : h0 + g.seg_h;
-    int a = g.pad - fh; if (a < h0) a = h0;
-    int b = g.H + g.pad - fh; if (b > h1) b = h1;
+    const int r = g.Rh > 0 ? fh % g.Rh : fh;
+    int a = g.pad - r; if (a < h0) a = h0;
+    int b = g.H + g.pad - r; if (b > h1) b = h1;
     *hs = a;
     *he = b > a ? b : a;
 }

@@ -232,3 +232,47 @@ def test_repeated_calls_bitwise(layer_name, env, monkeypatch):
     err = O.rel_max_err(W.as_krsc(first).cpu().numpy().astype(np.float64).ravel()[idx], ref)
     record_err(f"{layer_name} 400 cold-L2 calls bitwise equal {env}", err, p.kernel_name)
     assert err <= TOL[layer.dtype]
+
+
+# ====================================================== N-D (3-D) BFC (PAPER.md P@17805)
+ND = [
+    # N, C, D, H, W, K, T, R, S, pad, env
+    (1, 64, 16, 10, 11, 64, 3, 3, 3, 1, {}),
+    (2, 32, 16, 7, 9, 48, 3, 3, 3, 1, {"WINRS_FORCE_CSPLIT": "2"}),
+    (1, 128, 16, 6, 6, 128, 3, 3, 3, 1, {"WINRS_FORCE_TILE": "128x128"}),
+    (1, 64, 16, 8, 8, 64, 3, 3, 3, 1, {"WINRS_FORCE_TILE": "128x64"}),          # (t, r) rows stacked per CTA
+    (1, 256, 16, 5, 5, 256, 3, 3, 3, 1, {"WINRS_FORCE_TILE": "256x128"}),       # swapped CTA pair
+    (1, 40, 17, 9, 8, 24, 2, 2, 3, 1, {"WINRS_FORCE_Z": "3"}),                  # Do = 18 -> padded below
+    (2, 16, 18, 6, 6, 16, 3, 1, 3, 0, {}),                                      # pad 0, R = 1
+]
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+@pytest.mark.parametrize("case", ND, ids=[f"nd{i}" for i in range(len(ND))])
+def test_nd_bfc(case, dtype, monkeypatch):
+    N, C, D, H, Wd, K, T, R, S, pad, env = case
+    Do = D + 2 * pad - T + 1
+    if Do % 16:                       # the tc2 N-D path loads 16 depth slices per TMA box
+        D += 16 - Do % 16
+        Do = D + 2 * pad - T + 1
+    for k in ENV_KEYS:
+        monkeypatch.delenv(k, raising=False)
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    g = np.random.Generator(np.random.PCG64(1234 + N * 7 + C))
+    X = g.random((N, D, H, Wd, C), dtype=np.float32)
+    dY = (g.random((N, Do, H + 2 * pad - R + 1, Wd + 2 * pad - S + 1, K), dtype=np.float32) * 1e-2)
+    if dtype == "f16":
+        X, dY = X.astype(np.float16), dY.astype(np.float16)
+    else:
+        X, dY = wl.round_to_bf16(X), wl.round_to_bf16(dY)
+    p = W.plan3d(N, C, D, H, Wd, K, T, R, S, pad, dtype)
+    dW = W.as_krsc(W.bfc(p, _dev(X, dtype), _dev(dY, dtype)))
+    torch.cuda.synchronize()
+    got = dW.cpu().numpy().astype(np.float64)
+    ref = O.bfc3d_numpy(X.astype(np.float64), dY.astype(np.float64), T, R, S, pad)
+    err = O.rel_max_err(got, ref)
+    record_err(f"3-D N{N} C{C} D{D} {H}x{Wd} K{K} T{T}R{R}S{S} p{pad} [{dtype}] {env}", err,
+               f"{p.kernel_name} Z={p.info['Z']} cs={p.info['csplit']}")
+    assert got.shape == (K, T, R, S, C)
+    assert err <= TOL[dtype], (p.kernel_name, err)

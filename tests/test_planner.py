@@ -4,11 +4,13 @@ and of the C ABI surface (include/*.h)."""
 import os
 import re
 
+import numpy as np
 import pytest
 
 import paper_conf_icpp_zhangc0zx0025_b200 as W
 from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
 from paper_conf_icpp_zhangc0zx0025_b200._lib import WinrsError
+from oracle import oracle as O
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
@@ -194,3 +196,45 @@ def test_search_plan_is_valid(l):
     # R11: (Z - 1) buckets of |dW| <= floor(0.04 data / |dW|) buckets, i.e. <= 4 % of X + dY exactly
     assert i["workspace_bytes"] <= 0.04 * data
     assert i["csplit"] in (1, 2, 3, 4, 6, 8)
+
+
+# ============================================================== N-D (3-D) plans
+def test_plan3d_rules():
+    """winrs_plan3d: FP16 / BF16 plans on the second-generation kernel; FP32 and
+    Do % 16 != 0 are UNSUPPORTED; bad shapes INVALID_ARG."""
+    p = W.plan3d_for_device(2, 64, 16, 12, 12, 64, 3, 3, 3, 1, "f16")
+    i = p.info
+    assert (i["D"], i["T"], i["Do"]) == (16, 3, 16) and "_v2" in p.kernel_name
+    assert i["direct_flops"] == 2.0 * 2 * 16 * 64 * 64 * 12 * 12 * 27
+    with pytest.raises(WinrsError, match="UNSUPPORTED"):
+        W.plan3d_for_device(2, 64, 16, 12, 12, 64, 3, 3, 3, 1, "f32")
+    with pytest.raises(WinrsError, match="UNSUPPORTED"):
+        W.plan3d_for_device(2, 64, 10, 12, 12, 64, 3, 3, 3, 1, "f16")   # Do = 10
+    with pytest.raises(WinrsError, match="INVALID_ARG"):
+        W.plan3d_for_device(2, 64, 1, 12, 12, 64, 5, 3, 3, 1, "f16")    # Do < 1
+
+
+@pytest.mark.parametrize("shape,env", [
+    ((1, 16, 16, 6, 7, 24, 3, 3, 3, 1), {}),
+    ((2, 8, 16, 5, 6, 16, 2, 2, 3, 1), {}),                       # Do = 17 -> rejected below; see D
+    ((1, 24, 16, 5, 5, 8, 3, 3, 3, 1), {"WINRS_FORCE_CSPLIT": "2", "WINRS_FORCE_Z": "2"}),
+    ((1, 16, 16, 5, 5, 16, 3, 3, 3, 1), {"WINRS_FORCE_TILE": "128x64"}),   # two (t, r) rows stacked per CTA
+], ids=["t3", "t2", "split", "stacked"])
+def test_plan3d_decomposition_emulated(shape, env, monkeypatch):
+    """FP64 emulation of an N-D plan's decomposition (the T*R filter rows with
+    their depth taps, N*Do images, clipping, segments, buckets, cluster ranks)
+    equals the 3-D oracle."""
+    N, C, D, H, Wd, K, T, R, S, pad = shape
+    for k_, v_ in env.items():
+        monkeypatch.setenv(k_, v_)
+    Do = D + 2 * pad - T + 1
+    if Do % 16:
+        D += 16 - Do % 16
+        Do = D + 2 * pad - T + 1
+    p = W.plan3d_for_device(N, C, D, H, Wd, K, T, R, S, pad, "f16")
+    g = np.random.Generator(np.random.PCG64(5))
+    X = g.uniform(-1, 1, (N, D, H, Wd, C))
+    dY = g.uniform(-1, 1, (N, Do, H + 2 * pad - R + 1, Wd + 2 * pad - S + 1, K))
+    got = W.emulate(p, X, dY)
+    ref = O.bfc3d_numpy(X, dY, T, R, S, pad)
+    assert np.allclose(got, ref, rtol=1e-11, atol=1e-11), (p, np.max(np.abs(got - ref)))
