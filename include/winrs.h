@@ -126,8 +126,8 @@ WINRS_API winrs_status_t winrs_plan_for_device(int N, int C, int H, int W, int K
  * The T x R filter planes become T*R "filter rows" of the 2-D decomposition and
  * the N x Do dY slices its images; a row's depth offset t reads X slice d+t-pad
  * (zero outside [0, D)).  Run with winrs_bfc.  UNSUPPORTED beyond the 2-D rules
- * for FP32 and when Do % 16 != 0 (FP16 / BF16: the second-generation tensor-core
- * kernel loads 16 depth slices of one image per TMA box). */
+ * when Do % 16 != 0 for FP16 / BF16 (the second-generation tensor-core kernel
+ * loads 16 depth slices of one image per TMA box); FP32 runs the FP32 kernel. */
 WINRS_API winrs_status_t winrs_plan3d(int N, int C, int D, int H, int W, int K, int T, int R, int S, int pad,
                             winrs_dtype_t dtype, winrs_plan_t* out);
 WINRS_API winrs_status_t winrs_plan3d_for_device(int N, int C, int D, int H, int W, int K, int T, int R, int S,

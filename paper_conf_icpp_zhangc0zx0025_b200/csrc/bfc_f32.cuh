@@ -188,9 +188,19 @@ __device__ __forceinline__ void producer_phase(const Geometry& g, const float* _
         const bool dv = d < d_hi;
         const int w0 = P.w_first + u * RR;
         const float* gsrc = dY + (((long long)n * g.Ho + h) * g.Wo + w0) * g.ldy + k_base;
-        const int xrow = h + cc.fh - g.pad;
+        // filter row fh = (depth tap fh / Rh, height tap fh % Rh); for an N-D plan
+        // image n = (batch n / Do, dY depth slice n % Do) reads X slice
+        // (n % Do) + t - pad, zero outside [0, D) (PAPER.md P@17805)
+        const int xrow = h + cc.fh % g.Rh - g.pad;
         const int xcol0 = w0 + P.fw0 - g.pad;
-        const float* xsrc = X + (((long long)n * g.H + xrow) * g.W) * g.C + c_base;
+        long long ximg = n;
+        bool dok = true;
+        if (g.T > 1 || g.D > 1) {
+            const int dd = n % g.Do + cc.fh / g.Rh - g.pad;
+            dok = dd >= 0 && dd < g.D;
+            ximg = (long long)(n / g.Do) * g.D + dd;
+        }
+        const float* xsrc = X + ((ximg * g.H + xrow) * g.W) * g.C + c_base;
         float* gdst = rawG + ((buf * BD + ld_d) * RR) * BN;
         float* xdst = rawX + ((buf * BD + ld_d) * ALPHA) * BM;
         constexpr int GV = RR * (BN / 4);
@@ -211,7 +221,7 @@ __device__ __forceinline__ void producer_phase(const Geometry& g, const float* _
             if (XV % TPD == 0 || q < XV) {
                 const int t = q / (BM / 4), v4 = q % (BM / 4);
                 const int col = xcol0 + t;
-                const bool ok = dv && col >= 0 && col < g.W && c_base + v4 * 4 < g.C;
+                const bool ok = dv && dok && col >= 0 && col < g.W && c_base + v4 * 4 < g.C;
                 cp_async16(xdst + t * BM + v4 * 4, ok ? (const void*)(xsrc + (long long)col * g.C + v4 * 4) : (const void*)X,
                            ok);
             }

@@ -458,7 +458,8 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
             if (force_tile && (e->bn != fbn || e->bm != fbm)) continue;
             if (e->fhs > 0 && p.N % 16 != 0) continue;   // tc2: one 16-image TMA box per stage and atom
             const bool nd = p.T > 1 || p.D > 1;
-            if (nd && (e->fhs <= 0 || p.Do % 16 != 0)) continue;   // N-D: tc2 kernels, 16 slices of one image per box
+            // N-D: the FP32 kernel, or the tc2 kernels (16 depth slices of one image per TMA box)
+            if (nd && e->dtype != 0 && (e->fhs <= 0 || p.Do % 16 != 0)) continue;
             if (const char* v = getenv("WINRS_TC_GEN")) {   // debug: restrict to one tensor-core generation
                 if (e->dtype != 0 && ((atoi(v) == 2) != (e->fhs > 0))) continue;
             }

@@ -39,7 +39,6 @@ static winrs_status_t build_plan(int N, int C, int H, int W, int K, int R, int S
     const int align = dtype == WINRS_F32 ? 4 : 8;                                  // 16-byte vectors
     if (C % align || K % align) return WINRS_ERR_UNSUPPORTED;
     const bool nd = T > 1 || D > 1;
-    if (nd && dtype == WINRS_F32) return WINRS_ERR_UNSUPPORTED;   // N-D: the tensor-core kernels
     if ((long long)N * Do * Ho * Wo >= (1LL << 31) || (long long)R * T > (1 << 20))
         return WINRS_ERR_UNSUPPORTED;   // 32-bit depth index
     // N-D -> the 2-D decomposition: N*Do images, T*R filter rows

@@ -247,7 +247,7 @@ ND = [
 ]
 
 
-@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+@pytest.mark.parametrize("dtype", ["f16", "bf16", "f32"])
 @pytest.mark.parametrize("case", ND, ids=[f"nd{i}" for i in range(len(ND))])
 def test_nd_bfc(case, dtype, monkeypatch):
     N, C, D, H, Wd, K, T, R, S, pad, env = case
@@ -264,8 +264,10 @@ def test_nd_bfc(case, dtype, monkeypatch):
     dY = (g.random((N, Do, H + 2 * pad - R + 1, Wd + 2 * pad - S + 1, K), dtype=np.float32) * 1e-2)
     if dtype == "f16":
         X, dY = X.astype(np.float16), dY.astype(np.float16)
-    else:
+    elif dtype == "bf16":
         X, dY = wl.round_to_bf16(X), wl.round_to_bf16(dY)
+    elif "WINRS_FORCE_TILE" in env:   # the tensor-core tiles do not exist for FP32
+        monkeypatch.delenv("WINRS_FORCE_TILE", raising=False)
     p = W.plan3d(N, C, D, H, Wd, K, T, R, S, pad, dtype)
     dW = W.as_krsc(W.bfc(p, _dev(X, dtype), _dev(dY, dtype)))
     torch.cuda.synchronize()

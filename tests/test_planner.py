@@ -200,14 +200,13 @@ def test_search_plan_is_valid(l):
 
 # ============================================================== N-D (3-D) plans
 def test_plan3d_rules():
-    """winrs_plan3d: FP16 / BF16 plans on the second-generation kernel; FP32 and
-    Do % 16 != 0 are UNSUPPORTED; bad shapes INVALID_ARG."""
+    """winrs_plan3d: FP16 / BF16 plans on the second-generation kernel, FP32 on
+    the FP32 kernel; FP16 with Do % 16 != 0 is UNSUPPORTED; bad shapes INVALID_ARG."""
     p = W.plan3d_for_device(2, 64, 16, 12, 12, 64, 3, 3, 3, 1, "f16")
     i = p.info
     assert (i["D"], i["T"], i["Do"]) == (16, 3, 16) and "_v2" in p.kernel_name
     assert i["direct_flops"] == 2.0 * 2 * 16 * 64 * 64 * 12 * 12 * 27
-    with pytest.raises(WinrsError, match="UNSUPPORTED"):
-        W.plan3d_for_device(2, 64, 16, 12, 12, 64, 3, 3, 3, 1, "f32")
+    assert "f32_" in W.plan3d_for_device(2, 64, 16, 12, 12, 64, 3, 3, 3, 1, "f32").kernel_name
     with pytest.raises(WinrsError, match="UNSUPPORTED"):
         W.plan3d_for_device(2, 64, 10, 12, 12, 64, 3, 3, 3, 1, "f16")   # Do = 10
     with pytest.raises(WinrsError, match="INVALID_ARG"):
@@ -238,3 +237,7 @@ def test_plan3d_decomposition_emulated(shape, env, monkeypatch):
     got = W.emulate(p, X, dY)
     ref = O.bfc3d_numpy(X, dY, T, R, S, pad)
     assert np.allclose(got, ref, rtol=1e-11, atol=1e-11), (p, np.max(np.abs(got - ref)))
+    monkeypatch.delenv("WINRS_FORCE_TILE", raising=False)              # (tensor-core tile names)
+    p32 = W.plan3d_for_device(N, C, D, H, Wd, K, T, R, S, pad, "f32")    # FP32 kernel decomposition
+    got32 = W.emulate(p32, X, dY)
+    assert np.allclose(got32, ref, rtol=1e-11, atol=1e-11), (p32, np.max(np.abs(got32 - ref)))
