@@ -428,6 +428,46 @@ def measure(layers, args, ctx, primary=True):
                 clocks=clk, h2d=h2d, d2h=d2h, job_flops=job_flops, steps=steps)
 
 
+def measure_nd(args, dev, flush, peaks, reps=10):
+    """N-D (3-D) BFC layers: cold-L2 CUDA-event times of
+    winrs_bfc on winrs_plan3d plans, FP16, inputs resident in HBM."""
+    import torch
+    import paper_conf_icpp_zhangc0zx0025_b200 as W
+    from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+    stream = torch.cuda.current_stream(dev)
+    out, tot_ms, tot_flops = [], 0.0, 0.0
+    for shape in wl.ND_LAYERS:
+        name, N, C, D, H, Wd, K, T, R, S, pad = shape
+        X, dY = wl.make_inputs_nd(shape, "f16")
+        p = W.plan3d(N, C, D, H, Wd, K, T, R, S, pad, "f16")
+        Xg, Gg = torch.from_numpy(X).to(dev), torch.from_numpy(dY).to(dev)
+        dW = torch.empty((K, T, R, S, C), dtype=torch.float32, device=dev)
+        ws = torch.empty(max(16, p.workspace_bytes), dtype=torch.uint8, device=dev)
+        for _ in range(3):
+            W.bfc(p, Xg, Gg, dW, ws, stream)
+        ts = []
+        for _ in range(reps):
+            flush.fill_(7)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            W.bfc(p, Xg, Gg, dW, ws, stream)
+            b.record(stream)
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        ms = statistics.median(ts)
+        i = p.info
+        Z = i["Z"]
+        alg = 2 * (X.size + dY.size) + 4 * dW.numel() * (1 if Z == 1 else 2 * Z + 1)
+        t_roof = max(alg / (peaks["hbm_gbs"] * 1e9), i["ewm_flops"] / (peaks["bf16_tflops"] * 1e12))
+        out.append({"name": name, "ms": ms, "tflops": i["direct_flops"] / (ms * 1e-3) / 1e12,
+                    "kernel": p.kernel_name, "plan": repr(p), "roofline_frac": t_roof / (ms * 1e-3),
+                    "workspace_bytes": p.workspace_bytes})
+        tot_ms += ms
+        tot_flops += i["direct_flops"]
+    return {"workload": "nd_f16 (3-D BFC, winrs_plan3d)", "value": tot_flops / (tot_ms * 1e-3) / 1e12,
+            "unit": "TFLOPS", "ms_per_step": tot_ms, "steps": reps, "layers": out}
+
+
 def summarize(m, peaks, args):
     items = m["items"]
     layers = []
@@ -516,6 +556,8 @@ def run_winrs(args):
             cfg["compute_only_ms_per_step"] = m["compute_only_step_ms"]
             cfg["compute_only_tflops"] = m["job_flops"] / (m["compute_only_step_ms"] * 1e-3) / 1e12
             cfg["allreduce_share"] = 1.0 - m["compute_only_step_ms"] / m["step_ms"]
+        if world == 1 and not args.no_alongside and args.workload == "vgg":
+            cfg.setdefault("alongside", []).append(measure_nd(args, ctx["dev"], ctx["flush"], peaks))
         for wk, dt, a in alongside:
             cfg.setdefault("alongside", []).append({
                 "workload": f"{wk}_{dt}", "value": a["job_flops"] / (a["step_ms"] * 1e-3) / 1e12, "unit": "TFLOPS",

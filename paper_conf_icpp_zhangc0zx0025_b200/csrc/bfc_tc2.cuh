@@ -161,26 +161,31 @@ __device__ __forceinline__ void tma5(uint32_t dst, const CUtensorMap* m, uint64_
 // Image index img of the 2-D decomposition -> (inner, outer) TMA coordinates:
 // 2-D plans: (img, 0) of maps {ch, N, 1, H, W}; N-D plans (PAPER.md P@17805,
 // Level-2 dimension reduction): (depth slice img % Do, batch img / Do) of maps
-// {ch, D or Do, Nb, H, W}.  Past the end: outer = Nb (zero fill).
+// {ch, D or Do, Nb, H, W}.  Past the end: outer = Nb (zero fill).  Tracked
+// incrementally next to the producer's (n, u, h): a per-stage division on an
+// SM sub-partition shared with other warps cost ~30 % of the kernel (measured).
 struct ImgCoord {
     int a, b;
 };
-__device__ __forceinline__ ImgCoord img_coord(const Geometry& g, int img, bool in) {
-    const bool nd = g.T > 1 || g.D > 1;
-    const int inner = nd ? g.Do : g.N;
-    ImgCoord c;
-    c.a = in ? img % inner : 0;
-    c.b = in ? img / inner : (nd ? g.Nb : 1);
-    return c;
-}
-// X's inner coordinate for filter row fh: the depth slice shifted by the row's
-// depth tap fh / Rh (N-D), and the X row h + (fh % Rh) - pad.
-__device__ __forceinline__ int x_inner(const Geometry& g, int a, int fh) {
-    return (g.T > 1 || g.D > 1) ? a + fh / g.Rh - g.pad : a;
-}
-__device__ __forceinline__ int x_row(const Geometry& g, int h, int fh) {
-    return fh < g.R ? h + fh % g.Rh - g.pad : -(1 << 20);   // a slot past the last filter row: zero fill
-}
+struct ImgTracker {
+    int a, b, inner;
+    __device__ __forceinline__ void init(const Geometry& g, int img) {
+        inner = (g.T > 1 || g.D > 1) ? g.Do : g.N;
+        a = img % inner;
+        b = img / inner;
+    }
+    __device__ __forceinline__ void advance(int by, bool wrapped) {   // img += by (by divides inner)
+        a += by;
+        if (a >= inner) { a -= inner; ++b; }
+        if (wrapped) { a = 0; b = 0; }
+    }
+    __device__ __forceinline__ ImgCoord at(const Geometry& g, bool in) const {
+        ImgCoord c;
+        c.a = in ? a : 0;
+        c.b = in ? b : ((g.T > 1 || g.D > 1) ? g.Nb : 1);
+        return c;
+    }
+};
 __device__ __forceinline__ void fence_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void tc_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
@@ -405,6 +410,17 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         long long d = (long long)c_lo * KC;
         int n = 0, h = hs, u = 0;
         if (d < depth) depth_nhu((int)d, g.N, units, hs, &n, &h, &u);
+        ImgTracker itk;
+        itk.init(g, n);
+        // per X atom: depth-tap shift and height-tap row offset of its filter row
+        // (constant per CTA: no per-stage division)
+        int xdt[2], xdr[2];
+#pragma unroll
+        for (int a = 0; a < 2; ++a) {
+            const int fh = F == 2 ? fh_base + a : fh_base;
+            xdt[a] = (g.T > 1 || g.D > 1) ? fh / g.Rh - g.pad : 0;
+            xdr[a] = fh < g.R ? fh % g.Rh - g.pad : -(1 << 20);   // a slot past the last filter row: zero fill
+        }
         int s = 0;
         uint32_t ph = 0;
         for (int ch = c_lo; ch < c_hi; ++ch) {
@@ -414,7 +430,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             uint64_t* fb = &bars->full[s];
             const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
             const bool in = d < depth;               // past the end: outer image coordinate out of range (zero fill)
-            const ImgCoord ic = img_coord(g, n, in);
+            const ImgCoord ic = itk.at(g, in);
             const int hh = in ? h : hs;
             const int w0 = w_first + (in ? u : 0) * 2;
             if (elect_one()) {
@@ -426,10 +442,8 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 for (int a = 0; a < 2; ++a) {
                     // X window columns x0..x3 of atom a; an fh slot past the last
                     // filter row reads rows far outside (zero fill)
-                    const int fh = F == 2 ? fh_base + a : fh_base;
                     const int c0 = F == 2 ? c_base : c_base + a * 64;
-                    tma5(st + a * L::X_LBO, &tmX, fb, c0, x_inner(g, ic.a, fh), ic.b, x_row(g, hh, fh),
-                         w0 + fw0 - g.pad);
+                    tma5(st + a * L::X_LBO, &tmX, fb, c0, ic.a + xdt[a], ic.b, hh + xdr[a], w0 + fw0 - g.pad);
                 }
 #pragma unroll
                 for (int ka = 0; ka < L::NKL / 64; ++ka)   // dY unit columns w0, w0 + 1 of k atom ka
@@ -440,10 +454,13 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             TC2_TRACE(ch - c_lo, 1);
             d += KC;
             n += KC;
+            bool wrapped = false;
             while (n >= g.N) {
                 n -= g.N;
+                wrapped = true;
                 if (++u == units) { u = 0; ++h; }
             }
+            itk.advance(KC, wrapped);
             if (++s == L::S) { s = 0; ph ^= 1; }
         }
     } else if (warp == 1) {
@@ -743,6 +760,10 @@ bfc_tc2s_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
         long long d = (long long)c_lo * KC;
         int n = 0, h = hs, u = 0;
         if (d < depth) depth_nhu((int)d, g.N, units, hs, &n, &h, &u);
+        ImgTracker itk;
+        itk.init(g, n);
+        const int xdt = (g.T > 1 || g.D > 1) ? fh / g.Rh - g.pad : 0;   // per CTA, not per stage
+        const int xdr = fh < g.R ? fh % g.Rh - g.pad : -(1 << 20);
         int s = 0;
         uint32_t ph = 0;
         for (int ch = c_lo; ch < c_hi; ++ch) {
@@ -752,12 +773,12 @@ bfc_tc2s_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
             uint64_t* fb = &bars->full[s];
             const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
             const bool in = d < depth;
-            const ImgCoord ic = img_coord(g, n, in);
+            const ImgCoord ic = itk.at(g, in);
             const int hh = in ? h : hs;
             const int w0 = w_first + (in ? u : 0) * 2;
             if (elect_one()) {
                 mbar_expect_tx(fb, (uint32_t)L::TX_BYTES);
-                tma5(st + L::OFF_X, &tmX, fb, c_base, x_inner(g, ic.a, fh), ic.b, x_row(g, hh, fh), w0 + fw0 - g.pad);
+                tma5(st + L::OFF_X, &tmX, fb, c_base, ic.a + xdt, ic.b, hh + xdr, w0 + fw0 - g.pad);
                 tma5(st + L::OFF_Y, &tmY, fb, k_base, ic.a, ic.b, hh, w0);
                 tma5(st + L::OFF_Y + L::Y_LBO, &tmY, fb, k_base + 64, ic.a, ic.b, hh, w0);
             }
@@ -765,10 +786,13 @@ bfc_tc2s_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
             TC2_TRACE(ch - c_lo, 1);
             d += KC;
             n += KC;
+            bool wrapped = false;
             while (n >= g.N) {
                 n -= g.N;
+                wrapped = true;
                 if (++u == units) { u = 0; ++h; }
             }
+            itk.advance(KC, wrapped);
             if (++s == L::S) { s = 0; ph ^= 1; }
         }
     } else if (warp == 1) {

@@ -130,3 +130,30 @@ def sample_indices(layer: Layer, count: int, seed: int = 7) -> np.ndarray:
                     fixed.append(((k * R + r) * S + s) * C + c)
     rnd = g.integers(0, total, size=max(0, count - len(fixed)))
     return np.unique(np.concatenate([np.array(fixed, dtype=np.int64), rnd.astype(np.int64)]))
+
+
+# ---------------------------------------------------------------- N-D (3-D) layers
+# SURVEY §8(f) row 4 (PAPER.md P@17805, Level-2 dimension reduction): C3D-style
+# 3x3x3 layers, channels doubled when the map is halved (the paper's workload
+# structure), 16 depth slices, pad 1.  (name, N, C, D, H, W, K, T, R, S, pad)
+ND_LAYERS = [
+    ("c3d_128_28_f16", 8, 128, 16, 28, 28, 128, 3, 3, 3, 1),
+    ("c3d_256_14_f16", 8, 256, 16, 14, 14, 256, 3, 3, 3, 1),
+]
+
+
+def make_inputs_nd(shape, dtype: str = "f16", seed: int = 0):
+    """Seeded X [N,D,H,W,C] and dY [N,Do,Ho,Wo,K] for an N-D layer tuple of
+    ND_LAYERS: U[0,1) (dY x 1e-2 for 16-bit dtypes), rounded to the dtype."""
+    _, N, C, D, H, W, K, T, R, S, pad = shape
+    Do, Ho, Wo = D + 2 * pad - T + 1, H + 2 * pad - R + 1, W + 2 * pad - S + 1
+    gx = np.random.Generator(np.random.PCG64(3000017 + seed))
+    gy = np.random.Generator(np.random.PCG64(4000037 + seed))
+    X = gx.random((N, D, H, W, C), dtype=np.float32)
+    dY = gy.random((N, Do, Ho, Wo, K), dtype=np.float32)
+    if dtype in ("f16", "bf16"):
+        dY = dY * np.float32(1e-2)
+    if dtype == "bf16":
+        return round_to_bf16(X), round_to_bf16(dY)
+    dt = np_dtype(dtype)
+    return X.astype(dt), dY.astype(dt)
