@@ -32,6 +32,15 @@ an N-D BFC reduces to 2-D BFCs over the extra spatial axis)::
 ``bfc3d_numpy`` (one tensordot per filter tap) and ``bfc3d_bruteforce``; layouts
 NDHWC / NDHWC / KTRSC (Table 1 extended by the depth axis, R23).
 
+The forward and backward-data convolutions of PAPER.md §8 P@56407 ("with
+moderate modifications, WinRS can support FC and BDC"), plain definitions,
+stride 1, one symmetric pad (NHWC activations, KRSC weights)::
+
+    FC : Y[n, h, w, k]  = sum_{r, s, c} Xp[n, h + r - pad, w + s - pad, c] * Wt[k, r, s, c]
+    BDC: dX[n, i, j, c] = sum_{r, s, k} dYq[n, i - r + pad, j - s + pad, k] * Wt[k, r, s, c]
+
+(dYq = dY, zero outside [0, Ho) x [0, Wo)) — ``fc_numpy``, ``bdc_numpy``.
+
 Pins (tests/test_oracle.py): brute force == C == numpy (2-D and 3-D); torch
 conv3d_weight in FP64; the D = 1 reduction of the 3-D definition; impulse; all-ones
 closed form; adjoint identity against an independent forward convolution;
@@ -222,6 +231,44 @@ def bfc3d_bruteforce(X, dY, T: int, R: int, S: int, pad: int) -> np.ndarray:
                                             acc += Xl[n][a][i][j][c] * Gl[n][d][h][w][k]
                         out[k, t, r, s, c] = acc
     return out
+
+
+def fc_numpy(X: np.ndarray, Wt: np.ndarray, pad: int) -> np.ndarray:
+    """Forward convolution (correlation), FP64: one tensordot per filter tap."""
+    X = X.astype(np.float64)
+    Wt = Wt.astype(np.float64)
+    N, H, W, C = X.shape
+    K, R, S, C2 = Wt.shape
+    assert C2 == C
+    Ho, Wo = out_dims(H, W, R, S, pad)
+    Xp = np.zeros((N, H + 2 * pad, W + 2 * pad, C), dtype=np.float64)
+    Xp[:, pad:pad + H, pad:pad + W, :] = X
+    Y = np.zeros((N, Ho, Wo, K), dtype=np.float64)
+    for r in range(R):
+        for s in range(S):
+            Y += np.tensordot(Xp[:, r:r + Ho, s:s + Wo, :], Wt[:, r, s, :], axes=([3], [1]))
+    return Y
+
+
+def bdc_numpy(dY: np.ndarray, Wt: np.ndarray, pad: int, H: int, W: int) -> np.ndarray:
+    """Backward-data convolution (the adjoint of fc_numpy in X), FP64:
+    dX[n, i, j, c] = sum_{r, s, k} dY[n, i - r + pad, j - s + pad, k] Wt[k, r, s, c]."""
+    dY = dY.astype(np.float64)
+    Wt = Wt.astype(np.float64)
+    N, Ho, Wo, K = dY.shape
+    K2, R, S, C = Wt.shape
+    assert K2 == K and (Ho, Wo) == out_dims(H, W, R, S, pad)
+    dX = np.zeros((N, H, W, C), dtype=np.float64)
+    for r in range(R):
+        for s in range(S):
+            # output rows i with 0 <= i - r + pad < Ho
+            i0, i1 = max(0, r - pad), min(H, Ho + r - pad)
+            j0, j1 = max(0, s - pad), min(W, Wo + s - pad)
+            if i1 <= i0 or j1 <= j0:
+                continue
+            src = dY[:, i0 - r + pad:i1 - r + pad, j0 - s + pad:j1 - s + pad, :]
+            dX[:, i0:i1, j0:j1, :] += np.tensordot(src, Wt[:, r, s, :], axes=([3], [0]))
+    return dX
 
 
 def rel_max_err(got: np.ndarray, ref: np.ndarray) -> float:

@@ -217,3 +217,41 @@ def test_3d_impulse():
     Xp[:, pad:pad + D, pad:pad + H, pad:pad + W] = X
     assert np.array_equal(got[k0], Xp[n0, d0:d0 + T, h0:h0 + R, w0:w0 + S, :])
     assert np.all(got[1 - k0] == 0)
+
+
+# ============================================================== FC and BDC definitions
+CONV_SHAPES = [
+    # N, C, H, W, K, R, S, pad
+    (2, 3, 6, 7, 4, 3, 3, 1),
+    (1, 2, 5, 5, 3, 2, 3, 0),
+    (2, 4, 4, 6, 2, 3, 2, 2),
+]
+
+
+@pytest.mark.parametrize("shape", CONV_SHAPES)
+def test_fc_bdc_against_torch(shape):
+    """Library routines in FP64: torch conv2d (correlation) for FC and
+    torch.nn.grad.conv2d_input for BDC (NCHW / KCRS permuted to NHWC / KRSC)."""
+    N, C, H, W, K, R, S, pad = shape
+    Ho, Wo = O.out_dims(H, W, R, S, pad)
+    X = _rand((N, H, W, C), 21)
+    Wt = _rand((K, R, S, C), 22)
+    dY = _rand((N, Ho, Wo, K), 23)
+    tX, tW = torch.from_numpy(X).permute(0, 3, 1, 2), torch.from_numpy(Wt).permute(0, 3, 1, 2)
+    Y = torch.nn.functional.conv2d(tX, tW, padding=pad).permute(0, 2, 3, 1).numpy()
+    dX = torch.nn.grad.conv2d_input((N, C, H, W), tW, torch.from_numpy(dY).permute(0, 3, 1, 2),
+                                    padding=pad).permute(0, 2, 3, 1).numpy()
+    assert np.allclose(O.fc_numpy(X, Wt, pad), Y, rtol=1e-12, atol=1e-12)
+    assert np.allclose(O.bdc_numpy(dY, Wt, pad, H, W), dX, rtol=1e-12, atol=1e-12)
+
+
+def test_fc_bfc_bdc_adjoint_triangle():
+    """<FC(X, Wt), dY> = <X, BDC(dY, Wt)> = <Wt, BFC(X, dY)>: the three
+    convolutions of one layer are mutual adjoints."""
+    N, C, H, W, K, R, S, pad = 2, 3, 7, 6, 4, 3, 3, 1
+    Ho, Wo = O.out_dims(H, W, R, S, pad)
+    X, Wt, dY = _rand((N, H, W, C), 24), _rand((K, R, S, C), 25), _rand((N, Ho, Wo, K), 26)
+    a = float(np.sum(O.fc_numpy(X, Wt, pad) * dY))
+    b = float(np.sum(X * O.bdc_numpy(dY, Wt, pad, H, W)))
+    c = float(np.sum(Wt * O.bfc_c(X, dY, R, S, pad)))
+    assert abs(a - b) <= 1e-10 * abs(a) and abs(a - c) <= 1e-10 * abs(a)
