@@ -179,6 +179,53 @@ WINRS_API const char* winrs_version(void);
 /* Number of GPU kernel launches one winrs_bfc call of this plan issues. */
 WINRS_API int winrs_launch_count(winrs_plan_t plan);
 
+/* ---------------------------------------------------------------------------
+ * FC and BDC on the same machinery (§8 P@56407: "with moderate
+ * modifications, WinRS can support FC and BDC").  Stride 1, one symmetric pad,
+ * NHWC activations, KRSC weights, FP32 outputs:
+ *   FC : Y [N][Ho][Wo][K] = sum_{r,s,c} Xp[n][h+r-pad][w+s-pad][c] * Wt[k][r][s][c]
+ *   BDC: dX[N][H][W][C]   = sum_{r,s,k} dY[n][i-r+pad][j-s+pad][k] * Wt[k][r][s][c]
+ * (dY zero outside [0,Ho) x [0,Wo)).  Each is run as the BFC of a transposed
+ * problem (FC: N' = C, C' = N, R' x S' = Ho x Wo, the filter as dY'; BDC: the
+ * FC of dY with the spatially flipped filter and pad R-1-pad) between layout
+ * kernels; the BFC plan, kernels and reduction are the ones above unchanged.
+ * Constraints are the mapped BFC's: FC needs N % 4 (FP32) / % 8 (FP16, BF16),
+ * K likewise, and a kernel divisor n of Wo; BDC needs N and C aligned, a
+ * divisor n of W, R == S and pad <= R-1.  UNSUPPORTED otherwise. */
+typedef enum { WINRS_CONV_FC = 0, WINRS_CONV_BDC = 1 } winrs_conv_kind_t;
+typedef struct winrs_conv_plan_s* winrs_conv_plan_t;
+
+/* Plan an FC or BDC of the layer (N,C,H,W,K,R,S,pad) for the current device
+ * (or explicitly given properties).  On success *out owns a new plan. */
+WINRS_API winrs_status_t winrs_conv_plan(winrs_conv_kind_t kind, int N, int C, int H, int W, int K, int R, int S,
+                                         int pad, winrs_dtype_t dtype, winrs_conv_plan_t* out);
+WINRS_API winrs_status_t winrs_conv_plan_for_device(winrs_conv_kind_t kind, int N, int C, int H, int W, int K,
+                                                    int R, int S, int pad, winrs_dtype_t dtype,
+                                                    const winrs_device_t* dev, winrs_conv_plan_t* out);
+
+/* Workspace bytes (always > 0: it holds the transposed operands, the
+ * transposed FP32 result and the mapped BFC's bucket workspace). */
+WINRS_API size_t winrs_conv_workspace_bytes(winrs_conv_plan_t plan);
+
+/* The mapped BFC plan (owned by the conv plan; for winrs_plan_info). */
+WINRS_API winrs_status_t winrs_conv_bfc_plan(winrs_conv_plan_t plan, winrs_plan_t* bfc);
+
+/* GPU launches per winrs_fc / winrs_bdc call (3 layout kernels + the BFC's). */
+WINRS_API int winrs_conv_launch_count(winrs_conv_plan_t plan);
+
+/* Run asynchronously on `stream`.  X / dY / Wt device pointers in the plan's
+ * dtype; Y / dX device FP32, overwritten; workspace >= winrs_conv_workspace_bytes.
+ * All pointers 16-byte aligned, no aliasing.  INVALID_ARG for a null or
+ * misaligned pointer or a plan of the other kind, WORKSPACE for a null
+ * workspace, CUDA for a launch error. */
+WINRS_API winrs_status_t winrs_fc(winrs_conv_plan_t plan, const void* X, const void* Wt, float* Y,
+                                  void* workspace, void* stream);
+WINRS_API winrs_status_t winrs_bdc(winrs_conv_plan_t plan, const void* dY, const void* Wt, float* dX,
+                                   void* workspace, void* stream);
+
+/* Destroy a conv plan and its BFC plan (NULL is a no-op). */
+WINRS_API void winrs_conv_plan_destroy(winrs_conv_plan_t plan);
+
 #ifdef __cplusplus
 }
 #endif

@@ -20,15 +20,16 @@ from . import _lib
 from ._lib import WinrsError, DTYPES
 
 __all__ = ["Plan", "plan", "plan_for_device", "plan3d", "plan3d_for_device", "bfc", "bfc_host", "as_kcrs", "as_krsc", "bfc_data_parallel", "shard_range",
-           "bfc_k_sharded",
+           "bfc_k_sharded", "ConvPlan", "conv_plan", "conv_plan_for_device", "fc", "bdc", "emulate_conv",
            "WinrsError", "version", "emulate", "transform", "kernel_names"]
 
 
 class Plan:
     """Owns a winrs_plan_t.  `info` mirrors winrs_plan_info_t."""
 
-    def __init__(self, handle: ctypes.c_void_p):
+    def __init__(self, handle: ctypes.c_void_p, owned: bool = True):
         self._h = handle
+        self._owned = owned
         inf = _lib.PlanInfoT()
         _lib.check(_lib.lib().winrs_plan_info(self._h, ctypes.byref(inf)), "winrs_plan_info")
         self.info = {name: getattr(inf, name) for name, _ in _lib.PlanInfoT._fields_}
@@ -61,7 +62,7 @@ class Plan:
     def __del__(self):
         h, self._h = getattr(self, "_h", None), None
         try:
-            if h and _lib is not None and _lib._lib is not None:
+            if h and getattr(self, "_owned", False) and _lib is not None and _lib._lib is not None:
                 _lib._lib.winrs_plan_destroy(h)
         except Exception:   # interpreter shutdown
             pass
@@ -293,6 +294,118 @@ def bfc_data_parallel(X_shard, dY_shard, R: int, S: int, pad: int, dtype: str = 
     if dist.is_initialized() and dist.get_world_size(group) > 1:
         dist.all_reduce(as_krsc(dW), op=dist.ReduceOp.SUM, group=group)   # the contiguous KRSC storage
     return dW
+
+
+class ConvPlan:
+    """Owns a winrs_conv_plan_t (FC or BDC on the BFC machinery, include/winrs.h).
+    `bfc` is the mapped BFC Plan (owned by this object)."""
+
+    def __init__(self, handle: ctypes.c_void_p, kind: str, dims):
+        self._h = handle
+        self.kind = kind
+        self.N, self.C, self.H, self.W, self.K, self.R, self.S, self.pad, self.dtype = dims
+        self.Ho = self.H + 2 * self.pad - self.R + 1
+        self.Wo = self.W + 2 * self.pad - self.S + 1
+        b = ctypes.c_void_p()
+        _lib.check(_lib.lib().winrs_conv_bfc_plan(self._h, ctypes.byref(b)), "winrs_conv_bfc_plan")
+        self.bfc = Plan(b, owned=False)   # the mapped BFC plan, owned by the conv plan
+
+    @property
+    def workspace_bytes(self) -> int:
+        return int(_lib.lib().winrs_conv_workspace_bytes(self._h))
+
+    @property
+    def launch_count(self) -> int:
+        return int(_lib.lib().winrs_conv_launch_count(self._h))
+
+    @property
+    def kernel_name(self) -> str:
+        return self.bfc.kernel_name
+
+    def __del__(self):
+        h, self._h = getattr(self, "_h", None), None
+        try:
+            if h and _lib is not None and _lib._lib is not None:
+                _lib._lib.winrs_conv_plan_destroy(h)
+        except Exception:
+            pass
+
+
+_CONV_KINDS = {"fc": 0, "bdc": 1}
+
+
+def conv_plan(kind: str, N, C, H, W, K, R, S, pad, dtype: str = "f16") -> ConvPlan:
+    """winrs_conv_plan: FC ("fc") or BDC ("bdc") of the layer on the current device."""
+    h = ctypes.c_void_p()
+    _lib.check(_lib.lib().winrs_conv_plan(_CONV_KINDS[kind], N, C, H, W, K, R, S, pad, DTYPES[dtype],
+                                          ctypes.byref(h)), "winrs_conv_plan")
+    return ConvPlan(h, kind, (N, C, H, W, K, R, S, pad, dtype))
+
+
+def conv_plan_for_device(kind: str, N, C, H, W, K, R, S, pad, dtype: str = "f16", num_sms: int = 148,
+                         cc=(10, 0)) -> ConvPlan:
+    dev = _lib.DeviceT(num_sms, cc[0], cc[1])
+    h = ctypes.c_void_p()
+    _lib.check(_lib.lib().winrs_conv_plan_for_device(_CONV_KINDS[kind], N, C, H, W, K, R, S, pad, DTYPES[dtype],
+                                                     ctypes.byref(dev), ctypes.byref(h)),
+               "winrs_conv_plan_for_device")
+    return ConvPlan(h, kind, (N, C, H, W, K, R, S, pad, dtype))
+
+
+def _conv_run(cp: ConvPlan, fn: str, inp, Wt, out_shape, workspace, stream):
+    import torch
+    tdt = {"f32": torch.float32, "f16": torch.float16, "bf16": torch.bfloat16}[cp.dtype]
+    ishape = (cp.N, cp.H, cp.W, cp.C) if cp.kind == "fc" else (cp.N, cp.Ho, cp.Wo, cp.K)
+    In = _as_cl(inp, ishape, "input")
+    Wn = _as_krsc(Wt, cp.K, cp.C, cp.R, cp.S, "Wt")
+    if In.dtype != tdt or Wn.dtype != tdt:
+        raise TypeError(f"input and Wt must be {tdt} for this plan")
+    if not (In.is_cuda and Wn.is_cuda) or In.device != Wn.device:
+        raise ValueError("input and Wt must be CUDA tensors on one device")
+    if stream is None:
+        stream = torch.cuda.current_stream(In.device)
+    sp = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+    ts = stream if isinstance(stream, torch.cuda.Stream) else None
+    with torch.cuda.stream(ts) if ts is not None else _nullctx():
+        out = torch.empty(out_shape, dtype=torch.float32, device=In.device)
+        if workspace is None:
+            workspace = torch.empty(cp.workspace_bytes, dtype=torch.uint8, device=In.device)
+    if workspace.numel() * workspace.element_size() < cp.workspace_bytes or workspace.device != In.device:
+        raise ValueError(f"workspace must be >= {cp.workspace_bytes} bytes on the input's device")
+    _lib.check(getattr(_lib.lib(), fn)(cp._h, In.data_ptr(), Wn.data_ptr(), out.data_ptr(), workspace.data_ptr(),
+                                       sp), fn)
+    if ts is not None:
+        out.record_stream(ts)
+        workspace.record_stream(ts)
+    return out
+
+
+def fc(cp: ConvPlan, X, Wt, workspace=None, stream=None):
+    """winrs_fc: Y [N,Ho,Wo,K] FP32 (NHWC) = conv(X [N,H,W,C], Wt [K,R,S,C])."""
+    assert cp.kind == "fc"
+    return _conv_run(cp, "winrs_fc", X, Wt, (cp.N, cp.Ho, cp.Wo, cp.K), workspace, stream)
+
+
+def bdc(cp: ConvPlan, dY, Wt, workspace=None, stream=None):
+    """winrs_bdc: dX [N,H,W,C] FP32 (NHWC) from dY [N,Ho,Wo,K] and Wt [K,R,S,C]."""
+    assert cp.kind == "bdc"
+    return _conv_run(cp, "winrs_bdc", dY, Wt, (cp.N, cp.H, cp.W, cp.C), workspace, stream)
+
+
+def emulate_conv(cp: ConvPlan, inp, Wt):
+    """FP64 host emulation of winrs_fc / winrs_bdc: the C library's operand
+    mapping (include/winrs.h) in numpy, then winrs_debug_emulate of the mapped
+    BFC plan (numpy float64 in, NHWC out)."""
+    import numpy as np
+    inp = np.asarray(inp, dtype=np.float64)
+    Wt = np.asarray(Wt, dtype=np.float64)
+    Xp = np.ascontiguousarray(inp.transpose(3, 1, 2, 0))            # [ch][h][w][n]
+    if cp.kind == "fc":
+        Gp = np.ascontiguousarray(Wt.transpose(3, 1, 2, 0))         # [C][R][S][K]
+    else:
+        Gp = np.ascontiguousarray(Wt[:, ::-1, ::-1, :])             # [K][R][S][C], (r,s) reversed
+    out = emulate(cp.bfc, Xp, Gp)                             # [K'][R'][S'][N]
+    return np.ascontiguousarray(out.transpose(3, 1, 2, 0))
 
 
 def version() -> str:

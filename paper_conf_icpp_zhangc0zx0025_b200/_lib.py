@@ -58,6 +58,14 @@ SYMBOLS = [
     ("winrs_status_string", ctypes.c_char_p, [_i]),
     ("winrs_version", ctypes.c_char_p, []),
     ("winrs_launch_count", _i, [_p]),
+    ("winrs_conv_plan", _i, [_i] * 9 + [_i, ctypes.POINTER(_p)]),
+    ("winrs_conv_plan_for_device", _i, [_i] * 9 + [_i, ctypes.POINTER(DeviceT), ctypes.POINTER(_p)]),
+    ("winrs_conv_workspace_bytes", _s, [_p]),
+    ("winrs_conv_bfc_plan", _i, [_p, ctypes.POINTER(_p)]),
+    ("winrs_conv_launch_count", _i, [_p]),
+    ("winrs_fc", _i, [_p, _p, _p, _p, _p, _p]),
+    ("winrs_bdc", _i, [_p, _p, _p, _p, _p, _p]),
+    ("winrs_conv_plan_destroy", None, [_p]),
     # winrs_debug.h
     ("winrs_debug_emulate", _i, [_p, _p, _p, _p]),
     ("winrs_debug_transform", _i, [_i, _i, _i, _i, _p, _p]),
