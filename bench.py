@@ -214,7 +214,8 @@ def layer_roofline(l, p, ms, peaks):
         l2_bytes = depth / 16 * 2 * (8192 + 8192)         # per pair stage: each CTA X 8 KB + dY 8 KB
         alu_ops = depth * (256 + 128 * 2)                 # FT over 256 k, IT over 128 c (half2)
     elif "_v2" in name:
-        cg = int(name.split("_v2")[1][0])                 # CTAs per UMMA (2: cta_group::2 pair)
+        tag = name.split("_v2")[1][0]                     # CTAs per UMMA (2: cta_group::2 pair); t: Xhat in TMEM
+        cg = 1 if tag == "t" else int(tag)
         fhs = int(name.split("x")[-1].rstrip("fh")) * cg if bm == 64 else 1
         rows = sum(_rows_union(l, range(g, min(l.R, g + fhs))) for g in range(0, l.R, fhs))
         depth = rows * units * l.N * kb * cb * ft        # depth entries x (pair) tiles

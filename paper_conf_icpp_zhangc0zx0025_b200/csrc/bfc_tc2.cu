@@ -60,7 +60,7 @@ static int images_per_box(const Geometry& g) {
     return (nd ? g.Do : g.N) % KC == 0 ? KC : 0;
 }
 
-template <int F, int NK, bool BF, int CG>
+template <int F, int NK, bool BF, int CG, bool TA = false>
 cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
     using L = Lay<F, NK, CG>;
     const long long grid = num_ctas(g);
@@ -74,7 +74,7 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
     CUtensorMap mX, mY;
     if (!make_maps(g, X, dY, BF, &mX, &mY)) return cudaErrorInvalidValue;
     static std::atomic<unsigned long long> done{0};
-    auto k = bfc_tc2_kernel<F, NK, BF, CG>;
+    auto k = bfc_tc2_kernel<F, NK, BF, CG, TA>;
     cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
     if (e != cudaSuccess) return e;
     const int cluster = CG * g.csplit;
@@ -136,7 +136,12 @@ cudaError_t launch_sw(const Geometry& g, const void* X, const void* dY, float* d
     {DT, 4, 3, 2, 0, 0, 0, NK, (F == 1 ? ::winrs::tc2::MROWS * CG : ::winrs::tc2::MROWS / F),            \
      ::winrs::tc2::NTHREADS, 1, 1, (size_t)::winrs::tc2::Lay<F, NK, CG>::BYTES,                          \
      &::winrs::tc2::launch<F, NK, BF, CG>,                                                                \
-     PFX "_O4(3,2)_v2" #CG "_" #NK "x" #F "fh", (F == 1 ? 1 : F * CG), CG}
+     PFX "_O4(3,2)_v2" #CG "_" #NK "x" #F "fh", (F == 1 ? 1 : F * CG), CG, 0}
+// Xhat in TMEM (TA): single CTA, NK = 64
+#define WINRS_TC2T_ENTRY(DT, BF, PFX, F)                                                                  \
+    {DT, 4, 3, 2, 0, 0, 0, 64, ::winrs::tc2::MROWS / F, ::winrs::tc2::NTHREADS, 1, 1,                     \
+     (size_t)::winrs::tc2::Lay<F, 64, 1>::BYTES, &::winrs::tc2::launch<F, 64, BF, 1, true>,              \
+     PFX "_O4(3,2)_v2t_64x" #F "fh", F, 1, 1}
 
 #ifdef WINRS_TC2_TRACE
 extern "C" __attribute__((visibility("default"))) int winrs_tc2_trace(int cta, long long* out) {
@@ -162,9 +167,13 @@ const KernelEntry* tc2_entries(int* n) {
         WINRS_TC2_ENTRY(2, true, "bf16tc", 2, 128, 2),
         // swapped CTA pair: 256 k x 128 c (What rows split, the Xhat side shared)
         {1, 4, 3, 2, 0, 0, 0, 256, 128, ::winrs::tc2::NTHREADS, 1, 1, (size_t)::winrs::tc2::LaySw::BYTES,
-         &::winrs::tc2::launch_sw<false>, "f16tc_O4(3,2)_v2s_256x128", 1, 2},
+         &::winrs::tc2::launch_sw<false>, "f16tc_O4(3,2)_v2s_256x128", 1, 2, 0},
         {2, 4, 3, 2, 0, 0, 0, 256, 128, ::winrs::tc2::NTHREADS, 1, 1, (size_t)::winrs::tc2::LaySw::BYTES,
-         &::winrs::tc2::launch_sw<true>, "bf16tc_O4(3,2)_v2s_256x128", 1, 2},
+         &::winrs::tc2::launch_sw<true>, "bf16tc_O4(3,2)_v2s_256x128", 1, 2, 0},
+        WINRS_TC2T_ENTRY(1, false, "f16tc", 1),
+        WINRS_TC2T_ENTRY(1, false, "f16tc", 2),
+        WINRS_TC2T_ENTRY(2, true, "bf16tc", 1),
+        WINRS_TC2T_ENTRY(2, true, "bf16tc", 2),
     };
     *n = sizeof(e) / sizeof(e[0]);
     return e;

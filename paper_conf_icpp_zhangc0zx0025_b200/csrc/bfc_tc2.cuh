@@ -220,6 +220,36 @@ __device__ __forceinline__ void umma(uint32_t d, uint64_t a, uint64_t b, uint32_
             "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n"
             :: "r"(d), "l"(a), "l"(b), "r"(idesc<NK, BF, NEG, CG>()), "r"(acc));
 }
+// A operand from TMEM (the TA kernels): A K-major in 128 lanes x 8 columns
+// (lane = row m, column j = depth entries 2j, 2j + 1), B MN-major SW128.
+template <int NK, bool BF>
+__host__ __device__ constexpr uint32_t idesc_ta() {
+    return (1u << 4) | ((BF ? 1u : 0u) << 7) | ((BF ? 1u : 0u) << 10) | (1u << 16) | ((uint32_t)(NK >> 3) << 17) |
+           ((uint32_t)(MROWS >> 4) << 24);
+}
+template <int NK, bool BF>
+__device__ __forceinline__ void umma_ta(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t acc) {
+    asm volatile(
+        "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n"
+        :: "r"(d), "r"(a_tmem), "l"(b), "r"(idesc_ta<NK, BF>()), "r"(acc));
+}
+// ldmatrix.x4.trans: thread t receives, of matrix i (row addresses from
+// threads 8i..8i+7), the 16-bit elements (row 2(t%4), column t/4) and (row
+// 2(t%4) + 1, column t/4) packed -- rows = depth entries, columns = channels.
+__device__ __forceinline__ void ldsm_x4_t(uint32_t addr, uint32_t (&r)[4]) {
+    asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]) : "r"(addr));
+}
+// tcgen05.st 16x256b (probed on B200, tools/microbench/tmem_a.cu): thread t
+// writes r0, r1 to lane t/4, columns 2(t%4), 2(t%4) + 1 and r2, r3 to lane
+// t/4 + 8, same columns.
+__device__ __forceinline__ void tmem_st16x256(uint32_t taddr, const uint32_t (&r)[4]) {
+    asm volatile("tcgen05.st.sync.aligned.16x256b.x1.b32 [%0], {%1, %2, %3, %4};"
+                 :: "r"(taddr), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]) : "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
 // Commit: arrives on `bar` once every MMA issued so far completed; for a CTA
 // pair on the barrier at the same offset in both CTAs (mask = the pair).
 template <int CG = 1>
@@ -326,11 +356,18 @@ __device__ __forceinline__ void depth_nhu(int d, int N, int units, int hs, int* 
     *h = hs + t / units;
 }
 
-template <int F, int NK, bool BF, int CG = 1>
+// TA = true: the transformed X operand (Xhat) goes to TMEM (tcgen05.st) and
+// the MMAs read A from there: the IT's shared-memory write-back and the MMAs'
+// A reads leave the shared-memory port.  TMEM: 4 NK
+// accumulator columns + S ring slots x 4 xi x 8 columns (NK = 64: 256 + 256).
+template <int F, int NK, bool BF, int CG = 1, bool TA = false>
 __global__ void __launch_bounds__(NTHREADS, 1)
 bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX,
                const __grid_constant__ CUtensorMap tmY) {
     using L = Lay<F, NK, CG>;
+    static_assert(!TA || (CG == 1 && NK == 64 && L::S == 8), "TA: single CTA, NK = 64, 8-slot ring");
+    constexpr uint32_t TMEM_ALLOC = TA ? 512u : (uint32_t)L::TMEM_COLS;
+    constexpr uint32_t A_COL = 4 * NK;          // TA: first A ring column
     extern __shared__ uint8_t smem_raw[];
     // 1 KB-aligned base (SW128 atoms, TMA swizzle pattern)
     const uint32_t raw_s = su(smem_raw);
@@ -377,6 +414,8 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     }
     if (CG == 2 && threadIdx.x == 0 && e == 0)   // the leader's opfull gathers both CTAs' FT warps
         for (int s = 0; s < L::S; ++s) mbar_init(&bars->opfull[s], 2);
+    if (TA && threadIdx.x == 0)                  // TA: the four lane-quarter warps of a group
+        for (int s = 0; s < L::S; ++s) mbar_init(&bars->opfull[s], 4);
     if (warp == 0 && lane == 0) {
         asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
         asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
@@ -388,7 +427,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
         } else {
             asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
-                         :: "r"(su(&bars->tmem_base)), "r"(L::TMEM_COLS));
+                         :: "r"(su(&bars->tmem_base)), "r"(TMEM_ALLOC));
             asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
         }
     }
@@ -485,7 +524,13 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             const uint64_t w2d = desc_sw128(st + L::OFF_Y, L::Y_LBO, 1024), w3d = w2d + (L::ATOM >> 4);
             if (elect_one()) {
 #ifndef WINRS_TC2_NO_MMA   // debug ablation: no tensor-core work (barrier protocol kept)
-              if (!WINRS_TC2_ITM) {   // Xhat[xi] (IT done in place by the FT warps) x What[xi]
+              if (TA) {               // Xhat[xi] from the TMEM ring slot x What[xi]
+                const uint32_t a = tmem + A_COL + (uint32_t)(s * 32);
+                umma_ta<NK, BF>(tmem + 0 * NK, a + 0, w0d, acc);
+                umma_ta<NK, BF>(tmem + 1 * NK, a + 8, w1d, acc);
+                umma_ta<NK, BF>(tmem + 2 * NK, a + 16, w2d, acc);
+                umma_ta<NK, BF>(tmem + 3 * NK, a + 24, w3d, acc);
+              } else if (!WINRS_TC2_ITM) {   // Xhat[xi] (IT done in place by the FT warps) x What[xi]
                 umma<NK, BF, false, CG>(tmem + 0 * NK, x0, w0d, acc);
                 umma<NK, BF, false, CG>(tmem + 1 * NK, x1, w1d, acc);
                 umma<NK, BF, false, CG>(tmem + 2 * NK, x2, w2d, acc);
@@ -528,6 +573,69 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         constexpr int IPT = KO * KC / 32;           // items per lane: 8 (NK 128) / 4 (NK 64 or a pair)
         static_assert(L::S <= NTX, "one FT warp per ring slot");
         const int tw = warp - 2;
+        if constexpr (TA) {
+            // Two groups of four warps take alternate stages (group G: slots
+            // s = G, G + 2, ...); warp q = warp % 4 of a group owns TMEM lanes
+            // 32q..32q+31 = A rows (fh slot / channel half q / 2, channels
+            // 32 (q % 2) ..), the only lanes it may write.  Per 16-row half:
+            // four ldmatrix.x4.trans (x0..x3) give each thread two channels x
+            // four depth entries of every column, already in the 16x256b
+            // fragment order (matrix i: channel octet o0 + i/2, depth rows
+            // permuted so that lane t/4's columns 2(t%4), 2(t%4)+1 hold depth
+            // entries 4(t%4)..4(t%4)+3, i.e. column j = entries 2j, 2j+1); the
+            // IT runs on the packed registers and 4 stores fill the slot's
+            // xi = 0..3 A columns.  Ring safety as below: slot s is refilled
+            // only after the MMAs of this group's previous stage in it.
+            const int G = tw >> 2, q = warp & 3;
+            const int i4 = lane >> 3, rho = lane & 7;
+            const int img = 4 * (rho >> 1) + (rho & 1) + 2 * (i4 & 1);
+            uint32_t xoff[2];
+#pragma unroll
+            for (int hf = 0; hf < 2; ++hf) {
+                const int oct = 4 * (q & 1) + 2 * hf + (i4 >> 1);
+                xoff[hf] = (uint32_t)((q >> 1) * L::X_LBO) + opoff(oct, img, 0);
+            }
+            const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16) + A_COL;
+            const int it = q * 32 + lane;           // FT item: depth it / KO, k octet it % KO (KO * KC = 128)
+            const uint32_t foff = opoff(it % KO, it / KO, L::Y_LBO);
+            int s = G;
+            uint32_t ph = 0;
+            for (int ch = c_lo + G; ch < c_hi; ch += 2) {
+                mbar_wait(&bars->full[s], ph);
+                tc_after();
+                TC2_JITTER(ch, warp);
+                if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
+                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+#pragma unroll
+                for (int hf = 0; hf < 2; ++hf) {
+                    uint32_t x[4][4];
+#pragma unroll
+                    for (int c = 0; c < 4; ++c) ldsm_x4_t(st + xoff[hf] + c * L::ATOM, x[c]);
+                    uint32_t o[4][4];
+#pragma unroll
+                    for (int r = 0; r < 4; ++r) {
+                        o[0][r] = P16<BF>::add(x[1][r], x[2][r]);
+                        o[1][r] = P16<BF>::sub(x[2][r], x[1][r]);
+                        o[2][r] = P16<BF>::sub(x[0][r], x[2][r]);
+                        o[3][r] = P16<BF>::sub(x[3][r], x[1][r]);
+                    }
+                    const uint32_t ta = trow + ((uint32_t)(hf * 16) << 16) + (uint32_t)(s * 32);
+#pragma unroll
+                    for (int xi = 0; xi < 4; ++xi) tmem_st16x256(ta + xi * 8, o[xi]);
+                }
+                const uint4 w0 = lds16(st + L::OFF_Y + foff), w1 = lds16(st + L::OFF_Y + L::ATOM + foff);
+                sts16(st + L::OFF_F + foff, vadd<BF>(w0, w1));
+                sts16(st + L::OFF_F + L::ATOM + foff, vsub<BF>(w0, w1));
+                tmem_wait_st();
+                fence_async();
+                tc_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&bars->opfull[s]);
+                if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 3);
+                s += 2;
+                if (s >= L::S) { s -= L::S; ph ^= 1; }
+            }
+        } else {
         uint32_t ph = 0;
         for (int ch = c_lo + tw; tw < L::S && ch < c_hi; ch += L::S) {
             const int s = tw;
@@ -585,6 +693,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 else mbar_arrive(&bars->opfull[s]);
             }
             if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 3);
+        }
         }
         // ============================ epilogue ================================
         mbar_wait(&bars->accfull, 0);
@@ -661,7 +770,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         if constexpr (CG == 2)
             asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" :: "r"(tmem), "r"(L::TMEM_COLS));
         else
-            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem), "r"(L::TMEM_COLS));
+            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem), "r"(TMEM_ALLOC));
     }
 }
 

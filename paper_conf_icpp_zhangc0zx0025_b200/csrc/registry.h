@@ -25,6 +25,7 @@ struct KernelEntry {
     int fhs;                   // filter rows per tile (fh group; 0 = 1: one row); > 0 marks the
                                // second-generation tcgen05 kernels (bfc_tc2.cuh), which need N % 16 == 0
     int cg;                    // CTAs per UMMA: 2 = cta_group::2 pair (0 = 1)
+    int ta;                    // 1: tc2 kernel with the transformed X operand in TMEM (bfc_tc2.cuh TA)
 };
 
 // All entries (FP32 and FP16), terminated by count.

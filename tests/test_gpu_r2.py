@@ -21,7 +21,8 @@ from conftest import record_err
 pytestmark = pytest.mark.gpu
 
 TOL = {"f32": 1e-4, "f16": 2e-2, "bf16": 2e-2}
-ENV_KEYS = ("WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_TC_GEN", "WINRS_FORCE_CG")
+ENV_KEYS = ("WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_TC_GEN", "WINRS_FORCE_CG",
+            "WINRS_FORCE_TA")
 
 
 def _dev(a, dtype):
@@ -92,8 +93,45 @@ TC2 = [
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
 @pytest.mark.parametrize("name,ov,env", TC2, ids=[c[0] for c in TC2])
 def test_tc2(name, ov, env, dtype, monkeypatch):
+    """Xhat in shared memory (the TA variant is covered by test_tc2_ta)."""
     layer = BASE.with_(name="tc2_" + name, dtype=dtype, **ov)
-    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2"), expect_kernel="_v2")
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA="0"), expect_kernel="_v2")
+
+
+# Xhat in TMEM (bfc_tc2.cuh TA: ldmatrix.trans -> IT -> tcgen05.st, A operand from TMEM), NK = 64 tiles
+TA = [
+    ("l1", dict(N=16), {"WINRS_FORCE_TILE": "64x64"}),
+    ("l1_f1_cs2", dict(N=16), {"WINRS_FORCE_TILE": "64x128", "WINRS_FORCE_CSPLIT": "2"}),
+    ("l1_cs8", dict(N=32), {"WINRS_FORCE_TILE": "64x64", "WINRS_FORCE_CSPLIT": "8"}),
+    ("ragged_f2", dict(N=16, C=40, K=136, H=20, W=17), {"WINRS_FORCE_TILE": "64x64"}),
+    ("ragged_f1", dict(N=16, C=200, K=72, H=13, W=11), {"WINRS_FORCE_TILE": "64x128", "WINRS_FORCE_CSPLIT": "3"}),
+    ("pad0", dict(N=16, C=64, K=64, H=20, W=20, pad=0), {"WINRS_FORCE_TILE": "64x64"}),
+    ("s6_ftiles2", dict(N=16, C=64, K=64, H=16, W=16, R=3, S=6, pad=2), {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_TILE": "64x64"}),
+    ("r5_f2", dict(N=16, C=64, K=128, H=16, W=16, R=5, S=3, pad=2), {"WINRS_FORCE_TILE": "64x64"}),
+    ("r1", dict(N=16, C=64, K=64, H=12, W=12, R=1, S=3, pad=0), {"WINRS_FORCE_TILE": "64x128"}),
+    ("n32_z5", dict(N=32, C=64, K=64, H=30, W=30), {"WINRS_FORCE_Z": "5", "WINRS_FORCE_TILE": "64x64"}),
+    ("n48_cs4", dict(N=48, C=128, K=64, H=12, W=12), {"WINRS_FORCE_CSPLIT": "4", "WINRS_FORCE_TILE": "64x128"}),
+]
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+@pytest.mark.parametrize("name,ov,env", TA, ids=[c[0] for c in TA])
+def test_tc2_ta(name, ov, env, dtype, monkeypatch):
+    layer = BASE.with_(name="ta_" + name, dtype=dtype, **ov)
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA="1"), expect_kernel="_v2t_")
+
+
+@pytest.mark.parametrize("name,ov,env", TA[:4], ids=[c[0] for c in TA[:4]])
+def test_tc2_ta_matches_smem_variant(name, ov, env, monkeypatch):
+    """Same plan geometry, Xhat in TMEM vs in shared memory: the same packed
+    16-bit IT values and the same MMA depth order, so bitwise identical dW."""
+    layer = BASE.with_(name="ta_eq_" + name, **ov)
+    X, dY = wl.make_inputs(layer)
+    out = []
+    for ta in ("0", "1"):
+        p = _plan(layer, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA=ta), monkeypatch)
+        out.append(W.as_krsc(W.bfc(p, _dev(X, "f16"), _dev(dY, "f16"))).cpu().numpy())
+    assert np.array_equal(out[0], out[1])
 
 
 @pytest.mark.parametrize("name,ov,env", TC2[:8], ids=[c[0] for c in TC2[:8]])
@@ -244,6 +282,8 @@ ND = [
     (1, 256, 16, 5, 5, 256, 3, 3, 3, 1, {"WINRS_FORCE_TILE": "256x128"}),       # swapped CTA pair
     (1, 40, 17, 9, 8, 24, 2, 2, 3, 1, {"WINRS_FORCE_Z": "3"}),                  # Do = 18 -> padded below
     (2, 16, 18, 6, 6, 16, 3, 1, 3, 0, {}),                                      # pad 0, R = 1
+    (1, 64, 16, 10, 11, 64, 3, 3, 3, 1, {"WINRS_FORCE_TA": "0"}),              # Xhat in shared memory
+    (2, 64, 16, 7, 9, 64, 3, 3, 3, 1, {"WINRS_FORCE_TA": "1", "WINRS_FORCE_TILE": "64x64"}),   # Xhat in TMEM
 ]
 
 
