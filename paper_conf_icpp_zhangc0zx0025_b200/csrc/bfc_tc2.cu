@@ -46,9 +46,11 @@ static bool make_map(CUtensorMap* m, const void* base, int A, int B, int H, int 
               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 // The X and dY maps of a plan (2-D or N-D).
-static bool make_maps(const Geometry& g, const void* X, const void* dY, bool bf, CUtensorMap* mX, CUtensorMap* mY) {
+// xbn: images per X box (TA kernels: 8, two boxes per stage and atom).
+static bool make_maps(const Geometry& g, const void* X, const void* dY, bool bf, CUtensorMap* mX, CUtensorMap* mY,
+                      int xbn = KC) {
     const bool nd = g.T > 1 || g.D > 1;
-    return make_map(mX, X, nd ? g.D : g.N, nd ? g.Nb : 1, g.H, g.W, g.C, g.C, 4, KC, bf) &&
+    return make_map(mX, X, nd ? g.D : g.N, nd ? g.Nb : 1, g.H, g.W, g.C, g.C, 4, xbn, bf) &&
            make_map(mY, dY, nd ? g.Do : g.N, nd ? g.Nb : 1, g.Ho, g.Wo, g.K, g.ldy, 2, KC, bf);
 }
 
@@ -62,7 +64,7 @@ static int images_per_box(const Geometry& g) {
 
 template <int F, int NK, bool BF, int CG, bool TA = false>
 cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
-    using L = Lay<F, NK, CG>;
+    using L = Lay<F, NK, CG, TA>;
     const long long grid = num_ctas(g);
     if (grid <= 0) return cudaSuccess;
     Args a;
@@ -72,7 +74,7 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
     a.nb = images_per_box(g);
     if (a.nb == 0 || g.a0 != 4 || g.n0 != 3 || g.r0 != 2 || g.a1 != 0) return cudaErrorInvalidValue;
     CUtensorMap mX, mY;
-    if (!make_maps(g, X, dY, BF, &mX, &mY)) return cudaErrorInvalidValue;
+    if (!make_maps(g, X, dY, BF, &mX, &mY, TA ? 8 : KC)) return cudaErrorInvalidValue;
     static std::atomic<unsigned long long> done{0};
     auto k = bfc_tc2_kernel<F, NK, BF, CG, TA>;
     cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
@@ -140,7 +142,7 @@ cudaError_t launch_sw(const Geometry& g, const void* X, const void* dY, float* d
 // Xhat in TMEM (TA): single CTA, NK = 64
 #define WINRS_TC2T_ENTRY(DT, BF, PFX, F)                                                                  \
     {DT, 4, 3, 2, 0, 0, 0, 64, ::winrs::tc2::MROWS / F, ::winrs::tc2::NTHREADS, 1, 1,                     \
-     (size_t)::winrs::tc2::Lay<F, 64, 1>::BYTES, &::winrs::tc2::launch<F, 64, BF, 1, true>,              \
+     (size_t)::winrs::tc2::Lay<F, 64, 1, true>::BYTES, &::winrs::tc2::launch<F, 64, BF, 1, true>,              \
      PFX "_O4(3,2)_v2t_64x" #F "fh", F, 1, 1}
 
 #ifdef WINRS_TC2_TRACE

@@ -45,8 +45,8 @@
 //     phase-parity wait can alias (safe by construction; round 1's
 //     dynamically handed-out units needed a timing argument).
 //
-// Warp roles (320 threads, one CTA per SM):
-//   warp 0     TMA producer (one lane per box)
+// Warp roles (352 threads, one CTA per SM):
+//   warps 0,10 TMA producers (even / odd stages; one elected lane per box)
 //   warp 1     TMEM allocator + MMA issuer
 //   warps 2-9  FT (256 threads: at most one (k octet, depth) item per stage),
 //              then the epilogue (tcgen05.ld -> OT -> bucket, or -> shared
@@ -66,7 +66,8 @@ namespace tc2 {
 constexpr int KC = 16;                 // depth entries per stage = UMMA K
 constexpr int MROWS = 128;             // UMMA M = TMEM lanes
 constexpr int NTX = 8;                 // transformer warps
-constexpr int NTHREADS = 64 + 32 * NTX;
+constexpr int NTHREADS = 64 + 32 * NTX + 32;
+constexpr int PW2 = 2 + NTX;           // second TMA producer warp (odd stages; warp 0: even stages)
 constexpr int NSOUT = 3;               // n0: outputs per unit (S = 3)
 #ifndef WINRS_TC2_ITM
 #define WINRS_TC2_ITM 0    // 1: IT inside the tensor core (8 MMAs per stage on the raw X columns, by linearity);
@@ -74,7 +75,7 @@ constexpr int NSOUT = 3;               // n0: outputs per unit (S = 3)
                            //    alpha = 4 Winograd EWM).  A/B on B200 in DESIGN.md §6.4.
 #endif
 
-template <int F, int NK, int CG = 1>
+template <int F, int NK, int CG = 1, bool TA = false>
 struct Lay {
     static constexpr int BC = MROWS / F;                 // channels c per fh slot
     static constexpr int NKL = NK / CG;                  // k rows of the What operand held by this CTA
@@ -87,7 +88,16 @@ struct Lay {
     static constexpr int ATOM = KC * 128;                // 2 KB: 64 channels x 16 depth rows
     static constexpr int X_LBO = 4 * ATOM;               // 8 KB
     static constexpr int Y_LBO = 2 * ATOM;               // 4 KB
-    static constexpr int OFF_Y = 2 * X_LBO;              // 16 KB
+    // TA (Xhat in TMEM; X is read only by ldmatrix.trans): per X atom two
+    // boxes of 8 images x 4 cols (rows col * 8 + n, 4 KB), the upper-image box
+    // two 128-byte rows further (the TMA swizzle follows the absolute address
+    // bits [7:9]: probed, tools/microbench/tma_offset.cu), so that the 8 rows
+    // of every ldmatrix phase -- depth entries {4p, 4p+1} or {4p+2, 4p+3},
+    // p = 0..3, of one column -- fall in 8 distinct 16-byte bank groups.
+    static constexpr int XT_HI = 4096 + 256;             // upper 8 images
+    static constexpr int XT_GRP = 2 * 4096 + 256;        // between the two X atoms (66 rows)
+    static constexpr int X_GRP = TA ? XT_GRP : X_LBO;    // producer: X atom a at a * X_GRP
+    static constexpr int OFF_Y = TA ? 17 * 1024 : 2 * X_LBO;   // 16 KB (TA: 17 KB, 1 KB aligned)
     static constexpr int OFF_F = OFF_Y + (NKL / 64) * Y_LBO;
     static constexpr int STAGE = OFF_F + (NKL / 64) * Y_LBO;   // 32 / 24 KB (cta pair: 24 KB)
     static constexpr int LIMIT = 227 * 1024 - 1024 - 256;
@@ -96,7 +106,7 @@ struct Lay {
     static constexpr int OUT = NSOUT * NK * MROWS * 4;   // staging tile [s][k][m] fp32 (cluster split)
     static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
     static constexpr int BYTES = BAR_OFF + 256 + 1024;   // + alignment slack
-    static constexpr int TX_BYTES = OFF_F;               // TMA bytes per stage
+    static constexpr int TX_BYTES = 2 * X_LBO + (NKL / 64) * Y_LBO;   // TMA bytes per stage
     static constexpr int TMEM_COLS = 4 * NK;
     static_assert(STAGE % 1024 == 0, "stages must keep the 1 KB swizzle-atom alignment");
     static_assert(S >= 4, "ring too shallow");
@@ -174,10 +184,12 @@ struct ImgTracker {
         a = img % inner;
         b = img / inner;
     }
-    __device__ __forceinline__ void advance(int by, bool wrapped) {   // img += by (by divides inner)
-        a += by;
-        if (a >= inner) { a -= inner; ++b; }
-        if (wrapped) { a = 0; b = 0; }
+    // After the producer's n += by and its wrap loop: image n (n < by when
+    // wrapped, since n < N before the step); a < inner + by, so the loop runs
+    // at most by / 16 times (inner >= 16).
+    __device__ __forceinline__ void advance(int by, bool wrapped, int n) {
+        if (wrapped) { a = n; b = 0; } else { a += by; }
+        while (a >= inner) { a -= inner; ++b; }
     }
     __device__ __forceinline__ ImgCoord at(const Geometry& g, bool in) const {
         ImgCoord c;
@@ -364,7 +376,7 @@ template <int F, int NK, bool BF, int CG = 1, bool TA = false>
 __global__ void __launch_bounds__(NTHREADS, 1)
 bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX,
                const __grid_constant__ CUtensorMap tmY) {
-    using L = Lay<F, NK, CG>;
+    using L = Lay<F, NK, CG, TA>;
     static_assert(!TA || (CG == 1 && NK == 64 && L::S == 8), "TA: single CTA, NK = 64, 8-slot ring");
     constexpr uint32_t TMEM_ALLOC = TA ? 512u : (uint32_t)L::TMEM_COLS;
     constexpr uint32_t A_COL = 4 * NK;          // TA: first A ring column
@@ -438,15 +450,19 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     const uint32_t tmem = bars->tmem_base;
     if (threadIdx.x == 64) TC2_TRACE(511, 1);
 
-    if (warp == 0) {
-        // ============================ TMA producer ============================
-        // Converged warp, one elected lane issues the stage's boxes: X atoms
-        // 0 and 1 (c halves, or fh slots for F = 2) and the dY k atoms, each
-        // [64 ch][16 images][1 row][cols], i.e. one 128-byte swizzled row per
-        // (col, image) = the UMMA operand layout.  (n, u, h) advance
-        // incrementally (per-stage integer divisions cost ~700 cycles on an
-        // SM sub-partition shared with other warps: WINRS_TC2_TRACE timeline.)
-        long long d = (long long)c_lo * KC;
+    if (warp == 0 || warp == PW2) {
+        // ============================ TMA producers ===========================
+        // Two converged warps (warp 0: even stages, warp PW2: odd stages; the
+        // per-stage issue path is ~120 dependent instructions, which alone
+        // bounded the small-tile kernels: ncu source counters), one elected
+        // lane issues the stage's boxes: X atoms 0 and 1 (c halves, or fh
+        // slots for F = 2) and the dY k atoms, each [64 ch][16 images][1 row]
+        // [cols], i.e. one 128-byte swizzled row per (col, image) = the UMMA
+        // operand layout.  (n, u, h) advance incrementally (per-stage integer
+        // divisions cost ~700 cycles on an SM sub-partition shared with other
+        // warps: WINRS_TC2_TRACE timeline.)
+        const int pp = warp == 0 ? 0 : 1;
+        long long d = (long long)(c_lo + pp) * KC;
         int n = 0, h = hs, u = 0;
         if (d < depth) depth_nhu((int)d, g.N, units, hs, &n, &h, &u);
         ImgTracker itk;
@@ -460,9 +476,9 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             xdt[a] = (g.T > 1 || g.D > 1) ? fh / g.Rh - g.pad : 0;
             xdr[a] = fh < g.R ? fh % g.Rh - g.pad : -(1 << 20);   // a slot past the last filter row: zero fill
         }
-        int s = 0;
+        int s = pp;
         uint32_t ph = 0;
-        for (int ch = c_lo; ch < c_hi; ++ch) {
+        for (int ch = c_lo + pp; ch < c_hi; ch += 2) {
             mbar_wait(&bars->empty[s], ph ^ 1);
             TC2_JITTER(ch, 0);
             TC2_TRACE(ch - c_lo, 0);
@@ -482,7 +498,13 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     // X window columns x0..x3 of atom a; an fh slot past the last
                     // filter row reads rows far outside (zero fill)
                     const int c0 = F == 2 ? c_base : c_base + a * 64;
-                    tma5(st + a * L::X_LBO, &tmX, fb, c0, ic.a + xdt[a], ic.b, hh + xdr[a], w0 + fw0 - g.pad);
+                    if constexpr (TA) {   // two 8-image boxes (tmX box {64, 8, 1, 1, 4})
+                        tma5(st + a * L::X_GRP, &tmX, fb, c0, ic.a + xdt[a], ic.b, hh + xdr[a], w0 + fw0 - g.pad);
+                        tma5(st + a * L::X_GRP + L::XT_HI, &tmX, fb, c0, ic.a + 8 + xdt[a], ic.b, hh + xdr[a],
+                             w0 + fw0 - g.pad);
+                    } else {
+                        tma5(st + a * L::X_LBO, &tmX, fb, c0, ic.a + xdt[a], ic.b, hh + xdr[a], w0 + fw0 - g.pad);
+                    }
                 }
 #pragma unroll
                 for (int ka = 0; ka < L::NKL / 64; ++ka)   // dY unit columns w0, w0 + 1 of k atom ka
@@ -491,16 +513,17 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             }
             __syncwarp();
             TC2_TRACE(ch - c_lo, 1);
-            d += KC;
-            n += KC;
+            d += 2 * KC;
+            n += 2 * KC;
             bool wrapped = false;
             while (n >= g.N) {
                 n -= g.N;
                 wrapped = true;
                 if (++u == units) { u = 0; ++h; }
             }
-            itk.advance(KC, wrapped);
-            if (++s == L::S) { s = 0; ph ^= 1; }
+            itk.advance(2 * KC, wrapped, n);
+            s += 2;
+            if (s >= L::S) { s -= L::S; ph ^= 1; }
         }
     } else if (warp == 1) {
         // ============================ MMA issuer ==============================
@@ -593,7 +616,9 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
 #pragma unroll
             for (int hf = 0; hf < 2; ++hf) {
                 const int oct = 4 * (q & 1) + 2 * hf + (i4 >> 1);
-                xoff[hf] = (uint32_t)((q >> 1) * L::X_LBO) + opoff(oct, img, 0);
+                // row of (image img, column 0); columns are 8 rows (1 KB) apart
+                const uint32_t row = (uint32_t)((q >> 1) * L::X_GRP + (img >> 3) * L::XT_HI + (img & 7) * 128);
+                xoff[hf] = row + (uint32_t)((oct ^ ((row >> 7) & 7)) << 4);   // stages are 1 KB aligned
             }
             const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16) + A_COL;
             const int it = q * 32 + lane;           // FT item: depth it / KO, k octet it % KO (KO * KC = 128)
@@ -610,7 +635,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 for (int hf = 0; hf < 2; ++hf) {
                     uint32_t x[4][4];
 #pragma unroll
-                    for (int c = 0; c < 4; ++c) ldsm_x4_t(st + xoff[hf] + c * L::ATOM, x[c]);
+                    for (int c = 0; c < 4; ++c) ldsm_x4_t(st + xoff[hf] + c * 1024, x[c]);
                     uint32_t o[4][4];
 #pragma unroll
                     for (int r = 0; r < 4; ++r) {
@@ -864,18 +889,20 @@ bfc_tc2s_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     const uint32_t tmem = bars->tmem_base;
     if (threadIdx.x == 64) TC2_TRACE(511, 1);
 
-    if (warp == 0) {
-        // ---- TMA: X columns x0..x3 of this CTA's 64 channels; dY w0, w1 of its 128 k
-        long long d = (long long)c_lo * KC;
+    if (warp == 0 || warp == PW2) {
+        // ---- TMA (warp 0: even stages, warp PW2: odd stages): X columns x0..x3
+        // of this CTA's 64 channels; dY w0, w1 of its 128 k
+        const int pp = warp == 0 ? 0 : 1;
+        long long d = (long long)(c_lo + pp) * KC;
         int n = 0, h = hs, u = 0;
         if (d < depth) depth_nhu((int)d, g.N, units, hs, &n, &h, &u);
         ImgTracker itk;
         itk.init(g, n);
         const int xdt = (g.T > 1 || g.D > 1) ? fh / g.Rh - g.pad : 0;   // per CTA, not per stage
         const int xdr = fh < g.R ? fh % g.Rh - g.pad : -(1 << 20);
-        int s = 0;
+        int s = pp;
         uint32_t ph = 0;
-        for (int ch = c_lo; ch < c_hi; ++ch) {
+        for (int ch = c_lo + pp; ch < c_hi; ch += 2) {
             mbar_wait(&bars->empty[s], ph ^ 1);
             TC2_JITTER(ch, 0);
             TC2_TRACE(ch - c_lo, 0);
@@ -893,16 +920,17 @@ bfc_tc2s_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
             }
             __syncwarp();
             TC2_TRACE(ch - c_lo, 1);
-            d += KC;
-            n += KC;
+            d += 2 * KC;
+            n += 2 * KC;
             bool wrapped = false;
             while (n >= g.N) {
                 n -= g.N;
                 wrapped = true;
                 if (++u == units) { u = 0; ++h; }
             }
-            itk.advance(KC, wrapped);
-            if (++s == L::S) { s = 0; ph ^= 1; }
+            itk.advance(2 * KC, wrapped, n);
+            s += 2;
+            if (s >= L::S) { s -= L::S; ph ^= 1; }
         }
     } else if (warp == 1) {
         // ---- MMA (the pair's leader): D[xi] (256 k x 128 c) += What[xi] . Xhat[xi]

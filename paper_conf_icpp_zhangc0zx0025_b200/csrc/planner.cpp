@@ -249,8 +249,8 @@ static TimeModel time_model(const KernelEntry& e) {
         return {4.5e-6, 16.0e12};
     if (e.fhs > 0 && e.cg == 2)   // bfc_tc2.cuh CTA pair: rate of the pair over its 256-row tile
         return {4.5e-6, 11.0e12};
-    if (e.fhs > 0 && e.ta)   // bfc_tc2.cuh TA (Xhat in TMEM, NK = 64): 10-14 % faster than the SMEM twin
-        return {4.0e-6, 3.85e12};  // (tools/ta_ab.py: VGG L1 994 -> 855 us, R50 L1 58.3 -> 52.2 us)
+    if (e.fhs > 0 && e.ta)   // bfc_tc2.cuh TA (Xhat in TMEM, NK = 64, two TMA producer warps):
+        return {4.0e-6, 5.1e12};   // tools/ta_ab.py: VGG L1 988 -> 644 us, R50 L1 57.3 -> 44.0 us
     if (e.fhs > 0) {
         // bfc_tc2.cuh, rate over the whole 128-row UMMA tile (fhs filter rows).
         // Measured on B200 (tools/trace_tc2.py, WINRS_TC2_TRACE): a 16-deep stage
