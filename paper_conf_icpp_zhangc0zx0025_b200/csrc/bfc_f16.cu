@@ -130,26 +130,26 @@ const KernelEntry* f16_entries(int* n) {
         WINRS_F16_ENTRY(8, 3, 6, 4, 3, 2, 32),
         WINRS_F16_ENTRY(8, 3, 6, 0, 0, 0, 64),
         WINRS_F16_ENTRY(8, 3, 6, 0, 0, 0, 32),
-        WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 128),
-        WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 64),
-        WINRS_F16_ENTRY(4, 3, 2, 0, 0, 0, 32),
+        // Not registered: this family's stand-alone Omega_4(3,2) kernels (the
+        // deep-raw-ring variant, all B_M) and its B_M = 128 tiles -- at large
+        // depth they were not bitwise reproducible (VGG-16 conv2_2, N = 128:
+        // every call differed at ~2e-5 rel.) and failed with 3-8-rank clusters
+        // (tools/det_check.py).  Omega_4(3,2) runs on the tc2
+        // kernels (N % 16 == 0) or as the residual phase of Omega_8(3,6).
         // wider widths: F_W multiple of 5, 7, 4, 2
         WINRS_F16_ENTRY(8, 5, 4, 0, 0, 0, 64),
         WINRS_F16_ENTRY(8, 7, 2, 0, 0, 0, 64),
         WINRS_F16_ENTRY(8, 4, 5, 4, 2, 3, 64),
         WINRS_F16_ENTRY(8, 4, 5, 0, 0, 0, 64),
-        WINRS_F16_ENTRY(4, 2, 3, 0, 0, 0, 128),
         WINRS_F16_ENTRY(4, 2, 3, 0, 0, 0, 64),
         // BF16 inputs: the same kernels with bf16 operands
         WINRS_BF16_ENTRY(8, 3, 6, 4, 3, 2, 64),
         WINRS_BF16_ENTRY(8, 3, 6, 4, 3, 2, 32),
         WINRS_BF16_ENTRY(8, 3, 6, 0, 0, 0, 64),
-        WINRS_BF16_ENTRY(4, 3, 2, 0, 0, 0, 128),
-        WINRS_BF16_ENTRY(4, 3, 2, 0, 0, 0, 64),
         WINRS_BF16_ENTRY(8, 5, 4, 0, 0, 0, 64),
         WINRS_BF16_ENTRY(8, 7, 2, 0, 0, 0, 64),
         WINRS_BF16_ENTRY(8, 4, 5, 4, 2, 3, 64),
-        WINRS_BF16_ENTRY(4, 2, 3, 0, 0, 0, 128),
+        WINRS_BF16_ENTRY(4, 2, 3, 0, 0, 0, 64),
     };
     *n = sizeof(e) / sizeof(e[0]);
     return e;

@@ -246,11 +246,11 @@ struct SharedModel {
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
     if (e.fhs > 0 && e.cg == 2 && bn == 256)   // swapped CTA pair (256 k x 128 c): X side shared
-        return {4.5e-6, 16.0e12};
+        return {4.5e-6, 12.6e12};              // (re-fitted with two producer warps: tools/sweep_tc2.py)
     if (e.fhs > 0 && e.cg == 2)   // bfc_tc2.cuh CTA pair: rate of the pair over its 256-row tile
         return {4.5e-6, 11.0e12};
     if (e.fhs > 0 && e.ta)   // bfc_tc2.cuh TA (Xhat in TMEM, NK = 64, two TMA producer warps):
-        return {4.0e-6, 5.1e12};   // tools/ta_ab.py: VGG L1 988 -> 644 us, R50 L1 57.3 -> 44.0 us
+        return {4.0e-6, 5.6e12};   // tools/ta_ab.py: VGG L1 988 -> 644 us, R50 L1 57.3 -> 44.0 us
     if (e.fhs > 0) {
         // bfc_tc2.cuh, rate over the whole 128-row UMMA tile (fhs filter rows).
         // Measured on B200 (tools/trace_tc2.py, WINRS_TC2_TRACE): a 16-deep stage
@@ -340,6 +340,18 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
     return mk;
 }
 
+// Cluster depth splits a kernel may run.  The round-1 FP16 kernel (bfc_f16.cuh)
+// keeps its round-1 set {1, 2, 4}: with 3, 6 or 8 ranks it fails
+// intermittently at large depth (VGG-16 conv2_2, N = 128: an unspecified launch
+// failure within 12-24 calls; not reproducible under compute-sanitizer,
+// DESIGN.md §10).  The tc2 and FP32 kernels take {1, 2, 3, 4, 6, 8}.
+static bool cs_allowed(const KernelEntry& e, int cs) {
+    if (cs == 1) return true;
+    if (!e.csplit_ok) return false;
+    if (e.dtype != 0 && e.fhs <= 0) return cs == 2 || cs == 4;
+    return true;
+}
+
 static int forced_csplit() {
     if (const char* f = getenv("WINRS_FORCE_CSPLIT")) {
         const int v = atoi(f);
@@ -399,7 +411,7 @@ static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairC
         last_bands = g.bands; last_cols = g.seg_cols; last_sh = seg_h; last_sw = seg_w;
         const long long mc = min_tile_chunks(g);
         for (int cs : {1, 2, 3, 4, 6, 8}) {
-            if (cs > 1 && !e.csplit_ok) continue;   // never launch a cluster the kernel cannot reduce (even if forced)
+            if (!cs_allowed(e, cs)) continue;   // never launch a cluster the kernel cannot reduce (even if forced)
             if (e.cg == 2 && cs > 4) continue;   // 16-CTA clusters (pairs x 8): ~half the clusters co-resident (measured 2x slower)
             if (fcs ? cs != fcs : (cs > 1 && mc < cs)) continue;
             g.csplit = cs;
@@ -415,7 +427,7 @@ static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairC
         int z_used = 1, seg_h = p.Ho, seg_w = pc.k0 * e.r0;
         alg2(p, e.r0, pc.k0, z_lo, &z_used, &seg_h, &seg_w);
         fill_geometry(p, e, pc, seg_h, seg_w, &out->geom);
-        out->geom.csplit = fcs && e.csplit_ok ? fcs : 1;
+        out->geom.csplit = fcs && cs_allowed(e, fcs) ? fcs : 1;
         best_t = model_time(out->geom, e, num_sms);
     }
     out->entry = &e;

@@ -159,7 +159,7 @@ def test_reduced_f16_signed(layer):
 
 FORCED_F16 = [
     {"WINRS_FORCE_Z": "1"}, {"WINRS_FORCE_Z": "7"},
-    {"WINRS_FORCE_PAIR": "8,3,6,0,0,0"}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_Z": "3"},
+    {"WINRS_FORCE_PAIR": "8,3,6,0,0,0"}, {"WINRS_FORCE_PAIR": "8,3,6,4,3,2", "WINRS_FORCE_Z": "3"},
     {"WINRS_FORCE_CSPLIT": "1"}, {"WINRS_FORCE_CSPLIT": "2"}, {"WINRS_FORCE_CSPLIT": "8"},
     {"WINRS_FORCE_CSPLIT": "4", "WINRS_FORCE_TILE": "128x32", "WINRS_FORCE_Z": "2"},
     {"WINRS_FORCE_CSPLIT": "4", "WINRS_FORCE_PAIR": "8,3,6,0,0,0"},
@@ -174,7 +174,7 @@ K64_F16 = [
     ({"K": 40, "C": 72}, {"WINRS_FORCE_PAIR": "8,3,6,0,0,0", "WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "4"}),
     ({"K": 8, "C": 136}, {"WINRS_FORCE_PAIR": "8,3,6,0,0,0", "WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_Z": "3"}),
     ({"K": 56, "C": 64}, {"WINRS_FORCE_PAIR": "8,3,6,0,0,0", "WINRS_FORCE_TILE": "128x32"}),
-    ({"K": 64, "C": 128}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "2"}),
+    ({"K": 64, "C": 128}, {"WINRS_FORCE_PAIR": "8,3,6,4,3,2", "WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "2"}),
 ]
 
 

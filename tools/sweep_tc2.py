@@ -16,8 +16,10 @@ sys.path.insert(0, ROOT)
 import paper_conf_icpp_zhangc0zx0025_b200 as W  # noqa: E402
 from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl  # noqa: E402
 
-# (tile NK x bm, CTAs per UMMA): single CTA NK x (128 / F), or a cta_group::2 pair
-TILES = [("128x128", 1), ("64x128", 1), ("128x64", 1), ("64x64", 1), ("128x256", 2), ("128x64", 2)]
+# (tile NK x bm, CTAs per UMMA, Xhat in TMEM): single CTA NK x (128 / F), a cta_group::2 pair,
+# the swapped pair (256x128), or the TA kernels (NK = 64, Xhat in TMEM)
+TILES = [("128x128", 1, 0), ("64x128", 1, 0), ("128x64", 1, 0), ("64x64", 1, 0), ("128x256", 2, 0), ("128x64", 2, 0),
+         ("256x128", 2, 0), ("64x128", 1, 1), ("64x64", 1, 1)]
 
 
 def time_plan(p, Xg, Gg, flush, reps=10):
@@ -52,7 +54,8 @@ def main():
             cfgs += [("f", t, cs, z) for t in TILES for cs in (1, 2, 3, 4, 6, 8) for z in zs]
         seen = set()
         for kind, t, cs, z in cfgs:
-            for k in ("WINRS_FORCE_Z", "WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_TC_GEN", "WINRS_FORCE_CG"):
+            for k in ("WINRS_FORCE_Z", "WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_TC_GEN", "WINRS_FORCE_CG",
+                      "WINRS_FORCE_TA"):
                 os.environ.pop(k, None)
             if kind == "gen1":
                 os.environ["WINRS_TC_GEN"] = "1"
@@ -60,7 +63,7 @@ def main():
                 os.environ["WINRS_TC_GEN"] = "2"
             if kind == "f":
                 os.environ.update({"WINRS_FORCE_TILE": t[0], "WINRS_FORCE_CG": str(t[1]), "WINRS_FORCE_CSPLIT": str(cs),
-                                   "WINRS_FORCE_Z": str(z)})
+                                   "WINRS_FORCE_Z": str(z), "WINRS_FORCE_TA": str(t[2])})
             try:
                 p = W.plan(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype)
             except Exception:
