@@ -249,6 +249,8 @@ static TimeModel time_model(const KernelEntry& e) {
         return {4.5e-6, 12.6e12};              // (re-fitted with two producer warps: tools/sweep_tc2.py)
     if (e.fhs > 0 && e.cg == 2)   // bfc_tc2.cuh CTA pair: rate of the pair over its 256-row tile
         return {4.5e-6, 11.0e12};
+    if (e.fhs > 0 && e.tf32)   // bfc_tc3.cuh: FP32 inputs, 12 tf32 MMAs per 8-deep stage (3xTF32)
+        return {4.0e-6, 0.9e12};
     if (e.fhs > 0 && e.ta)   // bfc_tc2.cuh TA (Xhat in TMEM, NK = 64, two TMA producer warps):
         return {4.0e-6, 5.6e12};   // tools/ta_ab.py: VGG L1 988 -> 644 us, R50 L1 57.3 -> 44.0 us
     if (e.fhs > 0) {
@@ -470,8 +472,13 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
         });
         for (const KernelEntry* e : tiles) {
             if (force_tile && (e->bn != fbn || e->bm != fbm)) continue;
-            if (e->fhs > 0 && p.N % 16 != 0) continue;   // tc2: one 16-image TMA box per stage and atom
             const bool nd = p.T > 1 || p.D > 1;
+            // tcgen05 kernels: one 16-image (tc2) / 8-image (tc3, FP32) TMA box per stage
+            if (e->fhs > 0 && (nd ? p.Do : p.N) % (e->tf32 ? 8 : 16) != 0) continue;
+            if (e->fhs > 0 && p.N % (e->tf32 ? 8 : 16) != 0) continue;
+            if (const char* v = getenv("WINRS_FP32_TC")) {   // debug: FP32 on the tensor cores only (1) / never (0)
+                if (e->dtype == 0 && (atoi(v) != 0) != (e->tf32 != 0)) continue;
+            }
             // N-D: the FP32 kernel, or the tc2 kernels (16 depth slices of one image per TMA box)
             if (nd && e->dtype != 0 && (e->fhs <= 0 || p.Do % 16 != 0)) continue;
             if (const char* v = getenv("WINRS_TC_GEN")) {   // debug: restrict to one tensor-core generation

@@ -26,6 +26,7 @@ struct KernelEntry {
                                // second-generation tcgen05 kernels (bfc_tc2.cuh), which need N % 16 == 0
     int cg;                    // CTAs per UMMA: 2 = cta_group::2 pair (0 = 1)
     int ta;                    // 1: tc2 kernel with the transformed X operand in TMEM (bfc_tc2.cuh TA)
+    int tf32;                  // 1: FP32 inputs on the tensor cores, 3xTF32 split (bfc_tc3.cuh)
 };
 
 // All entries (FP32 and FP16), terminated by count.
