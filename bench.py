@@ -194,7 +194,12 @@ def layer_roofline(l, p, ms, peaks):
     fp32_peak = 148 * 128 * 2 * clk_ghz * 1e9            # FLOP/s (lanes x FMA)
     lanes = 148 * 128 * clk_ghz * 1e9                    # lane-ops/s
     t_hbm = alg_bytes / (peaks["hbm_gbs"] * 1e9)
-    if l.dtype == "f32":
+    if l.dtype == "f32" and p.kernel_name.startswith("f32tc_"):
+        # bfc_tc3.cuh: FP32 on the tensor cores, 3 tf32 MMAs per product (3xTF32);
+        # tf32 peak = the measured bf16 dense peak x the nominal 1.13 / 2.25 ratio
+        tf32 = peaks["bf16_tflops"] * 1.13 / 2.25
+        t_pipe, bound, pk = 3.0 * ewm / (tf32 * 1e12), "tensor", tf32
+    elif l.dtype == "f32":
         t_pipe, bound, pk = ewm / fp32_peak, "alu", fp32_peak / 1e12
     else:
         t_pipe, bound, pk = ewm / (peaks["bf16_tflops"] * 1e12), "tensor", peaks["bf16_tflops"]
@@ -213,6 +218,12 @@ def layer_roofline(l, p, ms, peaks):
         depth = rows * units * l.N * kb * cb * ft
         l2_bytes = depth / 16 * 2 * (8192 + 8192)         # per pair stage: each CTA X 8 KB + dY 8 KB
         alu_ops = depth * (256 + 128 * 2)                 # FT over 256 k, IT over 128 c (half2)
+    elif "_v3_" in name:                                  # FP32 tensor-core kernel: 8-deep stages
+        fhs = int(name.split("x")[-1].rstrip("fh"))
+        rows = sum(_rows_union(l, range(g, min(l.R, g + fhs))) for g in range(0, l.R, fhs))
+        depth = rows * units * l.N * kb * cb * ft
+        l2_bytes = depth / 8 * (16384 + bn * 64)          # per stage: X 16 KB + dY NK x 2 cols x 8 x 4 B
+        alu_ops = depth * (bn * 2 * 2 + 128 * 4 * 3)      # FT (+ lo split), IT 4 outputs (+ lo split)
     elif "_v2" in name:
         tag = name.split("_v2")[1][0]                     # CTAs per UMMA (2: cta_group::2 pair); t: Xhat in TMEM
         cg = 1 if tag == "t" else int(tag)

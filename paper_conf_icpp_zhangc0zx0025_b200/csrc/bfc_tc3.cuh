@@ -46,24 +46,41 @@ constexpr int NK = 64;     // k columns per tile (UMMA N)
 template <int F>
 struct Lay3 {
     static constexpr int BC = MROWS / F;                       // channels per fh slot
-    static constexpr int XSLOT = 4 * KT * BC * 4;              // raw X of one fh slot: [col][img][BC] fp32
-    static constexpr int OFF_X = 0;                            // 16 KB
-    static constexpr int OFF_Y = 4 * KT * MROWS * 4;           // raw dY [col 2][img 8][64 k]: 4 KB
-    static constexpr int ASLAB = MROWS * KT * 4;               // one K-major A slab (128 x 8 fp32): 4 KB
-    static constexpr int BSLAB = NK * KT * 4;                  // one K-major B slab (64 x 8): 2 KB
-    static constexpr int OFF_A = OFF_Y + 2 * KT * NK * 4;      // [hi, lo][xi 4] A slabs: 32 KB
-    static constexpr int OFF_B = OFF_A + 2 * 4 * ASLAB;        // [hi, lo][xi 4] B slabs: 16 KB
-    static constexpr int STAGE = OFF_B + 2 * 4 * BSLAB;        // 68 KB
-    static constexpr int LIMIT = 227 * 1024 - 1024 - 256;
-    static constexpr int S = LIMIT / STAGE > 8 ? 8 : LIMIT / STAGE;   // 3
-    static constexpr int RING = S * STAGE;
+    // Two rings (the raw TMA tiles are 20 KB, the hi / lo operands 48 KB, so
+    // separate rings give the TMA 4 stages of latency hiding next to 3
+    // operand stages instead of 3 combined ones):
+    //   raw  [SR]: X [fh slot][col 4][img 8][BC] fp32 (16 KB) + dY [col 2][img 8][64 k] (4 KB)
+    //   op   [SO]: A [hi, lo][xi 4] K-major slabs 128 x 8 (32 KB) + B [hi, lo][xi 4] 64 x 8 (16 KB)
+    static constexpr int XSLOT = 4 * KT * BC * 4;              // raw X of one fh slot
+    static constexpr int OFF_X = 0;
+    static constexpr int OFF_Y = 4 * KT * MROWS * 4;           // 16 KB
+    static constexpr int RAW = OFF_Y + 2 * KT * NK * 4;        // 20 KB
+    static constexpr int ASLAB = MROWS * KT * 4;               // 4 KB
+    static constexpr int BSLAB = NK * KT * 4;                  // 2 KB
+    static constexpr int OFF_A = 0;                            // within an operand stage
+    static constexpr int OFF_B = 2 * 4 * ASLAB;                // 32 KB
+    static constexpr int OP = OFF_B + 2 * 4 * BSLAB;           // 48 KB
+    static constexpr int LIMIT = 227 * 1024 - 1024 - 512;
+    static constexpr int SO = 3;
+    static constexpr int SR = (LIMIT - SO * OP) / RAW > 6 ? 6 : (LIMIT - SO * OP) / RAW;   // 4
+    static constexpr int OP_OFF = SR * RAW;
+    static constexpr int RING = OP_OFF + SO * OP;
     static constexpr int OUT = NSOUT * NK * MROWS * 4;         // cluster staging [s][k][m] fp32 (96 KB)
     static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
-    static constexpr int BYTES = BAR_OFF + 256 + 1024;
-    static constexpr int TX_BYTES = OFF_A;                     // TMA bytes per stage (20 KB)
+    static constexpr int BYTES = BAR_OFF + 512 + 1024;
+    static constexpr int TX_BYTES = RAW;                       // TMA bytes per stage
     static constexpr int TMEM_COLS = 4 * NK;                   // 256
-    static_assert(S >= 3, "ring too shallow");
-    static_assert(STAGE % 1024 == 0, "stage alignment");
+    static_assert(SR >= 3, "raw ring too shallow");
+    static_assert(RAW % 1024 == 0 && OP % 1024 == 0, "stage alignment");
+};
+
+struct Bars3 {
+    uint64_t full[8];      // raw stage landed (TMA)
+    uint64_t rempty[8];    // raw stage consumed (4 FT warps)
+    uint64_t opfull[8];    // operand stage written (4 FT warps)
+    uint64_t opempty[8];   // operand stage read by the MMAs (commit)
+    uint64_t accfull;
+    uint32_t tmem_base;
 };
 
 // K-major, no swizzle: element (row, k) of a slab at (row/8)*256 + (k/4)*128
@@ -104,7 +121,7 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     const uint32_t raw_s = su(smem_raw);
     uint8_t* smem = smem_raw + (((raw_s + 1023u) & ~1023u) - raw_s);
     const uint32_t sbase = su(smem);
-    Bars* bars = reinterpret_cast<Bars*>(smem + L::BAR_OFF);
+    Bars3* bars = reinterpret_cast<Bars3*>(smem + L::BAR_OFF);
     const Geometry& g = args.g;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
@@ -125,10 +142,13 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     const int fw0 = cc.ft * NSOUT;
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < L::S; ++s) {
+        for (int s = 0; s < L::SR; ++s) {
             mbar_init(&bars->full[s], 1);
-            mbar_init(&bars->opfull[s], 4);   // the four warps of an FT group
-            mbar_init(&bars->empty[s], 1);
+            mbar_init(&bars->rempty[s], 4);   // the four warps of an FT group
+        }
+        for (int s = 0; s < L::SO; ++s) {
+            mbar_init(&bars->opfull[s], 4);
+            mbar_init(&bars->opempty[s], 1);
         }
         mbar_init(&bars->accfull, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -165,9 +185,9 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         int s = pp;
         uint32_t ph = 0;
         for (int ch = c_lo + pp; ch < c_hi; ch += 2) {
-            mbar_wait(&bars->empty[s], ph ^ 1);
+            mbar_wait(&bars->rempty[s], ph ^ 1);
             uint64_t* fb = &bars->full[s];
-            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            const uint32_t st = sbase + (uint32_t)(s * L::RAW);
             const bool in = d < depth;
             const ImgCoord ic = itk.at(g, in);
             const int hh = in ? h : hs;
@@ -191,7 +211,7 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             }
             itk.advance(2 * KT, wrapped, n);
             s += 2;
-            if (s >= L::S) { s -= L::S; ph ^= 1; }
+            if (s >= L::SR) { s -= L::SR; ph ^= 1; }
         }
     } else if (warp == 1) {
         // ============================ MMA issuer ==============================
@@ -200,7 +220,7 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         for (int ch = c_lo; ch < c_hi; ++ch) {
             mbar_wait(&bars->opfull[s], ph);
             tc_after();
-            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            const uint32_t st = sbase + (uint32_t)(L::OP_OFF + s * L::OP);
             const uint32_t acc = ch > c_lo ? 1u : 0u;
             if (elect_one()) {
 #pragma unroll
@@ -213,10 +233,10 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     umma_tf32(tmem + x * NK, ah, bl, 1u);
                     umma_tf32(tmem + x * NK, al, bh, 1u);
                 }
-                umma_commit<1>(&bars->empty[s]);
+                umma_commit<1>(&bars->opempty[s]);
             }
             __syncwarp();
-            if (++s == L::S) { s = 0; ph ^= 1; }
+            if (++s == L::SO) { s = 0; ph ^= 1; }
         }
         if (elect_one()) umma_commit<1>(&bars->accfull);
         __syncwarp();
@@ -233,11 +253,13 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         const int f = m / L::BC, cm = m % L::BC;
         const uint32_t xrow = (uint32_t)(L::OFF_X + f * L::XSLOT + cm * 4);
         const int t = q * 32 + lane, kk = t % NK, dh = t / NK;
-        int s = G;
-        uint32_t ph = 0;
+        int s = G, so = G;                     // raw slot, operand slot
+        uint32_t ph = 0, pho = 0;
         for (int ch = c_lo + G; ch < c_hi; ch += 2) {
             mbar_wait(&bars->full[s], ph);
-            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            mbar_wait(&bars->opempty[so], pho ^ 1);   // the MMAs of this slot's previous stage are done
+            const uint32_t st = sbase + (uint32_t)(s * L::RAW);
+            const uint32_t ot = sbase + (uint32_t)(L::OP_OFF + so * L::OP);
 #pragma unroll
             for (int k4 = 0; k4 < 2; ++k4) {          // depth entries 4 k4 .. 4 k4 + 3
                 float hi[4][4], lo[4][4];
@@ -257,8 +279,8 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 const uint32_t o = koff(m, k4);
 #pragma unroll
                 for (int a = 0; a < 4; ++a) {
-                    sts4f(st + L::OFF_A + a * L::ASLAB + o, hi[a][0], hi[a][1], hi[a][2], hi[a][3]);
-                    sts4f(st + L::OFF_A + (4 + a) * L::ASLAB + o, lo[a][0], lo[a][1], lo[a][2], lo[a][3]);
+                    sts4f(ot + L::OFF_A + a * L::ASLAB + o, hi[a][0], hi[a][1], hi[a][2], hi[a][3]);
+                    sts4f(ot + L::OFF_A + (4 + a) * L::ASLAB + o, lo[a][0], lo[a][1], lo[a][2], lo[a][3]);
                 }
             }
             {
@@ -276,16 +298,21 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 const uint32_t o = koff(kk, dh);
 #pragma unroll
                 for (int a = 0; a < 4; ++a) {
-                    sts4f(st + L::OFF_B + a * L::BSLAB + o, w[a][0], w[a][1], w[a][2], w[a][3]);
-                    sts4f(st + L::OFF_B + (4 + a) * L::BSLAB + o, tf32_lo(w[a][0]), tf32_lo(w[a][1]),
+                    sts4f(ot + L::OFF_B + a * L::BSLAB + o, w[a][0], w[a][1], w[a][2], w[a][3]);
+                    sts4f(ot + L::OFF_B + (4 + a) * L::BSLAB + o, tf32_lo(w[a][0]), tf32_lo(w[a][1]),
                           tf32_lo(w[a][2]), tf32_lo(w[a][3]));
                 }
             }
             fence_async();     // generic-proxy stores -> visible to the tensor core (async proxy)
             __syncwarp();
-            if (lane == 0) mbar_arrive(&bars->opfull[s]);
+            if (lane == 0) {
+                mbar_arrive(&bars->rempty[s]);   // raw reads retired (the loads fed the stores above)
+                mbar_arrive(&bars->opfull[so]);
+            }
             s += 2;
-            if (s >= L::S) { s -= L::S; ph ^= 1; }
+            if (s >= L::SR) { s -= L::SR; ph ^= 1; }
+            so += 2;
+            if (so >= L::SO) { so -= L::SO; pho ^= 1; }
         }
         // ============================ epilogue (as bfc_tc2.cuh) ===============
         mbar_wait(&bars->accfull, 0);

@@ -22,7 +22,7 @@ pytestmark = pytest.mark.gpu
 
 TOL = {"f32": 1e-4, "f16": 2e-2, "bf16": 2e-2}
 ENV_KEYS = ("WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_TC_GEN", "WINRS_FORCE_CG",
-            "WINRS_FORCE_TA")
+            "WINRS_FORCE_TA", "WINRS_FP32_TC")
 
 
 def _dev(a, dtype):
@@ -146,6 +146,50 @@ def test_tc2_default_plans_use_tc2(monkeypatch):
     for l in wl.RESNET50_F16 + wl.VGG16_F16:
         p = _plan(l, {}, monkeypatch)
         assert "_v2" in p.kernel_name, (l.name, p.kernel_name)
+
+
+# ====================================================== bfc_tc3.cuh: FP32 inputs on the tensor cores (3xTF32)
+BASE32 = wl.LAYERS["r50_c64_56_f32"]
+TC3 = [
+    ("l1", dict(N=8), {}),
+    ("l1_f2", dict(N=8), {"WINRS_FORCE_TILE": "64x64"}),
+    ("l1_f1_cs2", dict(N=8), {"WINRS_FORCE_TILE": "64x128", "WINRS_FORCE_CSPLIT": "2"}),
+    ("l3", dict(N=8, C=256, K=256, H=14, W=14), {}),
+    ("ragged", dict(N=8, C=72, K=100, H=20, W=17), {}),
+    ("ragged_f2_cs3", dict(N=16, C=40, K=136, H=13, W=11), {"WINRS_FORCE_TILE": "64x64", "WINRS_FORCE_CSPLIT": "3"}),
+    ("pad0", dict(N=8, C=64, K=64, H=20, W=20, pad=0), {}),
+    ("r5", dict(N=8, C=64, K=64, H=16, W=16, R=5, S=3, pad=2), {}),
+    ("r1", dict(N=8, C=64, K=64, H=12, W=12, R=1, S=3, pad=0), {}),
+    ("s6", dict(N=8, C=64, K=64, H=16, W=16, R=3, S=6, pad=2), {"WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
+    ("s9_r9", dict(N=8, C=32, K=64, H=20, W=20, R=9, S=9, pad=4), {}),
+    ("z5", dict(N=16, C=64, K=64, H=30, W=30), {"WINRS_FORCE_Z": "5"}),
+    ("cs8", dict(N=24, C=128, K=64, H=12, W=12), {"WINRS_FORCE_CSPLIT": "8"}),
+    ("cs6_f2", dict(N=16, C=64, K=128, H=12, W=12), {"WINRS_FORCE_CSPLIT": "6", "WINRS_FORCE_TILE": "64x64"}),
+]
+
+
+@pytest.mark.parametrize("dist", ["u01", "signed"])
+@pytest.mark.parametrize("name,ov,env", TC3, ids=[c[0] for c in TC3])
+def test_tc3_fp32(name, ov, env, dist, monkeypatch):
+    """FP32 gate (1e-4) for the 3xTF32 tensor-core kernel, U[0,1) and signed inputs."""
+    layer = BASE32.with_(name="tc3_" + name, **ov)
+    _check(layer, monkeypatch, dict(env, WINRS_FP32_TC="1"), dist=dist, expect_kernel="f32tc_")
+
+
+def test_tc3_exact_all_ones(monkeypatch):
+    """X = dY = 1: every transformed operand is a small integer (exact in
+    tf32, lo = 0), so the 3xTF32 result is the closed form bit for bit."""
+    layer = BASE32.with_(N=8, C=64, K=64, H=18, W=17, name="tc3_ones")
+    X = np.ones((layer.N, layer.H, layer.W, layer.C), np.float32)
+    dY = np.ones((layer.N, layer.Ho, layer.Wo, layer.K), np.float32)
+    _check(layer, monkeypatch, {"WINRS_FP32_TC": "1"}, X=X, dY=dY, exact=True, expect_kernel="f32tc_")
+
+
+def test_fp32_default_plans_use_tc3(monkeypatch):
+    """The planner's picks for the ResNet-50 FP32 layers are the tensor-core kernel."""
+    for l in wl.RESNET50_F32:
+        p = _plan(l, {}, monkeypatch)
+        assert p.kernel_name.startswith("f32tc_"), (l.name, p.kernel_name)
 
 
 # ====================================================== pad = 0 (SURVEY §8(d): pad=0 variants of the wide config)
@@ -284,6 +328,8 @@ ND = [
     (2, 16, 18, 6, 6, 16, 3, 1, 3, 0, {}),                                      # pad 0, R = 1
     (1, 64, 16, 10, 11, 64, 3, 3, 3, 1, {"WINRS_FORCE_TA": "0"}),              # Xhat in shared memory
     (2, 64, 16, 7, 9, 64, 3, 3, 3, 1, {"WINRS_FORCE_TA": "1", "WINRS_FORCE_TILE": "64x64"}),   # Xhat in TMEM
+    (2, 48, 8, 7, 9, 64, 3, 3, 3, 1, {"WINRS_FP32_TC": "1"}),                 # FP32 on the tensor cores
+    (1, 64, 16, 6, 6, 64, 3, 3, 3, 1, {"WINRS_FP32_TC": "0"}),                # FP32 CUDA cores
 ]
 
 
@@ -328,8 +374,10 @@ STRESS = [
     ("vgg_128_128_112_f16", {"WINRS_FORCE_TA": "1", "WINRS_FORCE_CSPLIT": "6"}),
     ("vgg_128_128_112_f16", {"WINRS_FORCE_TA": "0", "WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "8"}),
     ("vgg_256_256_56_f16", {"WINRS_FORCE_TILE": "256x128", "WINRS_FORCE_CSPLIT": "3"}),
-    ("r50_c512_7_f32", {"WINRS_FORCE_CSPLIT": "6"}),
-    ("r50_c256_14_f32", {"WINRS_FORCE_CSPLIT": "8"}),
+    ("r50_c512_7_f32", {"WINRS_FORCE_CSPLIT": "6", "WINRS_FP32_TC": "0"}),
+    ("r50_c256_14_f32", {"WINRS_FORCE_CSPLIT": "8", "WINRS_FP32_TC": "0"}),
+    ("r50_c128_28_f32", {"WINRS_FORCE_CSPLIT": "8", "WINRS_FP32_TC": "1"}),
+    ("r50_c64_56_f32", {"WINRS_FORCE_CSPLIT": "3", "WINRS_FP32_TC": "1"}),
 ]
 
 

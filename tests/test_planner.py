@@ -201,12 +201,14 @@ def test_search_plan_is_valid(l):
 # ============================================================== N-D (3-D) plans
 def test_plan3d_rules():
     """winrs_plan3d: FP16 / BF16 plans on the second-generation kernel, FP32 on
-    the FP32 kernel; FP16 with Do % 16 != 0 is UNSUPPORTED; bad shapes INVALID_ARG."""
+    an FP32 kernel (tensor-core 3xTF32 when Do % 8 == 0, else CUDA-core); FP16
+    with Do % 16 != 0 is UNSUPPORTED; bad shapes INVALID_ARG."""
     p = W.plan3d_for_device(2, 64, 16, 12, 12, 64, 3, 3, 3, 1, "f16")
     i = p.info
     assert (i["D"], i["T"], i["Do"]) == (16, 3, 16) and "_v2" in p.kernel_name
     assert i["direct_flops"] == 2.0 * 2 * 16 * 64 * 64 * 12 * 12 * 27
-    assert "f32_" in W.plan3d_for_device(2, 64, 16, 12, 12, 64, 3, 3, 3, 1, "f32").kernel_name
+    assert W.plan3d_for_device(2, 64, 16, 12, 12, 64, 3, 3, 3, 1, "f32").kernel_name.startswith("f32")
+    assert W.plan3d_for_device(2, 64, 11, 12, 12, 64, 3, 3, 3, 1, "f32").kernel_name.startswith("f32_")   # Do = 11
     with pytest.raises(WinrsError, match="UNSUPPORTED"):
         W.plan3d_for_device(2, 64, 10, 12, 12, 64, 3, 3, 3, 1, "f16")   # Do = 10
     with pytest.raises(WinrsError, match="INVALID_ARG"):
