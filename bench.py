@@ -67,8 +67,9 @@ def _ncu_traffic(dtype: str, layer_name: str):
     with open(files[-1]) as f:
         t = json.load(f)
     base = layer_name.rsplit("_", 1)[0]
-    if dtype in t and base in t.get("layers", []):
-        i = t["layers"].index(base)
+    layers = t.get("layers_" + dtype, t.get("layers", []))
+    if dtype in t and base in layers:
+        i = layers.index(base)
         if i < len(t[dtype]):
             return t[dtype][i]["dram_bytes"], os.path.relpath(files[-1], ROOT) + " (ncu --set full)"
     return None, None
