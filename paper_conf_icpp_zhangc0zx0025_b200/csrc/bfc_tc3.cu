@@ -44,9 +44,9 @@ static bool make_map(CUtensorMap* m, const void* base, int A, int B, int H, int 
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-template <int F>
+template <int F, int NK>
 cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
-    using L = Lay3<F>;
+    using L = Lay3<F, NK>;
     const long long grid = num_ctas(g);
     if (grid <= 0) return cudaSuccess;
     const bool nd = g.T > 1 || g.D > 1;
@@ -62,7 +62,7 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
         !make_map(&mY, dY, nd ? g.Do : g.N, nd ? g.Nb : 1, g.Ho, g.Wo, g.K, g.ldy, NK, 2))
         return cudaErrorInvalidValue;
     static std::atomic<unsigned long long> done{0};
-    auto k = bfc_tc3_kernel<F>;
+    auto k = bfc_tc3_kernel<F, NK>;
     cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
     if (e != cudaSuccess) return e;
     if (g.csplit <= 1) {
@@ -74,16 +74,19 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
 
 }  // namespace tc3
 
-// tile = 64 k x (128 / F) c x F filter rows; fhs > 0 marks the tcgen05
+// tile = NK k x (128 / F) c x F filter rows; fhs > 0 marks the tcgen05
 // kernels, tf32 = 1 the FP32 (3xTF32) ones.
-#define WINRS_TC3_ENTRY(F)                                                                                 \
-    {0, 4, 3, 2, 0, 0, 0, 64, ::winrs::tc2::MROWS / F, ::winrs::tc2::NTHREADS, 1, 1,                       \
-     (size_t)::winrs::tc3::Lay3<F>::BYTES, &::winrs::tc3::launch<F>, "f32tc_O4(3,2)_v3_64x" #F "fh", F, 1, 0, 1}
+#define WINRS_TC3_ENTRY(F, NK)                                                                             \
+    {0, 4, 3, 2, 0, 0, 0, NK, ::winrs::tc2::MROWS / F, ::winrs::tc2::NTHREADS, 1, 1,                       \
+     (size_t)::winrs::tc3::Lay3<F, NK>::BYTES, &::winrs::tc3::launch<F, NK>,                              \
+     "f32tc_O4(3,2)_v3_" #NK "x" #F "fh", F, 1, 0, 1}
 
 const KernelEntry* tc3_entries(int* n) {
     static const KernelEntry e[] = {
-        WINRS_TC3_ENTRY(1),
-        WINRS_TC3_ENTRY(2),
+        WINRS_TC3_ENTRY(1, 128),
+        WINRS_TC3_ENTRY(2, 128),
+        WINRS_TC3_ENTRY(1, 64),
+        WINRS_TC3_ENTRY(2, 64),
     };
     *n = sizeof(e) / sizeof(e[0]);
     return e;

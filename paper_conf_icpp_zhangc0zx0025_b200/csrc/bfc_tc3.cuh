@@ -41,9 +41,10 @@ using tc2::NTHREADS;
 using tc2::PW2;
 
 constexpr int KT = 8;      // depth entries per stage = kind::tf32 UMMA K
-constexpr int NK = 64;     // k columns per tile (UMMA N)
 
-template <int F>
+// NK: k columns per tile (UMMA N): 64, or 128 (the MMAs' A reads -- A_hi is
+// read twice per xi -- amortised over twice the columns; 2 operand stages).
+template <int F, int NK>
 struct Lay3 {
     static constexpr int BC = MROWS / F;                       // channels per fh slot
     // Two rings (the raw TMA tiles are 20 KB, the hi / lo operands 48 KB, so
@@ -61,7 +62,7 @@ struct Lay3 {
     static constexpr int OFF_B = 2 * 4 * ASLAB;                // 32 KB
     static constexpr int OP = OFF_B + 2 * 4 * BSLAB;           // 48 KB
     static constexpr int LIMIT = 227 * 1024 - 1024 - 512;
-    static constexpr int SO = 3;
+    static constexpr int SO = NK == 64 ? 3 : 2;
     static constexpr int SR = (LIMIT - SO * OP) / RAW > 6 ? 6 : (LIMIT - SO * OP) / RAW;   // 4
     static constexpr int OP_OFF = SR * RAW;
     static constexpr int RING = OP_OFF + SO * OP;
@@ -89,15 +90,17 @@ __device__ __forceinline__ uint64_t desc_k(uint32_t addr) {
     return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)(128 >> 4) << 16) | ((uint64_t)(256 >> 4) << 32) |
            (1ull << 46);
 }
-// kind::tf32 instruction descriptor: D f32, A/B tf32 (2), both K-major, N = 64, M = 128.
+// kind::tf32 instruction descriptor: D f32, A/B tf32 (2), both K-major, N = NK, M = 128.
+template <int NK>
 __host__ __device__ constexpr uint32_t idesc_tf32() {
     return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(NK >> 3) << 17) | ((uint32_t)(MROWS >> 4) << 24);
 }
+template <int NK>
 __device__ __forceinline__ void umma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t acc) {
     asm volatile(
         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
         "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n"
-        :: "r"(d), "l"(a), "l"(b), "r"(idesc_tf32()), "r"(acc));
+        :: "r"(d), "l"(a), "l"(b), "r"(idesc_tf32<NK>()), "r"(acc));
 }
 // lo part of the 3xTF32 split (hi = the word itself: the tensor core reads its top 19 bits)
 __device__ __forceinline__ float tf32_lo(float x) { return x - __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
@@ -111,12 +114,12 @@ __device__ __forceinline__ void sts4f(uint32_t a, float x, float y, float z, flo
 }
 __device__ __forceinline__ uint32_t koff(int row, int k4) { return (uint32_t)((row >> 3) * 256 + k4 * 128 + (row & 7) * 16); }
 
-template <int F>
+template <int F, int NK>
 __global__ void __launch_bounds__(NTHREADS, 1)
 bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX,
                const __grid_constant__ CUtensorMap tmY) {
     using namespace tc2;
-    using L = Lay3<F>;
+    using L = Lay3<F, NK>;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw_s = su(smem_raw);
     uint8_t* smem = smem_raw + (((raw_s + 1023u) & ~1023u) - raw_s);
@@ -229,9 +232,9 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     const uint64_t al = desc_k(st + L::OFF_A + (4 + x) * L::ASLAB);
                     const uint64_t bh = desc_k(st + L::OFF_B + x * L::BSLAB);
                     const uint64_t bl = desc_k(st + L::OFF_B + (4 + x) * L::BSLAB);
-                    umma_tf32(tmem + x * NK, ah, bh, acc);   // fixed order: hi.hi, hi.lo, lo.hi
-                    umma_tf32(tmem + x * NK, ah, bl, 1u);
-                    umma_tf32(tmem + x * NK, al, bh, 1u);
+                    umma_tf32<NK>(tmem + x * NK, ah, bh, acc);   // fixed order: hi.hi, hi.lo, lo.hi
+                    umma_tf32<NK>(tmem + x * NK, ah, bl, 1u);
+                    umma_tf32<NK>(tmem + x * NK, al, bh, 1u);
                 }
                 umma_commit<1>(&bars->opempty[s]);
             }
@@ -252,7 +255,7 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         const int m = q * 32 + lane;
         const int f = m / L::BC, cm = m % L::BC;
         const uint32_t xrow = (uint32_t)(L::OFF_X + f * L::XSLOT + cm * 4);
-        const int t = q * 32 + lane, kk = t % NK, dh = t / NK;
+        const int t = q * 32 + lane;
         int s = G, so = G;                     // raw slot, operand slot
         uint32_t ph = 0, pho = 0;
         for (int ch = c_lo + G; ch < c_hi; ch += 2) {
@@ -283,7 +286,9 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     sts4f(ot + L::OFF_A + (4 + a) * L::ASLAB + o, lo[a][0], lo[a][1], lo[a][2], lo[a][3]);
                 }
             }
-            {
+#pragma unroll
+            for (int it2 = 0; it2 < NK / 64; ++it2) {   // dY items (k, depth half): NK x 2 over 128 threads
+                const int ti = t + it2 * 128, kk = ti % NK, dh = ti / NK;
                 float w[4][4];   // [xi][depth j]
 #pragma unroll
                 for (int j = 0; j < 4; ++j) {

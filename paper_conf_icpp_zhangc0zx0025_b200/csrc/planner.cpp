@@ -250,7 +250,7 @@ static TimeModel time_model(const KernelEntry& e) {
     if (e.fhs > 0 && e.cg == 2)   // bfc_tc2.cuh CTA pair: rate of the pair over its 256-row tile
         return {4.5e-6, 11.0e12};
     if (e.fhs > 0 && e.tf32)   // bfc_tc3.cuh: FP32 inputs, 12 tf32 MMAs per 8-deep stage (3xTF32)
-        return {4.0e-6, 1.05e12};  // tools/tc3_check.py --time (R50 FP32 L1-L4: 134/120/113/112 us)
+        return {4.0e-6, bn >= 128 ? 1.45e12 : 1.05e12};   // tools/tc3_check.py --time: NK = 128 ~1.4x per flop
     if (e.fhs > 0 && e.ta)   // bfc_tc2.cuh TA (Xhat in TMEM, NK = 64, two TMA producer warps):
         return {4.0e-6, 5.6e12};   // tools/ta_ab.py: VGG L1 988 -> 644 us, R50 L1 57.3 -> 44.0 us
     if (e.fhs > 0) {

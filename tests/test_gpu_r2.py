@@ -165,6 +165,10 @@ TC3 = [
     ("z5", dict(N=16, C=64, K=64, H=30, W=30), {"WINRS_FORCE_Z": "5"}),
     ("cs8", dict(N=24, C=128, K=64, H=12, W=12), {"WINRS_FORCE_CSPLIT": "8"}),
     ("cs6_f2", dict(N=16, C=64, K=128, H=12, W=12), {"WINRS_FORCE_CSPLIT": "6", "WINRS_FORCE_TILE": "64x64"}),
+    ("nk128", dict(N=8, C=128, K=128, H=14, W=14), {"WINRS_FORCE_TILE": "128x128"}),
+    ("nk128_f2_ragged_cs3", dict(N=16, C=40, K=200, H=13, W=11), {"WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "3"}),
+    ("nk128_z3_cs4", dict(N=16, C=64, K=128, H=30, W=30), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_Z": "3",
+                                                          "WINRS_FORCE_CSPLIT": "4"}),
 ]
 
 

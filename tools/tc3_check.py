@@ -28,6 +28,10 @@ CASES = [
     ("s6", dict(N=8, C=64, K=64, H=16, W=16, R=3, S=6, pad=2), {"WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
     ("z5", dict(N=16, C=64, K=64, H=30, W=30), {"WINRS_FORCE_Z": "5"}),
     ("cs8", dict(N=24, C=128, K=64, H=12, W=12), {"WINRS_FORCE_CSPLIT": "8"}),
+    ("nk128", dict(N=8, C=128, K=128, H=14, W=14), {"WINRS_FORCE_TILE": "128x128"}),
+    ("nk128_f2_ragged", dict(N=16, C=40, K=200, H=13, W=11), {"WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "3"}),
+    ("nk128_z3_cs4", dict(N=16, C=64, K=128, H=30, W=30), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_Z": "3",
+                                                          "WINRS_FORCE_CSPLIT": "4"}),
 ]
 KEYS = ("WINRS_FORCE_TILE", "WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_FP32_TC")
 
@@ -63,10 +67,12 @@ def timing():
     for l in wl.RESNET50_F32 + wl.WIDE_F32[-1:]:
         X, dY = wl.make_inputs(l)
         Xg, Gg = torch.from_numpy(X).cuda(), torch.from_numpy(dY).cuda()
-        for tc in ("0", "1"):
+        for tc, tile in (("0", None), ("1", None), ("1", "64x128"), ("1", "128x128"), ("1", "128x64"), ("1", "64x64")):
             for k in KEYS:
                 os.environ.pop(k, None)
             os.environ["WINRS_FP32_TC"] = tc
+            if tile:
+                os.environ["WINRS_FORCE_TILE"] = tile
             try:
                 p = W.plan(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, "f32")
             except Exception as e:
