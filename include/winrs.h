@@ -226,6 +226,38 @@ WINRS_API winrs_status_t winrs_bdc(winrs_conv_plan_t plan, const void* dY, const
 /* Destroy a conv plan and its BFC plan (NULL is a no-op). */
 WINRS_API void winrs_conv_plan_destroy(winrs_conv_plan_t plan);
 
+/* ---------------------------------------------------------------------------
+ * Data-parallel BFC with the bucket reduction and the cross-rank sum fused
+ * into one kernel over peer memory (§3
+ * P@17126 "launch a reduction kernel to sum all nabla W buckets", §5.2 P@39101
+ * FP32 Kahan summation).  Each rank runs winrs_bfc_allreduce on its batch
+ * shard; afterwards every rank's dW holds
+ *     dW = sum_{q = 0..world-1, in rank order} ( Kahan_z bucket_z of rank q )
+ * in FP32, bit-identical on all ranks and to the unfused path (winrs_bfc on
+ * each rank, then an FP32 sum of the ranks' dW in rank order).
+ * Buffers are shared between processes with CUDA IPC:
+ *   winrs_ipc_alloc  cudaMalloc + zero fill + the 64-byte IPC handle;
+ *   winrs_ipc_open   map a peer's handle (not one's own) into this process;
+ *   winrs_ipc_close / winrs_ipc_free.
+ * Per rank q: stage[q] and dW[q] of |dW| = K*R*S*C floats, flags[q] of
+ * winrs_allreduce_flag_bytes() bytes (zero-initialised, owned by rank q).
+ * peer_* are HOST arrays of world device pointers as seen by this process
+ * (peer_dW[rank] == dW).  epoch: 1, 2, 3, ... -- the same value on every rank
+ * for a given call, one larger than the previous call's.  world <= 8.
+ * The kernel is a cooperative launch whose barriers spin on the peers' flags;
+ * a rank that never arrives makes it trap after ~20 s (WINRS_ERR_CUDA or a
+ * sticky CUDA error) instead of hanging.  INVALID_ARG for a bad rank / world /
+ * epoch, a null or misaligned pointer, or peer_dW[rank] != dW. */
+WINRS_API winrs_status_t winrs_ipc_alloc(size_t bytes, void** ptr, unsigned char* handle);
+WINRS_API winrs_status_t winrs_ipc_open(const unsigned char* handle, void** ptr);
+WINRS_API winrs_status_t winrs_ipc_close(void* ptr);
+WINRS_API winrs_status_t winrs_ipc_free(void* ptr);
+WINRS_API size_t winrs_allreduce_flag_bytes(void);
+WINRS_API winrs_status_t winrs_bfc_allreduce(winrs_plan_t plan, const void* X, const void* dY, float* dW,
+                                             void* workspace, void* const* peer_stage, float* const* peer_dW,
+                                             void* const* peer_flags, int rank, int world, unsigned int epoch,
+                                             void* stream);
+
 #ifdef __cplusplus
 }
 #endif

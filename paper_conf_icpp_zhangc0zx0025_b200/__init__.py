@@ -20,7 +20,7 @@ from . import _lib
 from ._lib import WinrsError, DTYPES
 
 __all__ = ["Plan", "plan", "plan_for_device", "plan3d", "plan3d_for_device", "bfc", "bfc_host", "as_kcrs", "as_krsc", "bfc_data_parallel", "shard_range",
-           "bfc_k_sharded", "ConvPlan", "conv_plan", "conv_plan_for_device", "fc", "bdc", "emulate_conv",
+           "bfc_k_sharded", "PeerAllreduce", "ConvPlan", "conv_plan", "conv_plan_for_device", "fc", "bdc", "emulate_conv",
            "WinrsError", "version", "emulate", "transform", "kernel_names"]
 
 
@@ -294,6 +294,87 @@ def bfc_data_parallel(X_shard, dY_shard, R: int, S: int, pad: int, dtype: str = 
     if dist.is_initialized() and dist.get_world_size(group) > 1:
         dist.all_reduce(as_krsc(dW), op=dist.ReduceOp.SUM, group=group)   # the contiguous KRSC storage
     return dW
+
+
+class _CudaBuf:
+    """A raw device buffer exposed to torch through __cuda_array_interface__ (no copy)."""
+
+    def __init__(self, ptr, n):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": "<f4", "data": (int(ptr), False), "version": 2}
+
+
+class PeerAllreduce:
+    """Data-parallel BFC with the bucket reduction and the cross-rank sum fused
+    into one kernel over peer memory (winrs_bfc_allreduce, include/winrs.h;
+    SURVEY §8(f) row 1).  Collective constructor over a torch.distributed group
+    (any backend: only the 64-byte CUDA IPC handles are exchanged, with
+    all_gather_object).  `bfc(X, dY)` returns this rank's dW, logical [K,C,R,S]
+    channels_last like `bfc()`, identical on every rank."""
+
+    def __init__(self, p: Plan, group=None):
+        import torch.distributed as dist
+        self.p = p
+        self.rank = dist.get_rank(group) if dist.is_initialized() else 0
+        self.world = dist.get_world_size(group) if dist.is_initialized() else 1
+        i = p.info
+        self.n = i["K"] * i["T"] * i["R"] * i["S"] * i["C"]
+        L = _lib.lib()
+        self._own, handles = [], []
+        for nbytes in (4 * self.n, 4 * self.n, int(L.winrs_allreduce_flag_bytes())):   # stage, dW, flags
+            ptr, h = ctypes.c_void_p(), ctypes.create_string_buffer(64)
+            _lib.check(L.winrs_ipc_alloc(nbytes, ctypes.byref(ptr), h), "winrs_ipc_alloc")
+            self._own.append(ptr.value)
+            handles.append(h.raw)
+        allh = [None] * self.world
+        if self.world > 1:
+            dist.all_gather_object(allh, handles, group=group)
+        else:
+            allh = [handles]
+        self._opened = []
+        peers = [[None] * self.world for _ in range(3)]
+        for q in range(self.world):
+            for j in range(3):
+                if q == self.rank:
+                    peers[j][q] = self._own[j]
+                else:
+                    ptr = ctypes.c_void_p()
+                    _lib.check(L.winrs_ipc_open(allh[q][j], ctypes.byref(ptr)), "winrs_ipc_open")
+                    self._opened.append(ptr.value)
+                    peers[j][q] = ptr.value
+        arr = ctypes.c_void_p * self.world
+        self._stage, self._dW, self._flags = (arr(*peers[0]), arr(*peers[1]), arr(*peers[2]))
+        self.epoch = 0
+        self._group = group
+
+    def bfc(self, X, dY, workspace=None, stream=None):
+        import torch
+        i = self.p.info
+        tdt = {"f32": torch.float32, "f16": torch.float16, "bf16": torch.bfloat16}[self.p.dtype]
+        Xn = _as_nhwc(X, i["N"], i["H"], i["W"], i["C"], "X")
+        Gn = _as_nhwc(dY, i["N"], i["Ho"], i["Wo"], i["K"], "dY")
+        if Xn.dtype != tdt or Gn.dtype != tdt:
+            raise TypeError(f"X and dY must be {tdt} for this plan")
+        if stream is None:
+            stream = torch.cuda.current_stream(Xn.device)
+        sp = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+        wsb = self.p.workspace_bytes
+        if wsb and workspace is None:
+            workspace = torch.empty(wsb, dtype=torch.uint8, device=Xn.device)
+        self.epoch += 1
+        _lib.check(_lib.lib().winrs_bfc_allreduce(self.p.handle, Xn.data_ptr(), Gn.data_ptr(), self._own[1],
+                                                  workspace.data_ptr() if wsb else None, self._stage, self._dW,
+                                                  self._flags, self.rank, self.world, self.epoch, sp),
+                   "winrs_bfc_allreduce")
+        dW = torch.as_tensor(_CudaBuf(self._own[1], self.n), device=Xn.device).view(i["K"], i["R"], i["S"], i["C"])
+        return dW.permute(0, 3, 1, 2)
+
+    def close(self):
+        L = _lib.lib()
+        for ptr in getattr(self, "_opened", []):
+            L.winrs_ipc_close(ptr)
+        for ptr in getattr(self, "_own", []):
+            L.winrs_ipc_free(ptr)
+        self._opened, self._own = [], []
 
 
 class ConvPlan:

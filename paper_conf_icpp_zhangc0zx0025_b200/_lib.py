@@ -66,6 +66,13 @@ SYMBOLS = [
     ("winrs_fc", _i, [_p, _p, _p, _p, _p, _p]),
     ("winrs_bdc", _i, [_p, _p, _p, _p, _p, _p]),
     ("winrs_conv_plan_destroy", None, [_p]),
+    ("winrs_ipc_alloc", _i, [_s, ctypes.POINTER(_p), ctypes.c_char_p]),
+    ("winrs_ipc_open", _i, [ctypes.c_char_p, ctypes.POINTER(_p)]),
+    ("winrs_ipc_close", _i, [_p]),
+    ("winrs_ipc_free", _i, [_p]),
+    ("winrs_allreduce_flag_bytes", _s, []),
+    ("winrs_bfc_allreduce", _i, [_p, _p, _p, _p, _p, ctypes.POINTER(_p), ctypes.POINTER(_p), ctypes.POINTER(_p),
+                                 _i, _i, ctypes.c_uint, _p]),
     # winrs_debug.h
     ("winrs_debug_emulate", _i, [_p, _p, _p, _p]),
     ("winrs_debug_transform", _i, [_i, _i, _i, _i, _p, _p]),

@@ -35,4 +35,15 @@ const KernelEntry* kernel_entries(int* count);
 cudaError_t launch_bucket_reduce(float* dW, const float* ws, long long n, int Z, int num_sms,
                                  cudaStream_t stream);
 
+// Fused bucket reduction + cross-rank all-reduce over peer memory (allreduce.cu).
+constexpr int AR_MAX = 8;
+struct PeerArgs {
+    float* stage[AR_MAX];
+    float* dW[AR_MAX];
+    unsigned int* flags[AR_MAX];
+};
+cudaError_t launch_fused_reduce_allreduce(const float* dW_local, const float* ws, long long n, int Z,
+                                          const PeerArgs& pa, unsigned int* counter, int rank, int world,
+                                          unsigned int epoch, int num_sms, cudaStream_t stream);
+
 }  // namespace winrs

@@ -185,6 +185,83 @@ winrs_status_t winrs_bfc_host(winrs_plan_t plan, const void* host_X, const void*
     return WINRS_OK;
 }
 
+// ---------------------------------------------------------------------------
+// Fused bucket reduction + cross-rank all-reduce over peer memory (allreduce.cu).
+
+winrs_status_t winrs_ipc_alloc(size_t bytes, void** ptr, unsigned char* handle) {
+    if (!ptr || !handle || bytes == 0) return WINRS_ERR_INVALID_ARG;
+    *ptr = nullptr;
+    void* p = nullptr;
+    if (cudaMalloc(&p, bytes) != cudaSuccess) { cudaGetLastError(); return WINRS_ERR_CUDA; }
+    cudaIpcMemHandle_t h;
+    if (cudaMemset(p, 0, bytes) != cudaSuccess || cudaIpcGetMemHandle(&h, p) != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(p);
+        return WINRS_ERR_CUDA;
+    }
+    memcpy(handle, &h, sizeof(h));
+    *ptr = p;
+    return WINRS_OK;
+}
+
+winrs_status_t winrs_ipc_open(const unsigned char* handle, void** ptr) {
+    if (!ptr || !handle) return WINRS_ERR_INVALID_ARG;
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle, sizeof(h));
+    if (cudaIpcOpenMemHandle(ptr, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        cudaGetLastError();
+        *ptr = nullptr;
+        return WINRS_ERR_CUDA;
+    }
+    return WINRS_OK;
+}
+
+winrs_status_t winrs_ipc_close(void* ptr) {
+    if (!ptr) return WINRS_ERR_INVALID_ARG;
+    if (cudaIpcCloseMemHandle(ptr) != cudaSuccess) { cudaGetLastError(); return WINRS_ERR_CUDA; }
+    return WINRS_OK;
+}
+
+winrs_status_t winrs_ipc_free(void* ptr) {
+    if (!ptr) return WINRS_ERR_INVALID_ARG;
+    if (cudaFree(ptr) != cudaSuccess) { cudaGetLastError(); return WINRS_ERR_CUDA; }
+    return WINRS_OK;
+}
+
+size_t winrs_allreduce_flag_bytes(void) { return 128; }
+
+winrs_status_t winrs_bfc_allreduce(winrs_plan_t plan, const void* X, const void* dY, float* dW, void* workspace,
+                                   void* const* peer_stage, float* const* peer_dW, void* const* peer_flags,
+                                   int rank, int world, unsigned int epoch, void* stream) {
+    if (!plan || !X || !dY || !dW || !peer_stage || !peer_dW || !peer_flags) return WINRS_ERR_INVALID_ARG;
+    if (world < 1 || world > AR_MAX || rank < 0 || rank >= world || epoch == 0) return WINRS_ERR_INVALID_ARG;
+    if (peer_dW[rank] != dW) return WINRS_ERR_INVALID_ARG;
+    PeerArgs pa = {};
+    for (int q = 0; q < world; ++q) {
+        if (!peer_stage[q] || !peer_dW[q] || !peer_flags[q] || misaligned(peer_stage[q]) || misaligned(peer_dW[q]) ||
+            misaligned(peer_flags[q]))
+            return WINRS_ERR_INVALID_ARG;
+        pa.stage[q] = static_cast<float*>(peer_stage[q]);
+        pa.dW[q] = peer_dW[q];
+        pa.flags[q] = static_cast<unsigned int*>(peer_flags[q]);
+    }
+    if (misaligned(X) || misaligned(dY) || misaligned(dW)) return WINRS_ERR_INVALID_ARG;
+    Geometry g = plan->pr.geom;
+    g.ldy = plan->info.K;
+    if (plan->info.workspace_bytes > 0) {
+        if (!workspace) return WINRS_ERR_WORKSPACE;
+        if (misaligned(workspace)) return WINRS_ERR_INVALID_ARG;
+    }
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    cudaError_t e = plan->pr.entry->launch(g, X, dY, dW, static_cast<float*>(workspace), s);
+    if (e != cudaSuccess) return WINRS_ERR_CUDA;
+    // this rank's arrival counter lives after the 2 x AR_MAX flag words of its own block
+    unsigned int* counter = pa.flags[rank] + 2 * AR_MAX;
+    e = launch_fused_reduce_allreduce(dW, static_cast<const float*>(workspace), g.dw_elems, g.Z, pa, counter, rank,
+                                      world, epoch, plan->num_sms, s);
+    return e == cudaSuccess ? WINRS_OK : WINRS_ERR_CUDA;
+}
+
 void winrs_plan_destroy(winrs_plan_t plan) { delete plan; }
 
 const char* winrs_status_string(winrs_status_t s) {

@@ -243,3 +243,23 @@ def test_plan3d_decomposition_emulated(shape, env, monkeypatch):
     p32 = W.plan3d_for_device(N, C, D, H, Wd, K, T, R, S, pad, "f32")    # FP32 kernel decomposition
     got32 = W.emulate(p32, X, dY)
     assert np.allclose(got32, ref, rtol=1e-11, atol=1e-11), (p32, np.max(np.abs(got32 - ref)))
+
+
+def test_bfc_allreduce_validates_arguments():
+    """winrs_bfc_allreduce rejects a bad rank / world /
+    epoch, null peers and peer_dW[rank] != dW before any launch (no GPU needed)."""
+    import ctypes
+    from paper_conf_icpp_zhangc0zx0025_b200 import _lib
+    L = _lib.lib()
+    p = W.plan_for_device(2, 16, 8, 8, 16, 3, 3, 1, "f32")
+    fake = 1 << 20
+    arr = ctypes.c_void_p * 2
+    st, dw, fl = arr(fake, fake + 4096), arr(fake + 8192, fake + 12288), arr(fake + 16384, fake + 16512)
+    call = lambda rank, world, epoch, dW=fake + 8192: L.winrs_bfc_allreduce(
+        p.handle, fake, fake, dW, None, st, dw, fl, rank, world, epoch, None)
+    assert call(0, 9, 1) == 1          # world > 8
+    assert call(2, 2, 1) == 1          # rank >= world
+    assert call(0, 2, 0) == 1          # epoch 0 would pass the flags immediately
+    assert call(1, 2, 1) == 1          # peer_dW[rank] != dW
+    assert L.winrs_bfc_allreduce(p.handle, fake, fake, fake, None, None, dw, fl, 0, 2, 1, None) == 1
+    assert L.winrs_allreduce_flag_bytes() >= 4 * (2 * 8 + 1)
