@@ -281,9 +281,14 @@ def measure(layers, args, ctx, primary=True):
             Xt, Gt = Xt.to(torch.bfloat16), Gt.to(torch.bfloat16)
         dW = torch.empty((k1 - k0, l.R, l.S, l.C), dtype=torch.float32, device=dev)
         ws = torch.empty(max(p.workspace_bytes, 16), dtype=torch.uint8, device=dev)
-        items.append(dict(layer=l, local=ll, plan=p, X=Xt.to(dev), dY=Gt.to(dev), dW=dW, ws=ws,
-                          Xh=Xt.pin_memory(), Gh=Gt.pin_memory(), dWh=torch.empty(dW.shape).pin_memory(),
-                          k0=k0, k1=k1))
+        it = dict(layer=l, local=ll, plan=p, X=Xt.to(dev), dY=Gt.to(dev), dW=dW, ws=ws,
+                  Xh=Xt.pin_memory(), Gh=Gt.pin_memory(), dWh=torch.empty(dW.shape).pin_memory(), k0=k0, k1=k1)
+        if ctx.get("fused") and world > 1 and not kshard:
+            # bucket reduction + cross-rank sum in one kernel over peer memory (winrs_bfc_allreduce);
+            # dW is then the IPC-shared output buffer (collective setup: every rank, same order)
+            it["par"] = W.PeerAllreduce(p)
+            it["dW"] = W.as_krsc(it["par"].bfc(it["X"], it["dY"], ws))
+        items.append(it)
     stream = torch.cuda.current_stream(dev)
 
     def bfc_only(it, s):
@@ -297,6 +302,9 @@ def measure(layers, args, ctx, primary=True):
             W.bfc(it["plan"], it["X"], it["dY"], it["dW"], it["ws"], s)
 
     def run_bfc(it, s):
+        if "par" in it:                    # fused bucket reduction + all-reduce (one kernel, peer memory)
+            it["par"].bfc(it["X"], it["dY"], it["ws"], s)
+            return
         bfc_only(it, s)
         if world > 1 and not kshard:
             dist.all_reduce(it["dW"])      # the data-parallel step's one exchange (NCCL over NVLink)
@@ -523,7 +531,7 @@ def run_winrs(args):
     kshard = args.parallel == "kshard" and world > 1
     strong = args.workload == "r50l3" and world > 1 and not kshard
     ctx = dict(world=world, rank=rank, local=local, dev=dev, kshard=kshard, strong=strong,
-               flush=torch.empty(256 << 20, dtype=torch.uint8, device=dev))
+               fused=args.allreduce == "fused", flush=torch.empty(256 << 20, dtype=torch.uint8, device=dev))
     layers = _workload(args.workload, args.dtype)
     m = measure(layers, args, ctx, primary=True)
     alongside = []
@@ -556,6 +564,7 @@ def run_winrs(args):
         cfg = {"workload": f"{args.workload}_{args.dtype}: " + ", ".join(x["layer"].name for x in m["items"]),
                "global_batch": (m["items"][0]["layer"].N if (strong or kshard) else m["items"][0]["layer"].N * world),
                "parallelism": (f"kshard{world}" if kshard else f"dp{world}") if world > 1 else "single",
+               "allreduce": (args.allreduce if world > 1 and not kshard else None),
                "backend": backend,
                "l2": "flushed (256 MiB write) before every layer call; flush outside timed events",
                "workspace_cap": float(os.environ.get("WINRS_WS_CAP", "0.04")),
@@ -707,6 +716,9 @@ def main():
     ap.add_argument("--parallel", default="dp", choices=["dp", "kshard"],
                     help="N>1: dp = batch shards + one all_reduce of dW; kshard = output-channel "
                          "shards of the full batch, no communication (strong)")
+    ap.add_argument("--allreduce", default="nccl", choices=["nccl", "fused"],
+                    help="N>1 dp: nccl = bucket reduction, then one NCCL all_reduce; fused = both in one "
+                         "kernel over CUDA-IPC peer memory (winrs_bfc_allreduce)")
     ap.add_argument("--ws-cap", type=float, default=None,
                     help="planner workspace cap as a fraction of X+dY bytes (default: the paper's 4%%)")
     ap.add_argument("--dry-run", action="store_true", help="launch plumbing only (gloo, no GPU work)")
