@@ -25,7 +25,14 @@
 // zero-fill replaces texture -1 masking; 4-wide interleaved register tiles
 // replace the "contrapuntal" offsets; the residual kernel is fused into the
 // same launch instead of a separate block group.
+//
+// TI (input element type): float, or __half / __nv_bfloat16 for the FP16 /
+// BF16 plans whose kernel pair has no tensor-core kernel (the alpha = 16
+// widths, R26): 16-bit inputs are staged as they are and widened to
+// FP32 when the transforms read them; transforms, EWM and OT stay FP32.
 #pragma once
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include "dsmem.cuh"
@@ -74,6 +81,12 @@ __device__ __forceinline__ void cp_async16(void* dst, const void* src, bool vali
                  :: "r"(smem_u32(dst)), "l"(src), "r"(sz) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+// Two consecutive raw elements widened to FP32.
+__device__ __forceinline__ float2 ld2f(const float* p) { return *reinterpret_cast<const float2*>(p); }
+__device__ __forceinline__ float2 ld2f(const __half* p) { return __half22float2(*reinterpret_cast<const __half2*>(p)); }
+__device__ __forceinline__ float2 ld2f(const __nv_bfloat16* p) {
+    return __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(p));
+}
 template <int N_>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" :: "n"(N_) : "memory"); }
 
@@ -154,15 +167,16 @@ __device__ __forceinline__ void phase_chunks(const Geometry& g, const PhaseCtx& 
 }
 
 // ================= warpgroup 0: cp.async loads + FP32 transforms of one job =================
-template <int ALPHA, int NN, int RR, int BN, int BM, int S_RAW, int BD>
-__device__ __forceinline__ void producer_phase(const Geometry& g, const float* __restrict__ X,
-                                               const float* __restrict__ dY, const CtaCoord& cc, const PhaseCtx& P,
+template <int ALPHA, int NN, int RR, int BN, int BM, int S_RAW, int BD, typename TI = float>
+__device__ __forceinline__ void producer_phase(const Geometry& g, const TI* __restrict__ X,
+                                               const TI* __restrict__ dY, const CtaCoord& cc, const PhaseCtx& P,
                                                float* smem, TRing& ring, int& tcount) {
     using WT = Wino<ALPHA, NN, RR>;
     using SM = PhaseSmem<ALPHA, RR, BN, BM, S_RAW, BD>;
-    float* rawG = smem;                       // [S_RAW][BD][RR][BN]
-    float* rawX = rawG + SM::rawG;            // [S_RAW][BD][ALPHA][BM]
-    float* Gt = rawX + SM::rawX;              // [S_T][ALPHA][BD][BN]
+    constexpr int VE = 16 / (int)sizeof(TI);  // elements per 16-byte copy
+    TI* rawG = reinterpret_cast<TI*>(smem);   // [S_RAW][BD][RR][BN] (16-bit inputs use half the region)
+    TI* rawX = rawG + SM::rawG;               // [S_RAW][BD][ALPHA][BM]
+    float* Gt = smem + SM::rawG + SM::rawX;   // [S_T][ALPHA][BD][BN]
     float* Xt = Gt + SM::Gt;                  // [S_T][ALPHA][BD][BM]
     const int k_base = cc.kb * BN, c_base = cc.cb * BM;
     long long d_lo, d_hi;
@@ -187,7 +201,7 @@ __device__ __forceinline__ void producer_phase(const Geometry& g, const float* _
     auto issue = [&](int buf) {
         const bool dv = d < d_hi;
         const int w0 = P.w_first + u * RR;
-        const float* gsrc = dY + (((long long)n * g.Ho + h) * g.Wo + w0) * g.ldy + k_base;
+        const TI* gsrc = dY + (((long long)n * g.Ho + h) * g.Wo + w0) * g.ldy + k_base;
         // filter row fh = (depth tap fh / Rh, height tap fh % Rh); for an N-D plan
         // image n = (batch n / Do, dY depth slice n % Do) reads X slice
         // (n % Do) + t - pad, zero outside [0, D) (PAPER.md P@17805)
@@ -200,30 +214,30 @@ __device__ __forceinline__ void producer_phase(const Geometry& g, const float* _
             dok = dd >= 0 && dd < g.D;
             ximg = (long long)(n / g.Do) * g.D + dd;
         }
-        const float* xsrc = X + ((ximg * g.H + xrow) * g.W) * g.C + c_base;
-        float* gdst = rawG + ((buf * BD + ld_d) * RR) * BN;
-        float* xdst = rawX + ((buf * BD + ld_d) * ALPHA) * BM;
-        constexpr int GV = RR * (BN / 4);
+        const TI* xsrc = X + ((ximg * g.H + xrow) * g.W) * g.C + c_base;
+        TI* gdst = rawG + ((buf * BD + ld_d) * RR) * BN;
+        TI* xdst = rawX + ((buf * BD + ld_d) * ALPHA) * BM;
+        constexpr int GV = RR * (BN / VE);
 #pragma unroll
         for (int it = 0; it < (GV + TPD - 1) / TPD; ++it) {
             const int q = ld_l + it * TPD;
             if (GV % TPD == 0 || q < GV) {
-                const int i = q / (BN / 4), v4 = q % (BN / 4);
-                const bool ok = dv && (w0 + i < g.Wo) && (k_base + v4 * 4 < g.K);
-                cp_async16(gdst + i * BN + v4 * 4, ok ? (const void*)(gsrc + (long long)i * g.ldy + v4 * 4) : (const void*)dY,
-                           ok);
+                const int i = q / (BN / VE), v4 = q % (BN / VE);
+                const bool ok = dv && (w0 + i < g.Wo) && (k_base + v4 * VE < g.K);
+                cp_async16(gdst + i * BN + v4 * VE,
+                           ok ? (const void*)(gsrc + (long long)i * g.ldy + v4 * VE) : (const void*)dY, ok);
             }
         }
-        constexpr int XV = ALPHA * (BM / 4);
+        constexpr int XV = ALPHA * (BM / VE);
 #pragma unroll
         for (int it = 0; it < (XV + TPD - 1) / TPD; ++it) {
             const int q = ld_l + it * TPD;
             if (XV % TPD == 0 || q < XV) {
-                const int t = q / (BM / 4), v4 = q % (BM / 4);
+                const int t = q / (BM / VE), v4 = q % (BM / VE);
                 const int col = xcol0 + t;
-                const bool ok = dv && dok && col >= 0 && col < g.W && c_base + v4 * 4 < g.C;
-                cp_async16(xdst + t * BM + v4 * 4, ok ? (const void*)(xsrc + (long long)col * g.C + v4 * 4) : (const void*)X,
-                           ok);
+                const bool ok = dv && dok && col >= 0 && col < g.W && c_base + v4 * VE < g.C;
+                cp_async16(xdst + t * BM + v4 * VE,
+                           ok ? (const void*)(xsrc + (long long)col * g.C + v4 * VE) : (const void*)X, ok);
             }
         }
         // advance to this thread's entry of the next chunk
@@ -252,13 +266,13 @@ __device__ __forceinline__ void producer_phase(const Geometry& g, const float* _
         const int buf = ch % S_RAW;
         float* Gs = Gt + ts * SM::Gt1;
         float* Xs = Xt + ts * SM::Xt1;
-        const float* rg = rawG + buf * BD * RR * BN;
+        const TI* rg = rawG + buf * BD * RR * BN;
         for (int p = ptid; p < BD * (BN / 2); p += NP) {
             const int d = p / (BN / 2), k = 2 * (p % (BN / 2));
             F2 w[RR], o[ALPHA];
 #pragma unroll
             for (int i = 0; i < RR; ++i) {
-                const float2 t = *reinterpret_cast<const float2*>(rg + (d * RR + i) * BN + k);
+                const float2 t = ld2f(rg + (d * RR + i) * BN + k);
                 w[i] = F2{t.x, t.y};
             }
             WT::ft(w, o);
@@ -266,13 +280,13 @@ __device__ __forceinline__ void producer_phase(const Geometry& g, const float* _
             for (int x = 0; x < ALPHA; ++x)
                 *reinterpret_cast<float2*>(Gs + (x * BD + d) * BN + k) = make_float2(o[x].x, o[x].y);
         }
-        const float* rx = rawX + buf * BD * ALPHA * BM;
+        const TI* rx = rawX + buf * BD * ALPHA * BM;
         for (int p = ptid; p < BD * (BM / 2); p += NP) {
             const int d = p / (BM / 2), c = 2 * (p % (BM / 2));
             F2 xv[ALPHA], o[ALPHA];
 #pragma unroll
             for (int t = 0; t < ALPHA; ++t) {
-                const float2 q = *reinterpret_cast<const float2*>(rx + (d * ALPHA + t) * BM + c);
+                const float2 q = ld2f(rx + (d * ALPHA + t) * BM + c);
                 xv[t] = F2{q.x, q.y};
             }
             WT::it(xv, o);
@@ -458,9 +472,9 @@ constexpr size_t smem_bytes() {
 // cluster rank's share of the depth), CTAs of a band's last column segment
 // also run the residual Omega_a1 phase into the same staged tile, then the
 // tile (summed over the cluster) is written to the segment's bucket.
-template <int A0, int N0, int R0, int A1, int N1, int R1, int BN, int BM>
+template <int A0, int N0, int R0, int A1, int N1, int R1, int BN, int BM, typename TI = float>
 __global__ void __launch_bounds__(NTOT, 1)
-bfc_f32_kernel(const Geometry g, const float* __restrict__ X, const float* __restrict__ dY,
+bfc_f32_kernel(const Geometry g, const TI* __restrict__ X, const TI* __restrict__ dY,
                float* __restrict__ dW, float* __restrict__ ws) {
     extern __shared__ __align__(16) float smem[];
     float* Out = smem + pipe_floats<A0, N0, R0, A1, N1, R1, BN, BM>();
@@ -491,7 +505,7 @@ bfc_f32_kernel(const Geometry g, const float* __restrict__ X, const float* __res
     if (threadIdx.x < NP) {
         // the transformer warpgroup hands registers to the GEMM warpgroups
         asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" :: "n"(REG_P));
-        producer_phase<A0, N0, R0, BN, BM, C::SR, C::BD>(g, X, dY, cc, P0, smem, ring, tcount);
+        producer_phase<A0, N0, R0, BN, BM, C::SR, C::BD, TI>(g, X, dY, cc, P0, smem, ring, tcount);
         __syncwarp();   // bar.sync is .aligned: the warp must be converged
         asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");   // job boundary (ring reused by the OT)
         if constexpr (A1 != 0) {
@@ -499,8 +513,8 @@ bfc_f32_kernel(const Geometry g, const float* __restrict__ X, const float* __res
 #pragma unroll 1
                 for (int j = 0; j < NJ1; ++j) {
                     const PhaseCtx P1{hs, he, g.res_col0, g.k1, fw0 + j * N1, j * N1, rank, true};
-                    producer_phase<(A1 ? A1 : A0), (N1 ? N1 : N0), (R1 ? R1 : R0), BN, BM, C::SR, C::BD>(g, X, dY, cc, P1, smem, ring,
-                                                                                         tcount);
+                    producer_phase<(A1 ? A1 : A0), (N1 ? N1 : N0), (R1 ? R1 : R0), BN, BM, C::SR, C::BD, TI>(
+                        g, X, dY, cc, P1, smem, ring, tcount);
                     __syncwarp();   // bar.sync is .aligned: the warp must be converged
                     asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");
                 }

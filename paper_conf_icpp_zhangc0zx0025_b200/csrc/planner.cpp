@@ -262,7 +262,7 @@ static TimeModel time_model(const KernelEntry& e) {
         if (bn >= 128) return {4.5e-6, 5.5e12};
         return {4.0e-6, 3.4e12};
     }
-    if (dtype != 0) {
+    if (dtype != 0 && !e.cc16) {
         if (bm >= 128) return {11.02e-6, 3.095e12};
         if (bm >= 64) return {6.19e-6, 1.545e12};
         return {3.80e-6, 0.812e12};
@@ -291,7 +291,7 @@ static long long cluster_slots(int cs, int occ, int num_sms, const SharedModel& 
 
 static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
     const TimeModel m = time_model(e);
-    SharedModel sh = shared_model(e.dtype);
+    SharedModel sh = shared_model(e.cc16 ? 0 : e.dtype);
     const int fhs = e.fhs > 0 ? e.fhs : 1;
     const double per_chunk = (double)g.chunk * e.bn * e.bm * fhs * 2.0 / m.rate_sm;
     if (e.fhs > 0)   // rank skew + DSMEM reduction of the n0 x 128 x 128 (per SM) FP32 output tile (~20 B/clk/SM)
@@ -350,7 +350,7 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
 static bool cs_allowed(const KernelEntry& e, int cs) {
     if (cs == 1) return true;
     if (!e.csplit_ok) return false;
-    if (e.dtype != 0 && e.fhs <= 0) return cs == 2 || cs == 4;
+    if (e.dtype != 0 && e.fhs <= 0 && !e.cc16) return cs == 2 || cs == 4;
     return true;
 }
 
@@ -480,9 +480,9 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
                 if (e->dtype == 0 && (atoi(v) != 0) != (e->tf32 != 0)) continue;
             }
             // N-D: the FP32 kernel, or the tc2 kernels (16 depth slices of one image per TMA box)
-            if (nd && e->dtype != 0 && (e->fhs <= 0 || p.Do % 16 != 0)) continue;
+            if (nd && e->dtype != 0 && !e->cc16 && (e->fhs <= 0 || p.Do % 16 != 0)) continue;
             if (const char* v = getenv("WINRS_TC_GEN")) {   // debug: restrict to one tensor-core generation
-                if (e->dtype != 0 && ((atoi(v) == 2) != (e->fhs > 0))) continue;
+                if (e->dtype != 0 && !e->cc16 && ((atoi(v) == 2) != (e->fhs > 0))) continue;
             }
             if (const char* v = getenv("WINRS_FORCE_CG")) {  // debug: tc2 CTA pair (2) or single CTA (1)
                 if (e->fhs > 0 && atoi(v) != (e->cg > 0 ? e->cg : 1)) continue;

@@ -27,6 +27,7 @@ struct KernelEntry {
     int cg;                    // CTAs per UMMA: 2 = cta_group::2 pair (0 = 1)
     int ta;                    // 1: tc2 kernel with the transformed X operand in TMEM (bfc_tc2.cuh TA)
     int tf32;                  // 1: FP32 inputs on the tensor cores, 3xTF32 split (bfc_tc3.cuh)
+    int cc16;                  // 1: FP16 / BF16 inputs on the FP32 CUDA-core pipeline (bfc_f32.cuh, TI = 16-bit)
 };
 
 // All entries (FP32 and FP16), terminated by count.

@@ -414,3 +414,24 @@ def test_cluster_split_stress(layer_name, env, monkeypatch):
     err = O.rel_max_err(first.cpu().numpy().astype(np.float64).ravel()[idx], ref)
     record_err(f"{layer_name} 40-call stress {env}", err, f"{p.kernel_name} cs={p.info['csplit']}")
     assert err <= TOL[layer.dtype]
+
+
+# ====================================================== alpha = 16 with 16-bit inputs
+C16 = [
+    # layer overrides, forced pair
+    (dict(N=8, C=64, K=64, H=20, W=20, R=9, S=9, pad=4), "16,9,8,0,0,0"),
+    (dict(N=8, C=40, K=72, H=19, W=23, R=9, S=9, pad=4), "16,9,8,4,3,2"),      # residual Omega_4(3,2), ragged C/K
+    (dict(N=8, C=64, K=64, H=20, W=20, R=7, S=7, pad=3), "16,7,10,8,7,2"),
+    (dict(N=6, C=32, K=48, H=17, W=19, R=7, S=7, pad=0), "16,7,10,0,0,0"),     # pad 0, N % 16 != 0
+]
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+@pytest.mark.parametrize("ov,pair", C16, ids=[f"c16_{i}" for i in range(len(C16))])
+def test_alpha16_16bit_inputs(ov, pair, dtype, monkeypatch):
+    """Omega_16(9,8) / Omega_16(7,10) (eq. (7)-scaled transforms) on FP16 / BF16
+    inputs, gated at 2e-2 (Appendix B's FP16 check); both the U[0,1) protocol
+    and signed inputs."""
+    layer = wl.LAYERS["r50_c64_56_f16"].with_(name="c16", dtype=dtype, **ov)
+    p, err = _check(layer, monkeypatch, {"WINRS_FORCE_PAIR": pair}, expect_kernel="cc_O16")
+    _check(layer, monkeypatch, {"WINRS_FORCE_PAIR": pair}, dist="signed", expect_kernel="cc_O16")
