@@ -42,18 +42,23 @@ def main():
                 continue
             dW = torch.empty((l.K, l.R, l.S, l.C), device="cuda")
             ws = torch.empty(max(16, p.workspace_bytes), dtype=torch.uint8, device="cuda")
-            first, bad, maxd = None, 0, 0.0
+            first, bad, maxd, ts = None, 0, 0.0, []
             try:
                 for i in range(reps):
                     flush.fill_(i & 0xFF)
+                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record()
                     W.bfc(p, Xg, Gg, dW, ws)
+                    b.record()
                     torch.cuda.synchronize()
+                    ts.append(a.elapsed_time(b))
                     if first is None:
                         first = dW.clone()
                     elif not torch.equal(dW, first):
                         bad += 1
                         maxd = max(maxd, float((dW - first).abs().max() / first.abs().max()))
-                status = f"mismatching calls {bad}/{reps - 1} max rel diff {maxd:.2e}"
+                ts = sorted(ts[1:] or ts)
+                status = f"mismatching calls {bad}/{reps - 1} max rel diff {maxd:.2e}  median {ts[len(ts) // 2] * 1e3:.1f} us"
             except Exception as e:
                 status = f"ERROR {str(e)[:60]}"
                 print(f"{name:22s} {es:50s} {p.kernel_name:30s} cs={p.info['csplit']} Z={p.info['Z']} {status}", flush=True)
