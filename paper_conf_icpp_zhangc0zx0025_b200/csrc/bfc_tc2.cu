@@ -80,8 +80,9 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
     cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
     if (e != cudaSuccess) return e;
     const int cluster = CG * g.csplit;
+    constexpr unsigned NTH = (unsigned)tc2_threads<TA>();
     if (cluster <= 1) {
-        k<<<(unsigned)grid, NTHREADS, L::BYTES, stream>>>(a, mX, mY);
+        k<<<(unsigned)grid, NTH, L::BYTES, stream>>>(a, mX, mY);
         return cudaGetLastError();
     }
     if (cluster > 8) {   // 16-CTA clusters (a pair per rank of an 8-way depth split): non-portable size
@@ -94,7 +95,7 @@ cudaError_t launch(const Geometry& g, const void* X, const void* dY, float* dW, 
             np.fetch_or(1ull << (dev & 63));
         }
     }
-    return launch_cluster(k, (unsigned)grid, (unsigned)NTHREADS, (size_t)L::BYTES, stream, cluster, a, mX, mY);
+    return launch_cluster(k, (unsigned)grid, NTH, (size_t)L::BYTES, stream, cluster, a, mX, mY);
 }
 
 // The swapped CTA pair (bfc_tc2s_kernel): tile = 256 k x 128 c x 1 filter row.
@@ -141,7 +142,7 @@ cudaError_t launch_sw(const Geometry& g, const void* X, const void* dY, float* d
      PFX "_O4(3,2)_v2" #CG "_" #NK "x" #F "fh", (F == 1 ? 1 : F * CG), CG, 0}
 // Xhat in TMEM (TA): single CTA, NK = 64
 #define WINRS_TC2T_ENTRY(DT, BF, PFX, F)                                                                  \
-    {DT, 4, 3, 2, 0, 0, 0, 64, ::winrs::tc2::MROWS / F, ::winrs::tc2::NTHREADS, 1, 1,                     \
+    {DT, 4, 3, 2, 0, 0, 0, 64, ::winrs::tc2::MROWS / F, ::winrs::tc2::tc2_threads<true>(), 1, 1,          \
      (size_t)::winrs::tc2::Lay<F, 64, 1, true>::BYTES, &::winrs::tc2::launch<F, 64, BF, 1, true>,              \
      PFX "_O4(3,2)_v2t_64x" #F "fh", F, 1, 1}
 

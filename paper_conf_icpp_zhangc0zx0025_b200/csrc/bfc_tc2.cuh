@@ -68,6 +68,9 @@ constexpr int MROWS = 128;             // UMMA M = TMEM lanes
 constexpr int NTX = 8;                 // transformer warps
 constexpr int NTHREADS = 64 + 32 * NTX + 32;
 constexpr int PW2 = 2 + NTX;           // second TMA producer warp (odd stages; warp 0: even stages)
+// TA kernels: NTX_TA / 4 groups of four FT warps taking alternate stages
+constexpr int NTX_TA = 8;     // (16 measured: no gain, VGG conv1_2 650 -> 679 us)
+template <bool TA> __host__ __device__ constexpr int tc2_threads() { return 64 + 32 * (TA ? NTX_TA : NTX) + 32; }
 constexpr int NSOUT = 3;               // n0: outputs per unit (S = 3)
 #ifndef WINRS_TC2_ITM
 #define WINRS_TC2_ITM 0    // 1: IT inside the tensor core (8 MMAs per stage on the raw X columns, by linearity);
@@ -373,10 +376,14 @@ __device__ __forceinline__ void depth_nhu(int d, int N, int units, int hs, int* 
 // A reads leave the shared-memory port.  TMEM: 4 NK
 // accumulator columns + S ring slots x 4 xi x 8 columns (NK = 64: 256 + 256).
 template <int F, int NK, bool BF, int CG = 1, bool TA = false>
-__global__ void __launch_bounds__(NTHREADS, 1)
+__global__ void __launch_bounds__(tc2_threads<TA>(), 1)
 bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX,
                const __grid_constant__ CUtensorMap tmY) {
     using L = Lay<F, NK, CG, TA>;
+    constexpr int NTXK = TA ? NTX_TA : NTX;          // FT warps
+    constexpr int NTHK = tc2_threads<TA>();
+    constexpr int PW2K = 2 + NTXK;                   // second producer warp
+    constexpr int NG = NTXK / 4;                     // TA: FT groups of four warps
     static_assert(!TA || (CG == 1 && NK == 64 && L::S == 8), "TA: single CTA, NK = 64, 8-slot ring");
     constexpr uint32_t TMEM_ALLOC = TA ? 512u : (uint32_t)L::TMEM_COLS;
     constexpr uint32_t A_COL = 4 * NK;          // TA: first A ring column
@@ -450,7 +457,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     const uint32_t tmem = bars->tmem_base;
     if (threadIdx.x == 64) TC2_TRACE(511, 1);
 
-    if (warp == 0 || warp == PW2) {
+    if (warp == 0 || warp == PW2K) {
         // ============================ TMA producers ===========================
         // Two converged warps (warp 0: even stages, warp PW2: odd stages; the
         // per-stage issue path is ~120 dependent instructions, which alone
@@ -594,7 +601,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         // in it, so its parity wait can never see a phase two rounds ahead.
         constexpr int KO = L::NKL / 8;              // k octets of this CTA's What rows
         constexpr int IPT = KO * KC / 32;           // items per lane: 8 (NK 128) / 4 (NK 64 or a pair)
-        static_assert(L::S <= NTX, "one FT warp per ring slot");
+        static_assert(L::S <= NTXK, "one FT warp per ring slot");
         const int tw = warp - 2;
         if constexpr (TA) {
             // Two groups of four warps take alternate stages (group G: slots
@@ -609,6 +616,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             // IT runs on the packed registers and 4 stores fill the slot's
             // xi = 0..3 A columns.  Ring safety as below: slot s is refilled
             // only after the MMAs of this group's previous stage in it.
+            static_assert(L::S % NG == 0, "TA: each FT group owns every NG-th ring slot");
             const int G = tw >> 2, q = warp & 3;
             const int i4 = lane >> 3, rho = lane & 7;
             const int img = 4 * (rho >> 1) + (rho & 1) + 2 * (i4 & 1);
@@ -625,7 +633,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             const uint32_t foff = opoff(it % KO, it / KO, L::Y_LBO);
             int s = G;
             uint32_t ph = 0;
-            for (int ch = c_lo + G; ch < c_hi; ch += 2) {
+            for (int ch = c_lo + G; ch < c_hi; ch += NG) {
                 mbar_wait(&bars->full[s], ph);
                 tc_after();
                 TC2_JITTER(ch, warp);
@@ -657,7 +665,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&bars->opfull[s]);
                 if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 3);
-                s += 2;
+                s += NG;
                 if (s >= L::S) { s -= L::S; ph ^= 1; }
             }
         } else {
@@ -725,7 +733,8 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         tc_after();
         if (threadIdx.x == 64) TC2_TRACE(511, 2);
         const int q = warp & 3;                      // TMEM lane quarter of this warp
-        const int half = (warp - 2) >> 2;            // k half
+        constexpr int NPART = NTXK / 4;              // k column parts (one per group of four warps)
+        const int half = (warp - 2) >> 2;            // this warp's k part
         const int m = q * 32 + lane;
         const int fh = fh_base + m / L::BC;
         const int c = c_base + m % L::BC;
@@ -733,7 +742,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         float* Out = reinterpret_cast<float*>(smem);  // staging [s][k][m] (overlays the idle ring)
         const uint32_t lane_base = tmem + ((uint32_t)(q * 32) << 16);
 #pragma unroll 1
-        for (int k0 = half * (NK / 2); k0 < (half + 1) * (NK / 2); k0 += 8) {
+        for (int k0 = half * (NK / NPART); k0 < (half + 1) * (NK / NPART); k0 += 8) {
             float v[4][8];
             if (!empty_range) {
 #pragma unroll
@@ -776,7 +785,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         if (threadIdx.x == 64) TC2_TRACE(511, 4);
         const int r_lo = ROWS * rank / g.csplit, r_hi = ROWS * (rank + 1) / g.csplit;
         const uint32_t out_s = sbase;
-        for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHREADS) {
+        for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHK) {
             const int row = p / M4, m4 = p % M4;
             const int sidx = row / NK, kl = row % NK;
             const float4 acc = dsmem_sum4(out_s + (uint32_t)((row * MROWS + m4 * 4) * 4), g.csplit, CG, e);
