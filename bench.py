@@ -219,6 +219,12 @@ def layer_roofline(l, p, ms, peaks):
         depth = rows * units * l.N * kb * cb * ft
         l2_bytes = depth / 16 * 2 * (8192 + 8192)         # per pair stage: each CTA X 8 KB + dY 8 KB
         alu_ops = depth * (256 + 128 * 2)                 # FT over 256 k, IT over 128 c (half2)
+    elif "_v2x_" in name:                                 # xi-split pair: 128 k x 128 rows, xi {0,1} / {2,3}
+        fhs = int(name.split("x")[-1].rstrip("fh"))
+        rows = sum(_rows_union(l, range(g, min(l.R, g + fhs))) for g in range(0, l.R, fhs))
+        depth = rows * units * l.N * kb * cb * ft        # depth entries x pair tiles
+        l2_bytes = depth / 16 * (8192 + 16384 + 2 * 8192)  # per pair stage: X 8 + 16 KB, dY 8 KB per CTA
+        alu_ops = depth * (128 + 2 * 128 * 2)             # FT: W0, W1 over 128 k; IT: 2 outputs per row per half
     elif "_v3_" in name:                                  # FP32 tensor-core kernel: 8-deep stages
         fhs = int(name.split("x")[-1].rstrip("fh"))
         rows = sum(_rows_union(l, range(g, min(l.R, g + fhs))) for g in range(0, l.R, fhs))

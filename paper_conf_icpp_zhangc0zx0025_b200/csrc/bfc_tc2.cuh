@@ -72,6 +72,15 @@ constexpr int PW2 = 2 + NTX;           // second TMA producer warp (odd stages; 
 constexpr int NTX_TA = 8;     // (16 measured: no gain, VGG conv1_2 650 -> 679 us)
 template <bool TA> __host__ __device__ constexpr int tc2_threads() { return 64 + 32 * (TA ? NTX_TA : NTX) + 32; }
 constexpr int NSOUT = 3;               // n0: outputs per unit (S = 3)
+#ifndef WINRS_TC2_PF
+#define WINRS_TC2_PF 0     // TA producers: L2 prefetch (cp.async.bulk.prefetch.tensor) of the stage PF stages
+                           // ahead of the one being loaded (0: off).  Measured: PF = 8 / 16 / 32
+                           // all ~20 % SLOWER (ResNet-50 L4 33.8 -> 40 us, VGG conv1_2 656 -> 830 us): the
+                           // prefetch boxes cost TMA-engine time like loads; kept as a build option only.
+#endif
+#ifndef WINRS_TC2_STX4
+#define WINRS_TC2_STX4 1   // TA: one tcgen05.st .x4 per 16-row half (0: four .x1 stores)
+#endif
 #ifndef WINRS_TC2_ITM
 #define WINRS_TC2_ITM 0    // 1: IT inside the tensor core (8 MMAs per stage on the raw X columns, by linearity);
                            // 0: IT on the FT warps, in place over the raw X slabs (4 MMAs per stage: the
@@ -163,6 +172,11 @@ __device__ __forceinline__ bool elect_one() {
     uint32_t pred;
     asm volatile("{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\nselp.u32 %0, 1, 0, p;\n}\n" : "=r"(pred));
     return pred != 0;
+}
+// L2 prefetch of a box (no shared-memory destination, no barrier).
+__device__ __forceinline__ void tma5_pf(const CUtensorMap* m, int c0, int c1, int c2, int c3, int c4) {
+    asm volatile("cp.async.bulk.prefetch.tensor.5d.L2.global.tile [%0, {%1, %2, %3, %4, %5}];"
+                 :: "l"(reinterpret_cast<uint64_t>(m)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4) : "memory");
 }
 __device__ __forceinline__ void tma5(uint32_t dst, const CUtensorMap* m, uint64_t* bar, int c0, int c1, int c2, int c3,
                                      int c4) {
@@ -262,6 +276,23 @@ __device__ __forceinline__ void ldsm_x4_t(uint32_t addr, uint32_t (&r)[4]) {
 __device__ __forceinline__ void tmem_st16x256(uint32_t taddr, const uint32_t (&r)[4]) {
     asm volatile("tcgen05.st.sync.aligned.16x256b.x1.b32 [%0], {%1, %2, %3, %4};"
                  :: "r"(taddr), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]) : "memory");
+}
+// The same shape repeated over 4 consecutive 8-column chunks (.x4): registers
+// 4i..4i+3 go to columns 8i..8i+7 (one instruction for the four xi slabs of a
+// ring slot instead of four).
+__device__ __forceinline__ void tmem_st16x256_x4(uint32_t taddr, const uint32_t (&r)[4][4]) {
+    asm volatile("tcgen05.st.sync.aligned.16x256b.x4.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, "
+                 "%13, %14, %15, %16};"
+                 :: "r"(taddr), "r"(r[0][0]), "r"(r[0][1]), "r"(r[0][2]), "r"(r[0][3]), "r"(r[1][0]), "r"(r[1][1]),
+                    "r"(r[1][2]), "r"(r[1][3]), "r"(r[2][0]), "r"(r[2][1]), "r"(r[2][2]), "r"(r[2][3]), "r"(r[3][0]),
+                    "r"(r[3][1]), "r"(r[3][2]), "r"(r[3][3])
+                 : "memory");
+}
+__device__ __forceinline__ void tmem_st16x256_x2(uint32_t taddr, const uint32_t (&r)[2][4]) {
+    asm volatile("tcgen05.st.sync.aligned.16x256b.x2.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};"
+                 :: "r"(taddr), "r"(r[0][0]), "r"(r[0][1]), "r"(r[0][2]), "r"(r[0][3]), "r"(r[1][0]), "r"(r[1][1]),
+                    "r"(r[1][2]), "r"(r[1][3])
+                 : "memory");
 }
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
@@ -483,9 +514,52 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             xdt[a] = (g.T > 1 || g.D > 1) ? fh / g.Rh - g.pad : 0;
             xdr[a] = fh < g.R ? fh % g.Rh - g.pad : -(1 << 20);   // a slot past the last filter row: zero fill
         }
+        // TA, F = 2: the second fh slot lies past the last filter row (e.g. the
+        // {2, -} group of R = 3): its X boxes and IT are skipped; the MMAs still
+        // run M = 128, and the dead rows' accumulators are never written out.
+        const bool dead1 = F == 2 && fh_base + 1 >= g.R;
+        // L2 prefetch walker (TA): stages c_lo + pp + S, + S + 2, ... are
+        // prefetched while stage ch - PF + S .. ch is being loaded, so their
+        // TMA loads later hit L2 instead of waiting the HBM round trip.
+        constexpr int PF = TA ? WINRS_TC2_PF : 0;
+        int pch = c_lo + pp + L::S;
+        long long pd = (long long)pch * KC;
+        int pn = 0, ph_ = hs, pu = 0;
+        ImgTracker pitk;
+        if (PF > 0) {
+            if (pd < depth) depth_nhu((int)pd, g.N, units, hs, &pn, &ph_, &pu);
+            pitk.init(g, pn);
+        }
         int s = pp;
         uint32_t ph = 0;
         for (int ch = c_lo + pp; ch < c_hi; ch += 2) {
+            if constexpr (PF > 0) {
+                while (pch < c_hi && pch <= ch + PF) {
+                    const ImgCoord pc = pitk.at(g, true);
+                    const int pw0 = w_first + pu * 2;
+                    if (elect_one()) {
+#pragma unroll
+                        for (int a = 0; a < 2; ++a) {
+                            if (a == 1 && dead1) continue;
+                            const int c0 = F == 2 ? c_base : c_base + a * 64;
+                            tma5_pf(&tmX, c0, pc.a + xdt[a], pc.b, ph_ + xdr[a], pw0 + fw0 - g.pad);
+                            tma5_pf(&tmX, c0, pc.a + 8 + xdt[a], pc.b, ph_ + xdr[a], pw0 + fw0 - g.pad);
+                        }
+#pragma unroll
+                        for (int ka = 0; ka < L::NKL / 64; ++ka) tma5_pf(&tmY, k_base + ka * 64, pc.a, pc.b, ph_, pw0);
+                    }
+                    __syncwarp();
+                    pch += 2;
+                    pn += 2 * KC;
+                    bool pw = false;
+                    while (pn >= g.N) {
+                        pn -= g.N;
+                        pw = true;
+                        if (++pu == units) { pu = 0; ++ph_; }
+                    }
+                    pitk.advance(2 * KC, pw, pn);
+                }
+            }
             mbar_wait(&bars->empty[s], ph ^ 1);
             TC2_JITTER(ch, 0);
             TC2_TRACE(ch - c_lo, 0);
@@ -499,13 +573,14 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
 #ifdef WINRS_TC2_NO_TMA   // debug ablation: stages carry no data (barrier protocol kept)
                 mbar_arrive(fb);
 #else
-                mbar_expect_tx(fb, (uint32_t)L::TX_BYTES);
+                mbar_expect_tx(fb, (uint32_t)L::TX_BYTES - (TA && dead1 ? 8192u : 0u));
 #pragma unroll
                 for (int a = 0; a < 2; ++a) {
                     // X window columns x0..x3 of atom a; an fh slot past the last
                     // filter row reads rows far outside (zero fill)
                     const int c0 = F == 2 ? c_base : c_base + a * 64;
                     if constexpr (TA) {   // two 8-image boxes (tmX box {64, 8, 1, 1, 4})
+                        if (a == 1 && dead1) continue;   // no X rows for an fh slot past the last filter row
                         tma5(st + a * L::X_GRP, &tmX, fb, c0, ic.a + xdt[a], ic.b, hh + xdr[a], w0 + fw0 - g.pad);
                         tma5(st + a * L::X_GRP + L::XT_HI, &tmX, fb, c0, ic.a + 8 + xdt[a], ic.b, hh + xdr[a],
                              w0 + fw0 - g.pad);
@@ -629,6 +704,9 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 xoff[hf] = row + (uint32_t)((oct ^ ((row >> 7) & 7)) << 4);   // stages are 1 KB aligned
             }
             const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16) + A_COL;
+            // lanes of an fh slot past the last filter row: no X, no IT (their A
+            // rows stay stale; the rows they feed are never written out)
+            const bool xdead = F == 2 && fh_base + (q >> 1) >= g.R;
             const int it = q * 32 + lane;           // FT item: depth it / KO, k octet it % KO (KO * KC = 128)
             const uint32_t foff = opoff(it % KO, it / KO, L::Y_LBO);
             int s = G;
@@ -640,7 +718,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
                 const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
 #pragma unroll
-                for (int hf = 0; hf < 2; ++hf) {
+                for (int hf = 0; hf < 2 && !xdead; ++hf) {
                     uint32_t x[4][4];
 #pragma unroll
                     for (int c = 0; c < 4; ++c) ldsm_x4_t(st + xoff[hf] + c * 1024, x[c]);
@@ -653,8 +731,16 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                         o[3][r] = P16<BF>::sub(x[3][r], x[1][r]);
                     }
                     const uint32_t ta = trow + ((uint32_t)(hf * 16) << 16) + (uint32_t)(s * 32);
+#ifndef WINRS_TC2_NO_STTM   // debug ablation: no TMEM stores of the A operand (the MMAs read stale A)
+#if WINRS_TC2_STX4
+                    tmem_st16x256_x4(ta, o);   // the slot's four xi slabs are 4 consecutive 8-column chunks
+#else
 #pragma unroll
                     for (int xi = 0; xi < 4; ++xi) tmem_st16x256(ta + xi * 8, o[xi]);
+#endif
+#else
+                    asm volatile("" :: "r"(o[0][0] ^ o[1][1] ^ o[2][2] ^ o[3][3] ^ ta));
+#endif
                 }
                 const uint4 w0 = lds16(st + L::OFF_Y + foff), w1 = lds16(st + L::OFF_Y + L::ATOM + foff);
                 sts16(st + L::OFF_F + foff, vadd<BF>(w0, w1));

@@ -245,6 +245,8 @@ struct SharedModel {
 
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
+    if (e.fhs > 0 && e.ta == 2)   // bfc_tc2x.cuh xi-split pair (128 k x 128 rows, Xhat in TMEM): rate of the
+        return {4.0e-6, 9.0e12};   // pair over its tile (tools/sweep_tc2.py --xs: L4 41.8 us, VGG conv4_2 670 us)
     if (e.fhs > 0 && e.cg == 2 && bn == 256)   // swapped CTA pair (256 k x 128 c): X side shared
         return {4.5e-6, 12.6e12};              // (re-fitted with two producer warps: tools/sweep_tc2.py)
     if (e.fhs > 0 && e.cg == 2)   // bfc_tc2.cuh CTA pair: rate of the pair over its 256-row tile
@@ -333,7 +335,7 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
                     const double tr = m.fixed_s + a * t0 + (res ? jobs_res * (sh.job_s + b * t1) : 0.0);
                     t = std::max(t, tr);
                 }
-                if (g.csplit > 1) t += sh.cluster_s;
+                if (g.csplit > 1 || e.ta == 2) t += sh.cluster_s;   // xi-split: always a pair reduction
                 for (long long q = 0; q < mult; ++q) push_root(heap[0] + t);
             }
     double mk = 0;
@@ -487,8 +489,10 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
             if (const char* v = getenv("WINRS_FORCE_CG")) {  // debug: tc2 CTA pair (2) or single CTA (1)
                 if (e->fhs > 0 && atoi(v) != (e->cg > 0 ? e->cg : 1)) continue;
             }
-            if (const char* v = getenv("WINRS_FORCE_TA")) {  // debug: tc2 with Xhat in TMEM (1) or in SMEM (0)
-                if (e->fhs > 0 && (atoi(v) != 0) != (e->ta != 0)) continue;
+            if (const char* v = getenv("WINRS_FORCE_TA")) {  // debug: tc2 with Xhat in SMEM (0), in TMEM (1),
+                if (e->fhs > 0 && atoi(v) != e->ta) continue;  // or in TMEM with the xi split over a pair (2)
+            } else if (e->ta == 2) {
+                continue;   // the xi-split pair measured slower than TA on every layer: forced only
             }
             PlanResult r;
             const double t = plan_with_tile(p, *e, cand, num_sms, &r);

@@ -22,11 +22,14 @@ __device__ __forceinline__ void kahan_add(float& s, float& c, float x) {
     s = t;
 }
 
-// The bucket loads of a group of 8 are issued together (they are independent)
-// and then added in z order, so a thread waits for one memory latency per 8
+// The bucket loads of a group of ZB are issued together (they are independent)
+// and then added in z order, so a thread waits for one memory latency per ZB
 // buckets instead of one per bucket; small dW uses one float per thread so
-// the grid still covers the SMs.  The summation order is unchanged.
-constexpr int ZB = 8;
+// the grid still covers the SMs.  The summation order is unchanged.  ZB = 32
+// (float) / 16 (float4): with ~8 warps per SM for a small dW (VGG-16 conv1_2:
+// 36 864 floats, Z = 336) the batch depth sets the bytes in flight; ZB = 8
+// ran at ~1.5 TB/s (profiles/r02/launches_bench_r02.csv, 32 us).
+template <class V> constexpr int zbatch() { return sizeof(V) == 4 ? 32 : 16; }
 
 template <class V>
 __device__ __forceinline__ void kahan_v(V& s, V& c, const V& x);
@@ -50,6 +53,7 @@ template <class V>
 __global__ void __launch_bounds__(256)
 bucket_reduce_kernel(float* __restrict__ dW, const float* __restrict__ ws, long long n, int Z) {
     constexpr int W = sizeof(V) / 4;
+    constexpr int ZB = zbatch<V>();
     const long long nv = n / W;
     const long long stride = (long long)gridDim.x * blockDim.x;
     for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += stride) {

@@ -121,6 +121,51 @@ def test_tc2_ta(name, ov, env, dtype, monkeypatch):
     _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA="1"), expect_kernel="_v2t_")
 
 
+# xi-split pair (bfc_tc2x.cuh: xi {0,1} / {2,3} on the two CTAs of a pair, Xhat in TMEM, NK = 128 tiles,
+# the pair's partial OT tiles summed with the depth-split ranks in one DSMEM reduction)
+XS = [
+    ("l2", dict(N=16, C=128, K=128, H=28, W=28), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "1"}),
+    ("l2_cs2", dict(N=16, C=128, K=128, H=28, W=28), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "2"}),
+    ("l3_cs3", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "3"}),
+    ("l3_cs4", dict(N=32, C=256, K=256, H=14, W=14), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "4"}),
+    ("l4_odd_wo", dict(N=16, C=512, K=512, H=7, W=7), {"WINRS_FORCE_TILE": "128x128"}),
+    ("l1_f2", dict(N=16, C=64, K=128, H=20, W=20), {"WINRS_FORCE_TILE": "128x64"}),
+    ("f2_cs4", dict(N=32, C=64, K=128, H=16, W=16), {"WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "4"}),
+    ("ragged_f1", dict(N=16, C=200, K=136, H=13, W=11), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "3"}),
+    ("ragged_f2", dict(N=16, C=40, K=72, H=20, W=17), {"WINRS_FORCE_TILE": "128x64"}),
+    ("pad0", dict(N=16, C=128, K=128, H=20, W=20, pad=0), {"WINRS_FORCE_TILE": "128x128"}),
+    ("s6_ftiles2", dict(N=16, C=64, K=128, H=16, W=16, R=3, S=6, pad=2), {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_TILE": "128x64"}),
+    ("r5_f2", dict(N=16, C=64, K=128, H=16, W=16, R=5, S=3, pad=2), {"WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "2"}),
+    ("r1", dict(N=16, C=128, K=128, H=12, W=12, R=1, S=3, pad=0), {"WINRS_FORCE_TILE": "128x128"}),
+    ("n32_z5", dict(N=32, C=128, K=128, H=30, W=30), {"WINRS_FORCE_Z": "5", "WINRS_FORCE_TILE": "128x128"}),
+    ("n48_z3_cs2", dict(N=48, C=64, K=256, H=12, W=12), {"WINRS_FORCE_Z": "3", "WINRS_FORCE_CSPLIT": "2", "WINRS_FORCE_TILE": "128x64"}),
+]
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+@pytest.mark.parametrize("name,ov,env", XS, ids=[c[0] for c in XS])
+def test_tc2_xs(name, ov, env, dtype, monkeypatch):
+    layer = BASE.with_(name="xs_" + name, dtype=dtype, **ov)
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA="2"), expect_kernel="_v2x_")
+
+
+@pytest.mark.parametrize("name,ov,env", XS[:6], ids=[c[0] for c in XS[:6]])
+def test_tc2_xs_signed(name, ov, env, monkeypatch):
+    layer = BASE.with_(name="xss_" + name, **ov)
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA="2"), dist="signed", expect_kernel="_v2x_")
+
+
+def test_tc2_xs_exact_all_ones(monkeypatch):
+    """Small-integer inputs: every product and partial sum is exact in FP32,
+    so the xi-split result must equal the oracle bit for bit."""
+    layer = BASE.with_(name="xs_ones", N=16, C=128, K=128, H=14, W=14)
+    g = np.random.Generator(np.random.PCG64(5))
+    X = g.integers(0, 3, size=(layer.N, layer.H, layer.W, layer.C)).astype(np.float16)
+    dY = g.integers(0, 3, size=(layer.N, layer.Ho, layer.Wo, layer.K)).astype(np.float16)
+    _check(layer, monkeypatch, {"WINRS_TC_GEN": "2", "WINRS_FORCE_TA": "2", "WINRS_FORCE_TILE": "128x128",
+                                "WINRS_FORCE_CSPLIT": "2"}, X=X, dY=dY, exact=True, expect_kernel="_v2x_")
+
+
 @pytest.mark.parametrize("name,ov,env", TA[:4], ids=[c[0] for c in TA[:4]])
 def test_tc2_ta_matches_smem_variant(name, ov, env, monkeypatch):
     """Same plan geometry, Xhat in TMEM vs in shared memory: the same packed
@@ -251,6 +296,8 @@ EXACT = [
     ("f16", {"WINRS_TC_GEN": "2"}),
     ("bf16", {"WINRS_TC_GEN": "2"}),
     ("f16", {"WINRS_TC_GEN": "2", "WINRS_FORCE_TA": "1", "WINRS_FORCE_TILE": "64x64"}),
+    ("f16", {"WINRS_TC_GEN": "2", "WINRS_FORCE_TA": "2", "WINRS_FORCE_TILE": "128x64"}),
+    ("bf16", {"WINRS_TC_GEN": "2", "WINRS_FORCE_TA": "2", "WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "2"}),
 ]
 
 

@@ -23,7 +23,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
          "-I", os.path.join(ROOT, "include")]
 
-SOURCES = ["winrs_api.cpp", "planner.cpp", "registry.cpp", "reduce.cu", "allreduce.cu", "bfc_f16.cu", "bfc_tc2.cu", "bfc_tc3.cu", "conv_map.cu",
+SOURCES = ["winrs_api.cpp", "planner.cpp", "registry.cpp", "reduce.cu", "allreduce.cu", "bfc_f16.cu", "bfc_tc2.cu", "bfc_tc2x.cu", "bfc_tc3.cu", "conv_map.cu",
            "bfc_f32_part0.cu", "bfc_f32_part1.cu", "bfc_f32_part2.cu", "bfc_f32_part3.cu",
            "bfc_f32_part4.cu", "bfc_f32_part5.cu"]
 

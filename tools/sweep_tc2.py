@@ -2,7 +2,7 @@
 """Cold-L2 timing sweep of the second-generation tensor-core kernel
 (bfc_tc2.cuh) over its tiles x cluster splits x segment counts, for
 calibrating the planner's time model.  One JSON line per plan.
-Usage: python tools/sweep_tc2.py r50_c64_56_f16,r50_c128_28_f16 [--quick]"""
+Usage: python tools/sweep_tc2.py r50_c64_56_f16,r50_c128_28_f16 [--quick | --xs]"""
 import json
 import os
 import statistics
@@ -19,7 +19,8 @@ from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl  # noqa: E402
 # (tile NK x bm, CTAs per UMMA, Xhat in TMEM): single CTA NK x (128 / F), a cta_group::2 pair,
 # the swapped pair (256x128), or the TA kernels (NK = 64, Xhat in TMEM)
 TILES = [("128x128", 1, 0), ("64x128", 1, 0), ("128x64", 1, 0), ("64x64", 1, 0), ("128x256", 2, 0), ("128x64", 2, 0),
-         ("256x128", 2, 0), ("64x128", 1, 1), ("64x64", 1, 1)]
+         ("256x128", 2, 0), ("64x128", 1, 1), ("64x64", 1, 1), ("128x128", 2, 2), ("128x64", 2, 2)]
+XS_TILES = [("128x128", 2, 2), ("128x64", 2, 2)]   # the xi-split pair (bfc_tc2x.cuh)
 
 
 def time_plan(p, Xg, Gg, flush, reps=10):
@@ -49,8 +50,10 @@ def main():
         Xg, Gg = to(X), to(dY)
         data = l.N * (l.H * l.W * l.C + (l.H + 2 * l.pad - l.R + 1) * (l.W + 2 * l.pad - l.S + 1) * l.K) * 2
         cfgs = [("auto", None, None, None), ("gen1", None, None, None), ("gen2", None, None, None)]
-        if not quick:
-            zs = [1, 2, 4, 7, 8, 14, 16, 28, 56]
+        zs = [1, 2, 4, 7, 8, 14, 16, 28, 56]
+        if "--xs" in sys.argv:
+            cfgs = cfgs[:1] + [("f", t, cs, z) for t in XS_TILES for cs in (1, 2, 3, 4) for z in zs]
+        elif not quick:
             cfgs += [("f", t, cs, z) for t in TILES for cs in (1, 2, 3, 4, 6, 8) for z in zs]
         seen = set()
         for kind, t, cs, z in cfgs:
