@@ -352,6 +352,7 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
 static bool cs_allowed(const KernelEntry& e, int cs) {
     if (cs == 1) return true;
     if (!e.csplit_ok) return false;
+    if ((cs == 5 || cs == 7) && e.fhs <= 0) return false;   // 5 / 7 ranks: tc2 / tc3 kernels only
     if (e.dtype != 0 && e.fhs <= 0 && !e.cc16) return cs == 2 || cs == 4;
     return true;
 }
@@ -359,7 +360,7 @@ static bool cs_allowed(const KernelEntry& e, int cs) {
 static int forced_csplit() {
     if (const char* f = getenv("WINRS_FORCE_CSPLIT")) {
         const int v = atoi(f);
-        if (v >= 1 && v <= 8 && v != 5 && v != 7) return v;
+        if (v >= 1 && v <= 8) return v;
     }
     return 0;
 }
@@ -414,7 +415,8 @@ static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairC
         if (g.bands == last_bands && g.seg_cols == last_cols && seg_h == last_sh && seg_w == last_sw) continue;
         last_bands = g.bands; last_cols = g.seg_cols; last_sh = seg_h; last_sw = seg_w;
         const long long mc = min_tile_chunks(g);
-        for (int cs : {1, 2, 3, 4, 6, 8}) {
+        for (int cs : {1, 2, 3, 4, 5, 6, 7, 8}) {
+            if (cs == 7 && fcs != cs) continue;   // 7 ranks: measured slower everywhere (tools/sweep_tc2.py --cs57)
             if (!cs_allowed(e, cs)) continue;   // never launch a cluster the kernel cannot reduce (even if forced)
             if (e.cg == 2 && cs > 4) continue;   // 16-CTA clusters (pairs x 8): ~half the clusters co-resident (measured 2x slower)
             if (fcs ? cs != fcs : (cs > 1 && mc < cs)) continue;

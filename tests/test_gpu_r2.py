@@ -111,6 +111,9 @@ TA = [
     ("r1", dict(N=16, C=64, K=64, H=12, W=12, R=1, S=3, pad=0), {"WINRS_FORCE_TILE": "64x128"}),
     ("n32_z5", dict(N=32, C=64, K=64, H=30, W=30), {"WINRS_FORCE_Z": "5", "WINRS_FORCE_TILE": "64x64"}),
     ("n48_cs4", dict(N=48, C=128, K=64, H=12, W=12), {"WINRS_FORCE_CSPLIT": "4", "WINRS_FORCE_TILE": "64x128"}),
+    ("l1_cs5", dict(N=32), {"WINRS_FORCE_TILE": "64x64", "WINRS_FORCE_CSPLIT": "5"}),
+    ("ragged_f1_cs7", dict(N=16, C=200, K=72, H=13, W=11), {"WINRS_FORCE_TILE": "64x128", "WINRS_FORCE_CSPLIT": "7"}),
+    ("l3_cs5", dict(N=16, C=256, K=256, H=14, W=14), {"WINRS_FORCE_TILE": "64x128", "WINRS_FORCE_CSPLIT": "5"}),
 ]
 
 
@@ -202,6 +205,8 @@ TC3 = [
     ("l3", dict(N=8, C=256, K=256, H=14, W=14), {}),
     ("ragged", dict(N=8, C=72, K=100, H=20, W=17), {}),
     ("ragged_f2_cs3", dict(N=16, C=40, K=136, H=13, W=11), {"WINRS_FORCE_TILE": "64x64", "WINRS_FORCE_CSPLIT": "3"}),
+    ("l4_cs5", dict(N=8, C=512, K=512, H=7, W=7), {"WINRS_FORCE_CSPLIT": "5"}),
+    ("ragged_cs5", dict(N=8, C=72, K=100, H=20, W=17), {"WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "5"}),
     ("pad0", dict(N=8, C=64, K=64, H=20, W=20, pad=0), {}),
     ("r5", dict(N=8, C=64, K=64, H=16, W=16, R=5, S=3, pad=2), {}),
     ("r1", dict(N=8, C=64, K=64, H=12, W=12, R=1, S=3, pad=0), {}),

@@ -51,7 +51,10 @@ def main():
         data = l.N * (l.H * l.W * l.C + (l.H + 2 * l.pad - l.R + 1) * (l.W + 2 * l.pad - l.S + 1) * l.K) * 2
         cfgs = [("auto", None, None, None), ("gen1", None, None, None), ("gen2", None, None, None)]
         zs = [1, 2, 4, 7, 8, 14, 16, 28, 56]
-        if "--xs" in sys.argv:
+        if "--cs57" in sys.argv:   # odd cluster depth splits of the TA tiles
+            cfgs = cfgs[:1] + [("f", t, cs, z) for t in [("64x128", 1, 1), ("64x64", 1, 1)] for cs in (3, 4, 5, 6, 7)
+                               for z in zs]
+        elif "--xs" in sys.argv:
             cfgs = cfgs[:1] + [("f", t, cs, z) for t in XS_TILES for cs in (1, 2, 3, 4) for z in zs]
         elif not quick:
             cfgs += [("f", t, cs, z) for t in TILES for cs in (1, 2, 3, 4, 6, 8) for z in zs]
