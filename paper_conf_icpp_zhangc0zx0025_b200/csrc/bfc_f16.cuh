@@ -1255,8 +1255,8 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 tc_fence_after();
             }
         } else if (!direct) {
-            __syncwarp();   // bar.sync is .aligned: the warp must be converged
-            asm volatile("bar.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
+            __syncwarp();   // converged warp at the named barrier
+            asm volatile("barrier.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
             if (warp < 6) {
                 final_out<N0, BM, NAT>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));
                 if (threadIdx.x == 64) PTRACE(4);
@@ -1321,8 +1321,8 @@ bfc_f16_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         // staging tile (which overlays the rings) is written.  (Already implied
         // by acc_full -> all MMAs -> all op_full arrivals; made explicit.)
         if (threadIdx.x == 64) PTRACE(3);
-        __syncwarp();   // bar.sync is .aligned: the warp must be converged
-        asm volatile("bar.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
+        __syncwarp();   // converged warp at the named barrier
+        asm volatile("barrier.sync 1, %0;" :: "r"(32 * TX_WARPS) : "memory");
         if (warp < 6) {
             // every job's epilogue is done (this warp's own, in program order)
             final_out<N0, BM>(g, bucket, cc, fw0, tmem_base, warp, reinterpret_cast<float*>(smem));

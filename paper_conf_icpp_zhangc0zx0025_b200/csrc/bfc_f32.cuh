@@ -254,13 +254,13 @@ __device__ __forceinline__ void producer_phase(const Geometry& g, const TI* __re
     }
     for (int ch = 0; ch < nchunks; ++ch) {
         // the slot of chunk ch+S_RAW-1 was read by every thread's transform of ch-1
-        __syncwarp();   // bar.sync is .aligned: the warp must be converged
-        asm volatile("bar.sync 1, %0;" :: "n"(NP) : "memory");
+        __syncwarp();   // converged warp at the named barrier
+        asm volatile("barrier.sync 1, %0;" :: "n"(NP) : "memory");
         if (ch + S_RAW - 1 < nchunks) issue((ch + S_RAW - 1) % S_RAW);
         cp_async_commit();
         cp_async_wait<S_RAW - 1>();                                   // this thread's copies of chunk ch
-        __syncwarp();   // bar.sync is .aligned: the warp must be converged
-        asm volatile("bar.sync 1, %0;" :: "n"(NP) : "memory");       // everyone's copies of chunk ch
+        __syncwarp();   // converged warp at the named barrier
+        asm volatile("barrier.sync 1, %0;" :: "n"(NP) : "memory");       // everyone's copies of chunk ch
         const int ts = tcount % S_T;
         mbar_wait(&ring.t_empty[ts], ((tcount / S_T) & 1) ^ 1);
         const int buf = ch % S_RAW;
@@ -355,8 +355,8 @@ __device__ __forceinline__ void gemm_phase(const Geometry& g, float* __restrict_
     }
     // All of this job's ring writes are done (the producer only fills chunks of
     // this job, each consumed above), so the ring memory can hold the OT staging.
-    __syncwarp();   // bar.sync is .aligned: the warp must be converged
-    asm volatile("bar.sync 2, %0;" :: "n"(NT) : "memory");
+    __syncwarp();   // converged warp at the named barrier
+    asm volatile("barrier.sync 2, %0;" :: "n"(NT) : "memory");
 
     // ---- OT in rounds (one 4-wide k-group of every thread per round)
     float* As = smem;   // [ALPHA][TPK*4][BM]
@@ -372,8 +372,8 @@ __device__ __forceinline__ void gemm_phase(const Geometry& g, float* __restrict_
                 t.x = lo.x; t.y = lo.y; t.z = hi.x; t.w = hi.y;
                 *reinterpret_cast<float4*>(As + (xi * KR + tk * 4 + e) * BM + (gn * L::TPC + tc) * 4) = t;
             }
-        __syncwarp();   // bar.sync is .aligned: the warp must be converged
-        asm volatile("bar.sync 2, %0;" :: "n"(NT) : "memory");
+        __syncwarp();   // converged warp at the named barrier
+        asm volatile("barrier.sync 2, %0;" :: "n"(NT) : "memory");
         for (int p = gtid; p < KR * BM; p += NT) {
             const int kl = p / BM, c = p % BM;
             float vv[ALPHA], y[NN];
@@ -387,8 +387,8 @@ __device__ __forceinline__ void gemm_phase(const Geometry& g, float* __restrict_
                 *dst = P.accumulate ? *dst + y[j] : y[j];
             }
         }
-        __syncwarp();   // bar.sync is .aligned: the warp must be converged
-        asm volatile("bar.sync 2, %0;" :: "n"(NT) : "memory");
+        __syncwarp();   // converged warp at the named barrier
+        asm volatile("barrier.sync 2, %0;" :: "n"(NT) : "memory");
     }
 }
 
@@ -506,8 +506,8 @@ bfc_f32_kernel(const Geometry g, const TI* __restrict__ X, const TI* __restrict_
         // the transformer warpgroup hands registers to the GEMM warpgroups
         asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" :: "n"(REG_P));
         producer_phase<A0, N0, R0, BN, BM, C::SR, C::BD, TI>(g, X, dY, cc, P0, smem, ring, tcount);
-        __syncwarp();   // bar.sync is .aligned: the warp must be converged
-        asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");   // job boundary (ring reused by the OT)
+        __syncwarp();   // converged warp at the named barrier
+        asm volatile("barrier.sync 3, %0;" :: "n"(NTOT) : "memory");   // job boundary (ring reused by the OT)
         if constexpr (A1 != 0) {
             if (resid) {
 #pragma unroll 1
@@ -515,16 +515,16 @@ bfc_f32_kernel(const Geometry g, const TI* __restrict__ X, const TI* __restrict_
                     const PhaseCtx P1{hs, he, g.res_col0, g.k1, fw0 + j * N1, j * N1, rank, true};
                     producer_phase<(A1 ? A1 : A0), (N1 ? N1 : N0), (R1 ? R1 : R0), BN, BM, C::SR, C::BD, TI>(
                         g, X, dY, cc, P1, smem, ring, tcount);
-                    __syncwarp();   // bar.sync is .aligned: the warp must be converged
-                    asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");
+                    __syncwarp();   // converged warp at the named barrier
+                    asm volatile("barrier.sync 3, %0;" :: "n"(NTOT) : "memory");
                 }
             }
         }
     } else {
         asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" :: "n"(REG_G));
         gemm_phase<A0, N0, R0, BN, BM, C::SR, C::BD>(g, Out, cc, P0, smem, ring, tcount);
-        __syncwarp();   // bar.sync is .aligned: the warp must be converged
-        asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");
+        __syncwarp();   // converged warp at the named barrier
+        asm volatile("barrier.sync 3, %0;" :: "n"(NTOT) : "memory");
         if constexpr (A1 != 0) {
             if (resid) {
 #pragma unroll 1
@@ -532,8 +532,8 @@ bfc_f32_kernel(const Geometry g, const TI* __restrict__ X, const TI* __restrict_
                     const PhaseCtx P1{hs, he, g.res_col0, g.k1, fw0 + j * N1, j * N1, rank, true};
                     gemm_phase<(A1 ? A1 : A0), (N1 ? N1 : N0), (R1 ? R1 : R0), BN, BM, C::SR, C::BD>(g, Out, cc, P1, smem, ring,
                                                                                      tcount);
-                    __syncwarp();   // bar.sync is .aligned: the warp must be converged
-                    asm volatile("bar.sync 3, %0;" :: "n"(NTOT) : "memory");
+                    __syncwarp();   // converged warp at the named barrier
+                    asm volatile("barrier.sync 3, %0;" :: "n"(NTOT) : "memory");
                 }
             }
         }

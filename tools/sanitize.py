@@ -18,16 +18,19 @@ cases = [
     wl.LAYERS["r50_c64_56_f16"].with_(N=16, H=10, W=11),
     wl.LAYERS["r50_c256_14_f16"].with_(N=16, H=7, W=7, C=256, K=128),
     wl.LAYERS["r50_c256_14_f16"].with_(N=16, H=6, W=9, C=200, K=136, dtype="bf16"),
+    # bfc_tc3.cuh: FP32 on the tensor cores (N % 8 == 0)
+    wl.LAYERS["r50_c64_56_f32"].with_(N=8, H=10, W=11, C=72, K=100),
 ]
 envs = [{}, {"WINRS_FORCE_CSPLIT": "2"}, {"WINRS_FORCE_Z": "3"}, {"WINRS_FORCE_PAIR": "4,3,2,0,0,0", "WINRS_FORCE_CSPLIT": "4"},
-        {"WINRS_FORCE_CG": "2", "WINRS_FORCE_CSPLIT": "2"}]
+        {"WINRS_FORCE_CG": "2", "WINRS_FORCE_CSPLIT": "2"}, {"WINRS_FORCE_CSPLIT": "5"},
+        {"WINRS_FORCE_TA": "2", "WINRS_FORCE_CSPLIT": "2"}]
 for l in cases:
     for env in envs:
-        for k in ("WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_FORCE_CG"):
+        for k in ("WINRS_FORCE_CSPLIT", "WINRS_FORCE_Z", "WINRS_FORCE_PAIR", "WINRS_FORCE_CG", "WINRS_FORCE_TA"):
             os.environ.pop(k, None)
         if "WINRS_FORCE_PAIR" in env and l.dtype != "f16":
             continue
-        if "WINRS_FORCE_CG" in env and l.N % 16:
+        if ("WINRS_FORCE_CG" in env or "WINRS_FORCE_TA" in env) and (l.N % 16 or l.dtype == "f32"):
             continue
         os.environ.update(env)
         X, dY = wl.make_inputs(l)
