@@ -57,3 +57,28 @@ def test_emulated_f16_plans_equal_oracle(S, monkeypatch):
     X = g.uniform(-1, 1, (N, H, Wd, C))
     dY = g.uniform(-1, 1, (N, p.info["Ho"], p.info["Wo"], K))
     assert O.rel_max_err(W.emulate(p, X, dY), O.bfc_c(X, dY, S, S, pad)) < 1e-12
+
+
+XS_CS = [
+    ({"WINRS_FORCE_TA": "2", "WINRS_FORCE_TILE": "128x128", "WINRS_FORCE_CSPLIT": "1"}, 144, 40),
+    ({"WINRS_FORCE_TA": "2", "WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_CSPLIT": "3"}, 40, 136),
+    ({"WINRS_FORCE_TA": "1", "WINRS_FORCE_TILE": "64x128", "WINRS_FORCE_CSPLIT": "5"}, 136, 72),
+    ({"WINRS_FORCE_TA": "1", "WINRS_FORCE_TILE": "64x64", "WINRS_FORCE_CSPLIT": "7"}, 40, 72),
+]
+
+
+@pytest.mark.parametrize("env,C,K", XS_CS, ids=lambda v: str(v))
+def test_emulated_xs_and_odd_cluster_plans(env, C, K, monkeypatch):
+    """The xi-split pair's tiles (128 k x 128 / 64 rows, cg = 2) and 5- / 7-rank
+    cluster splits decompose the same BFC: the FP64 emulation of the plan's
+    tiles, segments and depth ranks equals the oracle."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    N, H, Wd, R, S, pad = 16, 9, 11, 3, 3, 1
+    p = W.plan_for_device(N, C, H, Wd, K, R, S, pad, "f16")
+    assert p.info["csplit"] == int(env["WINRS_FORCE_CSPLIT"]), p
+    assert ("_v2x_" in p.kernel_name) == (env["WINRS_FORCE_TA"] == "2"), p.kernel_name
+    g = np.random.default_rng(C + K)
+    X = g.uniform(-1, 1, (N, H, Wd, C))
+    dY = g.uniform(-1, 1, (N, p.info["Ho"], p.info["Wo"], K))
+    assert O.rel_max_err(W.emulate(p, X, dY), O.bfc_c(X, dY, R, S, pad)) < 1e-12

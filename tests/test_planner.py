@@ -195,7 +195,7 @@ def test_search_plan_is_valid(l):
     data = esz * (l.N * l.H * l.W * l.C + l.N * i["Ho"] * i["Wo"] * l.K)
     # R11: (Z - 1) buckets of |dW| <= floor(0.04 data / |dW|) buckets, i.e. <= 4 % of X + dY exactly
     assert i["workspace_bytes"] <= 0.04 * data
-    assert i["csplit"] in (1, 2, 3, 4, 6, 8)
+    assert i["csplit"] in (1, 2, 3, 4, 5, 6, 8)   # 7 ranks: forced only
 
 
 # ============================================================== N-D (3-D) plans
@@ -263,3 +263,25 @@ def test_bfc_allreduce_validates_arguments():
     assert call(1, 2, 1) == 1          # peer_dW[rank] != dW
     assert L.winrs_bfc_allreduce(p.handle, fake, fake, fake, None, None, dw, fl, 0, 2, 1, None) == 1
     assert L.winrs_allreduce_flag_bytes() >= 4 * (2 * 8 + 1)
+
+
+def test_default_plans_never_pick_the_xi_split_pair():
+    """The xi-split pair measured slower than TA on every layer (DESIGN.md
+    §6.10): the planner only runs it when WINRS_FORCE_TA=2."""
+    from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+    for l in wl.RESNET50_F16 + wl.VGG16_F16:
+        p = W.plan_for_device(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype)
+        assert "_v2x_" not in p.kernel_name, (l.name, p.kernel_name)
+        assert p.info["csplit"] != 7, (l.name, p)   # 7-rank clusters: forced only
+
+
+def test_five_rank_cluster_split_for_tensor_core_kernels_only(monkeypatch):
+    """cs = 5 (three 5-CTA clusters per GPC) is searched for the tc2 / tc3
+    kernels; the round-1 / CUDA-core kernels never run 5 or 7 ranks."""
+    from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
+    l = wl.LAYERS["r50_c256_14_f16"]
+    p = W.plan_for_device(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype)
+    assert p.info["csplit"] == 5 and "_v2t_" in p.kernel_name, p   # measured 31.7 vs 34.8 us at cs = 4
+    monkeypatch.setenv("WINRS_FORCE_CSPLIT", "5")
+    q = W.plan_for_device(2, 36, 13, 11, 40, 3, 3, 1, "f32")        # N % 8 != 0: FP32 CUDA-core kernel
+    assert q.kernel_name.startswith("f32_") and q.info["csplit"] != 5, q
