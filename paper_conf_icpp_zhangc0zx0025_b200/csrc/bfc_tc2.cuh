@@ -256,12 +256,13 @@ __host__ __device__ constexpr uint32_t idesc_ta() {
     return (1u << 4) | ((BF ? 1u : 0u) << 7) | ((BF ? 1u : 0u) << 10) | (1u << 16) | ((uint32_t)(NK >> 3) << 17) |
            ((uint32_t)(MROWS >> 4) << 24);
 }
-template <int NK, bool BF>
+template <int NK, bool BF, bool NEGB = false>
 __device__ __forceinline__ void umma_ta(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t acc) {
+    // bit 14: negate B
     asm volatile(
         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n"
-        :: "r"(d), "r"(a_tmem), "l"(b), "r"(idesc_ta<NK, BF>()), "r"(acc));
+        :: "r"(d), "r"(a_tmem), "l"(b), "r"(idesc_ta<NK, BF>() | (NEGB ? (1u << 14) : 0u)), "r"(acc));
 }
 // ldmatrix.x4.trans: thread t receives, of matrix i (row addresses from
 // threads 8i..8i+7), the 16-bit elements (row 2(t%4), column t/4) and (row

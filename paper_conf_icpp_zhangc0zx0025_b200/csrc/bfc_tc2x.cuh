@@ -31,6 +31,11 @@
 #pragma once
 #include "bfc_tc2.cuh"
 
+#ifndef WINRS_TC2X_LIN
+#define WINRS_TC2X_LIN 1   // e = 0 half: What[0,1] = w0 +- w1 applied by the tensor core (four MMAs on the raw
+                           // w0, w1 by linearity, negate-B for -w1) instead of the FT warps' stores (0: FT stores)
+#endif
+
 namespace winrs {
 namespace tc2 {
 
@@ -188,7 +193,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     } else if (warp == 1) {
         // ============================ MMA issuer ==============================
         // B: e = 0 What[0], What[1] (FT region); e = 1 the raw w0, w1.
-        const int off_b = e ? L::OFF_Y1 : L::OFF_F0;
+        const int off_b = e ? L::OFF_Y1 : (WINRS_TC2X_LIN ? L::OFF_Y0 : L::OFF_F0);
         int s = 0;
         uint32_t ph = 0;
         for (int ch = c_lo; ch < c_hi; ++ch) {
@@ -201,8 +206,15 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
             const uint64_t b0 = desc_sw128(st + off_b, L::Y_LBO, 1024), b1 = b0 + (L::ATOM >> 4);
             if (elect_one()) {
                 const uint32_t a = tmem + L::A_COL + (uint32_t)(s * 16);
-                umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
-                umma_ta<NK, BF>(tmem + NK, a + 8, b1, acc);
+                if (WINRS_TC2X_LIN && e == 0) {   // v0 += Xhat0 (w0 + w1), v1 += Xhat1 (w0 - w1)
+                    umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
+                    umma_ta<NK, BF>(tmem + 0, a + 0, b1, 1u);
+                    umma_ta<NK, BF>(tmem + NK, a + 8, b0, acc);
+                    umma_ta<NK, BF, true>(tmem + NK, a + 8, b1, 1u);
+                } else {
+                    umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
+                    umma_ta<NK, BF>(tmem + NK, a + 8, b1, acc);
+                }
                 umma_commit<1>(&bars->empty[s]);
             }
             __syncwarp();
@@ -268,7 +280,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 const uint32_t ta = trow + ((uint32_t)(hf * 16) << 16) + (uint32_t)(s * 16);
                 tmem_st16x256_x2(ta, o);
             }
-            if (e == 0) {   // What[0] = w0 + w1, What[1] = w0 - w1 (128 k x 16 depth)
+            if (e == 0 && !WINRS_TC2X_LIN) {   // What[0] = w0 + w1, What[1] = w0 - w1 (128 k x 16 depth)
                 const uint32_t y = st + L::OFF_Y0, f = st + L::OFF_F0;
                 const uint4 a0 = lds16(y + foff0), a1 = lds16(y + L::ATOM + foff0);
                 const uint4 b0 = lds16(y + foff1), b1 = lds16(y + L::ATOM + foff1);

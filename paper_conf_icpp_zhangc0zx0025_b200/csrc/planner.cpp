@@ -246,7 +246,7 @@ struct SharedModel {
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
     if (e.fhs > 0 && e.ta == 2)   // bfc_tc2x.cuh xi-split pair (128 k x 128 rows, Xhat in TMEM): rate of the
-        return {4.0e-6, 9.0e12};   // pair over its tile (tools/sweep_tc2.py --xs: L4 41.8 us, VGG conv4_2 670 us)
+        return {4.0e-6, 13.2e12};  // pair over its tile (tools/ab_xs.sh: VGG conv4_2 cs = 1, 3136 stages per pair in 508 us)
     if (e.fhs > 0 && e.cg == 2 && bn == 256)   // swapped CTA pair (256 k x 128 c): X side shared
         return {4.5e-6, 12.6e12};              // (re-fitted with two producer warps: tools/sweep_tc2.py)
     if (e.fhs > 0 && e.cg == 2)   // bfc_tc2.cuh CTA pair: rate of the pair over its 256-row tile
@@ -353,6 +353,7 @@ static bool cs_allowed(const KernelEntry& e, int cs) {
     if (cs == 1) return true;
     if (!e.csplit_ok) return false;
     if ((cs == 5 || cs == 7) && e.fhs <= 0) return false;   // 5 / 7 ranks: tc2 / tc3 kernels only
+    if (e.cg == 2 && cs > 4) return false;                  // CTA pairs: clusters of 2 x cs <= 8 CTAs
     if (e.dtype != 0 && e.fhs <= 0 && !e.cc16) return cs == 2 || cs == 4;
     return true;
 }
@@ -493,8 +494,6 @@ winrs_status_t make_plan(const Problem& p, int num_sms, PlanResult* out) {
             }
             if (const char* v = getenv("WINRS_FORCE_TA")) {  // debug: tc2 with Xhat in SMEM (0), in TMEM (1),
                 if (e->fhs > 0 && atoi(v) != e->ta) continue;  // or in TMEM with the xi split over a pair (2)
-            } else if (e->ta == 2) {
-                continue;   // the xi-split pair measured slower than TA on every layer: forced only
             }
             PlanResult r;
             const double t = plan_with_tile(p, *e, cand, num_sms, &r);

@@ -265,14 +265,18 @@ def test_bfc_allreduce_validates_arguments():
     assert L.winrs_allreduce_flag_bytes() >= 4 * (2 * 8 + 1)
 
 
-def test_default_plans_never_pick_the_xi_split_pair():
-    """The xi-split pair measured slower than TA on every layer (DESIGN.md
-    §6.10): the planner only runs it when WINRS_FORCE_TA=2."""
+def test_xi_split_pair_picks_follow_the_measurements():
+    """The xi-split pair wins only on the long VGG-16 layers
+    with enough tiles (conv2_2: 454 vs 480 us, tools/ab_xs.sh); on ResNet-50 it
+    measured slower, and 7-rank clusters are never picked."""
     from paper_conf_icpp_zhangc0zx0025_b200 import workloads as wl
     for l in wl.RESNET50_F16 + wl.VGG16_F16:
         p = W.plan_for_device(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype)
-        assert "_v2x_" not in p.kernel_name, (l.name, p.kernel_name)
+        if l.name.startswith("r50"):
+            assert "_v2x_" not in p.kernel_name, (l.name, p.kernel_name)
         assert p.info["csplit"] != 7, (l.name, p)   # 7-rank clusters: forced only
+    l = wl.LAYERS["vgg_128_128_112_f16"]
+    assert "_v2x_" in W.plan_for_device(l.N, l.C, l.H, l.W, l.K, l.R, l.S, l.pad, l.dtype).kernel_name
 
 
 def test_five_rank_cluster_split_for_tensor_core_kernels_only(monkeypatch):
