@@ -131,6 +131,11 @@ struct Args {
     float* dW;
     float* ws;
     int nb;            // images per TMA box (divides N and KC, >= 8)
+    // stream-K xi-split pairs (bfc_tc2x.cuh SK): number of pairs, per-tile
+    // chain flags (library-owned, zero-initialised) and this launch's epoch tag
+    int sk_pairs = 0;
+    unsigned int* sk_flags = nullptr;
+    unsigned int sk_epoch = 0;
 };
 
 struct Bars {

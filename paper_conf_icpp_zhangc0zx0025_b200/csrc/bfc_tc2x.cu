@@ -7,6 +7,8 @@
 #include "launch_util.cuh"
 #include "registry.h"
 #include "tc2_maps.cuh"
+#include <atomic>
+#include <mutex>
 
 namespace winrs {
 namespace tc2 {
@@ -36,7 +38,102 @@ cudaError_t launch_x(const Geometry& g, const void* X, const void* dY, float* dW
                           mX4, mX2, mY);
 }
 
+// Stream-K pairs (SK): the chain flags live in a library-owned, zero-initialised
+// per-device buffer (no workspace); each launch tags its flag values with a fresh
+// epoch so values left by an earlier launch never match a waiter.
+constexpr int SK_MAX_TILES = 1 << 16;
+static unsigned int* sk_flags_for_device(int dev) {
+    static std::mutex mu;
+    static unsigned int* bufs[64] = {};
+    std::lock_guard<std::mutex> lk(mu);
+    if (dev < 0 || dev >= 64) return nullptr;
+    if (!bufs[dev]) {
+        void* p = nullptr;
+        if (cudaMalloc(&p, SK_MAX_TILES * sizeof(unsigned int)) != cudaSuccess) return nullptr;
+        if (cudaMemset(p, 0, SK_MAX_TILES * sizeof(unsigned int)) != cudaSuccess) return nullptr;
+        if (cudaDeviceSynchronize() != cudaSuccess) return nullptr;
+        bufs[dev] = static_cast<unsigned int*>(p);
+    }
+    return bufs[dev];
+}
+
+template <int F, bool BF>
+cudaError_t launch_sk(const Geometry& g, const void* X, const void* dY, float* dW, float* ws, cudaStream_t stream) {
+    using L = LayX<F>;
+    const long long tiles = num_tiles(g);
+    if (tiles <= 0) return cudaSuccess;
+    Args a;
+    a.g = g;
+    a.dW = dW;
+    a.ws = ws;
+    a.nb = images_per_box(g);
+    if (a.nb == 0 || g.a0 != 4 || g.n0 != 3 || g.r0 != 2 || g.a1 != 0 || g.cg != 2 || g.fhs != F || g.csplit != 1 ||
+        g.Z != 1 || tiles > SK_MAX_TILES)
+        return cudaErrorInvalidValue;
+    const bool nd = g.T > 1 || g.D > 1;
+    CUtensorMap mX4, mX2, mY;
+    if (!make_maps(g, X, dY, BF, &mX4, &mY, 8)) return cudaErrorInvalidValue;
+    if (!make_map(&mX2, X, nd ? g.D : g.N, nd ? g.Nb : 1, g.H, g.W, g.C, g.C, 2, 8, BF)) return cudaErrorInvalidValue;
+    auto k = bfc_tc2x_kernel<F, BF, true>;
+    static std::atomic<unsigned long long> done{0};
+    cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
+    if (e != cudaSuccess) return e;
+    int dev = 0;
+    if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+    a.sk_flags = sk_flags_for_device(dev);
+    if (!a.sk_flags) return cudaErrorMemoryAllocation;
+    static std::atomic<unsigned int> epoch{0};
+    a.sk_epoch = (epoch.fetch_add(1) % 0xFFFFFEu) + 1u;   // 24-bit tag, never 0
+    // pairs: every co-resident 2-CTA cluster (all of them must be resident: the chain waits)
+    cudaLaunchConfig_t cfg = {};
+    cfg.blockDim = dim3((unsigned)tc2_threads<true>());
+    cfg.dynamicSmemBytes = (size_t)L::BYTES;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[2];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeCooperative;
+    attr[1].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    static int max_pairs[64] = {};
+    if (dev < 64 && max_pairs[dev] == 0) {
+        cfg.gridDim = dim3(2);
+        int n = 0;
+        if ((e = cudaOccupancyMaxActiveClusters(&n, k, &cfg)) != cudaSuccess) return e;
+        max_pairs[dev] = n > 0 ? n : 1;
+    }
+    int P = dev < 64 ? max_pairs[dev] : 1;
+    // a.sk_pairs <= the chunk count, so that every pair has work
+    long long chunks = 0;
+    for (int f = 0; f < g.fhg; ++f) {
+        int hs, he, wf, units;
+        group_rows(g, 0, f * g.fhs, &hs, &he);
+        seg_units(g, 0, &wf, &units);
+        chunks += (long long)g.kblocks * g.cblocks * g.ftiles * (((long long)(he > hs ? he - hs : 0) * units * g.N + KC - 1) / KC);
+    }
+    if (chunks <= 0) return cudaSuccess;
+    if (P > chunks) P = (int)chunks;
+    a.sk_pairs = P;
+    cfg.gridDim = dim3((unsigned)(2 * P));
+    cfg.numAttrs = 2;
+    e = cudaLaunchKernelEx(&cfg, k, a, mX4, mX2, mY);
+    if (e == cudaErrorCooperativeLaunchTooLarge || e == cudaErrorNotSupported || e == cudaErrorInvalidValue) {
+        (void)cudaGetLastError();   // cooperative + cluster unavailable: P <= the resident cluster count still holds
+        cfg.numAttrs = 1;
+        e = cudaLaunchKernelEx(&cfg, k, a, mX4, mX2, mY);
+    }
+    return e;
+}
+
 }  // namespace tc2
+
+#define WINRS_TC2K_ENTRY(DT, BF, PFX, F)                                                                  \
+    {DT, 4, 3, 2, 0, 0, 0, 128, ::winrs::tc2::MROWS / F, ::winrs::tc2::tc2_threads<true>(), 1, 1,         \
+     (size_t)::winrs::tc2::LayX<F>::BYTES, &::winrs::tc2::launch_sk<F, BF>, PFX "_O4(3,2)_v2k_128x" #F "fh", \
+     F, 2, 3}
 
 #define WINRS_TC2X_ENTRY(DT, BF, PFX, F)                                                                  \
     {DT, 4, 3, 2, 0, 0, 0, 128, ::winrs::tc2::MROWS / F, ::winrs::tc2::tc2_threads<true>(), 1, 1,         \
@@ -57,6 +154,11 @@ const KernelEntry* tc2x_entries(int* n) {
         WINRS_TC2X_ENTRY(1, false, "f16tc", 2),
         WINRS_TC2X_ENTRY(2, true, "bf16tc", 1),
         WINRS_TC2X_ENTRY(2, true, "bf16tc", 2),
+        // stream-K pairs (one launch of all co-resident pairs over the concatenated tile depths)
+        WINRS_TC2K_ENTRY(1, false, "f16tc", 1),
+        WINRS_TC2K_ENTRY(1, false, "f16tc", 2),
+        WINRS_TC2K_ENTRY(2, true, "bf16tc", 1),
+        WINRS_TC2K_ENTRY(2, true, "bf16tc", 2),
     };
     *n = sizeof(e) / sizeof(e[0]);
     return e;

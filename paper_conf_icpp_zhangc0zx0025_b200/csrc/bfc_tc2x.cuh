@@ -68,7 +68,65 @@ struct LayX {
     static_assert(BYTES <= 227 * 1024, "smem");
 };
 
-template <int F, bool BF>
+// ---- stream-K schedule (SK): the pairs take equal contiguous ranges of the
+// concatenated depth chunks of all tiles (Z = 1: one segment per tile; tiles
+// in decode_cta order, so the tiles of one fh group are a contiguous block of
+// equal depth).  A tile split over several pairs is combined in dW in a fixed
+// order -- the pair holding its last chunks first (plain store), then the
+// lower pairs in decreasing index (read-add-write) -- through one chain flag
+// per tile; a pair only ever waits for a higher pair, and all pairs are
+// co-resident (cooperative launch), so the chain cannot deadlock.
+struct SkTile {
+    long long t;       // tile index
+    long long g0;      // global chunk index of its first chunk
+    int depth;         // its chunks
+};
+__device__ __forceinline__ int sk_group_chunks(const Geometry& g, int fh) {
+    int hs, he, wf, units;
+    group_rows(g, 0, fh, &hs, &he);
+    seg_units(g, 0, &wf, &units);
+    const long long d = (long long)(he > hs ? he - hs : 0) * units * g.N;
+    return (int)((d + KC - 1) / KC);
+}
+__device__ __forceinline__ long long sk_total(const Geometry& g) {
+    const long long per = (long long)g.kblocks * g.cblocks * g.ftiles;
+    long long tot = 0;
+    for (int f = 0; f < g.fhg; ++f) tot += per * sk_group_chunks(g, f * g.fhs);
+    return tot;
+}
+// The tile holding global chunk gi.
+__device__ __forceinline__ SkTile sk_find(const Geometry& g, long long gi) {
+    const long long per = (long long)g.kblocks * g.cblocks * g.ftiles;
+    long long acc = 0;
+    SkTile r{0, 0, 0};
+    for (int f = 0; f < g.fhg; ++f) {
+        const int d = sk_group_chunks(g, f * g.fhs);
+        if (d > 0 && gi < acc + per * d) {
+            const long long i = (gi - acc) / d;
+            r.t = (long long)f * per + i;
+            r.g0 = acc + i * d;
+            r.depth = d;
+            return r;
+        }
+        acc += per * d;
+    }
+    return r;
+}
+__device__ __forceinline__ long long sk_start(long long tot, int p, int P) { return tot * p / P; }
+// The pair whose range holds global chunk gi: the largest p with sk_start(p) <= gi.
+__device__ __forceinline__ int sk_pair_of(long long tot, long long gi, int P) {
+    return (int)(((gi + 1) * P - 1) / tot);
+}
+__device__ __forceinline__ unsigned int ld_acquire(const unsigned int* p) {
+    unsigned int v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(unsigned int* p, unsigned int v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+
+template <int F, bool BF, bool SK = false>
 __global__ void __launch_bounds__(tc2_threads<true>(), 1)
 bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtensorMap tmX4,
                 const __grid_constant__ CUtensorMap tmX2, const __grid_constant__ CUtensorMap tmY) {
@@ -87,24 +145,10 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 64) TC2_TRACE(511, 0);
 
-    const int crank = (int)cluster_rank();               // cluster = 2 x csplit CTAs
+    const int crank = (int)cluster_rank();               // cluster = 2 x csplit CTAs (SK: one pair)
     const int nranks = 2 * g.csplit;
     const int e = crank & 1;                             // xi half
     const int rank = crank >> 1;                         // depth-split rank
-    const CtaCoord cc = decode_cta(g, blockIdx.x / nranks);
-    const int fh_base = cc.fh;
-    const int c_base = F == 2 ? cc.cb * 64 : cc.cb * 128;
-    const int k_base = cc.kb * NK;
-    const int seg = cc.band * g.seg_cols + cc.col;
-    float* bucket = seg == 0 ? args.dW : args.ws + (long long)(seg - 1) * g.dw_elems;
-    int hs, he, w_first, units;
-    group_rows(g, cc.band, cc.fh, &hs, &he);
-    seg_units(g, cc.col, &w_first, &units);
-    const long long depth = (long long)(he > hs ? he - hs : 0) * units * g.N;
-    int c_lo, c_hi;
-    split_chunks((int)((depth + KC - 1) / KC), rank, g.csplit, &c_lo, &c_hi);
-    const bool empty_range = c_hi <= c_lo;
-    const int fw0 = cc.ft * NSOUT;
     // per-half stage layout
     const int x_hi = e ? L::X4_HI : L::X2_HI, x_grp = e ? L::X4_GRP : L::X2_GRP;
     const int off_y = e ? L::OFF_Y1 : L::OFF_Y0;
@@ -133,228 +177,322 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     const uint32_t tmem = bars->tmem_base;
     if (threadIdx.x == 64) TC2_TRACE(511, 1);
 
-    if (warp == 0 || warp == PW2K) {
-        // ============================ TMA producers ===========================
-        const int pp = warp == 0 ? 0 : 1;
-        const CUtensorMap* mx = e ? &tmX4 : &tmX2;
-        const int xcol = e ? 0 : 1;                      // first X window column loaded
-        const uint32_t tx = e ? (uint32_t)L::TX1 : (uint32_t)L::TX0;
-        long long d = (long long)(c_lo + pp) * KC;
-        int n = 0, h = hs, u = 0;
-        if (d < depth) depth_nhu((int)d, g.N, units, hs, &n, &h, &u);
-        ImgTracker itk;
-        itk.init(g, n);
-        int xdt[2], xdr[2];
-#pragma unroll
-        for (int a = 0; a < 2; ++a) {
-            const int fh = F == 2 ? fh_base + a : fh_base;
-            xdt[a] = (g.T > 1 || g.D > 1) ? fh / g.Rh - g.pad : 0;
-            xdr[a] = fh < g.R ? fh % g.Rh - g.pad : -(1 << 20);   // a slot past the last filter row: zero fill
-        }
-        int s = pp;
-        uint32_t ph = 0;
-        for (int ch = c_lo + pp; ch < c_hi; ch += 2) {
-            mbar_wait(&bars->empty[s], ph ^ 1);
-            TC2_JITTER(ch, 0);
-            TC2_TRACE(ch - c_lo, 0);
-            uint64_t* fb = &bars->full[s];
-            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
-            const bool in = d < depth;
-            const ImgCoord ic = itk.at(g, in);
-            const int hh = in ? h : hs;
-            const int w0 = w_first + (in ? u : 0) * 2;
-            if (elect_one()) {
-                mbar_expect_tx(fb, tx);
-#pragma unroll
-                for (int a = 0; a < 2; ++a) {
-                    const int c0 = F == 2 ? c_base : c_base + a * 64;
-                    const int wx = w0 + fw0 - g.pad + xcol;
-                    tma5(st + a * x_grp, mx, fb, c0, ic.a + xdt[a], ic.b, hh + xdr[a], wx);
-                    tma5(st + a * x_grp + x_hi, mx, fb, c0, ic.a + 8 + xdt[a], ic.b, hh + xdr[a], wx);
+    // ---- the pieces this CTA works on: one (tile, depth-rank range) without
+    // SK; with SK the tiles (or tile parts) of this pair's chunk range
+    const int P = SK ? args.sk_pairs : 1;
+    const int pair = SK ? (int)(blockIdx.x >> 1) : 0;
+    const long long tot = SK ? sk_total(g) : 1;
+    long long gcur = SK ? sk_start(tot, pair, P) : 0;
+    const long long gend = SK ? sk_start(tot, pair + 1, P) : 1;
+    for (int piece = 0;; ++piece) {
+        long long tile;
+        int c_lo, c_hi, order = 0;
+        if constexpr (SK) {
+            if (gcur >= gend) break;
+            const SkTile st = sk_find(g, gcur);
+            tile = st.t;
+            c_lo = (int)(gcur - st.g0);
+            c_hi = (int)min((long long)st.depth, gend - st.g0);
+            order = sk_pair_of(tot, st.g0 + st.depth - 1, P) - pair;   // 0: the pair with the tile's last chunks
+            gcur += c_hi - c_lo;
+            if (piece > 0) {   // the previous piece drained: every barrier is quiescent
+                if (threadIdx.x == 0) {
+                    for (int s = 0; s < L::S; ++s) {
+                        asm volatile("mbarrier.inval.shared::cta.b64 [%0];" :: "r"(su(&bars->full[s])) : "memory");
+                        asm volatile("mbarrier.inval.shared::cta.b64 [%0];" :: "r"(su(&bars->opfull[s])) : "memory");
+                        asm volatile("mbarrier.inval.shared::cta.b64 [%0];" :: "r"(su(&bars->empty[s])) : "memory");
+                        mbar_init(&bars->full[s], 1);
+                        mbar_init(&bars->opfull[s], 4);
+                        mbar_init(&bars->empty[s], 1);
+                    }
+                    asm volatile("mbarrier.inval.shared::cta.b64 [%0];" :: "r"(su(&bars->accfull)) : "memory");
+                    mbar_init(&bars->accfull, 1);
+                    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
                 }
-#pragma unroll
-                for (int ka = 0; ka < 2; ++ka)
-                    tma5(st + off_y + ka * L::Y_LBO, &tmY, fb, k_base + ka * 64, ic.a, ic.b, hh, w0);
+                tc_before();
+                __syncthreads();
+                tc_after();
             }
-            __syncwarp();
-            TC2_TRACE(ch - c_lo, 1);
-            d += 2 * KC;
-            n += 2 * KC;
-            bool wrapped = false;
-            while (n >= g.N) {
-                n -= g.N;
-                wrapped = true;
-                if (++u == units) { u = 0; ++h; }
-            }
-            itk.advance(2 * KC, wrapped, n);
-            s += 2;
-            if (s >= L::S) { s -= L::S; ph ^= 1; }
+        } else {
+            if (piece > 0) break;
+            tile = blockIdx.x / nranks;
         }
-    } else if (warp == 1) {
-        // ============================ MMA issuer ==============================
-        // B: e = 0 What[0], What[1] (FT region); e = 1 the raw w0, w1.
-        const int off_b = e ? L::OFF_Y1 : (WINRS_TC2X_LIN ? L::OFF_Y0 : L::OFF_F0);
-        int s = 0;
-        uint32_t ph = 0;
-        for (int ch = c_lo; ch < c_hi; ++ch) {
-            mbar_wait(&bars->opfull[s], ph);
-            TC2_JITTER(ch, 1);
-            TC2_TRACE(ch - c_lo, 4);
-            tc_after();
-            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
-            const uint32_t acc = ch > c_lo ? 1u : 0u;
-            const uint64_t b0 = desc_sw128(st + off_b, L::Y_LBO, 1024), b1 = b0 + (L::ATOM >> 4);
-            if (elect_one()) {
-                const uint32_t a = tmem + L::A_COL + (uint32_t)(s * 16);
-                if (WINRS_TC2X_LIN && e == 0) {   // v0 += Xhat0 (w0 + w1), v1 += Xhat1 (w0 - w1)
-                    umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
-                    umma_ta<NK, BF>(tmem + 0, a + 0, b1, 1u);
-                    umma_ta<NK, BF>(tmem + NK, a + 8, b0, acc);
-                    umma_ta<NK, BF, true>(tmem + NK, a + 8, b1, 1u);
-                } else {
-                    umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
-                    umma_ta<NK, BF>(tmem + NK, a + 8, b1, acc);
+        const CtaCoord cc = decode_cta(g, tile);
+        const int fh_base = cc.fh;
+        const int c_base = F == 2 ? cc.cb * 64 : cc.cb * 128;
+        const int k_base = cc.kb * NK;
+        const int seg = cc.band * g.seg_cols + cc.col;
+        float* bucket = seg == 0 ? args.dW : args.ws + (long long)(seg - 1) * g.dw_elems;
+        int hs, he, w_first, units;
+        group_rows(g, cc.band, cc.fh, &hs, &he);
+        seg_units(g, cc.col, &w_first, &units);
+        const long long depth = (long long)(he > hs ? he - hs : 0) * units * g.N;
+        if constexpr (!SK) split_chunks((int)((depth + KC - 1) / KC), rank, g.csplit, &c_lo, &c_hi);
+        const bool empty_range = c_hi <= c_lo;
+        const int fw0 = cc.ft * NSOUT;
+        if (warp == 0 || warp == PW2K) {
+            // ============================ TMA producers ===========================
+            const int pp = warp == 0 ? 0 : 1;
+            const CUtensorMap* mx = e ? &tmX4 : &tmX2;
+            const int xcol = e ? 0 : 1;                      // first X window column loaded
+            const uint32_t tx = e ? (uint32_t)L::TX1 : (uint32_t)L::TX0;
+            long long d = (long long)(c_lo + pp) * KC;
+            int n = 0, h = hs, u = 0;
+            if (d < depth) depth_nhu((int)d, g.N, units, hs, &n, &h, &u);
+            ImgTracker itk;
+            itk.init(g, n);
+            int xdt[2], xdr[2];
+    #pragma unroll
+            for (int a = 0; a < 2; ++a) {
+                const int fh = F == 2 ? fh_base + a : fh_base;
+                xdt[a] = (g.T > 1 || g.D > 1) ? fh / g.Rh - g.pad : 0;
+                xdr[a] = fh < g.R ? fh % g.Rh - g.pad : -(1 << 20);   // a slot past the last filter row: zero fill
+            }
+            int s = pp;
+            uint32_t ph = 0;
+            for (int ch = c_lo + pp; ch < c_hi; ch += 2) {
+                mbar_wait(&bars->empty[s], ph ^ 1);
+                TC2_JITTER(ch, 0);
+                TC2_TRACE(ch - c_lo, 0);
+                uint64_t* fb = &bars->full[s];
+                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+                const bool in = d < depth;
+                const ImgCoord ic = itk.at(g, in);
+                const int hh = in ? h : hs;
+                const int w0 = w_first + (in ? u : 0) * 2;
+                if (elect_one()) {
+                    mbar_expect_tx(fb, tx);
+    #pragma unroll
+                    for (int a = 0; a < 2; ++a) {
+                        const int c0 = F == 2 ? c_base : c_base + a * 64;
+                        const int wx = w0 + fw0 - g.pad + xcol;
+                        tma5(st + a * x_grp, mx, fb, c0, ic.a + xdt[a], ic.b, hh + xdr[a], wx);
+                        tma5(st + a * x_grp + x_hi, mx, fb, c0, ic.a + 8 + xdt[a], ic.b, hh + xdr[a], wx);
+                    }
+    #pragma unroll
+                    for (int ka = 0; ka < 2; ++ka)
+                        tma5(st + off_y + ka * L::Y_LBO, &tmY, fb, k_base + ka * 64, ic.a, ic.b, hh, w0);
                 }
-                umma_commit<1>(&bars->empty[s]);
+                __syncwarp();
+                TC2_TRACE(ch - c_lo, 1);
+                d += 2 * KC;
+                n += 2 * KC;
+                bool wrapped = false;
+                while (n >= g.N) {
+                    n -= g.N;
+                    wrapped = true;
+                    if (++u == units) { u = 0; ++h; }
+                }
+                itk.advance(2 * KC, wrapped, n);
+                s += 2;
+                if (s >= L::S) { s -= L::S; ph ^= 1; }
             }
+        } else if (warp == 1) {
+            // ============================ MMA issuer ==============================
+            // B: e = 0 What[0], What[1] (FT region); e = 1 the raw w0, w1.
+            const int off_b = e ? L::OFF_Y1 : (WINRS_TC2X_LIN ? L::OFF_Y0 : L::OFF_F0);
+            int s = 0;
+            uint32_t ph = 0;
+            for (int ch = c_lo; ch < c_hi; ++ch) {
+                mbar_wait(&bars->opfull[s], ph);
+                TC2_JITTER(ch, 1);
+                TC2_TRACE(ch - c_lo, 4);
+                tc_after();
+                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+                const uint32_t acc = ch > c_lo ? 1u : 0u;
+                const uint64_t b0 = desc_sw128(st + off_b, L::Y_LBO, 1024), b1 = b0 + (L::ATOM >> 4);
+                if (elect_one()) {
+                    const uint32_t a = tmem + L::A_COL + (uint32_t)(s * 16);
+                    if (WINRS_TC2X_LIN && e == 0) {   // v0 += Xhat0 (w0 + w1), v1 += Xhat1 (w0 - w1)
+                        umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
+                        umma_ta<NK, BF>(tmem + 0, a + 0, b1, 1u);
+                        umma_ta<NK, BF>(tmem + NK, a + 8, b0, acc);
+                        umma_ta<NK, BF, true>(tmem + NK, a + 8, b1, 1u);
+                    } else {
+                        umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
+                        umma_ta<NK, BF>(tmem + NK, a + 8, b1, acc);
+                    }
+                    umma_commit<1>(&bars->empty[s]);
+                }
+                __syncwarp();
+                TC2_TRACE(ch - c_lo, 5);
+                if (++s == L::S) { s = 0; ph ^= 1; }
+            }
+            if (elect_one()) umma_commit<1>(&bars->accfull);
             __syncwarp();
-            TC2_TRACE(ch - c_lo, 5);
-            if (++s == L::S) { s = 0; ph ^= 1; }
-        }
-        if (elect_one()) umma_commit<1>(&bars->accfull);
-        __syncwarp();
-    } else {
-        // ================================= FT =================================
-        // Group G takes stages G, G + NG, ...; warp q owns TMEM lanes 32q..
-        // (A rows: fh slot / channel half q / 2, channels 32 (q % 2) ..).  Per
-        // 16-row half, ldmatrix.x4.trans of the needed columns gives each
-        // thread two channels x four depth entries in the tcgen05.st 16x256b
-        // fragment order (bfc_tc2.cuh TA), the IT runs on the packed
-        // registers and two stores fill the slot's two xi A columns.
-        const int tw = warp - 2;
-        const int G = tw >> 2, q = warp & 3;
-        const int i4 = lane >> 3, rho = lane & 7;
-        const int img = 4 * (rho >> 1) + (rho & 1) + 2 * (i4 & 1);
-        uint32_t xoff[2];
-#pragma unroll
-        for (int hf = 0; hf < 2; ++hf) {
-            const int oct = 4 * (q & 1) + 2 * hf + (i4 >> 1);
-            const uint32_t row = (uint32_t)((q >> 1) * x_grp + (img >> 3) * x_hi + (img & 7) * 128);
-            xoff[hf] = row + (uint32_t)((oct ^ ((row >> 7) & 7)) << 4);   // stages are 1 KB aligned
-        }
-        const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16) + L::A_COL;
-        // FT items (e = 0): 16 k octets x 16 depth entries = 256 per stage, 2 per lane
-        const int it0 = q * 32 + lane;
-        const uint32_t foff0 = opoff(it0 % 16, it0 / 16, L::Y_LBO);
-        const uint32_t foff1 = opoff((it0 + 128) % 16, (it0 + 128) / 16, L::Y_LBO);
-        int s = G;
-        uint32_t ph = 0;
-        for (int ch = c_lo + G; ch < c_hi; ch += NG) {
-            mbar_wait(&bars->full[s], ph);
-            tc_after();
-            TC2_JITTER(ch, warp);
-            if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
-            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
-#pragma unroll
+        } else {
+            // ================================= FT =================================
+            // Group G takes stages G, G + NG, ...; warp q owns TMEM lanes 32q..
+            // (A rows: fh slot / channel half q / 2, channels 32 (q % 2) ..).  Per
+            // 16-row half, ldmatrix.x4.trans of the needed columns gives each
+            // thread two channels x four depth entries in the tcgen05.st 16x256b
+            // fragment order (bfc_tc2.cuh TA), the IT runs on the packed
+            // registers and two stores fill the slot's two xi A columns.
+            const int tw = warp - 2;
+            const int G = tw >> 2, q = warp & 3;
+            const int i4 = lane >> 3, rho = lane & 7;
+            const int img = 4 * (rho >> 1) + (rho & 1) + 2 * (i4 & 1);
+            uint32_t xoff[2];
+    #pragma unroll
             for (int hf = 0; hf < 2; ++hf) {
-                uint32_t o[2][4];
-                if (e == 0) {
-                    uint32_t x1[4], x2[4];
-                    ldsm_x4_t(st + xoff[hf], x1);
-                    ldsm_x4_t(st + xoff[hf] + 1024, x2);
-#pragma unroll
-                    for (int r = 0; r < 4; ++r) {
-                        o[0][r] = P16<BF>::add(x1[r], x2[r]);
-                        o[1][r] = P16<BF>::sub(x2[r], x1[r]);
+                const int oct = 4 * (q & 1) + 2 * hf + (i4 >> 1);
+                const uint32_t row = (uint32_t)((q >> 1) * x_grp + (img >> 3) * x_hi + (img & 7) * 128);
+                xoff[hf] = row + (uint32_t)((oct ^ ((row >> 7) & 7)) << 4);   // stages are 1 KB aligned
+            }
+            const uint32_t trow = tmem + ((uint32_t)(q * 32) << 16) + L::A_COL;
+            // FT items (e = 0): 16 k octets x 16 depth entries = 256 per stage, 2 per lane
+            const int it0 = q * 32 + lane;
+            const uint32_t foff0 = opoff(it0 % 16, it0 / 16, L::Y_LBO);
+            const uint32_t foff1 = opoff((it0 + 128) % 16, (it0 + 128) / 16, L::Y_LBO);
+            int s = G;
+            uint32_t ph = 0;
+            for (int ch = c_lo + G; ch < c_hi; ch += NG) {
+                mbar_wait(&bars->full[s], ph);
+                tc_after();
+                TC2_JITTER(ch, warp);
+                if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
+                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+    #pragma unroll
+                for (int hf = 0; hf < 2; ++hf) {
+                    uint32_t o[2][4];
+                    if (e == 0) {
+                        uint32_t x1[4], x2[4];
+                        ldsm_x4_t(st + xoff[hf], x1);
+                        ldsm_x4_t(st + xoff[hf] + 1024, x2);
+    #pragma unroll
+                        for (int r = 0; r < 4; ++r) {
+                            o[0][r] = P16<BF>::add(x1[r], x2[r]);
+                            o[1][r] = P16<BF>::sub(x2[r], x1[r]);
+                        }
+                    } else {
+                        uint32_t x[4][4];
+    #pragma unroll
+                        for (int c = 0; c < 4; ++c) ldsm_x4_t(st + xoff[hf] + c * 1024, x[c]);
+    #pragma unroll
+                        for (int r = 0; r < 4; ++r) {
+                            o[0][r] = P16<BF>::sub(x[0][r], x[2][r]);
+                            o[1][r] = P16<BF>::sub(x[3][r], x[1][r]);
+                        }
                     }
+                    const uint32_t ta = trow + ((uint32_t)(hf * 16) << 16) + (uint32_t)(s * 16);
+                    tmem_st16x256_x2(ta, o);
+                }
+                if (e == 0 && !WINRS_TC2X_LIN) {   // What[0] = w0 + w1, What[1] = w0 - w1 (128 k x 16 depth)
+                    const uint32_t y = st + L::OFF_Y0, f = st + L::OFF_F0;
+                    const uint4 a0 = lds16(y + foff0), a1 = lds16(y + L::ATOM + foff0);
+                    const uint4 b0 = lds16(y + foff1), b1 = lds16(y + L::ATOM + foff1);
+                    sts16(f + foff0, vadd<BF>(a0, a1));
+                    sts16(f + L::ATOM + foff0, vsub<BF>(a0, a1));
+                    sts16(f + foff1, vadd<BF>(b0, b1));
+                    sts16(f + L::ATOM + foff1, vsub<BF>(b0, b1));
+                }
+                tmem_wait_st();
+                fence_async();
+                tc_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&bars->opfull[s]);
+                if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 3);
+                s += NG;
+                if (s >= L::S) { s -= L::S; ph ^= 1; }
+            }
+            // ============================ epilogue ================================
+            // This half's share of the OT into the staging tile [s][k][m]; e = 1
+            // has no y1 term (its rows are skipped by the reduction).
+            mbar_wait(&bars->accfull, 0);
+            tc_after();
+            if (threadIdx.x == 64) TC2_TRACE(511, 2);
+            const int m = q * 32 + lane;
+            float* Out = reinterpret_cast<float*>(smem);      // overlays the idle ring
+            const uint32_t lane_base = tmem + ((uint32_t)(q * 32) << 16);
+    #pragma unroll 1
+            for (int k0 = G * (NK / NG); k0 < (G + 1) * (NK / NG); k0 += 8) {
+                float va[8], vb[8];
+                if (!empty_range) {
+                    tmem_ld8(lane_base + (uint32_t)k0, va);
+                    tmem_ld8(lane_base + (uint32_t)(NK + k0), vb);
+                    tmem_wait_ld();
                 } else {
-                    uint32_t x[4][4];
-#pragma unroll
-                    for (int c = 0; c < 4; ++c) ldsm_x4_t(st + xoff[hf] + c * 1024, x[c]);
-#pragma unroll
-                    for (int r = 0; r < 4; ++r) {
-                        o[0][r] = P16<BF>::sub(x[0][r], x[2][r]);
-                        o[1][r] = P16<BF>::sub(x[3][r], x[1][r]);
+    #pragma unroll
+                    for (int i = 0; i < 8; ++i) va[i] = vb[i] = 0.f;
+                }
+    #pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    if (e == 0) {
+                        const float sp = 0.5f * (va[i] + vb[i]);
+                        Out[(0 * NK + k0 + i) * MROWS + m] = sp;
+                        Out[(1 * NK + k0 + i) * MROWS + m] = 0.5f * (va[i] - vb[i]);
+                        Out[(2 * NK + k0 + i) * MROWS + m] = sp;
+                    } else {
+                        Out[(0 * NK + k0 + i) * MROWS + m] = va[i];
+                        Out[(2 * NK + k0 + i) * MROWS + m] = vb[i];
                     }
                 }
-                const uint32_t ta = trow + ((uint32_t)(hf * 16) << 16) + (uint32_t)(s * 16);
-                tmem_st16x256_x2(ta, o);
             }
-            if (e == 0 && !WINRS_TC2X_LIN) {   // What[0] = w0 + w1, What[1] = w0 - w1 (128 k x 16 depth)
-                const uint32_t y = st + L::OFF_Y0, f = st + L::OFF_F0;
-                const uint4 a0 = lds16(y + foff0), a1 = lds16(y + L::ATOM + foff0);
-                const uint4 b0 = lds16(y + foff1), b1 = lds16(y + L::ATOM + foff1);
-                sts16(f + foff0, vadd<BF>(a0, a1));
-                sts16(f + L::ATOM + foff0, vsub<BF>(a0, a1));
-                sts16(f + foff1, vadd<BF>(b0, b1));
-                sts16(f + L::ATOM + foff1, vsub<BF>(b0, b1));
-            }
-            tmem_wait_st();
-            fence_async();
-            tc_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&bars->opfull[s]);
-            if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 3);
-            s += NG;
-            if (s >= L::S) { s -= L::S; ph ^= 1; }
         }
-        // ============================ epilogue ================================
-        // This half's share of the OT into the staging tile [s][k][m]; e = 1
-        // has no y1 term (its rows are skipped by the reduction).
-        mbar_wait(&bars->accfull, 0);
-        tc_after();
-        if (threadIdx.x == 64) TC2_TRACE(511, 2);
-        const int m = q * 32 + lane;
-        float* Out = reinterpret_cast<float*>(smem);      // overlays the idle ring
-        const uint32_t lane_base = tmem + ((uint32_t)(q * 32) << 16);
-#pragma unroll 1
-        for (int k0 = G * (NK / NG); k0 < (G + 1) * (NK / NG); k0 += 8) {
-            float va[8], vb[8];
-            if (!empty_range) {
-                tmem_ld8(lane_base + (uint32_t)k0, va);
-                tmem_ld8(lane_base + (uint32_t)(NK + k0), vb);
-                tmem_wait_ld();
+        tc_before();
+        __syncthreads();
+        if (threadIdx.x == 64) TC2_TRACE(511, 3);
+        // ---- deterministic cluster reduction over the 2 x csplit ranks: cluster
+        // rank r sums rows (s, k) of its slice over ranks 0..nranks-1 in order
+        // (the y1 rows over the e = 0 ranks only) and writes them to the bucket.
+        {
+            constexpr int ROWS = NSOUT * NK, M4 = MROWS / 4;
+            cluster_sync_all();
+            if (threadIdx.x == 64) TC2_TRACE(511, 4);
+            unsigned int* flag = SK ? args.sk_flags + tile : nullptr;
+            const int r_lo = ROWS * crank / nranks, r_hi = ROWS * (crank + 1) / nranks;
+            if constexpr (SK) {
+                // 1. the pair's sum of this CTA's row slice, written back in place (only
+                //    this CTA reads its own slice rows); 2. wait for this tile's chain
+                //    turn; 3. read-add-write (or store, order 0) from shared memory.
+                for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHK) {
+                    const int row = p / M4, m4 = p % M4;
+                    const uint32_t addr = sbase + (uint32_t)((row * MROWS + m4 * 4) * 4);
+                    const float4 acc = row / NK == 1 ? dsmem_sum4(addr, 1, 2, 0) : dsmem_sum4(addr, 2);
+                    *reinterpret_cast<float4*>(smem + (size_t)(row * MROWS + m4 * 4) * 4) = acc;
+                }
+                if (order > 0 && threadIdx.x == 0) {
+                    const unsigned int want = (args.sk_epoch << 8) | (unsigned int)order;
+                    const long long t0 = clock64();
+                    while (ld_acquire(flag) != want) {
+                        __nanosleep(64);
+                        if (clock64() - t0 > 8000000000LL) __trap();   // ~4 s: a broken chain fails loudly, never hangs
+                    }
+                }
+                __syncthreads();
+#pragma unroll 4
+                for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHK) {
+                    const int row = p / M4, m4 = p % M4;
+                    const int sidx = row / NK, kl = row % NK;
+                    float4 acc = *reinterpret_cast<const float4*>(smem + (size_t)(row * MROWS + m4 * 4) * 4);
+                    const int mm = m4 * 4;
+                    const int fh = fh_base + mm / L::BC, c = c_base + mm % L::BC, k = k_base + kl;
+                    if (fh < g.R && c < g.C && k < g.K) {
+                        float4* o = reinterpret_cast<float4*>(bucket + (((long long)k * g.R + fh) * g.S + fw0 + sidx) * g.C + c);
+                        if (order > 0) {   // the tile's later parts first, this part added last (fixed order)
+                            const float4 prev = __ldcg(o);
+                            acc = make_float4(prev.x + acc.x, prev.y + acc.y, prev.z + acc.z, prev.w + acc.w);
+                        }
+                        *o = acc;
+                    }
+                }
             } else {
-#pragma unroll
-                for (int i = 0; i < 8; ++i) va[i] = vb[i] = 0.f;
-            }
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                if (e == 0) {
-                    const float sp = 0.5f * (va[i] + vb[i]);
-                    Out[(0 * NK + k0 + i) * MROWS + m] = sp;
-                    Out[(1 * NK + k0 + i) * MROWS + m] = 0.5f * (va[i] - vb[i]);
-                    Out[(2 * NK + k0 + i) * MROWS + m] = sp;
-                } else {
-                    Out[(0 * NK + k0 + i) * MROWS + m] = va[i];
-                    Out[(2 * NK + k0 + i) * MROWS + m] = vb[i];
+                for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHK) {
+                    const int row = p / M4, m4 = p % M4;
+                    const int sidx = row / NK, kl = row % NK;
+                    const uint32_t addr = sbase + (uint32_t)((row * MROWS + m4 * 4) * 4);
+                    const float4 acc = sidx == 1 ? dsmem_sum4(addr, g.csplit, 2, 0) : dsmem_sum4(addr, nranks);
+                    const int mm = m4 * 4;
+                    const int fh = fh_base + mm / L::BC, c = c_base + mm % L::BC, k = k_base + kl;
+                    if (fh < g.R && c < g.C && k < g.K)
+                        *reinterpret_cast<float4*>(bucket + (((long long)k * g.R + fh) * g.S + fw0 + sidx) * g.C + c) = acc;
                 }
             }
+            if (threadIdx.x == 64) TC2_TRACE(511, 5);
+            if (SK) __threadfence();
+            cluster_sync_all();
+            if (SK && crank == 0 && threadIdx.x == 0) st_release(flag, (args.sk_epoch << 8) | (unsigned int)(order + 1));
         }
-    }
-    tc_before();
-    __syncthreads();
-    if (threadIdx.x == 64) TC2_TRACE(511, 3);
-    // ---- deterministic cluster reduction over the 2 x csplit ranks: cluster
-    // rank r sums rows (s, k) of its slice over ranks 0..nranks-1 in order
-    // (the y1 rows over the e = 0 ranks only) and writes them to the bucket.
-    {
-        constexpr int ROWS = NSOUT * NK, M4 = MROWS / 4;
-        cluster_sync_all();
-        if (threadIdx.x == 64) TC2_TRACE(511, 4);
-        const int r_lo = ROWS * crank / nranks, r_hi = ROWS * (crank + 1) / nranks;
-        for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHK) {
-            const int row = p / M4, m4 = p % M4;
-            const int sidx = row / NK, kl = row % NK;
-            const uint32_t addr = sbase + (uint32_t)((row * MROWS + m4 * 4) * 4);
-            const float4 acc = sidx == 1 ? dsmem_sum4(addr, g.csplit, 2, 0) : dsmem_sum4(addr, nranks);
-            const int mm = m4 * 4;
-            const int fh = fh_base + mm / L::BC, c = c_base + mm % L::BC, k = k_base + kl;
-            if (fh < g.R && c < g.C && k < g.K)
-                *reinterpret_cast<float4*>(bucket + (((long long)k * g.R + fh) * g.S + fw0 + sidx) * g.C + c) = acc;
-        }
-        if (threadIdx.x == 64) TC2_TRACE(511, 5);
-        cluster_sync_all();
     }
     if (threadIdx.x == 64) TC2_TRACE(511, 6);
     if (warp == 1) {

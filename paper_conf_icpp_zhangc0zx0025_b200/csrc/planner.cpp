@@ -245,6 +245,8 @@ struct SharedModel {
 
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
+    if (e.fhs > 0 && e.ta == 3)   // stream-K xi-split pairs, all 74 pairs busy (tools/ab_sk.sh)
+        return {4.0e-6, 10.3e12};
     if (e.fhs > 0 && e.ta == 2)   // bfc_tc2x.cuh xi-split pair (128 k x 128 rows, Xhat in TMEM): rate of the
         return {4.0e-6, 13.2e12};  // pair over its tile (tools/ab_xs.sh: VGG conv4_2 cs = 1, 3136 stages per pair in 508 us)
     if (e.fhs > 0 && e.cg == 2 && bn == 256)   // swapped CTA pair (256 k x 128 c): X side shared
@@ -293,6 +295,25 @@ static long long cluster_slots(int cs, int occ, int num_sms, const SharedModel& 
 
 static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
     const TimeModel m = time_model(e);
+    if (e.ta == 3) {
+        // stream-K pairs (bfc_tc2x.cuh SK): every co-resident pair takes an equal share
+        // of the concatenated tile depths; each tile part ends with the pair's OT /
+        // DSMEM reduction and a read-add-write of dW in the chain order.
+        long long chunks = 0;
+        for (int fh = 0; fh < g.R; fh += g.fhs) {
+            int hs, he, wf, units;
+            group_rows(g, 0, fh, &hs, &he);
+            seg_units(g, 0, &wf, &units);
+            chunks += (long long)g.kblocks * g.cblocks * g.ftiles * (((long long)(he - hs) * units * g.N + g.chunk - 1) / g.chunk);
+        }
+        // Fitted on B200 (tools/ab_sk.sh, profiles/r02/ablations/ab_sk2.txt): ~203 ns per
+        // chunk per pair with every pair busy, ~8 us per step of a tile's chain (the
+        // parts of one tile are written one after another, all near the end).
+        const double pairs = std::max(1.0, std::min((double)chunks, std::floor(num_sms / 2.0)));
+        const double per_chunk = (double)g.chunk * e.bn * e.bm * e.fhs * 2.0 * g.a0 / m.rate_sm;
+        const double chain = 1.0 + std::ceil(pairs / (double)num_tiles(g));
+        return m.fixed_s + std::ceil(chunks / pairs) * per_chunk + chain * 8.0e-6;
+    }
     SharedModel sh = shared_model(e.cc16 ? 0 : e.dtype);
     const int fhs = e.fhs > 0 ? e.fhs : 1;
     const double per_chunk = (double)g.chunk * e.bn * e.bm * fhs * 2.0 / m.rate_sm;
@@ -354,6 +375,7 @@ static bool cs_allowed(const KernelEntry& e, int cs) {
     if (!e.csplit_ok) return false;
     if ((cs == 5 || cs == 7) && e.fhs <= 0) return false;   // 5 / 7 ranks: tc2 / tc3 kernels only
     if (e.cg == 2 && cs > 4) return false;                  // CTA pairs: clusters of 2 x cs <= 8 CTAs
+    if (e.ta == 3) return false;                            // stream-K pairs: no cluster depth split
     if (e.dtype != 0 && e.fhs <= 0 && !e.cc16) return cs == 2 || cs == 4;
     return true;
 }
@@ -398,6 +420,7 @@ static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairC
         const int v = atoi(fz);
         if (v >= 1) { z_lo = z_hi = v; zmax = 1 << 30; }
     }
+    if (e.ta == 3) z_lo = z_hi = 1;   // stream-K pairs: one segment per tile (the pairs split the depth)
     int zhat_used = 1, sh0 = p.Ho, sw0 = pc.k0 * e.r0;
     alg2(p, e.r0, pc.k0, std::min(z_alg1, zmax), &zhat_used, &sh0, &sw0);
     const int fcs = forced_csplit();

@@ -152,6 +152,43 @@ def test_tc2_xs(name, ov, env, dtype, monkeypatch):
     _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA="2"), expect_kernel="_v2x_")
 
 
+# stream-K xi-split pairs (bfc_tc2x.cuh SK): all co-resident pairs split the concatenated tile depths;
+# tiles cut between pairs are combined in dW in a fixed chain order
+XSK = [
+    ("l2", dict(N=16, C=128, K=128, H=28, W=28), {}),
+    ("l3", dict(N=16, C=256, K=256, H=14, W=14), {}),
+    ("l4_many_tiles", dict(N=16, C=512, K=512, H=7, W=7), {}),
+    ("f2", dict(N=16, C=64, K=128, H=20, W=20), {"WINRS_FORCE_TILE": "128x64"}),
+    ("ragged", dict(N=16, C=200, K=136, H=13, W=11), {}),
+    ("tiny_fewer_chunks_than_pairs", dict(N=16, C=64, K=64, H=4, W=5), {"WINRS_FORCE_TILE": "128x128"}),
+    ("pad0_s6", dict(N=16, C=128, K=128, H=16, W=16, S=6, pad=0), {"WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
+    ("r5_f2", dict(N=32, C=64, K=128, H=16, W=16, R=5, S=3, pad=2), {"WINRS_FORCE_TILE": "128x64"}),
+    ("vgg_like_long", dict(N=32, C=128, K=256, H=56, W=56), {}),
+]
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+@pytest.mark.parametrize("name,ov,env", XSK, ids=[c[0] for c in XSK])
+def test_tc2_xsk(name, ov, env, dtype, monkeypatch):
+    layer = BASE.with_(name="xsk_" + name, dtype=dtype, **ov)
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA="3"), expect_kernel="_v2k_")
+
+
+def test_tc2_xsk_exact_and_repeatable(monkeypatch):
+    """Integer inputs: the chained read-add-write of tiles cut between pairs is
+    exact; 20 repeated calls are bitwise identical (fixed chain order)."""
+    layer = BASE.with_(name="xsk_ints", N=32, C=256, K=256, H=14, W=14)
+    g = np.random.Generator(np.random.PCG64(9))
+    X = g.integers(0, 3, size=(layer.N, layer.H, layer.W, layer.C)).astype(np.float16)
+    dY = g.integers(0, 3, size=(layer.N, layer.Ho, layer.Wo, layer.K)).astype(np.float16)
+    p, _ = _check(layer, monkeypatch, {"WINRS_TC_GEN": "2", "WINRS_FORCE_TA": "3"}, X=X, dY=dY, exact=True,
+                  expect_kernel="_v2k_")
+    Xg, Gg = _dev(X, "f16"), _dev(dY, "f16")
+    first = W.bfc(p, Xg, Gg).clone()
+    for _ in range(20):
+        assert torch.equal(W.bfc(p, Xg, Gg), first)
+
+
 @pytest.mark.parametrize("name,ov,env", XS[:6], ids=[c[0] for c in XS[:6]])
 def test_tc2_xs_signed(name, ov, env, monkeypatch):
     layer = BASE.with_(name="xss_" + name, **ov)
