@@ -217,6 +217,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
             if (piece > 0) break;
             tile = blockIdx.x / nranks;
         }
+        if (SK && threadIdx.x == 64 && piece < 3) TC2_TRACE(490 + piece * 6, 0);
         const CtaCoord cc = decode_cta(g, tile);
         const int fh_base = cc.fh;
         const int c_base = F == 2 ? cc.cb * 64 : cc.cb * 128;
@@ -451,6 +452,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                     const float4 acc = row / NK == 1 ? dsmem_sum4(addr, 1, 2, 0) : dsmem_sum4(addr, 2);
                     *reinterpret_cast<float4*>(smem + (size_t)(row * MROWS + m4 * 4) * 4) = acc;
                 }
+                if (threadIdx.x == 64 && piece < 3) TC2_TRACE(490 + piece * 6 + 1, 0);
                 if (order > 0 && threadIdx.x == 0) {
                     const unsigned int want = (args.sk_epoch << 8) | (unsigned int)order;
                     const long long t0 = clock64();
@@ -460,6 +462,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                     }
                 }
                 __syncthreads();
+                if (threadIdx.x == 64 && piece < 3) TC2_TRACE(490 + piece * 6 + 2, 0);
 #pragma unroll 4
                 for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHK) {
                     const int row = p / M4, m4 = p % M4;
@@ -492,6 +495,13 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
             if (SK) __threadfence();
             cluster_sync_all();
             if (SK && crank == 0 && threadIdx.x == 0) st_release(flag, (args.sk_epoch << 8) | (unsigned int)(order + 1));
+            if (SK && threadIdx.x == 64 && piece < 3) {
+                TC2_TRACE(490 + piece * 6 + 3, 0);
+                TC2_TRACE(490 + piece * 6 + 4, 0);
+#ifdef WINRS_TC2_TRACE
+                if (blockIdx.x == (unsigned)g_tc2_trace_cta) { g_tc2_trace[490 + piece * 6 + 5][0] = order; g_tc2_trace[490 + piece * 6 + 5][1] = c_hi - c_lo; }
+#endif
+            }
         }
     }
     if (threadIdx.x == 64) TC2_TRACE(511, 6);
