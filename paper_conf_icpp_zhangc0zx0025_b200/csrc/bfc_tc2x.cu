@@ -41,7 +41,6 @@ cudaError_t launch_x(const Geometry& g, const void* X, const void* dY, float* dW
 // Stream-K pairs (SK): the chain flags live in a library-owned, zero-initialised
 // per-device buffer (no workspace); each launch tags its flag values with a fresh
 // epoch so values left by an earlier launch never match a waiter.
-constexpr int SK_MAX_TILES = 1 << 16;
 static unsigned int* sk_flags_for_device(int dev) {
     static std::mutex mu;
     static unsigned int* bufs[64] = {};
@@ -49,12 +48,19 @@ static unsigned int* sk_flags_for_device(int dev) {
     if (dev < 0 || dev >= 64) return nullptr;
     if (!bufs[dev]) {
         void* p = nullptr;
-        if (cudaMalloc(&p, SK_MAX_TILES * sizeof(unsigned int)) != cudaSuccess) return nullptr;
-        if (cudaMemset(p, 0, SK_MAX_TILES * sizeof(unsigned int)) != cudaSuccess) return nullptr;
+        if (cudaMalloc(&p, (SK_MAX_TILES + 2) * sizeof(unsigned int)) != cudaSuccess) return nullptr;
+        if (cudaMemset(p, 0, (SK_MAX_TILES + 2) * sizeof(unsigned int)) != cudaSuccess) return nullptr;
         if (cudaDeviceSynchronize() != cudaSuccess) return nullptr;
         bufs[dev] = static_cast<unsigned int*>(p);
     }
     return bufs[dev];
+}
+
+// One epoch counter for every instantiation (f16 / bf16, F = 1 / 2): the flags and
+// the ticket counter are shared, so two launches must never carry the same tag.
+static unsigned int sk_next_epoch() {
+    static std::atomic<unsigned int> epoch{0};
+    return (epoch.fetch_add(1) % 0xFFFFFEu) + 1u;   // 24-bit tag, never 0
 }
 
 template <int F, bool BF>
@@ -82,20 +88,19 @@ cudaError_t launch_sk(const Geometry& g, const void* X, const void* dY, float* d
     if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
     a.sk_flags = sk_flags_for_device(dev);
     if (!a.sk_flags) return cudaErrorMemoryAllocation;
-    static std::atomic<unsigned int> epoch{0};
-    a.sk_epoch = (epoch.fetch_add(1) % 0xFFFFFEu) + 1u;   // 24-bit tag, never 0
-    // pairs: every co-resident 2-CTA cluster (all of them must be resident: the chain waits)
+    a.sk_epoch = sk_next_epoch();
+    // pairs: the co-resident 2-CTA clusters (one wave; the chain itself only waits for
+    // lower, already running pairs -- ticketed in the kernel -- so residency is not
+    // required for progress)
     cudaLaunchConfig_t cfg = {};
     cfg.blockDim = dim3((unsigned)tc2_threads<true>());
     cfg.dynamicSmemBytes = (size_t)L::BYTES;
     cfg.stream = stream;
-    cudaLaunchAttribute attr[2];
+    cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = 2;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
-    attr[1].id = cudaLaunchAttributeCooperative;
-    attr[1].val.cooperative = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     static int max_pairs[64] = {};
@@ -118,14 +123,7 @@ cudaError_t launch_sk(const Geometry& g, const void* X, const void* dY, float* d
     if (P > chunks) P = (int)chunks;
     a.sk_pairs = P;
     cfg.gridDim = dim3((unsigned)(2 * P));
-    cfg.numAttrs = 2;
-    e = cudaLaunchKernelEx(&cfg, k, a, mX4, mX2, mY);
-    if (e == cudaErrorCooperativeLaunchTooLarge || e == cudaErrorNotSupported || e == cudaErrorInvalidValue) {
-        (void)cudaGetLastError();   // cooperative + cluster unavailable: P <= the resident cluster count still holds
-        cfg.numAttrs = 1;
-        e = cudaLaunchKernelEx(&cfg, k, a, mX4, mX2, mY);
-    }
-    return e;
+    return cudaLaunchKernelEx(&cfg, k, a, mX4, mX2, mY);
 }
 
 }  // namespace tc2

@@ -72,10 +72,9 @@ struct LayX {
 // concatenated depth chunks of all tiles (Z = 1: one segment per tile; tiles
 // in decode_cta order, so the tiles of one fh group are a contiguous block of
 // equal depth).  A tile split over several pairs is combined in dW in a fixed
-// order -- the pair holding its last chunks first (plain store), then the
-// lower pairs in decreasing index (read-add-write) -- through one chain flag
-// per tile; a pair only ever waits for a higher pair, and all pairs are
-// co-resident (cooperative launch), so the chain cannot deadlock.
+// order -- the pair holding its first chunks first (plain store), then the
+// higher pairs in increasing index (read-add-write) -- through one chain flag
+// per tile; a pair only ever waits for a lower pair (see the piece loop).
 struct SkTile {
     long long t;       // tile index
     long long g0;      // global chunk index of its first chunk
@@ -112,6 +111,8 @@ __device__ __forceinline__ SkTile sk_find(const Geometry& g, long long gi) {
     }
     return r;
 }
+constexpr int SK_MAX_TILES = 1 << 16;   // flag slots; then the pair-ticket and finished-pair counters
+constexpr int SK_TICKET = SK_MAX_TILES;
 __device__ __forceinline__ long long sk_start(long long tot, int p, int P) { return tot * p / P; }
 // The pair whose range holds global chunk gi: the largest p with sk_start(p) <= gi.
 __device__ __forceinline__ int sk_pair_of(long long tot, long long gi, int P) {
@@ -180,21 +181,41 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     // ---- the pieces this CTA works on: one (tile, depth-rank range) without
     // SK; with SK the tiles (or tile parts) of this pair's chunk range
     const int P = SK ? args.sk_pairs : 1;
-    const int pair = SK ? (int)(blockIdx.x >> 1) : 0;
+    // SK pair index = a ticket taken in dispatch order (rank 0 of the cluster takes
+    // it, rank 1 reads it over DSMEM): every lower pair is already running when a
+    // pair starts, so waiting only on lower pairs is safe whatever the residency.
+    int pair = 0;
+    if constexpr (SK) {
+        uint32_t* slot = reinterpret_cast<uint32_t*>(&bars->accfull) + 3;   // spare word after tmem_base
+        if (crank == 0 && threadIdx.x == 0)   // arrival order; the last pair to finish resets the counters
+            *slot = atomicAdd(args.sk_flags + SK_TICKET, 1u) % (unsigned)P;
+        cluster_sync_all();
+        uint32_t remote, v;
+        asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(su(slot)), "r"(0));
+        asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(remote) : "memory");
+        pair = (int)v;
+        cluster_sync_all();   // rank 0's slot is not reused before rank 1 read it
+    }
     const long long tot = SK ? sk_total(g) : 1;
-    long long gcur = SK ? sk_start(tot, pair, P) : 0;
-    const long long gend = SK ? sk_start(tot, pair + 1, P) : 1;
+    // SK: the pair walks its range BACKWARDS (the head of its last tile first), and
+    // a tile's parts are combined in increasing pair order: the pair holding the
+    // tile's first chunks stores (that part is its first piece, done early), each
+    // higher pair adds when its turn comes (its part of the tile is its last
+    // piece).  A pair only ever waits for LOWER pairs, which are dispatched no
+    // later than it, so the chain needs no co-residency guarantee.
+    const long long gbeg = SK ? sk_start(tot, pair, P) : 0;
+    long long gcur = SK ? sk_start(tot, pair + 1, P) : 1;   // exclusive end of the part still to do
     for (int piece = 0;; ++piece) {
         long long tile;
         int c_lo, c_hi, order = 0;
         if constexpr (SK) {
-            if (gcur >= gend) break;
-            const SkTile st = sk_find(g, gcur);
+            if (gcur <= gbeg) break;
+            const SkTile st = sk_find(g, gcur - 1);
             tile = st.t;
-            c_lo = (int)(gcur - st.g0);
-            c_hi = (int)min((long long)st.depth, gend - st.g0);
-            order = sk_pair_of(tot, st.g0 + st.depth - 1, P) - pair;   // 0: the pair with the tile's last chunks
-            gcur += c_hi - c_lo;
+            c_lo = (int)(max(st.g0, gbeg) - st.g0);
+            c_hi = (int)(gcur - st.g0);
+            order = pair - sk_pair_of(tot, st.g0, P);   // 0: the pair holding the tile's first chunks
+            gcur -= c_hi - c_lo;
             if (piece > 0) {   // the previous piece drained: every barrier is quiescent
                 if (threadIdx.x == 0) {
                     for (int s = 0; s < L::S; ++s) {
@@ -472,7 +493,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                     const int fh = fh_base + mm / L::BC, c = c_base + mm % L::BC, k = k_base + kl;
                     if (fh < g.R && c < g.C && k < g.K) {
                         float4* o = reinterpret_cast<float4*>(bucket + (((long long)k * g.R + fh) * g.S + fw0 + sidx) * g.C + c);
-                        if (order > 0) {   // the tile's later parts first, this part added last (fixed order)
+                        if (order > 0) {   // the tile's earlier parts first, this part added last (fixed order)
                             const float4 prev = __ldcg(o);
                             acc = make_float4(prev.x + acc.x, prev.y + acc.y, prev.z + acc.z, prev.w + acc.w);
                         }
@@ -505,6 +526,12 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
         }
     }
     if (threadIdx.x == 64) TC2_TRACE(511, 6);
+    if (SK && crank == 0 && threadIdx.x == 0) {   // every ticket is taken: the last pair out resets both counters
+        if (atomicAdd(args.sk_flags + SK_TICKET + 1, 1u) == (unsigned)P - 1u) {
+            atomicExch(args.sk_flags + SK_TICKET, 0u);
+            atomicExch(args.sk_flags + SK_TICKET + 1, 0u);
+        }
+    }
     if (warp == 1) {
         tc_after();
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(tmem), "r"(512));

@@ -246,7 +246,7 @@ struct SharedModel {
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
     if (e.fhs > 0 && e.ta == 3)   // stream-K xi-split pairs, all 74 pairs busy (tools/ab_sk.sh)
-        return {4.0e-6, 10.3e12};
+        return {0.0, 11.46e12};
     if (e.fhs > 0 && e.ta == 2)   // bfc_tc2x.cuh xi-split pair (128 k x 128 rows, Xhat in TMEM): rate of the
         return {4.0e-6, 13.2e12};  // pair over its tile (tools/ab_xs.sh: VGG conv4_2 cs = 1, 3136 stages per pair in 508 us)
     if (e.fhs > 0 && e.cg == 2 && bn == 256)   // swapped CTA pair (256 k x 128 c): X side shared
@@ -306,13 +306,16 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
             seg_units(g, 0, &wf, &units);
             chunks += (long long)g.kblocks * g.cblocks * g.ftiles * (((long long)(he - hs) * units * g.N + g.chunk - 1) / g.chunk);
         }
-        // Fitted on B200 (tools/ab_sk.sh, profiles/r02/ablations/ab_sk2.txt): ~203 ns per
-        // chunk per pair with every pair busy, ~8 us per step of a tile's chain (the
-        // parts of one tile are written one after another, all near the end).
+        // Fitted on B200 (tools/ab_sk.sh, profiles/r02/ablations/ab_sk3.txt): ~183 ns per
+        // chunk per pair with every pair busy, ~9 us per tile part a pair walks (ring
+        // fill, OT, DSMEM pair reduction) and ~6.5 us per step of a tile's chain.
         const double pairs = std::max(1.0, std::min((double)chunks, std::floor(num_sms / 2.0)));
         const double per_chunk = (double)g.chunk * e.bn * e.bm * e.fhs * 2.0 * g.a0 / m.rate_sm;
-        const double chain = 1.0 + std::ceil(pairs / (double)num_tiles(g));
-        return m.fixed_s + std::ceil(chunks / pairs) * per_chunk + chain * 8.0e-6;
+        const double tiles = (double)num_tiles(g);
+        const double parts = 1.0 + std::ceil(tiles / pairs), chain = 1.0 + std::ceil(pairs / tiles);
+        // (long chains -- few tiles -- also leave the middle parts waiting: +3 us per step past 4)
+        return m.fixed_s + std::ceil(chunks / pairs) * per_chunk + parts * 9.0e-6 + chain * 6.5e-6 +
+               std::max(0.0, chain - 4.0) * 3.0e-6;
     }
     SharedModel sh = shared_model(e.cc16 ? 0 : e.dtype);
     const int fhs = e.fhs > 0 ? e.fhs : 1;
