@@ -248,7 +248,9 @@ static TimeModel time_model(const KernelEntry& e) {
     if (e.fhs > 0 && e.ta == 3)   // stream-K xi-split pairs, all 74 pairs busy (tools/ab_sk.sh)
         return {0.0, 11.46e12};
     if (e.fhs > 0 && e.ta == 2)   // bfc_tc2x.cuh xi-split pair (128 k x 128 rows, Xhat in TMEM): rate of the
-        return {4.0e-6, 13.2e12};  // pair over its tile (tools/ab_xs.sh: VGG conv4_2 cs = 1, 3136 stages per pair in 508 us)
+        // pair over its tile (tools/ab_xs.sh: VGG conv4_2 cs = 1, 3136 stages per pair in 508 us); the
+        // F = 2 tiles carry the dead fh slot of R = 3 through every MMA (VGG conv2_1: 343 vs TA 331 us)
+        return {4.0e-6, e.fhs == 2 ? 12.4e12 : 13.2e12};
     if (e.fhs > 0 && e.cg == 2 && bn == 256)   // swapped CTA pair (256 k x 128 c): X side shared
         return {4.5e-6, 12.6e12};              // (re-fitted with two producer warps: tools/sweep_tc2.py)
     if (e.fhs > 0 && e.cg == 2)   // bfc_tc2.cuh CTA pair: rate of the pair over its 256-row tile
