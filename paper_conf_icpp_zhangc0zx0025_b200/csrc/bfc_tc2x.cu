@@ -41,6 +41,11 @@ cudaError_t launch_x(const Geometry& g, const void* X, const void* dY, float* dW
 // Stream-K pairs (SK): the chain flags live in a library-owned, zero-initialised
 // per-device buffer (no workspace); each launch tags its flag values with a fresh
 // epoch so values left by an earlier launch never match a waiter.
+// SK_REGIONS independent flag / ticket regions per device, used in rotation (one per
+// launch): launches that overlap on different streams use different regions (up to
+// SK_REGIONS in flight); launches on one stream are serialised anyway.
+constexpr int SK_REGIONS = 8;
+constexpr size_t SK_REGION_WORDS = SK_MAX_TILES + 64;   // flags, ticket counters, 256-byte aligned
 static unsigned int* sk_flags_for_device(int dev) {
     static std::mutex mu;
     static unsigned int* bufs[64] = {};
@@ -48,8 +53,8 @@ static unsigned int* sk_flags_for_device(int dev) {
     if (dev < 0 || dev >= 64) return nullptr;
     if (!bufs[dev]) {
         void* p = nullptr;
-        if (cudaMalloc(&p, (SK_MAX_TILES + 2) * sizeof(unsigned int)) != cudaSuccess) return nullptr;
-        if (cudaMemset(p, 0, (SK_MAX_TILES + 2) * sizeof(unsigned int)) != cudaSuccess) return nullptr;
+        if (cudaMalloc(&p, SK_REGIONS * SK_REGION_WORDS * sizeof(unsigned int)) != cudaSuccess) return nullptr;
+        if (cudaMemset(p, 0, SK_REGIONS * SK_REGION_WORDS * sizeof(unsigned int)) != cudaSuccess) return nullptr;
         if (cudaDeviceSynchronize() != cudaSuccess) return nullptr;
         bufs[dev] = static_cast<unsigned int*>(p);
     }
@@ -86,9 +91,10 @@ cudaError_t launch_sk(const Geometry& g, const void* X, const void* dY, float* d
     if (e != cudaSuccess) return e;
     int dev = 0;
     if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
-    a.sk_flags = sk_flags_for_device(dev);
-    if (!a.sk_flags) return cudaErrorMemoryAllocation;
+    unsigned int* base = sk_flags_for_device(dev);
+    if (!base) return cudaErrorMemoryAllocation;
     a.sk_epoch = sk_next_epoch();
+    a.sk_flags = base + (size_t)(a.sk_epoch % SK_REGIONS) * SK_REGION_WORDS;
     // pairs: the co-resident 2-CTA clusters (one wave; the chain itself only waits for
     // lower, already running pairs -- ticketed in the kernel -- so residency is not
     // required for progress)

@@ -174,6 +174,27 @@ def test_tc2_xsk(name, ov, env, dtype, monkeypatch):
     _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA="3"), expect_kernel="_v2k_")
 
 
+def test_tc2_xsk_two_streams(monkeypatch):
+    """Two stream-K launches in flight on different streams (separate flag / ticket
+    regions): both results equal the single-stream ones bit for bit."""
+    layer = BASE.with_(name="xsk_streams", N=16, C=256, K=256, H=14, W=14)
+    X, dY = wl.make_inputs(layer)
+    p = _plan(layer, {"WINRS_TC_GEN": "2", "WINRS_FORCE_TA": "3"}, monkeypatch)
+    assert "_v2k_" in p.kernel_name
+    Xg, Gg = _dev(X, "f16"), _dev(dY, "f16")
+    ref = W.bfc(p, Xg, Gg).clone()
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    torch.cuda.synchronize()
+    outs = []
+    for _ in range(10):
+        a = W.bfc(p, Xg, Gg, stream=s1)
+        b = W.bfc(p, Xg, Gg, stream=s2)
+        outs += [a, b]
+    torch.cuda.synchronize()
+    for o in outs:
+        assert torch.equal(o, ref)
+
+
 def test_tc2_xsk_exact_and_repeatable(monkeypatch):
     """Integer inputs: the chained read-add-write of tiles cut between pairs is
     exact; 20 repeated calls are bitwise identical (fixed chain order)."""
