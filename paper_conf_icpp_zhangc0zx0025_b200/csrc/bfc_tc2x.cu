@@ -79,7 +79,7 @@ cudaError_t launch_sk(const Geometry& g, const void* X, const void* dY, float* d
     a.ws = ws;
     a.nb = images_per_box(g);
     if (a.nb == 0 || g.a0 != 4 || g.n0 != 3 || g.r0 != 2 || g.a1 != 0 || g.cg != 2 || g.fhs != F || g.csplit != 1 ||
-        g.Z != 1 || tiles > SK_MAX_TILES)
+        tiles > SK_MAX_TILES || g.bands * g.seg_cols * g.fhg > 4096)
         return cudaErrorInvalidValue;
     const bool nd = g.T > 1 || g.D > 1;
     CUtensorMap mX4, mX2, mY;
@@ -119,10 +119,11 @@ cudaError_t launch_sk(const Geometry& g, const void* X, const void* dY, float* d
     int P = dev < 64 ? max_pairs[dev] : 1;
     // a.sk_pairs <= the chunk count, so that every pair has work
     long long chunks = 0;
-    for (int f = 0; f < g.fhg; ++f) {
+    for (int bi = 0; bi < g.bands * g.seg_cols * g.fhg; ++bi) {
         int hs, he, wf, units;
-        group_rows(g, 0, f * g.fhs, &hs, &he);
-        seg_units(g, 0, &wf, &units);
+        const int sc = bi / g.fhg;
+        group_rows(g, sc / g.seg_cols, (bi % g.fhg) * g.fhs, &hs, &he);
+        seg_units(g, sc % g.seg_cols, &wf, &units);
         chunks += (long long)g.kblocks * g.cblocks * g.ftiles * (((long long)(he > hs ? he - hs : 0) * units * g.N + KC - 1) / KC);
     }
     if (chunks <= 0) return cudaSuccess;

@@ -69,9 +69,9 @@ struct LayX {
 };
 
 // ---- stream-K schedule (SK): the pairs take equal contiguous ranges of the
-// concatenated depth chunks of all tiles (Z = 1: one segment per tile; tiles
-// in decode_cta order, so the tiles of one fh group are a contiguous block of
-// equal depth).  A tile split over several pairs is combined in dW in a fixed
+// concatenated depth chunks of all tiles (tiles = segments x fh groups x tile
+// coordinates in decode_cta order; a segment's tiles of one fh group form a
+// contiguous block of equal depth; Z > 1 segments write their own buckets).  A tile split over several pairs is combined in dW in a fixed
 // order -- the pair holding its first chunks first (plain store), then the
 // higher pairs in increasing index (read-add-write) -- through one chain flag
 // per tile; a pair only ever waits for a lower pair (see the piece loop).
@@ -80,29 +80,35 @@ struct SkTile {
     long long g0;      // global chunk index of its first chunk
     int depth;         // its chunks
 };
-__device__ __forceinline__ int sk_group_chunks(const Geometry& g, int fh) {
+// Blocks of equal-depth tiles: block bi = (band * seg_cols + col) * fhg + fh group
+// holds the kblocks x cblocks x ftiles tiles of one segment and filter-row group
+// (decode_cta order), each `sk_block_chunks` deep.
+__device__ __forceinline__ int sk_block_chunks(const Geometry& g, int bi) {
+    const int fgrp = bi % g.fhg, sc = bi / g.fhg;
     int hs, he, wf, units;
-    group_rows(g, 0, fh, &hs, &he);
-    seg_units(g, 0, &wf, &units);
+    group_rows(g, sc / g.seg_cols, fgrp * g.fhs, &hs, &he);
+    seg_units(g, sc % g.seg_cols, &wf, &units);
     const long long d = (long long)(he > hs ? he - hs : 0) * units * g.N;
     return (int)((d + KC - 1) / KC);
 }
 __device__ __forceinline__ long long sk_total(const Geometry& g) {
     const long long per = (long long)g.kblocks * g.cblocks * g.ftiles;
+    const int nb = g.bands * g.seg_cols * g.fhg;
     long long tot = 0;
-    for (int f = 0; f < g.fhg; ++f) tot += per * sk_group_chunks(g, f * g.fhs);
+    for (int bi = 0; bi < nb; ++bi) tot += per * sk_block_chunks(g, bi);
     return tot;
 }
 // The tile holding global chunk gi.
 __device__ __forceinline__ SkTile sk_find(const Geometry& g, long long gi) {
     const long long per = (long long)g.kblocks * g.cblocks * g.ftiles;
+    const int nb = g.bands * g.seg_cols * g.fhg;
     long long acc = 0;
     SkTile r{0, 0, 0};
-    for (int f = 0; f < g.fhg; ++f) {
-        const int d = sk_group_chunks(g, f * g.fhs);
+    for (int bi = 0; bi < nb; ++bi) {
+        const int d = sk_block_chunks(g, bi);
         if (d > 0 && gi < acc + per * d) {
             const long long i = (gi - acc) / d;
-            r.t = (long long)f * per + i;
+            r.t = (long long)bi * per + i;
             r.g0 = acc + i * d;
             r.depth = d;
             return r;

@@ -245,8 +245,8 @@ struct SharedModel {
 
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
-    if (e.fhs > 0 && e.ta == 3)   // stream-K xi-split pairs, all 74 pairs busy (tools/ab_sk.sh)
-        return {0.0, 11.46e12};
+    if (e.fhs > 0 && e.ta == 3)   // stream-K xi-split pairs, all 74 pairs busy (tools/ab_sk.sh); F = 2 tiles
+        return {0.0, e.fhs == 2 ? 8.0e12 : 11.46e12};   // carry the dead fh slot (VGG conv2_1: 402 vs TA 331 us)
     if (e.fhs > 0 && e.ta == 2)   // bfc_tc2x.cuh xi-split pair (128 k x 128 rows, Xhat in TMEM): rate of the
         // pair over its tile (tools/ab_xs.sh: VGG conv4_2 cs = 1, 3136 stages per pair in 508 us); the
         // F = 2 tiles carry the dead fh slot of R = 3 through every MMA (VGG conv2_1: 343 vs TA 331 us)
@@ -302,12 +302,15 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
         // of the concatenated tile depths; each tile part ends with the pair's OT /
         // DSMEM reduction and a read-add-write of dW in the chain order.
         long long chunks = 0;
-        for (int fh = 0; fh < g.R; fh += g.fhs) {
-            int hs, he, wf, units;
-            group_rows(g, 0, fh, &hs, &he);
-            seg_units(g, 0, &wf, &units);
-            chunks += (long long)g.kblocks * g.cblocks * g.ftiles * (((long long)(he - hs) * units * g.N + g.chunk - 1) / g.chunk);
-        }
+        for (int band = 0; band < g.bands; ++band)
+            for (int col = 0; col < g.seg_cols; ++col)
+                for (int fh = 0; fh < g.R; fh += g.fhs) {
+                    int hs, he, wf, units;
+                    group_rows(g, band, fh, &hs, &he);
+                    seg_units(g, col, &wf, &units);
+                    chunks += (long long)g.kblocks * g.cblocks * g.ftiles *
+                              (((long long)(he - hs) * units * g.N + g.chunk - 1) / g.chunk);
+                }
         // Fitted on B200 (tools/ab_sk.sh, profiles/r02/ablations/ab_sk3.txt): ~183 ns per
         // chunk per pair with every pair busy, ~9 us per tile part a pair walks (ring
         // fill, OT, DSMEM pair reduction) and ~6.5 us per step of a tile's chain.
@@ -316,8 +319,13 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
         const double tiles = (double)num_tiles(g);
         const double parts = 1.0 + std::ceil(tiles / pairs), chain = 1.0 + std::ceil(pairs / tiles);
         // (long chains -- few tiles -- also leave the middle parts waiting: +3 us per step past 4)
-        return m.fixed_s + std::ceil(chunks / pairs) * per_chunk + parts * 9.0e-6 + chain * 6.5e-6 +
-               std::max(0.0, chain - 4.0) * 3.0e-6;
+        double t = m.fixed_s + std::ceil(chunks / pairs) * per_chunk + parts * 9.0e-6 + chain * 6.5e-6 +
+                   std::max(0.0, chain - 4.0) * 3.0e-6;
+        if (g.Z > 1) {   // the segments' buckets are summed by the reduction launch
+            const SharedModel sh = shared_model(e.dtype);
+            t += sh.reduce_s + 2.0 * g.Z * (double)g.dw_elems * 4.0 / sh.reduce_bw;
+        }
+        return t;
     }
     SharedModel sh = shared_model(e.cc16 ? 0 : e.dtype);
     const int fhs = e.fhs > 0 ? e.fhs : 1;
@@ -425,7 +433,7 @@ static double plan_with_tile(const Problem& p, const KernelEntry& e, const PairC
         const int v = atoi(fz);
         if (v >= 1) { z_lo = z_hi = v; zmax = 1 << 30; }
     }
-    if (e.ta == 3) z_lo = z_hi = 1;   // stream-K pairs: one segment per tile (the pairs split the depth)
+
     int zhat_used = 1, sh0 = p.Ho, sw0 = pc.k0 * e.r0;
     alg2(p, e.r0, pc.k0, std::min(z_alg1, zmax), &zhat_used, &sh0, &sw0);
     const int fcs = forced_csplit();

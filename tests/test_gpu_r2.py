@@ -164,6 +164,10 @@ XSK = [
     ("pad0_s6", dict(N=16, C=128, K=128, H=16, W=16, S=6, pad=0), {"WINRS_FORCE_PAIR": "4,3,2,0,0,0"}),
     ("r5_f2", dict(N=32, C=64, K=128, H=16, W=16, R=5, S=3, pad=2), {"WINRS_FORCE_TILE": "128x64"}),
     ("vgg_like_long", dict(N=32, C=128, K=256, H=56, W=56), {}),
+    # Z > 1: segments' buckets summed by the reduction launch
+    ("z4", dict(N=16, C=128, K=128, H=28, W=28), {"WINRS_FORCE_Z": "4"}),
+    ("z7_ragged", dict(N=16, C=200, K=136, H=30, W=29), {"WINRS_FORCE_Z": "7"}),
+    ("f2_z6", dict(N=32, C=64, K=128, H=24, W=24), {"WINRS_FORCE_TILE": "128x64", "WINRS_FORCE_Z": "6"}),
 ]
 
 
