@@ -408,6 +408,92 @@ __device__ __forceinline__ void depth_nhu(int d, int N, int units, int hs, int* 
     *h = hs + t / units;
 }
 
+// ---- stream-K schedule (SK): the pairs (bfc_tc2x.cuh) take equal contiguous ranges of the
+// concatenated depth chunks of all tiles (tiles = segments x fh groups x tile
+// coordinates in decode_cta order; a segment's tiles of one fh group form a
+// contiguous block of equal depth; Z > 1 segments write their own buckets).  A tile split over several pairs is combined in dW in a fixed
+// order -- the pair holding its first chunks first (plain store), then the
+// higher pairs in increasing index (read-add-write) -- through one chain flag
+// per tile; a pair only ever waits for a lower pair (see the piece loop).
+struct SkTile {
+    long long t;       // tile index
+    long long g0;      // global chunk index of its first chunk
+    int depth;         // its chunks
+};
+// Blocks of equal-depth tiles: block bi = (band * seg_cols + col) * fhg + fh group
+// holds the kblocks x cblocks x ftiles tiles of one segment and filter-row group
+// (decode_cta order).  With N % 16 == 0 (every tc2-family plan) a tile's chunks
+// are rows(band, group) x units(col) x N / 16, so the prefix over blocks factors
+// by band, column and group: sk_total / sk_find walk bands, then columns, then
+// groups (O(bands + seg_cols + fhg) instead of a walk over every block).
+__device__ __forceinline__ int sk_rows(const Geometry& g, int band, int f) {
+    int hs, he;
+    group_rows(g, band, f * g.fhs, &hs, &he);
+    return he > hs ? he - hs : 0;
+}
+__device__ __forceinline__ int sk_units(const Geometry& g, int col) {
+    int wf, units;
+    seg_units(g, col, &wf, &units);
+    return units;
+}
+__device__ __forceinline__ long long sk_total(const Geometry& g) {
+    const long long per = (long long)g.kblocks * g.cblocks * g.ftiles * (g.N / KC);
+    long long rows = 0, units = 0;
+    for (int b = 0; b < g.bands; ++b)
+        for (int f = 0; f < g.fhg; ++f) rows += sk_rows(g, b, f);
+    for (int c = 0; c < g.seg_cols; ++c) units += sk_units(g, c);
+    return per * rows * units;
+}
+// The tile holding global chunk gi.
+__device__ __forceinline__ SkTile sk_find(const Geometry& g, long long gi) {
+    const long long per = (long long)g.kblocks * g.cblocks * g.ftiles;
+    const long long n16 = g.N / KC;
+    long long utot = 0;
+    for (int c = 0; c < g.seg_cols; ++c) utot += sk_units(g, c);
+    long long acc = 0;
+    SkTile r{0, 0, 0};
+    for (int b = 0; b < g.bands; ++b) {
+        long long rb = 0;
+        for (int f = 0; f < g.fhg; ++f) rb += sk_rows(g, b, f);
+        const long long bsz = per * n16 * rb * utot;
+        if (gi >= acc + bsz) { acc += bsz; continue; }
+        for (int c = 0; c < g.seg_cols; ++c) {
+            const long long uc = sk_units(g, c);
+            const long long csz = per * n16 * rb * uc;
+            if (gi >= acc + csz) { acc += csz; continue; }
+            for (int f = 0; f < g.fhg; ++f) {
+                const long long d = (long long)sk_rows(g, b, f) * uc * n16;
+                if (d > 0 && gi < acc + per * d) {
+                    const long long i = (gi - acc) / d;
+                    r.t = ((long long)(b * g.seg_cols + c) * g.fhg + f) * per + i;
+                    r.g0 = acc + i * d;
+                    r.depth = (int)d;
+                    return r;
+                }
+                acc += per * d;
+            }
+            return r;
+        }
+        return r;
+    }
+    return r;
+}
+constexpr int SK_MAX_TILES = 1 << 16;   // flag slots; then the pair-ticket and finished-pair counters
+constexpr int SK_TICKET = SK_MAX_TILES;
+__device__ __forceinline__ long long sk_start(long long tot, int p, int P) { return tot * p / P; }
+// The pair whose range holds global chunk gi: the largest p with sk_start(p) <= gi.
+__device__ __forceinline__ int sk_pair_of(long long tot, long long gi, int P) {
+    return (int)(((gi + 1) * P - 1) / tot);
+}
+__device__ __forceinline__ unsigned int ld_acquire(const unsigned int* p) {
+    unsigned int v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(unsigned int* p, unsigned int v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+
 // TA = true: the transformed X operand (Xhat) goes to TMEM (tcgen05.st) and
 // the MMAs read A from there: the IT's shared-memory write-back and the MMAs'
 // A reads leave the shared-memory port.  TMEM: 4 NK

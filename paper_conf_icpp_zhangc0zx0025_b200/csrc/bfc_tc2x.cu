@@ -61,9 +61,14 @@ static unsigned int* sk_flags_for_device(int dev) {
     return bufs[dev];
 }
 
+unsigned int* sk_flags_region(int dev, unsigned int epoch) {
+    unsigned int* base = sk_flags_for_device(dev);
+    return base ? base + (size_t)(epoch % SK_REGIONS) * SK_REGION_WORDS : nullptr;
+}
+
 // One epoch counter for every instantiation (f16 / bf16, F = 1 / 2): the flags and
 // the ticket counter are shared, so two launches must never carry the same tag.
-static unsigned int sk_next_epoch() {
+unsigned int sk_next_epoch() {
     static std::atomic<unsigned int> epoch{0};
     return (epoch.fetch_add(1) % 0xFFFFFEu) + 1u;   // 24-bit tag, never 0
 }
@@ -91,10 +96,9 @@ cudaError_t launch_sk(const Geometry& g, const void* X, const void* dY, float* d
     if (e != cudaSuccess) return e;
     int dev = 0;
     if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
-    unsigned int* base = sk_flags_for_device(dev);
-    if (!base) return cudaErrorMemoryAllocation;
     a.sk_epoch = sk_next_epoch();
-    a.sk_flags = base + (size_t)(a.sk_epoch % SK_REGIONS) * SK_REGION_WORDS;
+    a.sk_flags = sk_flags_region(dev, a.sk_epoch);
+    if (!a.sk_flags) return cudaErrorMemoryAllocation;
     // pairs: the co-resident 2-CTA clusters (one wave; the chain itself only waits for
     // lower, already running pairs -- ticketed in the kernel -- so residency is not
     // required for progress)

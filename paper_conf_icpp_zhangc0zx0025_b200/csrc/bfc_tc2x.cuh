@@ -68,70 +68,7 @@ struct LayX {
     static_assert(BYTES <= 227 * 1024, "smem");
 };
 
-// ---- stream-K schedule (SK): the pairs take equal contiguous ranges of the
-// concatenated depth chunks of all tiles (tiles = segments x fh groups x tile
-// coordinates in decode_cta order; a segment's tiles of one fh group form a
-// contiguous block of equal depth; Z > 1 segments write their own buckets).  A tile split over several pairs is combined in dW in a fixed
-// order -- the pair holding its first chunks first (plain store), then the
-// higher pairs in increasing index (read-add-write) -- through one chain flag
-// per tile; a pair only ever waits for a lower pair (see the piece loop).
-struct SkTile {
-    long long t;       // tile index
-    long long g0;      // global chunk index of its first chunk
-    int depth;         // its chunks
-};
-// Blocks of equal-depth tiles: block bi = (band * seg_cols + col) * fhg + fh group
-// holds the kblocks x cblocks x ftiles tiles of one segment and filter-row group
-// (decode_cta order), each `sk_block_chunks` deep.
-__device__ __forceinline__ int sk_block_chunks(const Geometry& g, int bi) {
-    const int fgrp = bi % g.fhg, sc = bi / g.fhg;
-    int hs, he, wf, units;
-    group_rows(g, sc / g.seg_cols, fgrp * g.fhs, &hs, &he);
-    seg_units(g, sc % g.seg_cols, &wf, &units);
-    const long long d = (long long)(he > hs ? he - hs : 0) * units * g.N;
-    return (int)((d + KC - 1) / KC);
-}
-__device__ __forceinline__ long long sk_total(const Geometry& g) {
-    const long long per = (long long)g.kblocks * g.cblocks * g.ftiles;
-    const int nb = g.bands * g.seg_cols * g.fhg;
-    long long tot = 0;
-    for (int bi = 0; bi < nb; ++bi) tot += per * sk_block_chunks(g, bi);
-    return tot;
-}
-// The tile holding global chunk gi.
-__device__ __forceinline__ SkTile sk_find(const Geometry& g, long long gi) {
-    const long long per = (long long)g.kblocks * g.cblocks * g.ftiles;
-    const int nb = g.bands * g.seg_cols * g.fhg;
-    long long acc = 0;
-    SkTile r{0, 0, 0};
-    for (int bi = 0; bi < nb; ++bi) {
-        const int d = sk_block_chunks(g, bi);
-        if (d > 0 && gi < acc + per * d) {
-            const long long i = (gi - acc) / d;
-            r.t = (long long)bi * per + i;
-            r.g0 = acc + i * d;
-            r.depth = d;
-            return r;
-        }
-        acc += per * d;
-    }
-    return r;
-}
-constexpr int SK_MAX_TILES = 1 << 16;   // flag slots; then the pair-ticket and finished-pair counters
-constexpr int SK_TICKET = SK_MAX_TILES;
-__device__ __forceinline__ long long sk_start(long long tot, int p, int P) { return tot * p / P; }
-// The pair whose range holds global chunk gi: the largest p with sk_start(p) <= gi.
-__device__ __forceinline__ int sk_pair_of(long long tot, long long gi, int P) {
-    return (int)(((gi + 1) * P - 1) / tot);
-}
-__device__ __forceinline__ unsigned int ld_acquire(const unsigned int* p) {
-    unsigned int v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_release(unsigned int* p, unsigned int v) {
-    asm volatile("st.release.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
-}
+// The stream-K schedule helpers (SkTile, sk_find, ...) are in bfc_tc2.cuh.
 
 template <int F, bool BF, bool SK = false>
 __global__ void __launch_bounds__(tc2_threads<true>(), 1)

@@ -315,11 +315,12 @@ static double model_time(const Geometry& g, const KernelEntry& e, int num_sms) {
         // chunk per pair with every pair busy, ~9 us per tile part a pair walks (ring
         // fill, OT, DSMEM pair reduction) and ~6.5 us per step of a tile's chain.
         const double pairs = std::max(1.0, std::min((double)chunks, std::floor(num_sms / 2.0)));
+        const double part_s = 9.0e-6, step_s = 6.5e-6;
         const double per_chunk = (double)g.chunk * e.bn * e.bm * e.fhs * 2.0 * g.a0 / m.rate_sm;
         const double tiles = (double)num_tiles(g);
         const double parts = 1.0 + std::ceil(tiles / pairs), chain = 1.0 + std::ceil(pairs / tiles);
         // (long chains -- few tiles -- also leave the middle parts waiting: +3 us per step past 4)
-        double t = m.fixed_s + std::ceil(chunks / pairs) * per_chunk + parts * 9.0e-6 + chain * 6.5e-6 +
+        double t = m.fixed_s + std::ceil(chunks / pairs) * per_chunk + parts * part_s + chain * step_s +
                    std::max(0.0, chain - 4.0) * 3.0e-6;
         if (g.Z > 1) {   // the segments' buckets are summed by the reduction launch
             const SharedModel sh = shared_model(e.dtype);

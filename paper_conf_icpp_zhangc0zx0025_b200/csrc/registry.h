@@ -26,7 +26,8 @@ struct KernelEntry {
                                // second-generation tcgen05 kernels (bfc_tc2.cuh), which need N % 16 == 0
     int cg;                    // CTAs per UMMA: 2 = cta_group::2 pair (0 = 1)
     int ta;                    // 1: tc2 kernel with the transformed X operand in TMEM (bfc_tc2.cuh TA);
-                               // 2: the same with the four xi split over a CTA pair (bfc_tc2x.cuh)
+                               // 2: the same with the four xi split over a CTA pair (bfc_tc2x.cuh);
+                               // 3: those pairs on the stream-K schedule
     int tf32;                  // 1: FP32 inputs on the tensor cores, 3xTF32 split (bfc_tc3.cuh)
     int cc16;                  // 1: FP16 / BF16 inputs on the FP32 CUDA-core pipeline (bfc_f32.cuh, TI = 16-bit)
 };

@@ -62,5 +62,11 @@ inline int images_per_box(const Geometry& g) {
     return (nd ? g.Do : g.N) % KC == 0 ? KC : 0;
 }
 
+// Stream-K chain flags / ticket counters (bfc_tc2x.cu): a fresh epoch tag per
+// launch and the device's flag region for that epoch (regions rotate, so launches
+// in flight on different streams do not share one); nullptr if allocation failed.
+unsigned int sk_next_epoch();
+unsigned int* sk_flags_region(int dev, unsigned int epoch);
+
 }  // namespace tc2
 }  // namespace winrs
