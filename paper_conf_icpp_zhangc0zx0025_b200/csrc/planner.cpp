@@ -246,7 +246,7 @@ struct SharedModel {
 static TimeModel time_model(const KernelEntry& e) {
     const int dtype = e.dtype, bn = e.bn, bm = e.bm;
     if (e.fhs > 0 && e.ta == 3)   // stream-K xi-split pairs, all 74 pairs busy (tools/ab_sk.sh); F = 2 tiles
-        return {0.0, e.fhs == 2 ? 8.0e12 : 11.46e12};   // carry the dead fh slot (VGG conv2_1: 402 vs TA 331 us)
+        return {0.0, e.fhs == 2 ? 11.0e12 : 11.46e12};   // carry the dead fh slot (VGG conv2_1: 312 vs TA 329 us)
     if (e.fhs > 0 && e.ta == 2)   // bfc_tc2x.cuh xi-split pair (128 k x 128 rows, Xhat in TMEM): rate of the
         // pair over its tile (tools/ab_xs.sh: VGG conv4_2 cs = 1, 3136 stages per pair in 508 us); the
         // F = 2 tiles carry the dead fh slot of R = 3 through every MMA (VGG conv2_1: 343 vs TA 331 us)
