@@ -7,7 +7,7 @@ set -u
 mkdir -p gpurun_out
 timeout 900 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
 echo "bench rc=$?"
-for L in vgg_64_64_224_f16 vgg_128_128_112_f16 vgg_256_256_56_f16 vgg_512_512_28_f16 r50_c64_56_f16 r50_c256_14_f16 r50_c512_7_f16 r50_c256_14_f32; do
+for L in vgg_64_64_224_f16 vgg_64_128_112_f16 vgg_128_128_112_f16 vgg_256_256_56_f16 vgg_512_512_28_f16 r50_c64_56_f16 r50_c256_14_f16 r50_c512_7_f16 r50_c256_14_f32; do
   timeout 300 ncu --set full --import-source on --clock-control none -k regex:"bfc_tc[23]" -c 1 \
       -o gpurun_out/prof_$L python tools/run_layer.py $L 2 > gpurun_out/prof_$L.log 2>&1
   echo "ncu $L rc=$?"
