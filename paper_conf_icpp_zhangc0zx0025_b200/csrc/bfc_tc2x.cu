@@ -139,6 +139,8 @@ cudaError_t launch_sk(const Geometry& g, const void* X, const void* dY, float* d
 
 }  // namespace tc2
 
+cudaError_t sk_prepare(int dev) { return tc2::sk_flags_region(dev, 0) ? cudaSuccess : cudaErrorMemoryAllocation; }
+
 #define WINRS_TC2K_ENTRY(DT, BF, PFX, F)                                                                  \
     {DT, 4, 3, 2, 0, 0, 0, 128, ::winrs::tc2::MROWS / F, ::winrs::tc2::tc2_threads<true>(), 1, 1,         \
      (size_t)::winrs::tc2::LayX<F>::BYTES, &::winrs::tc2::launch_sk<F, BF>, PFX "_O4(3,2)_v2k_128x" #F "fh", \

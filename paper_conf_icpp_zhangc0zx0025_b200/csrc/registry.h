@@ -35,6 +35,9 @@ struct KernelEntry {
 // All entries (FP32 and FP16), terminated by count.
 const KernelEntry* kernel_entries(int* count);
 
+// Allocates the stream-K chain-flag regions of device `dev` (bfc_tc2x.cu), once.
+cudaError_t sk_prepare(int dev);
+
 cudaError_t launch_bucket_reduce(float* dW, const float* ws, long long n, int Z, int num_sms,
                                  cudaStream_t stream);
 

@@ -95,7 +95,16 @@ winrs_status_t winrs_plan(int N, int C, int H, int W, int K, int R, int S, int p
         cudaGetLastError();
         return WINRS_ERR_CUDA;
     }
-    return build_plan(N, C, H, W, K, R, S, pad, dtype, &dev, out);
+    const winrs_status_t st = build_plan(N, C, H, W, K, R, S, pad, dtype, &dev, out);
+    // stream-K plans: allocate the device's chain-flag regions now (not inside a
+    // later launch that a caller may be capturing into a CUDA graph)
+    if (st == WINRS_OK && (*out)->pr.entry->ta == 3 && sk_prepare(d) != cudaSuccess) {
+        cudaGetLastError();
+        winrs_plan_destroy(*out);
+        *out = nullptr;
+        return WINRS_ERR_CUDA;
+    }
+    return st;
 }
 
 winrs_status_t winrs_plan3d_for_device(int N, int C, int D, int H, int W, int K, int T, int R, int S, int pad,
