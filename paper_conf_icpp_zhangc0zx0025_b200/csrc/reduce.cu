@@ -25,11 +25,11 @@ __device__ __forceinline__ void kahan_add(float& s, float& c, float x) {
 // The bucket loads of a group of ZB are issued together (they are independent)
 // and then added in z order, so a thread waits for one memory latency per ZB
 // buckets instead of one per bucket; small dW uses one float per thread so
-// the grid still covers the SMs.  The summation order is unchanged.  ZB = 32
-// (float) / 16 (float4): with ~8 warps per SM for a small dW (VGG-16 conv1_2:
-// 36 864 floats, Z = 336) the batch depth sets the bytes in flight; ZB = 8
-// ran at ~1.5 TB/s (profiles/r02/launches_bench_r02.csv, 32 us).
-template <class V> constexpr int zbatch() { return sizeof(V) == 4 ? 32 : 16; }
+// the grid still covers the SMs.  The summation order is unchanged.
+#ifndef WINRS_REDUCE_ZB
+#define WINRS_REDUCE_ZB 8   // layer times with the reduction (tools/ab_reduce_zb.sh): VGG conv1_2 (Z = 336)
+#endif                      // 652 / 761 / 660 us at ZB = 8 / 16 / 32 -- deeper batches did not pay
+template <class V> constexpr int zbatch() { return sizeof(V) == 4 ? WINRS_REDUCE_ZB : (WINRS_REDUCE_ZB < 16 ? WINRS_REDUCE_ZB : 16); }
 
 template <class V>
 __device__ __forceinline__ void kahan_v(V& s, V& c, const V& x);
