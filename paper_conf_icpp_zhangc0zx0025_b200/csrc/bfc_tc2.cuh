@@ -78,6 +78,9 @@ constexpr int NSOUT = 3;               // n0: outputs per unit (S = 3)
                            // all ~20 % SLOWER (ResNet-50 L4 33.8 -> 40 us, VGG conv1_2 656 -> 830 us): the
                            // prefetch boxes cost TMA-engine time like loads; kept as a build option only.
 #endif
+#ifndef WINRS_TC2_TA_S
+#define WINRS_TC2_TA_S 8   // TA ring depth (A/B only: 6 / 7 measure how latency-bound the 8-slot ring is)
+#endif
 #ifndef WINRS_TC2_STX4
 #define WINRS_TC2_STX4 1   // TA: one tcgen05.st .x4 per 16-row half (0: four .x1 stores)
 #endif
@@ -113,7 +116,7 @@ struct Lay {
     static constexpr int OFF_F = OFF_Y + (NKL / 64) * Y_LBO;
     static constexpr int STAGE = OFF_F + (NKL / 64) * Y_LBO;   // 32 / 24 KB (cta pair: 24 KB)
     static constexpr int LIMIT = 227 * 1024 - 1024 - 256;
-    static constexpr int S = LIMIT / STAGE > 8 ? 8 : LIMIT / STAGE;
+    static constexpr int S = (TA && WINRS_TC2_TA_S < 8) ? WINRS_TC2_TA_S : (LIMIT / STAGE > 8 ? 8 : LIMIT / STAGE);
     static constexpr int RING = S * STAGE;
     static constexpr int OUT = NSOUT * NK * MROWS * 4;   // staging tile [s][k][m] fp32 (cluster split)
     static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
@@ -507,7 +510,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     constexpr int NTHK = tc2_threads<TA>();
     constexpr int PW2K = 2 + NTXK;                   // second producer warp
     constexpr int NG = NTXK / 4;                     // TA: FT groups of four warps
-    static_assert(!TA || (CG == 1 && NK == 64 && L::S == 8), "TA: single CTA, NK = 64, 8-slot ring");
+    static_assert(!TA || (CG == 1 && NK == 64 && L::S <= 8 && L::S % 2 == 0), "TA: single CTA, NK = 64, <= 8-slot ring");
     constexpr uint32_t TMEM_ALLOC = TA ? 512u : (uint32_t)L::TMEM_COLS;
     constexpr uint32_t A_COL = 4 * NK;          // TA: first A ring column
     extern __shared__ uint8_t smem_raw[];
