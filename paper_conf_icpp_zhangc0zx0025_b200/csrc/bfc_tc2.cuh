@@ -79,7 +79,9 @@ constexpr int NSOUT = 3;               // n0: outputs per unit (S = 3)
                            // prefetch boxes cost TMA-engine time like loads; kept as a build option only.
 #endif
 #ifndef WINRS_TC2_TA_S
-#define WINRS_TC2_TA_S 8   // TA ring depth (A/B only: 6 / 7 measure how latency-bound the 8-slot ring is)
+#define WINRS_TC2_TA_S 8   // TA shared-memory ring depth (6 / 8 / 9; at 9 the TMEM A ring keeps 8 slots with its
+                           // own release barrier and the FT groups an extra opfull guard: measured slower,
+                           // DESIGN.md §6.4b)
 #endif
 #ifndef WINRS_TC2_STX4
 #define WINRS_TC2_STX4 1   // TA: one tcgen05.st .x4 per 16-row half (0: four .x1 stores)
@@ -115,12 +117,13 @@ struct Lay {
     static constexpr int OFF_Y = TA ? 17 * 1024 : 2 * X_LBO;   // 16 KB (TA: 17 KB, 1 KB aligned)
     static constexpr int OFF_F = OFF_Y + (NKL / 64) * Y_LBO;
     static constexpr int STAGE = OFF_F + (NKL / 64) * Y_LBO;   // 32 / 24 KB (cta pair: 24 KB)
-    static constexpr int LIMIT = 227 * 1024 - 1024 - 256;
-    static constexpr int S = (TA && WINRS_TC2_TA_S < 8) ? WINRS_TC2_TA_S : (LIMIT / STAGE > 8 ? 8 : LIMIT / STAGE);
+    static constexpr int LIMIT = 227 * 1024 - 1024 - 512;
+    static constexpr int SCAP = TA ? (WINRS_TC2_TA_S < 9 ? WINRS_TC2_TA_S : 9) : 8;
+    static constexpr int S = LIMIT / STAGE > SCAP ? SCAP : LIMIT / STAGE;
     static constexpr int RING = S * STAGE;
     static constexpr int OUT = NSOUT * NK * MROWS * 4;   // staging tile [s][k][m] fp32 (cluster split)
     static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
-    static constexpr int BYTES = BAR_OFF + 256 + 1024;   // + alignment slack
+    static constexpr int BYTES = BAR_OFF + 512 + 1024;   // + alignment slack
     static constexpr int TX_BYTES = 2 * X_LBO + (NKL / 64) * Y_LBO;   // TMA bytes per stage
     static constexpr int TMEM_COLS = 4 * NK;
     static_assert(STAGE % 1024 == 0, "stages must keep the 1 KB swizzle-atom alignment");
@@ -142,12 +145,15 @@ struct Args {
 };
 
 struct Bars {
-    uint64_t full[8];       // TMA data landed
-    uint64_t opfull[8];     // FT operands stored (one warp per stage)
-    uint64_t empty[8];      // MMAs of the stage done (commit)
+    uint64_t full[9];       // TMA data landed
+    uint64_t opfull[9];     // FT operands stored (one warp per stage)
+    uint64_t empty[9];      // MMAs of the stage done (commit)
     uint64_t accfull;
     uint32_t tmem_base;
+    uint32_t spare;
+    uint64_t aempty[8];     // TA with a 9-slot ring: MMAs that read TMEM A slot a done (commit)
 };
+static_assert(sizeof(Bars) <= 512, "barrier block");
 
 // ----------------------------------------------------------------------------- PTX helpers
 __device__ __forceinline__ uint32_t su(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
@@ -510,7 +516,8 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     constexpr int NTHK = tc2_threads<TA>();
     constexpr int PW2K = 2 + NTXK;                   // second producer warp
     constexpr int NG = NTXK / 4;                     // TA: FT groups of four warps
-    static_assert(!TA || (CG == 1 && NK == 64 && L::S <= 8 && L::S % 2 == 0), "TA: single CTA, NK = 64, <= 8-slot ring");
+    static_assert(!TA || (CG == 1 && NK == 64 && L::S <= 9), "TA: single CTA, NK = 64, <= 9-slot ring");
+    constexpr bool ASEP = TA && L::S != 8;          // TMEM A ring (8 slots) decoupled from the SMEM ring
     constexpr uint32_t TMEM_ALLOC = TA ? 512u : (uint32_t)L::TMEM_COLS;
     constexpr uint32_t A_COL = 4 * NK;          // TA: first A ring column
     extern __shared__ uint8_t smem_raw[];
@@ -559,8 +566,10 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     }
     if (CG == 2 && threadIdx.x == 0 && e == 0)   // the leader's opfull gathers both CTAs' FT warps
         for (int s = 0; s < L::S; ++s) mbar_init(&bars->opfull[s], 2);
-    if (TA && threadIdx.x == 0)                  // TA: the four lane-quarter warps of a group
+    if (TA && threadIdx.x == 0) {                // TA: the four lane-quarter warps of a group
         for (int s = 0; s < L::S; ++s) mbar_init(&bars->opfull[s], 4);
+        for (int a = 0; a < 8; ++a) mbar_init(&bars->aempty[a], 1);
+    }
     if (warp == 0 && lane == 0) {
         asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmX)) : "memory");
         asm volatile("prefetch.tensormap [%0];" :: "l"(reinterpret_cast<uint64_t>(&tmY)) : "memory");
@@ -725,7 +734,8 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             if (elect_one()) {
 #ifndef WINRS_TC2_NO_MMA   // debug ablation: no tensor-core work (barrier protocol kept)
               if (TA) {               // Xhat[xi] from the TMEM ring slot x What[xi]
-                const uint32_t a = tmem + A_COL + (uint32_t)(s * 32);
+                const int aslot = ASEP ? (ch - c_lo) % 8 : s;
+                const uint32_t a = tmem + A_COL + (uint32_t)(aslot * 32);
                 umma_ta<NK, BF>(tmem + 0 * NK, a + 0, w0d, acc);
                 umma_ta<NK, BF>(tmem + 1 * NK, a + 8, w1d, acc);
                 umma_ta<NK, BF>(tmem + 2 * NK, a + 16, w2d, acc);
@@ -749,6 +759,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 (void)x0; (void)x1; (void)x2; (void)x3; (void)w0d; (void)w1d; (void)w2d; (void)w3d; (void)acc;
 #endif
                 umma_commit<CG>(&bars->empty[s], pair_mask);
+                if (ASEP) umma_commit<1>(&bars->aempty[(ch - c_lo) % 8]);
             }
             __syncwarp();
             TC2_TRACE(ch - c_lo, 5);
@@ -771,7 +782,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         // in it, so its parity wait can never see a phase two rounds ahead.
         constexpr int KO = L::NKL / 8;              // k octets of this CTA's What rows
         constexpr int IPT = KO * KC / 32;           // items per lane: 8 (NK 128) / 4 (NK 64 or a pair)
-        static_assert(L::S <= NTXK, "one FT warp per ring slot");
+        static_assert(TA || L::S <= NTXK, "one FT warp per ring slot");
         const int tw = warp - 2;
         if constexpr (TA) {
             // Two groups of four warps take alternate stages (group G: slots
@@ -786,7 +797,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             // IT runs on the packed registers and 4 stores fill the slot's
             // xi = 0..3 A columns.  Ring safety as below: slot s is refilled
             // only after the MMAs of this group's previous stage in it.
-            static_assert(L::S % NG == 0, "TA: each FT group owns every NG-th ring slot");
+            static_assert(ASEP || L::S % NG == 0, "TA: each FT group owns every NG-th ring slot");
             const int G = tw >> 2, q = warp & 3;
             const int i4 = lane >> 3, rho = lane & 7;
             const int img = 4 * (rho >> 1) + (rho & 1) + 2 * (i4 & 1);
@@ -807,11 +818,20 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             int s = G;
             uint32_t ph = 0;
             for (int ch = c_lo + G; ch < c_hi; ch += NG) {
+                // odd ring depth (ASEP, S = 9): a group meets each slot every other
+                // round, so first wait for the other group's stage in this slot to be
+                // through (its opfull): the full wait below then never sees a phase
+                // two rounds old (parity aliasing)
+                if (ASEP && ch - c_lo >= L::S)
+                    mbar_wait(&bars->opfull[s], (uint32_t)(((ch - c_lo - L::S) / L::S) & 1));
                 mbar_wait(&bars->full[s], ph);
                 tc_after();
                 TC2_JITTER(ch, warp);
                 if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
                 const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+                const int aslot = ASEP ? (ch - c_lo) % 8 : s;
+                if (ASEP && ch - c_lo >= 8)   // the MMAs of stage ch - 8 read this A slot
+                    mbar_wait(&bars->aempty[aslot], (uint32_t)(((ch - c_lo) / 8 - 1) & 1));
 #pragma unroll
                 for (int hf = 0; hf < 2 && !xdead; ++hf) {
                     uint32_t x[4][4];
@@ -825,7 +845,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                         o[2][r] = P16<BF>::sub(x[0][r], x[2][r]);
                         o[3][r] = P16<BF>::sub(x[3][r], x[1][r]);
                     }
-                    const uint32_t ta = trow + ((uint32_t)(hf * 16) << 16) + (uint32_t)(s * 32);
+                    const uint32_t ta = trow + ((uint32_t)(hf * 16) << 16) + (uint32_t)(aslot * 32);
 #ifndef WINRS_TC2_NO_STTM   // debug ablation: no TMEM stores of the A operand (the MMAs read stale A)
 #if WINRS_TC2_STX4
                     tmem_st16x256_x4(ta, o);   // the slot's four xi slabs are 4 consecutive 8-column chunks
@@ -1013,7 +1033,7 @@ struct LaySw {
                                                          // lanes on consecutive k rows hit distinct banks
     static constexpr int OUT = NSOUT * 128 * OUT_LD * 4;  // staging [s][k 128][c 128 (+4)] fp32, 198 KB
     static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
-    static constexpr int BYTES = BAR_OFF + 256 + 1024;
+    static constexpr int BYTES = BAR_OFF + 512 + 1024;
     static constexpr int TX_BYTES = OFF_F;               // 16 KB per stage
     static constexpr int TMEM_COLS = 512;                // 4 xi x N = 128
     static_assert(BYTES <= 227 * 1024, "smem");

@@ -58,7 +58,7 @@ struct LayX {
     static constexpr int RING = S * STAGE;               // 200 KB
     static constexpr int OUT = NSOUT * NK * MROWS * 4;   // staging [s][k][m] fp32, 192 KB
     static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
-    static constexpr int BYTES = BAR_OFF + 256 + 1024;
+    static constexpr int BYTES = BAR_OFF + 512 + 1024;
     static constexpr int TX0 = 4 * 2048 + 2 * Y_LBO;     // TMA bytes per stage: 16 KB (e = 0)
     static constexpr int TX1 = 4 * 4096 + 2 * Y_LBO;     //                      24 KB (e = 1)
     static constexpr uint32_t A_COL = 2 * NK;            // first A ring column (after 2 x 128 accumulators)
