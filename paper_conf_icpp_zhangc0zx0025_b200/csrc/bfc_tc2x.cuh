@@ -422,7 +422,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                     const long long t0 = clock64();
                     while (ld_acquire(flag) != want) {
                         __nanosleep(64);
-                        if (clock64() - t0 > 8000000000LL) __trap();   // ~4 s: a broken chain fails loudly, never hangs
+                        if (clock64() - t0 > 40000000000LL) __trap();   // ~20 s: a broken chain fails loudly, never hangs
                     }
                 }
                 __syncthreads();
