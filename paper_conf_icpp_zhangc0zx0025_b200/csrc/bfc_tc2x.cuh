@@ -6,16 +6,20 @@
 //     IT  Xhat = (x1 + x2, x2 - x1, x0 - x2, x3 - x1)
 //     OT  y0 = (v0 + v1)/2 + v2,  y1 = (v0 - v1)/2,  y2 = (v0 + v1)/2 + v3
 // but the four Winograd points xi of one tile are split over a CTA pair:
-//     half e = 0: xi = 0, 1 (X columns x1, x2; the FT'd What[0], What[1])
+//     half e = 0: xi = 0, 1 (X columns x1, x2; What[0], What[1] = w0 +- w1)
 //     half e = 1: xi = 2, 3 (X columns x0..x3; the raw dY columns w0, w1)
 // Each CTA keeps only two accumulators in TMEM, so the tile can be NK = 128
 // k wide with the transformed X operand still in TMEM (TA):
-// 2 x 128 accumulator columns + an 8-slot ring of 2 x 8 A columns.  Per
-// 16-deep stage each CTA issues two A-from-TMEM MMAs at N = 128 (~92 cycles
-// each, §6.5) instead of four at N = 64 (~84 each), and moves 16 + 8 KB (e=0:
-// 8 KB X fill + 8 KB ldmatrix, 8 KB dY fill, 8 + 8 KB FT) or 16 + 16 + 8 KB
-// (e=1, no FT) through the shared-memory port, against 44 KB for the same
-// MACs in the NK = 64 TA kernel.
+// 2 x 128 accumulator columns + an 8-slot ring of 2 x 8 A columns, and the
+// A-from-TMEM MMAs run at N = 128 (~92 cycles, §6.5) instead of N = 64 (~84,
+// bound by the 4 KB TMEM read of A, §6.4b).  The e = 0 half applies its FT by
+// linearity in the tensor core (WINRS_TC2X_LIN, default): v0 += Xhat0 w0 +
+// Xhat0 w1, v1 += Xhat1 w0 - Xhat1 w1 (negate-B bit) -- four MMAs on the raw
+// w0, w1 and no FT stores / proxy fence on its critical path; e = 1 issues two.
+// The pair moves 8 + 8 + 8 KB (e = 0: X fill, ldmatrix, dY fill) and
+// 16 + 16 + 8 KB (e = 1) per stage through the shared-memory port (DESIGN.md
+// §6.10).  On the stream-K schedule (SK = true, §6.11) one wave of pairs takes
+// equal ranges of all tiles' depth chunks.
 //
 // The OT is linear in v, so each half applies its share of A^T to its own
 // accumulators (e=0: y0 = y2 = (v0+v1)/2, y1 = (v0-v1)/2; e=1: y0 = v2,
