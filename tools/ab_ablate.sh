@@ -1,4 +1,6 @@
 # A/B of TA builds (cold-L2 layer times): usage ab_ablate.sh variant...  ("" = libwinrs.so)
+# build the variants first, e.g. python tools/build.py --variant nosttm --define WINRS_TC2_NO_STTM
+#   (nomma: WINRS_TC2_NO_MMA, notma: WINRS_TC2_NO_TMA, pf16: WINRS_TC2_PF=16, stx1: WINRS_TC2_STX4=0)
 mkdir -p gpurun_out
 for V in "$@"; do
   [ "$V" = base ] && V=""
