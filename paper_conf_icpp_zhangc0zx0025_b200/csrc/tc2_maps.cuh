@@ -7,6 +7,10 @@
 #include <mutex>
 #include "bfc_tc2.cuh"
 
+#ifndef WINRS_TMA_L2PROMO
+#define WINRS_TMA_L2PROMO CU_TENSOR_MAP_L2_PROMOTION_L2_256B   // L2 sector promotion of the X / dY boxes (A/B knob)
+#endif
+
 namespace winrs {
 namespace tc2 {
 
@@ -43,7 +47,7 @@ inline bool make_map(CUtensorMap* m, const void* base, int A, int B, int H, int 
     const cuuint32_t es[5] = {1u, 1u, 1u, 1u, 1u};
     return fn(m, bf ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 5, const_cast<void*>(base),
               dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+              WINRS_TMA_L2PROMO, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 // The X and dY maps of a plan (2-D or N-D).
 // xbn: images per X box (TA kernels: 8, two boxes per stage and atom).
