@@ -145,9 +145,9 @@ struct Args {
 };
 
 struct Bars {
-    uint64_t full[9];       // TMA data landed
-    uint64_t opfull[9];     // FT operands stored (one warp per stage)
-    uint64_t empty[9];      // MMAs of the stage done (commit)
+    uint64_t full[12];      // TMA data landed
+    uint64_t opfull[12];    // FT operands stored (one warp per stage)
+    uint64_t empty[12];     // MMAs of the stage done (commit)
     uint64_t accfull;
     uint32_t tmem_base;
     uint32_t spare;

@@ -35,6 +35,9 @@
 #pragma once
 #include "bfc_tc2.cuh"
 
+#ifndef WINRS_TC2X_S0
+#define WINRS_TC2X_S0 12   // ring depth of the e = 0 half (17 KB stages without the FT region); e = 1: 8 x 25 KB
+#endif
 #ifndef WINRS_TC2X_LIN
 #define WINRS_TC2X_LIN 1   // e = 0 half: What[0,1] = w0 +- w1 applied by the tensor core (four MMAs on the raw
                            // w0, w1 by linearity, negate-B for -w1) instead of the FT warps' stores (0: FT stores)
@@ -60,9 +63,16 @@ struct LayX {
     static constexpr int STAGE = 25 * 1024;
     static constexpr int S = 8;
     static constexpr int RING = S * STAGE;               // 200 KB
+    // e = 0 with the FT by linearity needs no FT region: 17 KB stages, a deeper ring
+    static constexpr int STAGE0 = WINRS_TC2X_LIN ? 17 * 1024 : STAGE;
+    static constexpr int S0 = WINRS_TC2X_LIN ? WINRS_TC2X_S0 : S;
+    static constexpr int SMAX = S0 > S ? S0 : S;
+    static constexpr int RING0 = S0 * STAGE0;
     static constexpr int OUT = NSOUT * NK * MROWS * 4;   // staging [s][k][m] fp32, 192 KB
-    static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
+    static constexpr int RINGM = RING > RING0 ? RING : RING0;
+    static constexpr int BAR_OFF = RINGM > OUT ? RINGM : OUT;
     static constexpr int BYTES = BAR_OFF + 512 + 1024;
+    static_assert(SMAX <= 12 && 2 * NK + SMAX * 16 <= 512 && BYTES <= 227 * 1024, "ring / TMEM / smem budget");
     static constexpr int TX0 = 4 * 2048 + 2 * Y_LBO;     // TMA bytes per stage: 16 KB (e = 0)
     static constexpr int TX1 = 4 * 4096 + 2 * Y_LBO;     //                      24 KB (e = 1)
     static constexpr uint32_t A_COL = 2 * NK;            // first A ring column (after 2 x 128 accumulators)
@@ -83,7 +93,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     constexpr int NTHK = tc2_threads<true>();
     constexpr int PW2K = 2 + NTX_TA;                     // second producer warp
     constexpr int NG = NTX_TA / 4;                       // FT groups
-    static_assert(L::S % NG == 0, "each FT group owns every NG-th ring slot");
+    static_assert(L::S % NG == 0 && L::S0 % NG == 0, "each FT group owns every NG-th ring slot");
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw_s = su(smem_raw);
     uint8_t* smem = smem_raw + (((raw_s + 1023u) & ~1023u) - raw_s);
@@ -100,9 +110,11 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     // per-half stage layout
     const int x_hi = e ? L::X4_HI : L::X2_HI, x_grp = e ? L::X4_GRP : L::X2_GRP;
     const int off_y = e ? L::OFF_Y1 : L::OFF_Y0;
+    const int RS = e ? L::S : L::S0;                     // this half's ring depth and stage size
+    const uint32_t RSTAGE = e ? (uint32_t)L::STAGE : (uint32_t)L::STAGE0;
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < L::S; ++s) {
+        for (int s = 0; s < L::SMAX; ++s) {
             mbar_init(&bars->full[s], 1);
             mbar_init(&bars->opfull[s], 4);              // the four lane-quarter warps of a group
             mbar_init(&bars->empty[s], 1);
@@ -165,7 +177,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
             gcur -= c_hi - c_lo;
             if (piece > 0) {   // the previous piece drained: every barrier is quiescent
                 if (threadIdx.x == 0) {
-                    for (int s = 0; s < L::S; ++s) {
+                    for (int s = 0; s < L::SMAX; ++s) {
                         asm volatile("mbarrier.inval.shared::cta.b64 [%0];" :: "r"(su(&bars->full[s])) : "memory");
                         asm volatile("mbarrier.inval.shared::cta.b64 [%0];" :: "r"(su(&bars->opfull[s])) : "memory");
                         asm volatile("mbarrier.inval.shared::cta.b64 [%0];" :: "r"(su(&bars->empty[s])) : "memory");
@@ -224,7 +236,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 TC2_JITTER(ch, 0);
                 TC2_TRACE(ch - c_lo, 0);
                 uint64_t* fb = &bars->full[s];
-                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+                const uint32_t st = sbase + (uint32_t)s * RSTAGE;
                 const bool in = d < depth;
                 const ImgCoord ic = itk.at(g, in);
                 const int hh = in ? h : hs;
@@ -254,7 +266,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 }
                 itk.advance(2 * KC, wrapped, n);
                 s += 2;
-                if (s >= L::S) { s -= L::S; ph ^= 1; }
+                if (s >= RS) { s -= RS; ph ^= 1; }
             }
         } else if (warp == 1) {
             // ============================ MMA issuer ==============================
@@ -267,7 +279,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 TC2_JITTER(ch, 1);
                 TC2_TRACE(ch - c_lo, 4);
                 tc_after();
-                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+                const uint32_t st = sbase + (uint32_t)s * RSTAGE;
                 const uint32_t acc = ch > c_lo ? 1u : 0u;
                 const uint64_t b0 = desc_sw128(st + off_b, L::Y_LBO, 1024), b1 = b0 + (L::ATOM >> 4);
                 if (elect_one()) {
@@ -285,7 +297,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 }
                 __syncwarp();
                 TC2_TRACE(ch - c_lo, 5);
-                if (++s == L::S) { s = 0; ph ^= 1; }
+                if (++s == RS) { s = 0; ph ^= 1; }
             }
             if (elect_one()) umma_commit<1>(&bars->accfull);
             __syncwarp();
@@ -320,7 +332,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 tc_after();
                 TC2_JITTER(ch, warp);
                 if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
-                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+                const uint32_t st = sbase + (uint32_t)s * RSTAGE;
     #pragma unroll
                 for (int hf = 0; hf < 2; ++hf) {
                     uint32_t o[2][4];
@@ -362,7 +374,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 if (lane == 0) mbar_arrive(&bars->opfull[s]);
                 if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 3);
                 s += NG;
-                if (s >= L::S) { s -= L::S; ph ^= 1; }
+                if (s >= RS) { s -= RS; ph ^= 1; }
             }
             // ============================ epilogue ================================
             // This half's share of the OT into the staging tile [s][k][m]; e = 1
