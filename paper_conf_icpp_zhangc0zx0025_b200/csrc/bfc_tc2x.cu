@@ -29,7 +29,9 @@ cudaError_t launch_x(const Geometry& g, const void* X, const void* dY, float* dW
     CUtensorMap mX4, mX2, mY;
     if (!make_maps(g, X, dY, BF, &mX4, &mY, 8)) return cudaErrorInvalidValue;
     // x1, x2 only (the e = 0 half): box {64, 8, 1, 1, 2}
-    if (!make_map(&mX2, X, nd ? g.D : g.N, nd ? g.Nb : 1, g.H, g.W, g.C, g.C, 2, 8, BF)) return cudaErrorInvalidValue;
+    if (!make_map(&mX2, X, nd ? g.D : g.N, nd ? g.Nb : 1, g.H, g.W, g.C, g.C, LayX<F>::BAL ? 3 : 2, 8, BF))
+        return cudaErrorInvalidValue;
+    if (LayX<F>::BAL) mX4 = mX2;   // balanced split: both halves load three columns
     static std::atomic<unsigned long long> done{0};
     auto k = bfc_tc2x_kernel<F, BF>;
     cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);
@@ -89,7 +91,9 @@ cudaError_t launch_sk(const Geometry& g, const void* X, const void* dY, float* d
     const bool nd = g.T > 1 || g.D > 1;
     CUtensorMap mX4, mX2, mY;
     if (!make_maps(g, X, dY, BF, &mX4, &mY, 8)) return cudaErrorInvalidValue;
-    if (!make_map(&mX2, X, nd ? g.D : g.N, nd ? g.Nb : 1, g.H, g.W, g.C, g.C, 2, 8, BF)) return cudaErrorInvalidValue;
+    if (!make_map(&mX2, X, nd ? g.D : g.N, nd ? g.Nb : 1, g.H, g.W, g.C, g.C, LayX<F>::BAL ? 3 : 2, 8, BF))
+        return cudaErrorInvalidValue;
+    if (LayX<F>::BAL) mX4 = mX2;   // balanced split: both halves load three columns
     auto k = bfc_tc2x_kernel<F, BF, true>;
     static std::atomic<unsigned long long> done{0};
     cudaError_t e = ensure_smem_attr(k, (size_t)L::BYTES, done);

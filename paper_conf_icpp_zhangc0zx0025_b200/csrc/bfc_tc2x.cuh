@@ -35,6 +35,11 @@
 #pragma once
 #include "bfc_tc2.cuh"
 
+#ifndef WINRS_TC2X_BAL
+#define WINRS_TC2X_BAL 2   // balanced split (e = 0: xi 0, 2 from x0..x2; e = 1: xi 1, 3 from x1..x3; three MMAs
+                           // each, 21 KB stages, 10-deep rings on both halves): 0 never, 1 always, 2 for the F = 2
+                           // tiles only (measured: VGG conv2_1 294 vs 310 us; slower on the F = 1 layers)
+#endif
 #ifndef WINRS_TC2X_S0
 #define WINRS_TC2X_S0 12   // ring depth of the e = 0 half (17 KB stages without the FT region); e = 1: 8 x 25 KB
 #endif
@@ -48,6 +53,7 @@ namespace tc2 {
 
 template <int F>
 struct LayX {
+    static constexpr bool BAL = WINRS_TC2X_BAL == 1 || (WINRS_TC2X_BAL == 2 && F == 2);
     static constexpr int NK = 128;                       // k per tile (both halves)
     static constexpr int BC = MROWS / F;                 // channels per fh slot
     static constexpr int ATOM = KC * 128;                // 2 KB: 64 channels x 16 depth rows
@@ -66,10 +72,13 @@ struct LayX {
     // e = 0 with the FT by linearity needs no FT region: 17 KB stages, a deeper ring
     static constexpr int STAGE0 = WINRS_TC2X_LIN ? 17 * 1024 : STAGE;
     static constexpr int S0 = WINRS_TC2X_LIN ? WINRS_TC2X_S0 : S;
-    static constexpr int SMAX = S0 > S ? S0 : S;
+    static constexpr int SMAX = BAL ? 10 : (S0 > S ? S0 : S);
     static constexpr int RING0 = S0 * STAGE0;
     static constexpr int OUT = NSOUT * NK * MROWS * 4;   // staging [s][k][m] fp32, 192 KB
-    static constexpr int RINGM = RING > RING0 ? RING : RING0;
+    static constexpr int X3_HI = 3072 + 256, X3_GRP = 2 * X3_HI;   // balanced split: 3 columns per half
+    static constexpr int OFF_Y3 = 13 * 1024, STAGE3 = 21 * 1024, S3 = 10, RING3 = S3 * STAGE3;
+    static constexpr int TX3 = 4 * 3072 + 2 * Y_LBO;
+    static constexpr int RINGM = BAL ? RING3 : (RING > RING0 ? RING : RING0);
     static constexpr int BAR_OFF = RINGM > OUT ? RINGM : OUT;
     static constexpr int BYTES = BAR_OFF + 512 + 1024;
     static_assert(SMAX <= 12 && 2 * NK + SMAX * 16 <= 512 && BYTES <= 227 * 1024, "ring / TMEM / smem budget");
@@ -93,7 +102,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     constexpr int NTHK = tc2_threads<true>();
     constexpr int PW2K = 2 + NTX_TA;                     // second producer warp
     constexpr int NG = NTX_TA / 4;                       // FT groups
-    static_assert(L::S % NG == 0 && L::S0 % NG == 0, "each FT group owns every NG-th ring slot");
+    static_assert(L::S % NG == 0 && L::S0 % NG == 0 && L::S3 % NG == 0, "each FT group owns every NG-th ring slot");
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw_s = su(smem_raw);
     uint8_t* smem = smem_raw + (((raw_s + 1023u) & ~1023u) - raw_s);
@@ -108,10 +117,11 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     const int e = crank & 1;                             // xi half
     const int rank = crank >> 1;                         // depth-split rank
     // per-half stage layout
-    const int x_hi = e ? L::X4_HI : L::X2_HI, x_grp = e ? L::X4_GRP : L::X2_GRP;
-    const int off_y = e ? L::OFF_Y1 : L::OFF_Y0;
-    const int RS = e ? L::S : L::S0;                     // this half's ring depth and stage size
-    const uint32_t RSTAGE = e ? (uint32_t)L::STAGE : (uint32_t)L::STAGE0;
+    const int x_hi = L::BAL ? L::X3_HI : (e ? L::X4_HI : L::X2_HI);
+    const int x_grp = L::BAL ? L::X3_GRP : (e ? L::X4_GRP : L::X2_GRP);
+    const int off_y = L::BAL ? L::OFF_Y3 : (e ? L::OFF_Y1 : L::OFF_Y0);
+    const int RS = L::BAL ? L::S3 : (e ? L::S : L::S0);          // this half's ring depth and stage size
+    const uint32_t RSTAGE = L::BAL ? (uint32_t)L::STAGE3 : (e ? (uint32_t)L::STAGE : (uint32_t)L::STAGE0);
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < L::SMAX; ++s) {
@@ -215,8 +225,8 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
             // ============================ TMA producers ===========================
             const int pp = warp == 0 ? 0 : 1;
             const CUtensorMap* mx = e ? &tmX4 : &tmX2;
-            const int xcol = e ? 0 : 1;                      // first X window column loaded
-            const uint32_t tx = e ? (uint32_t)L::TX1 : (uint32_t)L::TX0;
+            const int xcol = L::BAL ? e : (e ? 0 : 1);   // first X window column loaded
+            const uint32_t tx = L::BAL ? (uint32_t)L::TX3 : (e ? (uint32_t)L::TX1 : (uint32_t)L::TX0);
             long long d = (long long)(c_lo + pp) * KC;
             int n = 0, h = hs, u = 0;
             if (d < depth) depth_nhu((int)d, g.N, units, hs, &n, &h, &u);
@@ -271,7 +281,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
         } else if (warp == 1) {
             // ============================ MMA issuer ==============================
             // B: e = 0 What[0], What[1] (FT region); e = 1 the raw w0, w1.
-            const int off_b = e ? L::OFF_Y1 : (WINRS_TC2X_LIN ? L::OFF_Y0 : L::OFF_F0);
+            const int off_b = L::BAL ? L::OFF_Y3 : (e ? L::OFF_Y1 : (WINRS_TC2X_LIN ? L::OFF_Y0 : L::OFF_F0));
             int s = 0;
             uint32_t ph = 0;
             for (int ch = c_lo; ch < c_hi; ++ch) {
@@ -284,7 +294,15 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 const uint64_t b0 = desc_sw128(st + off_b, L::Y_LBO, 1024), b1 = b0 + (L::ATOM >> 4);
                 if (elect_one()) {
                     const uint32_t a = tmem + L::A_COL + (uint32_t)(s * 16);
-                    if (WINRS_TC2X_LIN && e == 0) {   // v0 += Xhat0 (w0 + w1), v1 += Xhat1 (w0 - w1)
+                    if (L::BAL && e == 0) {   // v0 += Xhat0 (w0 + w1), v2 += Xhat2 w0
+                        umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
+                        umma_ta<NK, BF>(tmem + 0, a + 0, b1, 1u);
+                        umma_ta<NK, BF>(tmem + NK, a + 8, b0, acc);
+                    } else if (L::BAL) {       // v1 += Xhat1 (w0 - w1), v3 += Xhat3 w1
+                        umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
+                        umma_ta<NK, BF, true>(tmem + 0, a + 0, b1, 1u);
+                        umma_ta<NK, BF>(tmem + NK, a + 8, b1, acc);
+                    } else if (WINRS_TC2X_LIN && e == 0) {   // v0 += Xhat0 (w0 + w1), v1 += Xhat1 (w0 - w1)
                         umma_ta<NK, BF>(tmem + 0, a + 0, b0, acc);
                         umma_ta<NK, BF>(tmem + 0, a + 0, b1, 1u);
                         umma_ta<NK, BF>(tmem + NK, a + 8, b0, acc);
@@ -336,7 +354,21 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     #pragma unroll
                 for (int hf = 0; hf < 2; ++hf) {
                     uint32_t o[2][4];
-                    if (e == 0) {
+                    if (L::BAL) {   // box columns p0..p2 = x0..x2 (e = 0) / x1..x3 (e = 1)
+                        uint32_t x[3][4];
+#pragma unroll
+                        for (int c = 0; c < 3; ++c) ldsm_x4_t(st + xoff[hf] + c * 1024, x[c]);
+#pragma unroll
+                        for (int r = 0; r < 4; ++r) {
+                            if (e == 0) {
+                                o[0][r] = P16<BF>::add(x[1][r], x[2][r]);   // Xhat0 = x1 + x2
+                                o[1][r] = P16<BF>::sub(x[0][r], x[2][r]);   // Xhat2 = x0 - x2
+                            } else {
+                                o[0][r] = P16<BF>::sub(x[1][r], x[0][r]);   // Xhat1 = x2 - x1
+                                o[1][r] = P16<BF>::sub(x[2][r], x[0][r]);   // Xhat3 = x3 - x1
+                            }
+                        }
+                    } else if (e == 0) {
                         uint32_t x1[4], x2[4];
                         ldsm_x4_t(st + xoff[hf], x1);
                         ldsm_x4_t(st + xoff[hf] + 1024, x2);
@@ -398,7 +430,12 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 }
     #pragma unroll
                 for (int i = 0; i < 8; ++i) {
-                    if (e == 0) {
+                    if (L::BAL) {   // e = 0: (v0 / 2 + v2, v0 / 2, v0 / 2); e = 1: (v1 / 2, -v1 / 2, v1 / 2 + v3)
+                        const float h = 0.5f * va[i];
+                        Out[(0 * NK + k0 + i) * MROWS + m] = e == 0 ? h + vb[i] : h;
+                        Out[(1 * NK + k0 + i) * MROWS + m] = e == 0 ? h : -h;
+                        Out[(2 * NK + k0 + i) * MROWS + m] = e == 0 ? h : h + vb[i];
+                    } else if (e == 0) {
                         const float sp = 0.5f * (va[i] + vb[i]);
                         Out[(0 * NK + k0 + i) * MROWS + m] = sp;
                         Out[(1 * NK + k0 + i) * MROWS + m] = 0.5f * (va[i] - vb[i]);
@@ -429,7 +466,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                 for (int p = r_lo * M4 + (int)threadIdx.x; p < r_hi * M4; p += NTHK) {
                     const int row = p / M4, m4 = p % M4;
                     const uint32_t addr = sbase + (uint32_t)((row * MROWS + m4 * 4) * 4);
-                    const float4 acc = row / NK == 1 ? dsmem_sum4(addr, 1, 2, 0) : dsmem_sum4(addr, 2);
+                    const float4 acc = (!L::BAL && row / NK == 1) ? dsmem_sum4(addr, 1, 2, 0) : dsmem_sum4(addr, 2);
                     *reinterpret_cast<float4*>(smem + (size_t)(row * MROWS + m4 * 4) * 4) = acc;
                 }
                 if (threadIdx.x == 64 && piece < 3) TC2_TRACE(490 + piece * 6 + 1, 0);
@@ -464,7 +501,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
                     const int row = p / M4, m4 = p % M4;
                     const int sidx = row / NK, kl = row % NK;
                     const uint32_t addr = sbase + (uint32_t)((row * MROWS + m4 * 4) * 4);
-                    const float4 acc = sidx == 1 ? dsmem_sum4(addr, g.csplit, 2, 0) : dsmem_sum4(addr, nranks);
+                    const float4 acc = (!L::BAL && sidx == 1) ? dsmem_sum4(addr, g.csplit, 2, 0) : dsmem_sum4(addr, nranks);
                     const int mm = m4 * 4;
                     const int fh = fh_base + mm / L::BC, c = c_base + mm % L::BC, k = k_base + kl;
                     if (fh < g.R && c < g.C && k < g.K)
