@@ -231,6 +231,23 @@ def test_tc2_xs_exact_all_ones(monkeypatch):
                                 "WINRS_FORCE_CSPLIT": "2"}, X=X, dY=dY, exact=True, expect_kernel="_v2x_")
 
 
+@pytest.mark.parametrize("ta,tag", [("2", "_v2x_"), ("3", "_v2k_")])
+@pytest.mark.parametrize("shape,env", [
+    (dict(N=16, C=64, K=128, H=20, W=20), {}),
+    (dict(N=16, C=40, K=72, H=17, W=19), {}),
+    (dict(N=32, C=64, K=128, H=24, W=24), {"WINRS_FORCE_Z": "6"}),
+], ids=["f2", "f2_ragged", "f2_z6"])
+def test_tc2_xs_balanced_f2_exact(ta, tag, shape, env, monkeypatch):
+    """F = 2 tiles run the balanced split (xi {0,2} / {1,3}, three MMAs per half):
+    small-integer inputs, so the pair sum must equal the oracle bit for bit."""
+    layer = BASE.with_(name="xs_bal_ints", **shape)
+    g = np.random.Generator(np.random.PCG64(11))
+    X = g.integers(0, 3, size=(layer.N, layer.H, layer.W, layer.C)).astype(np.float16)
+    dY = g.integers(-2, 3, size=(layer.N, layer.Ho, layer.Wo, layer.K)).astype(np.float16)
+    _check(layer, monkeypatch, dict(env, WINRS_TC_GEN="2", WINRS_FORCE_TA=ta, WINRS_FORCE_TILE="128x64"),
+           X=X, dY=dY, exact=True, expect_kernel=tag + "128x2fh")
+
+
 @pytest.mark.parametrize("name,ov,env", TA[:4], ids=[c[0] for c in TA[:4]])
 def test_tc2_ta_matches_smem_variant(name, ov, env, monkeypatch):
     """Same plan geometry, Xhat in TMEM vs in shared memory: the same packed
