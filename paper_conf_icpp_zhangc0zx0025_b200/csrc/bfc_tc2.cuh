@@ -232,6 +232,11 @@ struct ImgTracker {
 __device__ __forceinline__ void fence_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void tc_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+// Programmatic dependent launch: once every CTA of this grid has started, the
+// bucket reduction queued behind it (reduce.cu, launched with programmatic
+// stream serialisation) may be scheduled; it waits in griddepcontrol.wait
+// until this grid has completed and its writes are visible.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 // UMMA shared-memory descriptor, MN-major, 128-byte swizzle: atoms of 64 MN
 // elements x 8 K rows (1 KB); LBO = MN-atom stride, SBO = K-atom stride
@@ -589,6 +594,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     __syncthreads();
     if (CG == 2) cluster_sync_all();   // peer barriers initialised before any remote arrive / multicast commit
     tc_after();
+    if (threadIdx.x == 0) pdl_trigger();
     const uint32_t tmem = bars->tmem_base;
     if (threadIdx.x == 64) TC2_TRACE(511, 1);
 
@@ -1096,6 +1102,7 @@ bfc_tc2s_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     __syncthreads();
     cluster_sync_all();
     tc_after();
+    if (threadIdx.x == 0) pdl_trigger();
     const uint32_t tmem = bars->tmem_base;
     if (threadIdx.x == 64) TC2_TRACE(511, 1);
 

@@ -144,6 +144,7 @@ bfc_tc2x_kernel(const __grid_constant__ Args args, const __grid_constant__ CUten
     tc_before();
     __syncthreads();
     tc_after();
+    if (threadIdx.x == 0) pdl_trigger();
     const uint32_t tmem = bars->tmem_base;
     if (threadIdx.x == 64) TC2_TRACE(511, 1);
 

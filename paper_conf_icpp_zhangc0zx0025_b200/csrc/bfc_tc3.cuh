@@ -168,6 +168,7 @@ bfc_tc3_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     tc_before();
     __syncthreads();
     tc_after();
+    if (threadIdx.x == 0) pdl_trigger();
     const uint32_t tmem = bars->tmem_base;
 
     if (warp == 0 || warp == PW2) {

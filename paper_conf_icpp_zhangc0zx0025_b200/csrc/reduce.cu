@@ -8,6 +8,7 @@
 // grid sized to a multiple of the SM count, deterministic (no atomics).
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 namespace winrs {
 
@@ -54,6 +55,9 @@ __global__ void __launch_bounds__(256)
 bucket_reduce_kernel(float* __restrict__ dW, const float* __restrict__ ws, long long n, int Z) {
     constexpr int W = sizeof(V) / 4;
     constexpr int ZB = zbatch<V>();
+    // Launched as a programmatic dependent of the BFC kernel: wait until that
+    // grid has completed and its bucket writes are visible (a no-op otherwise).
+    asm volatile("griddepcontrol.wait;" ::: "memory");
     const long long nv = n / W;
     const long long stride = (long long)gridDim.x * blockDim.x;
     for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += stride) {
@@ -89,11 +93,25 @@ cudaError_t launch_bucket_reduce(float* dW, const float* ws, long long n, int Z,
     long long blocks = (items + 255) / 256;
     if (blocks > cap) blocks = cap - cap % num_sms;
     if (blocks < 1) blocks = 1;
+    // Programmatic stream serialisation: the reduction is scheduled once every
+    // CTA of the BFC kernel ahead of it has started (griddepcontrol.launch_dependents
+    // in the tc kernels; kernels without it trigger at exit) and waits on the
+    // device, so its launch latency overlaps the BFC kernel's tail.
+    // WINRS_PDL=0 launches it plainly (A/B).
+    static const bool pdl = [] { const char* v = getenv("WINRS_PDL"); return !(v && v[0] == '0'); }();
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.gridDim = dim3((unsigned)blocks);
+    cfg.blockDim = dim3(256);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = stream;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl ? 1 : 0;
     if (scalar)
-        bucket_reduce_kernel<float><<<(unsigned)blocks, 256, 0, stream>>>(dW, ws, n, Z);
-    else
-        bucket_reduce_kernel<float4><<<(unsigned)blocks, 256, 0, stream>>>(dW, ws, n, Z);
-    return cudaGetLastError();
+        return cudaLaunchKernelEx(&cfg, bucket_reduce_kernel<float>, dW, ws, n, Z);
+    return cudaLaunchKernelEx(&cfg, bucket_reduce_kernel<float4>, dW, ws, n, Z);
 }
 
 }  // namespace winrs
