@@ -278,7 +278,7 @@ static TimeModel time_model(const KernelEntry& e) {
     return {4.02e-6, 1.95e11};
 }
 static SharedModel shared_model(int dtype) {
-    if (dtype != 0) return {2.02e-6, 2.13e-6, 10.8e-6, 7.86e12, 33.1, 14.0};
+    if (dtype != 0) return {2.02e-6, 2.13e-6, 8.3e-6, 7.86e12, 33.1, 14.0};   // reduce_s: 10.8 us before the PDL launch (ablations/ab_pdl.txt: -2..4 us)
     return {0.0, 2.01e-6, 20.8e-6, 2.0e13, 34.8, 15.6};
 }
 
