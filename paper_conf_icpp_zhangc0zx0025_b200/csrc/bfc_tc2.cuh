@@ -83,6 +83,10 @@ constexpr int NSOUT = 3;               // n0: outputs per unit (S = 3)
                            // own release barrier and the FT groups an extra opfull guard: measured slower,
                            // DESIGN.md §6.4b)
 #endif
+#ifndef WINRS_TC2_TA_DEAD_S
+#define WINRS_TC2_TA_DEAD_S 0   // TA, F = 2: ring depth of the CTAs whose second fh slot is dead (the {2, -}
+                                // group of R = 3): one X atom, 17 KB stages; 0 = same ring as the live groups
+#endif
 #ifndef WINRS_TC2_STX4
 #define WINRS_TC2_STX4 1   // TA: one tcgen05.st .x4 per 16-row half (0: four .x1 stores)
 #endif
@@ -120,7 +124,15 @@ struct Lay {
     static constexpr int LIMIT = 227 * 1024 - 1024 - 512;
     static constexpr int SCAP = TA ? (WINRS_TC2_TA_S < 9 ? WINRS_TC2_TA_S : 9) : 8;
     static constexpr int S = LIMIT / STAGE > SCAP ? SCAP : LIMIT / STAGE;
-    static constexpr int RING = S * STAGE;
+    // TA, F = 2, dead second fh slot: X atom 0 only (two 4 KB boxes, 8.25 KB), so What / FT move
+    // up and a stage is 17 KB; S_D of them (the TMEM A ring stays 8 slots: its own release barrier)
+    static constexpr bool DRING = TA && F == 2 && WINRS_TC2_TA_DEAD_S > 0;
+    static constexpr int OFF_Y_D = 9 * 1024;
+    static constexpr int OFF_F_D = OFF_Y_D + (NKL / 64) * Y_LBO;
+    static constexpr int STAGE_D = OFF_F_D + (NKL / 64) * Y_LBO;
+    static constexpr int S_D = DRING ? WINRS_TC2_TA_DEAD_S : S;
+    static constexpr int RING_D = DRING ? S_D * STAGE_D : 0;
+    static constexpr int RING = S * STAGE > RING_D ? S * STAGE : RING_D;
     static constexpr int OUT = NSOUT * NK * MROWS * 4;   // staging tile [s][k][m] fp32 (cluster split)
     static constexpr int BAR_OFF = RING > OUT ? RING : OUT;
     static constexpr int BYTES = BAR_OFF + 512 + 1024;   // + alignment slack
@@ -128,6 +140,8 @@ struct Lay {
     static constexpr int TMEM_COLS = 4 * NK;
     static_assert(STAGE % 1024 == 0, "stages must keep the 1 KB swizzle-atom alignment");
     static_assert(S >= 4, "ring too shallow");
+    static_assert(!DRING || (S_D % 2 == 0 && S_D <= 12 && STAGE_D % 1024 == 0 && RING_D <= LIMIT),
+                  "dead-slot ring: even depth (two FT groups), <= 12 barrier slots, fits");
     static_assert(MROWS == F * BC && BC % 64 == 0, "fh slots of whole 64-channel atoms");
     static_assert(NKL % 64 == 0, "whole 64-channel k atoms per CTA");
 };
@@ -547,6 +561,14 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     // F = 2: fh slots fh_base, fh_base + 1 of channels c_base..c_base + 63.
     // A pair covers 256 channels (F = 1) or 4 filter rows (F = 2).
     const int fh_base = cc.fh + (F == 2 ? 2 * e : 0);
+    // TA, F = 2: a CTA whose second fh slot lies past the last filter row runs the deeper
+    // ring of 17 KB stages (Lay::DRING; its TMEM A ring keeps 8 slots and its own release)
+    const bool dring = L::DRING && fh_base + 1 >= g.R;
+    const int RS = dring ? L::S_D : L::S;
+    const uint32_t RSTAGE = dring ? (uint32_t)L::STAGE_D : (uint32_t)L::STAGE;
+    const uint32_t OFFY = dring ? (uint32_t)L::OFF_Y_D : (uint32_t)L::OFF_Y;
+    const uint32_t OFFF = dring ? (uint32_t)L::OFF_F_D : (uint32_t)L::OFF_F;
+    const bool asep = ASEP || dring;
     const int c_base = F == 2 ? cc.cb * 64 : cc.cb * (128 * CG) + e * 128;
     const int k_base = cc.kb * NK + e * L::NKL;              // this CTA's What rows
     const int seg = cc.band * g.seg_cols + cc.col;
@@ -561,7 +583,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
     const int fw0 = cc.ft * NSOUT;       // first output column of this fw-tile (S = 3 * ftiles)
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < L::S; ++s) {
+        for (int s = 0; s < RS; ++s) {
             mbar_init(&bars->full[s], 1);
             mbar_init(&bars->opfull[s], 1);
             mbar_init(&bars->empty[s], 1);
@@ -570,9 +592,9 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (CG == 2 && threadIdx.x == 0 && e == 0)   // the leader's opfull gathers both CTAs' FT warps
-        for (int s = 0; s < L::S; ++s) mbar_init(&bars->opfull[s], 2);
+        for (int s = 0; s < RS; ++s) mbar_init(&bars->opfull[s], 2);
     if (TA && threadIdx.x == 0) {                // TA: the four lane-quarter warps of a group
-        for (int s = 0; s < L::S; ++s) mbar_init(&bars->opfull[s], 4);
+        for (int s = 0; s < RS; ++s) mbar_init(&bars->opfull[s], 4);
         for (int a = 0; a < 8; ++a) mbar_init(&bars->aempty[a], 1);
     }
     if (warp == 0 && lane == 0) {
@@ -632,7 +654,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
         // prefetched while stage ch - PF + S .. ch is being loaded, so their
         // TMA loads later hit L2 instead of waiting the HBM round trip.
         constexpr int PF = TA ? WINRS_TC2_PF : 0;
-        int pch = c_lo + pp + L::S;
+        int pch = c_lo + pp + RS;
         long long pd = (long long)pch * KC;
         int pn = 0, ph_ = hs, pu = 0;
         ImgTracker pitk;
@@ -674,7 +696,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             TC2_JITTER(ch, 0);
             TC2_TRACE(ch - c_lo, 0);
             uint64_t* fb = &bars->full[s];
-            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            const uint32_t st = sbase + (uint32_t)(s * RSTAGE);
             const bool in = d < depth;               // past the end: outer image coordinate out of range (zero fill)
             const ImgCoord ic = itk.at(g, in);
             const int hh = in ? h : hs;
@@ -700,7 +722,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 }
 #pragma unroll
                 for (int ka = 0; ka < L::NKL / 64; ++ka)   // dY unit columns w0, w0 + 1 of k atom ka
-                    tma5(st + L::OFF_Y + ka * L::Y_LBO, &tmY, fb, k_base + ka * 64, ic.a, ic.b, hh, w0);
+                    tma5(st + OFFY + ka * L::Y_LBO, &tmY, fb, k_base + ka * 64, ic.a, ic.b, hh, w0);
 #endif
             }
             __syncwarp();
@@ -715,7 +737,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             }
             itk.advance(2 * KC, wrapped, n);
             s += 2;
-            if (s >= L::S) { s -= L::S; ph ^= 1; }
+            if (s >= RS) { s -= RS; ph ^= 1; }
         }
     } else if (warp == 1) {
         // ============================ MMA issuer ==============================
@@ -730,17 +752,17 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
             TC2_JITTER(ch, 1);
             TC2_TRACE(ch - c_lo, 4);
             tc_after();
-            const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
+            const uint32_t st = sbase + (uint32_t)(s * RSTAGE);
             const uint32_t acc = ch > c_lo ? 1u : 0u;
             // A: raw X column x_t (M = 128: two atoms X_LBO apart); B: What[xi]
             const uint64_t x0 = desc_sw128(st, L::X_LBO, 1024);
             const uint64_t x1 = x0 + (L::ATOM >> 4), x2 = x0 + (2 * L::ATOM >> 4), x3 = x0 + (3 * L::ATOM >> 4);
-            const uint64_t w0d = desc_sw128(st + L::OFF_F, L::Y_LBO, 1024), w1d = w0d + (L::ATOM >> 4);
-            const uint64_t w2d = desc_sw128(st + L::OFF_Y, L::Y_LBO, 1024), w3d = w2d + (L::ATOM >> 4);
+            const uint64_t w0d = desc_sw128(st + OFFF, L::Y_LBO, 1024), w1d = w0d + (L::ATOM >> 4);
+            const uint64_t w2d = desc_sw128(st + OFFY, L::Y_LBO, 1024), w3d = w2d + (L::ATOM >> 4);
             if (elect_one()) {
 #ifndef WINRS_TC2_NO_MMA   // debug ablation: no tensor-core work (barrier protocol kept)
               if (TA) {               // Xhat[xi] from the TMEM ring slot x What[xi]
-                const int aslot = ASEP ? (ch - c_lo) % 8 : s;
+                const int aslot = asep ? (ch - c_lo) % 8 : s;
                 const uint32_t a = tmem + A_COL + (uint32_t)(aslot * 32);
                 umma_ta<NK, BF>(tmem + 0 * NK, a + 0, w0d, acc);
                 umma_ta<NK, BF>(tmem + 1 * NK, a + 8, w1d, acc);
@@ -765,11 +787,11 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 (void)x0; (void)x1; (void)x2; (void)x3; (void)w0d; (void)w1d; (void)w2d; (void)w3d; (void)acc;
 #endif
                 umma_commit<CG>(&bars->empty[s], pair_mask);
-                if (ASEP) umma_commit<1>(&bars->aempty[(ch - c_lo) % 8]);
+                if (asep) umma_commit<1>(&bars->aempty[(ch - c_lo) % 8]);
             }
             __syncwarp();
             TC2_TRACE(ch - c_lo, 5);
-            if (++s == L::S) { s = 0; ph ^= 1; }
+            if (++s == RS) { s = 0; ph ^= 1; }
         }
         if (elect_one()) umma_commit<CG>(&bars->accfull, pair_mask);   // arrives once all issued MMAs completed
         __syncwarp();
@@ -834,9 +856,9 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 tc_after();
                 TC2_JITTER(ch, warp);
                 if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 2);
-                const uint32_t st = sbase + (uint32_t)(s * L::STAGE);
-                const int aslot = ASEP ? (ch - c_lo) % 8 : s;
-                if (ASEP && ch - c_lo >= 8)   // the MMAs of stage ch - 8 read this A slot
+                const uint32_t st = sbase + (uint32_t)(s * RSTAGE);
+                const int aslot = asep ? (ch - c_lo) % 8 : s;
+                if (asep && ch - c_lo >= 8)   // the MMAs of stage ch - 8 read this A slot
                     mbar_wait(&bars->aempty[aslot], (uint32_t)(((ch - c_lo) / 8 - 1) & 1));
 #pragma unroll
                 for (int hf = 0; hf < 2 && !xdead; ++hf) {
@@ -863,9 +885,9 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                     asm volatile("" :: "r"(o[0][0] ^ o[1][1] ^ o[2][2] ^ o[3][3] ^ ta));
 #endif
                 }
-                const uint4 w0 = lds16(st + L::OFF_Y + foff), w1 = lds16(st + L::OFF_Y + L::ATOM + foff);
-                sts16(st + L::OFF_F + foff, vadd<BF>(w0, w1));
-                sts16(st + L::OFF_F + L::ATOM + foff, vsub<BF>(w0, w1));
+                const uint4 w0 = lds16(st + OFFY + foff), w1 = lds16(st + OFFY + L::ATOM + foff);
+                sts16(st + OFFF + foff, vadd<BF>(w0, w1));
+                sts16(st + OFFF + L::ATOM + foff, vsub<BF>(w0, w1));
                 tmem_wait_st();
                 fence_async();
                 tc_before();
@@ -873,7 +895,7 @@ bfc_tc2_kernel(const __grid_constant__ Args args, const __grid_constant__ CUtens
                 if (lane == 0) mbar_arrive(&bars->opfull[s]);
                 if (tw == 0 && lane == 0) TC2_TRACE(ch - c_lo, 3);
                 s += NG;
-                if (s >= L::S) { s -= L::S; ph ^= 1; }
+                if (s >= RS) { s -= RS; ph ^= 1; }
             }
         } else {
         uint32_t ph = 0;
